@@ -1,0 +1,199 @@
+"""CPU oracle for the RecFlex hot path -- TEST INFRASTRUCTURE ONLY.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s
+``cpu_baseline`` / ``--impl reference`` legs may import this package.  The
+product path never imports it and shares no code with it.
+
+The arithmetic lives in ``oracle.c`` (plain C, fp64 accumulation); this file
+only builds it with gcc, marshals numpy arrays through ctypes and, for the
+full-size sampled checks, extracts the bags to check into a compact sub-batch
+(pure input selection -- the pooled values are still computed by the C code).
+
+Functions and the passages they follow (PAPER.md "P:n"):
+  embedding_bag  -- P:41, P:51 (§II-A): gather the rows named by each sample's
+                    lookup IDs, pool them by elementwise reduction, concatenate
+                    per-feature outputs.  Readings C1, C2, C6.
+  task_map       -- Fig. 8: d_blocks_map and d_task_map, reading C12.
+  nnz_task_ranges-- reading C12 for nnz-partitioned schedules.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+import threading
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, 'oracle.c')
+_LIB = os.path.join(_HERE, 'liboracle.so')
+_lock = threading.Lock()
+_lib = None
+
+POOL_SUM = 0
+POOL_MEAN = 1
+
+
+def build(force: bool = False) -> str:
+    """Compile oracle.c -> liboracle.so (gcc -O2 -fopenmp, no fast-math)."""
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        tmp = _LIB + f'.tmp{os.getpid()}'
+        subprocess.check_call(['gcc', '-O2', '-fopenmp', '-fPIC', '-shared', '-std=c11', '-Wall',
+                               '-o', tmp, _SRC])
+        os.replace(tmp, _LIB)
+    return _LIB
+
+
+def lib():
+    global _lib
+    with _lock:
+        if _lib is None:
+            build()
+            L = ctypes.CDLL(_LIB)
+            P = ctypes.POINTER
+            L.oracle_embedding_bag.restype = ctypes.c_int
+            L.oracle_embedding_bag.argtypes = [
+                ctypes.c_int, ctypes.c_int, P(ctypes.c_int), P(ctypes.c_int),
+                P(ctypes.c_void_p), P(ctypes.c_int64), P(ctypes.c_int32), P(ctypes.c_int32),
+                P(ctypes.c_double), ctypes.c_int]
+            L.oracle_task_map.restype = ctypes.c_int
+            L.oracle_task_map.argtypes = [
+                ctypes.c_int, ctypes.c_int, P(ctypes.c_int), P(ctypes.c_int), P(ctypes.c_int),
+                P(ctypes.c_int32), P(ctypes.c_int), P(ctypes.c_int), P(ctypes.c_int),
+                ctypes.c_int64, P(ctypes.c_int64)]
+            L.oracle_nnz_task_ranges.restype = ctypes.c_int
+            L.oracle_nnz_task_ranges.argtypes = [
+                ctypes.c_int, ctypes.c_int, P(ctypes.c_int32), ctypes.c_int, P(ctypes.c_int), P(ctypes.c_int)]
+            L.oracle_max_threads.restype = ctypes.c_int
+            _lib = L
+    return _lib
+
+
+def _ptr(a, ct):
+    return a.ctypes.data_as(ctypes.POINTER(ct))
+
+
+class OracleError(RuntimeError):
+    pass
+
+
+def max_threads() -> int:
+    return int(lib().oracle_max_threads())
+
+
+def embedding_bag(tables, dims, pools, indices, offsets, B, nthreads: int = 0) -> np.ndarray:
+    """fp64 pooled output [B][sum(dims)].
+
+    tables: list of F float32 arrays [rows_f][d_f] (one per feature; aliasing allowed)
+    """
+    F = len(dims)
+    tabs = [np.ascontiguousarray(t, dtype=np.float32) for t in tables]
+    for f in range(F):
+        if tabs[f].ndim != 2 or tabs[f].shape[1] != dims[f]:
+            raise ValueError(f'table {f} shape {tabs[f].shape} vs dim {dims[f]}')
+    dims_a = np.asarray(dims, np.intc)
+    pools_a = np.asarray(pools, np.intc)
+    rows_a = np.asarray([t.shape[0] for t in tabs], np.int64)
+    ptrs = (ctypes.c_void_p * F)(*[t.ctypes.data for t in tabs])
+    idx = np.ascontiguousarray(indices, np.int32)
+    off = np.ascontiguousarray(offsets, np.int32)
+    if off.shape[0] != F * B + 1:
+        raise ValueError('offsets must have F*B+1 entries')
+    out = np.zeros((B, int(dims_a.sum())), np.float64)
+    if idx.size == 0:
+        idx = np.zeros(1, np.int32)
+    rc = lib().oracle_embedding_bag(F, B, _ptr(dims_a, ctypes.c_int), _ptr(pools_a, ctypes.c_int),
+                                    ptrs, _ptr(rows_a, ctypes.c_int64), _ptr(idx, ctypes.c_int32),
+                                    _ptr(off, ctypes.c_int32), _ptr(out, ctypes.c_double), int(nthreads))
+    if rc != 0:
+        raise OracleError({-1: 'index out of range', -2: 'bad offsets', -3: 'bad argument'}.get(rc, rc))
+    return out
+
+
+def task_map(B, mode, per_block, offsets, cap=None):
+    """Fig. 8 arrays: (blocks_map[F], task_feature[T], task_rel[T])."""
+    F = len(mode)
+    mode_a = np.asarray(mode, np.intc)
+    pb = np.asarray(per_block, np.intc)
+    cap_a = np.asarray(cap if cap is not None else [0] * F, np.intc)
+    off = np.ascontiguousarray(offsets, np.int32)
+    # upper bound on tasks for the output buffers
+    ub = 0
+    for f in range(F):
+        if mode[f] == 0:
+            ub += (B + pb[f] - 1) // pb[f]
+        else:
+            ub += (int(off[(f + 1) * B]) - int(off[f * B])) // pb[f] + 1
+    ub = max(ub, 1)
+    blocks = np.zeros(F, np.intc)
+    tf = np.zeros(ub, np.intc)
+    tr = np.zeros(ub, np.intc)
+    n = ctypes.c_int64(0)
+    rc = lib().oracle_task_map(F, B, _ptr(mode_a, ctypes.c_int), _ptr(pb, ctypes.c_int),
+                               _ptr(cap_a, ctypes.c_int), _ptr(off, ctypes.c_int32),
+                               _ptr(blocks, ctypes.c_int), _ptr(tf, ctypes.c_int), _ptr(tr, ctypes.c_int),
+                               ub, ctypes.byref(n))
+    if rc != 0:
+        raise OracleError(rc)
+    return blocks, tf[:n.value].copy(), tr[:n.value].copy()
+
+
+def block_start_from_task_map(F, task_feature):
+    """Exclusive-scan view of d_task_map: first task index of every feature, plus total."""
+    counts = np.bincount(np.asarray(task_feature, np.int64), minlength=F)[:F]
+    bs = np.zeros(F + 1, np.int64)
+    np.cumsum(counts, out=bs[1:])
+    return bs
+
+
+def nnz_task_ranges(B, npb, feature_offsets, blocks):
+    off = np.ascontiguousarray(feature_offsets, np.int32)
+    s0 = np.zeros(max(blocks, 1), np.intc)
+    s1 = np.zeros(max(blocks, 1), np.intc)
+    rc = lib().oracle_nnz_task_ranges(int(B), int(npb), _ptr(off, ctypes.c_int32), int(blocks),
+                                      _ptr(s0, ctypes.c_int), _ptr(s1, ctypes.c_int))
+    if rc != 0:
+        raise OracleError(rc)
+    return s0[:blocks].copy(), s1[:blocks].copy()
+
+
+# ---------------------------------------------------------------------------
+# Full-size sampled checks: compute selected samples one by one.
+# ---------------------------------------------------------------------------
+
+def sampled_forward(model, batch, samples, table_getter):
+    """Oracle output rows for the given sample ids of a (possibly huge) batch.
+
+    table_getter(feature_index, unique_row_ids) -> float32 [n][d_f] rows of that
+    feature's table (from the seeded generator).  Returns fp64 [len(samples)][D_tot]
+    and the per-(sample, feature) bag lengths [len(samples)][F].
+    """
+    F, B = batch.F, batch.B
+    samples = np.asarray(samples, np.int64)
+    S = samples.size
+    offs = batch.offsets.astype(np.int64)
+    sub_off = [0]
+    sub_idx = []
+    tables = []
+    lens = np.zeros((S, F), np.int64)
+    for f in range(F):
+        bags = []
+        for k, s in enumerate(samples):
+            a, b = offs[f * B + s], offs[f * B + s + 1]
+            bags.append(batch.indices[a:b])
+            lens[k, f] = b - a
+        allids = np.concatenate(bags) if bags else np.zeros(0, np.int32)
+        uniq, inv = np.unique(allids, return_inverse=True)
+        if uniq.size == 0:
+            uniq = np.zeros(1, np.int64)
+        tables.append(np.asarray(table_getter(f, uniq), np.float32).reshape(uniq.size, model.features[f].dim))
+        pos = 0
+        for bag in bags:
+            sub_idx.append(inv[pos:pos + bag.size].astype(np.int32))
+            pos += bag.size
+            sub_off.append(sub_off[-1] + bag.size)
+    idx = np.concatenate(sub_idx) if sub_idx else np.zeros(0, np.int32)
+    off = np.asarray(sub_off, np.int32)
+    out = embedding_bag(tables, model.dims, [f.pool for f in model.features], idx, off, S)
+    return out, lens

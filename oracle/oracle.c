@@ -1,0 +1,190 @@
+/*
+ * oracle.c -- CPU oracle for the RecFlex hot path.
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and
+ * bench.py's cpu_baseline / --impl reference legs may load this library.
+ * The product path (paper_conf_sc_panzzxwslr0d24_b200/) never links,
+ * imports or calls it, and shares no code, header or constant with it.
+ *
+ * Plain, slow, obviously correct: fp64 accumulation, loops in the order the
+ * definition states, no blocking, no fusion, no reordering.
+ *
+ * Functions and the passages they follow (PAPER.md line numbers, "P:n"):
+ *
+ *   oracle_embedding_bag  -- the embedding-bag operation, P:41 (§II-A, Fig. 1)
+ *       and P:51: "An input sample of the operation consists of single or
+ *       multiple lookup IDs, which are used to retrieve corresponding rows in
+ *       the embedding table.  Then, the retrieved embedding vectors of the
+ *       same sample will be applied by a pooling operation (i.e., elementwise
+ *       reduction)"; per-feature outputs "are then concatenated".
+ *       Readings: C1 pool = SUM or MEAN, empty bag -> 0;
+ *       C2 duplicate IDs counted with multiplicity; C6 output row-major
+ *       [B][D_tot], feature f at column col_f = sum_{g<f} d_g.
+ *       Pinned by tests/test_oracle.py (worked example in tests/golden,
+ *       torch.nn.functional.embedding_bag, brute force, closed-form invariants).
+ *
+ *   oracle_task_map       -- the runtime thread map of Fig. 8:
+ *       d_blocks_map[f] = feature_blocks, and d_task_map[b] = (feature_idx,
+ *       rel_bidx) enumerating, feature by feature, rel = 0..feature_blocks-1.
+ *       feature_blocks follows reading C12 (blocks "adaptive" to the batch's
+ *       workload): sample-partitioned schedules take ceil(B/spb),
+ *       nnz-partitioned schedules take floor(nnz_f/npb) + 1; an optional cap
+ *       (tuning padding) limits it.  Pinned by brute-force enumeration
+ *       and invariants in tests/test_oracle.py.
+ *
+ *   oracle_nnz_task_ranges -- for an nnz-partitioned feature, the samples a
+ *       task owns: {s : floor((off[s]-off[0]) / npb) == rel}, written out by
+ *       brute force over s for every task (reading C12).
+ */
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+#ifdef _OPENMP
+#include <omp.h>
+#endif
+
+#define ORACLE_OK 0
+#define ORACLE_ERR_INDEX -1
+#define ORACLE_ERR_OFFSETS -2
+#define ORACLE_ERR_ARG -3
+
+#define POOL_SUM 0
+#define POOL_MEAN 1
+
+int oracle_version(void) { return 1; }
+
+int oracle_max_threads(void) {
+#ifdef _OPENMP
+    return omp_get_max_threads();
+#else
+    return 1;
+#endif
+}
+
+/*
+ * F features, batch B.
+ * dims[f], pools[f], rows[f]; tables[f] -> float32 [rows[f]][dims[f]] row-major.
+ * indices int32[nnz], offsets int32[F*B+1] (feature-major KJT CSR).
+ * out -> double [B][sum(dims)].
+ * nthreads <= 0: library default.
+ */
+int oracle_embedding_bag(int F, int B, const int *dims, const int *pools,
+                         const float *const *tables, const int64_t *rows,
+                         const int32_t *indices, const int32_t *offsets,
+                         double *out, int nthreads) {
+    if (F <= 0 || B < 0) return ORACLE_ERR_ARG;
+    int64_t d_tot = 0;
+    int64_t *col = (int64_t *)malloc(sizeof(int64_t) * (size_t)F);
+    if (!col) return ORACLE_ERR_ARG;
+    for (int f = 0; f < F; ++f) {          /* col_f = sum_{g<f} d_g  (P:41 concatenation) */
+        col[f] = d_tot;
+        d_tot += dims[f];
+    }
+    /* validate the CSR once, sequentially (reading C3: precondition) */
+    if (offsets[0] != 0) { free(col); return ORACLE_ERR_OFFSETS; }
+    for (int64_t k = 0; k < (int64_t)F * B; ++k)
+        if (offsets[k + 1] < offsets[k]) { free(col); return ORACLE_ERR_OFFSETS; }
+    for (int f = 0; f < F; ++f) {
+        int64_t a = offsets[(int64_t)f * B], b = offsets[(int64_t)(f + 1) * B];
+        for (int64_t j = a; j < b; ++j)
+            if (indices[j] < 0 || (int64_t)indices[j] >= rows[f]) { free(col); return ORACLE_ERR_INDEX; }
+    }
+#ifdef _OPENMP
+    if (nthreads > 0) omp_set_num_threads(nthreads);
+#else
+    (void)nthreads;
+#endif
+    /* features write disjoint output columns -> identical result for any thread count */
+#pragma omp parallel for schedule(dynamic)
+    for (int f = 0; f < F; ++f) {
+        const int d = dims[f];
+        const float *T = tables[f];
+        double *acc = (double *)malloc(sizeof(double) * (size_t)(d > 0 ? d : 1));
+        for (int s = 0; s < B; ++s) {
+            const int64_t lo = offsets[(int64_t)f * B + s];
+            const int64_t hi = offsets[(int64_t)f * B + s + 1];
+            const int64_t L = hi - lo;
+            for (int c = 0; c < d; ++c) acc[c] = 0.0;
+            for (int64_t j = lo; j < hi; ++j) {             /* ascending j */
+                const float *row = T + (int64_t)indices[j] * d;
+                for (int c = 0; c < d; ++c) acc[c] += (double)row[c];
+            }
+            double *o = out + (int64_t)s * d_tot + col[f];
+            for (int c = 0; c < d; ++c) {
+                if (pools[f] == POOL_MEAN)
+                    o[c] = (L > 0) ? acc[c] / (double)L : 0.0;   /* reading C1: empty -> 0 */
+                else
+                    o[c] = acc[c];
+            }
+        }
+        free(acc);
+    }
+    free(col);
+    return ORACLE_OK;
+}
+
+/*
+ * Task map of Fig. 8.
+ *   mode[f]: 0 = sample-partitioned (per_block[f] = samples per block)
+ *            1 = nnz-partitioned    (per_block[f] = lookups per block)
+ *   cap[f]:  0 = none, else feature_blocks = min(feature_blocks, cap[f])
+ * Outputs blocks_map[F] (d_blocks_map), task_feature/task_rel[max_tasks]
+ * (d_task_map .x/.y), *num_tasks.  Returns ORACLE_ERR_ARG if max_tasks is short.
+ */
+int oracle_task_map(int F, int B, const int *mode, const int *per_block, const int *cap,
+                    const int32_t *offsets, int *blocks_map, int *task_feature, int *task_rel,
+                    int64_t max_tasks, int64_t *num_tasks) {
+    int64_t n = 0;
+    for (int f = 0; f < F; ++f) {
+        int64_t blocks;
+        if (mode[f] == 0) {
+            blocks = ((int64_t)B + per_block[f] - 1) / per_block[f];
+        } else {
+            int64_t nnz_f = (int64_t)offsets[(int64_t)(f + 1) * B] - offsets[(int64_t)f * B];
+            blocks = nnz_f / per_block[f] + 1;
+            if (B == 0) blocks = 0;
+        }
+        if (cap && cap[f] > 0 && blocks > cap[f]) blocks = cap[f];
+        blocks_map[f] = (int)blocks;
+        for (int64_t rel = 0; rel < blocks; ++rel) {
+            if (n >= max_tasks) return ORACLE_ERR_ARG;
+            task_feature[n] = f;
+            task_rel[n] = (int)rel;
+            ++n;
+        }
+    }
+    *num_tasks = n;
+    return ORACLE_OK;
+}
+
+/*
+ * Sample range owned by each task of one nnz-partitioned feature:
+ * off -> the feature's B+1 offsets (absolute), npb lookups per block.
+ * For task q in [0, blocks): s0[q] = min{s : floor((off[s]-off[0])/npb) >= q}
+ * (B if none) and s1[q] = s0[q+1]-style end, computed by brute force as
+ * the first and one-past-last s whose floor equals q (empty range -> s0=s1).
+ */
+int oracle_nnz_task_ranges(int B, int npb, const int32_t *off, int blocks, int *s0, int *s1) {
+    for (int q = 0; q < blocks; ++q) {
+        int first = -1, last = -1;
+        for (int s = 0; s < B; ++s) {
+            int64_t t = ((int64_t)off[s] - off[0]) / npb;
+            if (t == q) {
+                if (first < 0) first = s;
+                last = s;
+            }
+        }
+        if (first < 0) {
+            /* no bag starts in this task: empty range positioned at the first later bag */
+            int pos = B;
+            for (int s = 0; s < B; ++s)
+                if (((int64_t)off[s] - off[0]) / npb > q) { pos = s; break; }
+            s0[q] = pos;
+            s1[q] = pos;
+        } else {
+            s0[q] = first;
+            s1[q] = last + 1;
+        }
+    }
+    return ORACLE_OK;
+}

@@ -1,0 +1,342 @@
+"""Seeded synthetic inputs shared by the CUDA path's tests/bench and the oracle.
+
+This module holds NONE of the method's arithmetic (no gather, no pooling, no
+thread mapping).  It only draws the inputs the paper says its data-synthesis
+script draws: per-feature pooling factors from a stated distribution, lookup
+IDs uniform over each table, and table contents (PAPER.md P:260, P:505 --
+"indices with specified pooling factor distribution and embedding table
+shape"; coverage as in Fig. 3).
+
+Readings:
+  C9  coverage c = P(L > 0); L = 0 w.p. 1-c, else a draw from the length model,
+      rounded half-to-even (numpy ``rint``) and clipped to [1, Lmax].
+  C10 lookup IDs i.i.d. uniform over [0, rows_f) with replacement.
+  C11 table contents are a counter-based hash of (table, row, column):
+        'float' mode -> U[-1, 1) on a 2^-23 grid (exactly representable in fp32)
+        'int'   mode -> integers in [-8, 7] (every fp32 partial sum is exact)
+      The hash uses only int64 ops whose products stay < 2^63, so torch on CPU
+      and torch on CUDA produce identical bits; any row can be regenerated on
+      the host for sampled oracle checks without copying it from the device.
+  C25 heavy: 100 fields whose 10M-row index ranges alias 16 physical tables.
+
+Layout produced (KJT feature-major CSR):
+  indices int32[nnz], offsets int32[F*B + 1]; bag (f, s) is
+  indices[offsets[f*B+s] : offsets[f*B+s+1]].
+"""
+from __future__ import annotations
+
+import dataclasses
+import math
+from typing import List, Optional
+
+import numpy as np
+
+POOL_SUM = 0
+POOL_MEAN = 1
+
+MODEL_SEED = 1234
+M32 = 0xFFFFFFFF
+
+
+@dataclasses.dataclass
+class Feature:
+    rows: int                 # index range of the field (== rows of its physical table)
+    dim: int
+    pool: int                 # POOL_SUM / POOL_MEAN
+    kind: str                 # 'onehot' | 'normal' | 'lognormal' | 'uniform' | 'fixed'
+    coverage: float = 1.0
+    mu: float = 1.0           # mean of the length model (normal / lognormal) or fixed L
+    sigma: float = 0.0        # normal: std; lognormal: sigma of log
+    lo: int = 0               # uniform model: L ~ U{lo..hi}
+    hi: int = 0
+    lmax: int = 1
+    table: int = 0            # physical table id (aliasing, C25)
+
+    # hotness stats an operator would pass to recflex_plan_create (from history)
+    def mean_len(self) -> float:
+        if self.kind == 'onehot':
+            return 1.0
+        if self.kind == 'uniform':
+            # E[L | L > 0] for U{lo..hi}
+            vals = [v for v in range(self.lo, self.hi + 1) if v > 0]
+            return float(sum(vals)) / max(1, len(vals))
+        if self.kind == 'fixed':
+            return float(self.mu)
+        return float(min(self.mu, self.lmax))
+
+    def max_len(self) -> float:
+        if self.kind == 'onehot':
+            return 1.0
+        if self.kind == 'uniform':
+            return float(self.hi)
+        if self.kind == 'fixed':
+            return float(self.mu)
+        return float(self.lmax)
+
+
+@dataclasses.dataclass
+class Model:
+    name: str
+    features: List[Feature]
+    tables: List[tuple]       # (rows, dim) per physical table
+    batch: int
+    seed: int = MODEL_SEED
+
+    @property
+    def F(self) -> int:
+        return len(self.features)
+
+    @property
+    def dims(self) -> List[int]:
+        return [f.dim for f in self.features]
+
+    @property
+    def d_tot(self) -> int:
+        return sum(self.dims)
+
+
+# ---------------------------------------------------------------------------
+# Model definitions (SURVEY §8d generator table; BASELINE.json "configs")
+# ---------------------------------------------------------------------------
+
+def _log_uniform(rng, lo, hi, size=None):
+    return np.exp(rng.uniform(math.log(lo), math.log(hi), size=size))
+
+
+def make_model(name: str, seed: int = MODEL_SEED) -> Model:
+    rng = np.random.Generator(np.random.PCG64([seed, _name_key(name)]))
+    feats: List[Feature] = []
+    if name == 'tiny':
+        # 4 fields (2 one-hot, 2 multi-hot L<=8 incl. empty bags), 1k rows, dim 16, sum, B=64
+        for f in range(4):
+            if f < 2:
+                feats.append(Feature(rows=1000, dim=16, pool=POOL_SUM, kind='onehot', coverage=1.0, lmax=1, table=f))
+            else:
+                feats.append(Feature(rows=1000, dim=16, pool=POOL_SUM, kind='uniform', lo=0, hi=8, lmax=8, table=f))
+        B = 64
+    elif name == 'medium':
+        # 50 fields alternating one-hot / multi-hot, dims cycle 16/32/64, 1M rows, sum, B=1024
+        for f in range(50):
+            dim = (16, 32, 64)[f % 3]
+            if f % 2 == 0:
+                feats.append(Feature(rows=1_000_000, dim=dim, pool=POOL_SUM, kind='onehot',
+                                     coverage=float(rng.uniform(0.9, 1.0)), lmax=1, table=f))
+            else:
+                mu = float(rng.uniform(5, 50))
+                feats.append(Feature(rows=1_000_000, dim=dim, pool=POOL_SUM, kind='normal', mu=mu, sigma=mu / 4,
+                                     coverage=float(rng.uniform(0.3, 1.0)), lmax=int(round(3 * mu)), table=f))
+        B = 1024
+    elif name == 'industrial':
+        # 300 fields (120 one-hot / 180 multi-hot), skewed lognormal lengths 1..200,
+        # dims {8,16,32,64,128} p=.3/.3/.2/.1/.1, rows log-uniform [1e4, 2e6], even f sum / odd f mean
+        onehot = set(rng.permutation(300)[:120].tolist())
+        for f in range(300):
+            dim = int(rng.choice([8, 16, 32, 64, 128], p=[.3, .3, .2, .1, .1]))
+            rows = int(_log_uniform(rng, 1e4, 2e6))
+            pool = POOL_SUM if f % 2 == 0 else POOL_MEAN
+            if f in onehot:
+                feats.append(Feature(rows=rows, dim=dim, pool=pool, kind='onehot',
+                                     coverage=float(rng.uniform(0.5, 1.0)), lmax=1, table=f))
+            else:
+                mu = float(_log_uniform(rng, 2, 200))
+                feats.append(Feature(rows=rows, dim=dim, pool=pool, kind='lognormal', mu=mu, sigma=0.9,
+                                     coverage=float(rng.uniform(0.3, 1.0)), lmax=200, table=f))
+        B = 4096
+    elif name == 'heavy':
+        # 100 multi-hot fields, lognormal mean 100 sigma .9 clipped [1,1000], coverage 1, dim 128,
+        # 10M-row index ranges aliased onto 16 physical tables (C25), sum, B=8192
+        for f in range(100):
+            feats.append(Feature(rows=10_000_000, dim=128, pool=POOL_SUM, kind='lognormal', mu=100.0, sigma=0.9,
+                                 coverage=1.0, lmax=1000, table=f % 16))
+        B = 8192
+    elif name == 'sharded1000':
+        # model-A-shaped 1000 fields (500/500), dims {4..128}, rows log-uniform [1e4, 1e6], sum, B=16384
+        onehot = set(rng.permutation(1000)[:500].tolist())
+        for f in range(1000):
+            dim = int(rng.choice([4, 8, 16, 32, 64, 128], p=[.1, .25, .25, .2, .1, .1]))
+            rows = int(_log_uniform(rng, 1e4, 1e6))
+            if f in onehot:
+                feats.append(Feature(rows=rows, dim=dim, pool=POOL_SUM, kind='onehot',
+                                     coverage=float(rng.uniform(0.5, 1.0)), lmax=1, table=f))
+            else:
+                mu = float(_log_uniform(rng, 2, 100))
+                feats.append(Feature(rows=rows, dim=dim, pool=POOL_SUM, kind='normal', mu=mu, sigma=mu / 4,
+                                     coverage=float(rng.uniform(0.3, 1.0)), lmax=max(1, int(round(3 * mu))),
+                                     table=f))
+        B = 16384
+    elif name == 'fig3':
+        # Fig. 3: two dim-32 fields; f0 N(50,10^2) at coverage 0.3, f1 fixed 50
+        feats.append(Feature(rows=1_000_000, dim=32, pool=POOL_SUM, kind='normal', mu=50, sigma=10,
+                             coverage=0.3, lmax=100, table=0))
+        feats.append(Feature(rows=1_000_000, dim=32, pool=POOL_SUM, kind='fixed', mu=50, lmax=50, table=1))
+        B = 512
+    else:
+        raise ValueError(f'unknown model {name!r}')
+    ntab = max(f.table for f in feats) + 1
+    tables = [None] * ntab
+    for f in feats:
+        tables[f.table] = (f.rows, f.dim)
+    return Model(name=name, features=feats, tables=tables, batch=B, seed=seed)
+
+
+def custom_model(name: str, features: List[Feature], batch: int) -> Model:
+    ntab = max(f.table for f in features) + 1
+    tables = [None] * ntab
+    for f in features:
+        if tables[f.table] is not None and tables[f.table] != (f.rows, f.dim):
+            raise ValueError('aliased features must share table shape')
+        tables[f.table] = (f.rows, f.dim)
+    return Model(name=name, features=features, tables=tables, batch=batch)
+
+
+CONFIG_NAMES = ('tiny', 'medium', 'industrial', 'heavy', 'sharded1000', 'fig3')
+
+
+def _name_key(name: str) -> int:
+    return sum((i + 1) * ord(ch) for i, ch in enumerate(name))
+
+
+# ---------------------------------------------------------------------------
+# Batches: pooling factors and lookup IDs
+# ---------------------------------------------------------------------------
+
+def _lengths(rng, feat: Feature, B: int) -> np.ndarray:
+    present = rng.random(B) < feat.coverage
+    if feat.kind == 'onehot':
+        L = np.ones(B, np.int64)
+    elif feat.kind == 'fixed':
+        L = np.full(B, int(feat.mu), np.int64)
+    elif feat.kind == 'uniform':
+        L = rng.integers(feat.lo, feat.hi + 1, size=B).astype(np.int64)
+        return L  # U{lo..hi} already includes empty bags (tiny config)
+    elif feat.kind == 'normal':
+        L = np.clip(np.rint(rng.normal(feat.mu, feat.sigma, size=B)), 1, feat.lmax).astype(np.int64)
+    elif feat.kind == 'lognormal':
+        m = math.log(feat.mu) - 0.5 * feat.sigma ** 2
+        L = np.clip(np.rint(np.exp(rng.normal(m, feat.sigma, size=B))), 1, feat.lmax).astype(np.int64)
+    else:
+        raise ValueError(feat.kind)
+    return np.where(present, L, 0)
+
+
+@dataclasses.dataclass
+class Batch:
+    indices: np.ndarray   # int32 [nnz]
+    offsets: np.ndarray   # int32 [F*B + 1]
+    B: int
+    F: int
+
+    @property
+    def nnz(self) -> int:
+        return int(self.offsets[-1])
+
+    def lengths(self) -> np.ndarray:
+        return np.diff(self.offsets.astype(np.int64)).reshape(self.F, self.B)
+
+
+def make_batch(model: Model, batch_seed: int = 7, B: Optional[int] = None) -> Batch:
+    """One synthetic batch (seed 7+i for the i-th batch)."""
+    B = model.batch if B is None else int(B)
+    rng = np.random.Generator(np.random.PCG64([model.seed, _name_key(model.name), batch_seed]))
+    F = model.F
+    lens = np.empty((F, B), np.int64)
+    for f, feat in enumerate(model.features):
+        lens[f] = _lengths(rng, feat, B)
+    offsets = np.zeros(F * B + 1, np.int64)
+    np.cumsum(lens.reshape(-1), out=offsets[1:])
+    nnz = int(offsets[-1])
+    if nnz >= 2 ** 31:
+        raise ValueError('nnz exceeds int32 (reading C4)')
+    indices = np.empty(nnz, np.int32)
+    for f, feat in enumerate(model.features):
+        a, b = int(offsets[f * B]), int(offsets[(f + 1) * B])
+        if b > a:
+            indices[a:b] = rng.integers(0, feat.rows, size=b - a, dtype=np.int64).astype(np.int32)
+    return Batch(indices=indices, offsets=offsets.astype(np.int32), B=B, F=F)
+
+
+def batch_from_lengths(lengths: np.ndarray, rows: List[int], seed: int = 0) -> Batch:
+    """Hand-shaped batch: lengths[F][B] given, IDs uniform (for edge-case tests)."""
+    lengths = np.asarray(lengths, np.int64)
+    F, B = lengths.shape
+    rng = np.random.Generator(np.random.PCG64(seed))
+    offsets = np.zeros(F * B + 1, np.int64)
+    np.cumsum(lengths.reshape(-1), out=offsets[1:])
+    indices = np.empty(int(offsets[-1]), np.int32)
+    for f in range(F):
+        a, b = int(offsets[f * B]), int(offsets[(f + 1) * B])
+        indices[a:b] = rng.integers(0, rows[f], size=b - a).astype(np.int32)
+    return Batch(indices=indices, offsets=offsets.astype(np.int32), B=B, F=F)
+
+
+# ---------------------------------------------------------------------------
+# Table contents: counter-based hash (identical on CPU and CUDA)
+# ---------------------------------------------------------------------------
+
+_K1 = 0x7FEB352D
+_K2 = 0x6C8E9CF5
+
+
+def _mix32(x):
+    """32-bit avalanche on a non-negative int64 tensor holding values < 2^32."""
+    x = x ^ (x >> 16)
+    x = (x * _K1) & M32
+    x = x ^ (x >> 15)
+    x = (x * _K2) & M32
+    x = x ^ (x >> 16)
+    return x
+
+
+def table_rows(table_id: int, row_start: int, row_end: int, dim: int, mode: str = 'float',
+               device='cpu', seed: int = MODEL_SEED):
+    """Rows [row_start, row_end) of physical table ``table_id`` as a float32 torch tensor."""
+    import torch
+    r = torch.arange(row_start, row_end, dtype=torch.int64, device=device)
+    h0 = _mix32(torch.tensor(((table_id * 0x27D4EB2F) + (seed * 0x165667B1)) & M32, dtype=torch.int64,
+                             device=device))
+    h1 = _mix32((h0 ^ (r & M32)) & M32)                      # [rows]
+    c = torch.arange(dim, dtype=torch.int64, device=device)
+    ck = (c * 0x61C88647) & M32                               # [dim]
+    h2 = _mix32((h1[:, None] + ck[None, :]) & M32)            # [rows, dim]
+    if mode == 'float':
+        out = (h2 >> 8).to(torch.float64) * (2.0 ** -23) - 1.0
+    elif mode == 'int':
+        out = ((h2 >> 28) - 8).to(torch.float64)
+    else:
+        raise ValueError(mode)
+    return out.to(torch.float32)
+
+
+def make_table(table_id: int, rows: int, dim: int, mode: str = 'float', device='cpu',
+               seed: int = MODEL_SEED, chunk_rows: Optional[int] = None):
+    import torch
+    out = torch.empty((rows, dim), dtype=torch.float32, device=device)
+    if chunk_rows is None:
+        chunk_rows = max(1, (1 << 25) // max(1, dim))
+    for a in range(0, rows, chunk_rows):
+        b = min(rows, a + chunk_rows)
+        out[a:b] = table_rows(table_id, a, b, dim, mode, device, seed)
+    return out
+
+
+def make_tables(model: Model, mode: str = 'float', device='cpu'):
+    """Physical tables of a model (list indexed by table id)."""
+    return [make_table(t, rows, dim, mode, device, model.seed) for t, (rows, dim) in enumerate(model.tables)]
+
+
+# ---------------------------------------------------------------------------
+# Byte accounting (C26): what the method must move per batch
+# ---------------------------------------------------------------------------
+
+def algorithmic_bytes(model: Model, batch: Batch) -> dict:
+    """indices + gathered rows + outputs (reading C26); offsets reported apart."""
+    F, B = batch.F, batch.B
+    offs = batch.offsets.astype(np.int64)
+    nnz_f = offs[np.arange(1, F + 1) * B] - offs[np.arange(0, F) * B]
+    dims = np.asarray(model.dims, np.int64)
+    idx_b = 4 * int(nnz_f.sum())
+    row_b = 4 * int((dims * nnz_f).sum())
+    out_b = 4 * B * int(dims.sum())
+    off_b = 4 * (F * B + 1)
+    return {'index': idx_b, 'rows': row_b, 'out': out_b, 'offsets': off_b,
+            'total': idx_b + row_b + out_b}

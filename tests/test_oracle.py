@@ -1,0 +1,300 @@
+"""Pins for the CPU oracle (no GPU).  Each test names what fixes the value
+independently of the oracle's own code: the paper's definition worked by hand
+(tests/golden), a library routine (torch embedding_bag in fp64), brute force
+in Python loops, or a closed-form invariant."""
+import json
+import os
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from paper_conf_sc_panzzxwslr0d24_b200 import synth
+
+GOLD = os.path.join(os.path.dirname(__file__), 'golden', 'worked_example.json')
+
+
+def _gold():
+    with open(GOLD) as fh:
+        return json.load(fh)
+
+
+# ---------------------------------------------------------------- worked examples (hand-computed)
+
+@pytest.mark.parametrize('pool', [0, 1])
+def test_worked_example_single_feature(pool):
+    g = _gold()['single_feature']
+    T = np.asarray(g['table'], np.float32)
+    out = oracle.embedding_bag([T], [4], [pool], g['indices'], g['offsets'], g['B'])
+    if pool == 0:
+        exp = np.asarray(g['sum'], np.float64)
+    else:
+        exp = np.asarray(g['mean_num'], np.float64) / np.asarray(g['mean_den'], np.float64)
+        exp[1] = 0.0  # empty bag -> 0 (reading C1)
+    assert np.array_equal(out, exp)
+
+
+def test_worked_example_two_features_concat():
+    g = _gold()['two_features']
+    tabs = [np.asarray(t, np.float32) for t in g['tables']]
+    out = oracle.embedding_bag(tabs, g['dims'], g['pools'], g['indices'], g['offsets'], g['B'])
+    exp = np.asarray(g['out_num'], np.float64) / np.asarray(g['out_den'], np.float64)
+    assert np.array_equal(out, exp)
+
+
+def test_worked_task_map_p338():
+    g = _gold()['task_map_static_example']
+    F = len(g['mode'])
+    off = np.zeros(F * g['B'] + 1, np.int32)
+    blocks, tf, tr = oracle.task_map(g['B'], g['mode'], g['per_block'], off)
+    assert blocks.tolist() == g['blocks_map']
+    assert tf.tolist() == g['task_feature']
+    assert tr.tolist() == g['task_rel']
+
+
+# ---------------------------------------------------------------- library routine: torch embedding_bag fp64
+
+def _torch_ref(tables, dims, pools, indices, offsets, B):
+    F = len(dims)
+    outs = []
+    for f in range(F):
+        off = torch.as_tensor(offsets[f * B:(f + 1) * B + 1].astype(np.int64))
+        base = int(off[0])
+        idx = torch.as_tensor(indices[base:int(off[-1])].astype(np.int64))
+        W = torch.as_tensor(np.asarray(tables[f], np.float64))
+        mode = 'sum' if pools[f] == 0 else 'mean'
+        outs.append(torch.nn.functional.embedding_bag(idx, W, off - base, mode=mode,
+                                                      include_last_offset=True).numpy())
+    return np.concatenate(outs, axis=1)
+
+
+@pytest.mark.parametrize('name', ['tiny', 'fig3'])
+def test_vs_torch_embedding_bag_configs(name):
+    m = synth.make_model(name)
+    b = synth.make_batch(m, 7, B=min(m.batch, 256))
+    tabs_np = []
+    for f in m.features:
+        tabs_np.append(synth.make_table(f.table, min(f.rows, 5000), f.dim).numpy())
+    # keep ids in range of the truncated tables
+    idx = b.indices % np.int32(5000)   # keep ids inside the truncated tables
+    pools = [f.pool for f in m.features]
+    out = oracle.embedding_bag(tabs_np, m.dims, pools, idx, b.offsets, b.B)
+    ref = _torch_ref(tabs_np, m.dims, pools, idx, b.offsets, b.B)
+    np.testing.assert_allclose(out, ref, rtol=1e-12, atol=1e-12)
+
+
+def test_vs_torch_embedding_bag_mixed_dims_pools():
+    rng = np.random.default_rng(3)
+    F, B = 7, 37
+    dims = [4, 8, 12, 16, 3, 128, 1]
+    pools = [0, 1, 0, 1, 1, 0, 1]
+    rows = [11, 50, 7, 300, 5, 64, 9]
+    lens = rng.integers(0, 9, size=(F, B))
+    lens[2, :5] = 0
+    b = synth.batch_from_lengths(lens, rows, seed=5)
+    tabs = [rng.standard_normal((rows[f], dims[f])).astype(np.float32) for f in range(F)]
+    out = oracle.embedding_bag(tabs, dims, pools, b.indices, b.offsets, B)
+    ref = _torch_ref(tabs, dims, pools, b.indices, b.offsets, B)
+    np.testing.assert_allclose(out, ref, rtol=1e-12, atol=1e-12)
+
+
+# ---------------------------------------------------------------- brute force (pure Python loops)
+
+def test_brute_force_tiny():
+    rng = np.random.default_rng(11)
+    F, B = 3, 5
+    dims = [2, 3, 4]
+    pools = [1, 0, 1]
+    rows = [4, 6, 3]
+    tabs = [rng.integers(-5, 6, size=(rows[f], dims[f])).astype(np.float32) for f in range(F)]
+    lens = rng.integers(0, 4, size=(F, B))
+    b = synth.batch_from_lengths(lens, rows, seed=2)
+    out = oracle.embedding_bag(tabs, dims, pools, b.indices, b.offsets, B)
+    D = sum(dims)
+    exp = [[0.0] * D for _ in range(B)]
+    col = 0
+    for f in range(F):
+        for s in range(B):
+            a, e = int(b.offsets[f * B + s]), int(b.offsets[f * B + s + 1])
+            for c in range(dims[f]):
+                acc = 0.0
+                for j in range(a, e):
+                    acc += float(tabs[f][int(b.indices[j])][c])
+                if pools[f] == 1:
+                    acc = acc / (e - a) if e > a else 0.0
+                exp[s][col + c] = acc
+        col += dims[f]
+    assert np.array_equal(out, np.asarray(exp))
+
+
+# ---------------------------------------------------------------- closed-form invariants
+
+def _rand_case(seed=0, F=4, B=20, maxlen=6, dims=(4, 8, 16, 5), rows=(10, 20, 30, 7)):
+    rng = np.random.default_rng(seed)
+    lens = rng.integers(0, maxlen + 1, size=(F, B))
+    b = synth.batch_from_lengths(lens, list(rows), seed=seed + 1)
+    tabs = [rng.uniform(-1, 1, size=(rows[f], dims[f])).astype(np.float32) for f in range(F)]
+    return b, tabs, list(dims)
+
+
+def test_one_hot_is_row_copy():
+    b, tabs, dims = _rand_case(maxlen=1)
+    lens = b.lengths()
+    out = oracle.embedding_bag(tabs, dims, [0] * 4, b.indices, b.offsets, b.B)
+    col = np.cumsum([0] + dims)
+    for f in range(4):
+        for s in range(b.B):
+            a = int(b.offsets[f * b.B + s])
+            piece = out[s, col[f]:col[f + 1]]
+            if lens[f, s] == 1:
+                assert np.array_equal(piece, tabs[f][b.indices[a]].astype(np.float64))
+            else:
+                assert np.all(piece == 0.0)
+
+
+def test_empty_bags_zero_both_pools():
+    F, B = 2, 6
+    lens = np.zeros((F, B), np.int64)
+    b = synth.batch_from_lengths(lens, [3, 3])
+    tabs = [np.ones((3, 4), np.float32)] * 2
+    for pool in (0, 1):
+        out = oracle.embedding_bag(tabs, [4, 4], [pool, pool], b.indices, b.offsets, B)
+        assert np.all(out == 0.0) and not np.any(np.isnan(out))
+
+
+def test_mean_is_sum_over_len():
+    b, tabs, dims = _rand_case(seed=4)
+    s = oracle.embedding_bag(tabs, dims, [0] * 4, b.indices, b.offsets, b.B)
+    m = oracle.embedding_bag(tabs, dims, [1] * 4, b.indices, b.offsets, b.B)
+    lens = b.lengths()
+    col = np.cumsum([0] + dims)
+    for f in range(4):
+        L = lens[f][:, None].astype(np.float64)
+        exp = np.where(L > 0, s[:, col[f]:col[f + 1]] / np.maximum(L, 1), 0.0)
+        assert np.array_equal(m[:, col[f]:col[f + 1]], exp)
+
+
+def test_linearity_scaling_by_two_exact():
+    b, tabs, dims = _rand_case(seed=5)
+    o1 = oracle.embedding_bag(tabs, dims, [0, 1, 0, 1], b.indices, b.offsets, b.B)
+    o2 = oracle.embedding_bag([2 * t for t in tabs], dims, [0, 1, 0, 1], b.indices, b.offsets, b.B)
+    assert np.array_equal(o2, 2 * o1)
+
+
+def test_permutation_within_bag_invariant_integer_tables():
+    rng = np.random.default_rng(6)
+    b, tabs, dims = _rand_case(seed=6, maxlen=9)
+    tabs = [np.round(t * 8).astype(np.float32) for t in tabs]   # integer values -> exact fp64 sums
+    o1 = oracle.embedding_bag(tabs, dims, [0, 1, 0, 1], b.indices, b.offsets, b.B)
+    idx2 = b.indices.copy()
+    for k in range(b.F * b.B):
+        a, e = int(b.offsets[k]), int(b.offsets[k + 1])
+        idx2[a:e] = rng.permutation(idx2[a:e])
+    o2 = oracle.embedding_bag(tabs, dims, [0, 1, 0, 1], idx2, b.offsets, b.B)
+    assert np.array_equal(o1, o2)
+
+
+def test_batch_split_invariance():
+    b, tabs, dims = _rand_case(seed=7, B=24)
+    full = oracle.embedding_bag(tabs, dims, [0, 1, 1, 0], b.indices, b.offsets, b.B)
+    # split samples [0,10) and [10,24): rebuild each half's KJT from the full one
+    for lo, hi in ((0, 10), (10, 24)):
+        Bh = hi - lo
+        idx, off = [], [0]
+        for f in range(b.F):
+            for s in range(lo, hi):
+                a, e = int(b.offsets[f * b.B + s]), int(b.offsets[f * b.B + s + 1])
+                idx.extend(b.indices[a:e].tolist())
+                off.append(off[-1] + e - a)
+        part = oracle.embedding_bag(tabs, dims, [0, 1, 1, 0], np.asarray(idx, np.int32),
+                                    np.asarray(off, np.int32), Bh)
+        assert np.array_equal(part, full[lo:hi])
+
+
+def test_integer_mode_tables_give_exact_integers():
+    m = synth.make_model('tiny')
+    b = synth.make_batch(m, 7)
+    tabs = [synth.make_table(f.table, f.rows, f.dim, mode='int').numpy() for f in m.features]
+    assert all(t.min() >= -8 and t.max() <= 7 for t in tabs)
+    out = oracle.embedding_bag(tabs, m.dims, [0] * 4, b.indices, b.offsets, b.B)
+    assert np.array_equal(out, np.round(out))
+
+
+def test_duplicate_ids_counted_with_multiplicity():
+    T = np.arange(12, dtype=np.float32).reshape(3, 4)
+    out = oracle.embedding_bag([T], [4], [0], [1, 1, 1], [0, 3], 1)
+    assert np.array_equal(out[0], 3 * T[1].astype(np.float64))
+
+
+def test_out_of_range_index_rejected():
+    T = np.zeros((3, 4), np.float32)
+    with pytest.raises(oracle.OracleError):
+        oracle.embedding_bag([T], [4], [0], [3], [0, 1], 1)
+    with pytest.raises(oracle.OracleError):
+        oracle.embedding_bag([T], [4], [0], [0, 1], [0, 2, 1], 2)
+
+
+def test_thread_count_does_not_change_result():
+    b, tabs, dims = _rand_case(seed=8, B=64)
+    o1 = oracle.embedding_bag(tabs, dims, [0, 1, 0, 1], b.indices, b.offsets, b.B, nthreads=1)
+    o4 = oracle.embedding_bag(tabs, dims, [0, 1, 0, 1], b.indices, b.offsets, b.B, nthreads=4)
+    assert np.array_equal(o1, o4)
+
+
+# ---------------------------------------------------------------- task map (Fig. 8) pins
+
+def _brute_task_map(B, mode, pb, off, cap):
+    F = len(mode)
+    tasks = []
+    blocks = []
+    for f in range(F):
+        if mode[f] == 0:
+            n = -(-B // pb[f])
+        else:
+            nnz = int(off[(f + 1) * B]) - int(off[f * B])
+            n = nnz // pb[f] + 1
+        if cap[f] > 0:
+            n = min(n, cap[f])
+        blocks.append(n)
+        tasks += [(f, r) for r in range(n)]
+    return blocks, tasks
+
+
+@pytest.mark.parametrize('seed', range(5))
+def test_task_map_vs_brute_force(seed):
+    rng = np.random.default_rng(seed)
+    F, B = int(rng.integers(1, 9)), int(rng.integers(1, 70))
+    lens = rng.integers(0, 30, size=(F, B))
+    b = synth.batch_from_lengths(lens, [100] * F, seed=seed)
+    mode = rng.integers(0, 2, size=F).tolist()
+    pb = [int(rng.integers(1, 40)) for _ in range(F)]
+    cap = [int(rng.integers(0, 4)) if rng.random() < 0.3 else 0 for _ in range(F)]
+    blocks, tf, tr = oracle.task_map(B, mode, pb, b.offsets, cap)
+    eb, et = _brute_task_map(B, mode, pb, b.offsets, cap)
+    assert blocks.tolist() == eb
+    assert list(zip(tf.tolist(), tr.tolist())) == et
+    bs = oracle.block_start_from_task_map(F, tf)
+    assert bs[-1] == sum(eb) and np.all(np.diff(bs) == np.asarray(eb))
+
+
+def test_nnz_task_ranges_partition():
+    rng = np.random.default_rng(9)
+    for trial in range(20):
+        B = int(rng.integers(1, 50))
+        lens = rng.integers(0, 40, size=B)
+        lens[rng.random(B) < 0.2] = 0
+        off = np.zeros(B + 1, np.int32)
+        off[1:] = np.cumsum(lens) + 5
+        off[0] = 5
+        npb = int(rng.integers(1, 60))
+        nnz = int(off[-1] - off[0])
+        blocks = nnz // npb + 1
+        s0, s1 = oracle.nnz_task_ranges(B, npb, off, blocks)
+        # ranges are ordered, contiguous, cover [0, B) exactly once
+        assert s0[0] == 0 and s1[-1] == B
+        assert np.all(s1 >= s0)
+        assert np.all(s0[1:] == s1[:-1])
+        for s in range(B):
+            q = (int(off[s]) - int(off[0])) // npb
+            assert s0[q] <= s < s1[q]
