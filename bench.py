@@ -1,0 +1,437 @@
+#!/usr/bin/env python
+"""bench.py -- RecFlex hot path on B200: fused heterogeneous-schedule
+embedding-bag forward (map + fused kernels), table-wise sharded with a pooled-
+output NCCL all-to-all at N > 1.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config sharded1000]
+    torchrun --nproc-per-node N bench.py --gpus N ...       (N > 1)
+    python bench.py --impl reference ...                      (CPU oracle arm)
+
+One step = one pass of the whole hot path over one synthetic batch already
+resident in HBM: device-side workload map -> fused kernel (-> alltoallv ->
+relayout at N > 1).  Batches rotate over --batches distinct seeded batches
+whose index arrays alone exceed L2 (sharded1000: 0.55 GB per batch, tables
+28.5 GB), so no L2 flush is needed between steps (configs whose working set
+fits in L2 are flushed between steps by a kernel outside the timed events).
+Rank 0 prints ONE JSON line.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import tempfile
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+FALLBACK_HBM_GBS = 6650.0   # B200_PROFILING.md fallback, used only if MEASURED_PEAKS.json is absent
+L2_BYTES = 126 * 2 ** 20
+
+
+def _baseline_metric():
+    try:
+        with open(os.path.join(ROOT, 'BASELINE.json')) as fh:
+            return json.load(fh)['metric']
+    except Exception:
+        return 'pooled samples/s and effective HBM GB/s (% of 8 TB/s) at 1/2/4/8 B200'
+
+
+def _peaks():
+    p = os.path.join(ROOT, 'MEASURED_PEAKS.json')
+    if os.path.exists(p):
+        with open(p) as fh:
+            d = json.load(fh)
+        return float(d['hbm_gbs']), 'measured (MEASURED_PEAKS.json hbm_gbs, copy read+write)'
+    return FALLBACK_HBM_GBS, 'fallback (B200_PROFILING.md)'
+
+
+# ------------------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi clocks/throttle sampling DURING the timed region."""
+    Q = ('index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,'
+         'clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,'
+         'clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap')
+
+    def __init__(self, gpu_index: int):
+        self.gpu = gpu_index
+        self.proc = None
+        self.path = None
+
+    def start(self):
+        try:
+            fd, self.path = tempfile.mkstemp(suffix='.csv')
+            os.close(fd)
+            self.proc = subprocess.Popen(['nvidia-smi', f'--id={self.gpu}', f'--query-gpu={self.Q}',
+                                          '--format=csv,noheader,nounits', '-lms', '100'],
+                                         stdout=open(self.path, 'w'), stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return None
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        rows = []
+        for line in open(self.path):
+            parts = [x.strip() for x in line.split(',')]
+            if len(parts) < 9:
+                continue
+            try:
+                rows.append(dict(sm=float(parts[1]), smmax=float(parts[2]), reasons=parts[5:9]))
+            except ValueError:
+                continue
+        os.unlink(self.path)
+        if not rows:
+            return None
+        names = ['hw_slowdown', 'hw_thermal_slowdown', 'sw_thermal_slowdown', 'sw_power_cap']
+        seen = set()
+        for r in rows:
+            for n, v in zip(names, r['reasons']):
+                if v.lower().startswith('active'):
+                    seen.add(n)
+        return {'sm_mhz': float(np.median([r['sm'] for r in rows])), 'sm_max_mhz': rows[0]['smmax'],
+                'reasons': sorted(seen), 'samples': len(rows)}
+
+
+# ------------------------------------------------------------------------- CPU oracle arm
+def oracle_sample_rate(model, batch, n_samples: int, seed: int = 0, nthreads: int = 0):
+    """Time the oracle (as it stands) on a bounded sample of the workload.
+
+    Input preparation (regenerating the referenced table rows from the seeded
+    generator) is outside the timed region; the timed call is the oracle's
+    embedding-bag over the sampled bags of every feature."""
+    import oracle
+    from paper_conf_sc_panzzxwslr0d24_b200 import synth
+    rng = np.random.default_rng(seed)
+    samples = np.sort(rng.choice(batch.B, size=min(n_samples, batch.B), replace=False))
+    F, B = batch.F, batch.B
+    offs = batch.offsets.astype(np.int64)
+    tables, sub_idx, sub_off = [], [], [0]
+    for f in range(F):
+        bags = [batch.indices[offs[f * B + s]:offs[f * B + s + 1]] for s in samples]
+        ids = np.concatenate(bags) if bags else np.zeros(0, np.int32)
+        uniq, inv = np.unique(ids, return_inverse=True)
+        if uniq.size == 0:
+            uniq = np.zeros(1, np.int64)
+        feat = model.features[f]
+        tables.append(synth.table_rows_at(feat.table, uniq, feat.dim, 'float', seed=model.seed).numpy())
+        pos = 0
+        for bag in bags:
+            sub_idx.append(inv[pos:pos + bag.size].astype(np.int32))
+            pos += bag.size
+            sub_off.append(sub_off[-1] + bag.size)
+    idx = np.concatenate(sub_idx) if sub_idx else np.zeros(0, np.int32)
+    off = np.asarray(sub_off, np.int32)
+    S = len(samples)
+    # algorithmic bytes of the sample (C26)
+    nnz_f = np.asarray([off[(f + 1) * S] - off[f * S] for f in range(F)], np.int64)
+    dims = np.asarray(model.dims, np.int64)
+    alg = 4 * int(nnz_f.sum()) + 4 * int((dims * nnz_f).sum()) + 4 * S * int(dims.sum())
+    t0 = time.perf_counter()
+    oracle.embedding_bag(tables, model.dims, [f.pool for f in model.features], idx, off, S, nthreads=nthreads)
+    dt = time.perf_counter() - t0
+    return S, dt, alg
+
+
+def run_reference(args, rank, world):
+    """--impl reference: the CPU oracle timed on the host cores (rank 0 only)."""
+    if rank != 0:
+        return 0
+    import oracle
+    from paper_conf_sc_panzzxwslr0d24_b200 import synth
+    model = synth.make_model(args.config)
+    batch = synth.make_batch(model, 7)
+    cores = len(os.sched_getaffinity(0))
+    n = args.ref_samples
+    for _ in range(args.warmup):
+        oracle_sample_rate(model, batch, max(8, n // 8), seed=99, nthreads=cores)
+    tot_s, tot_t, tot_b = 0, 0.0, 0
+    for i in range(args.steps):
+        S, dt, alg = oracle_sample_rate(model, batch, n, seed=i, nthreads=cores)
+        tot_s += S
+        tot_t += dt
+        tot_b += alg
+    value = tot_s / tot_t
+    line = {
+        'impl': 'reference', 'metric': _baseline_metric(), 'value': value, 'unit': 'samples/s',
+        'n_gpus': world, 'steps': args.steps, 'warmup': args.warmup, 'ms_per_step': 1e3 * tot_t / args.steps,
+        'higher_is_better': True, 'scaling': 'strong' if world > 1 else 'weak', 'vs_baseline': None,
+        'dtype': 'f64', 'data': 'synthetic',
+        'config': {'workload': args.config, 'global_batch': model.batch, 'fields': model.F,
+                   'parallelism': f'tablewise{world}'},
+        'effective_gbs': tot_b / tot_t / 1e9,
+        'cpu_baseline': {'value': value, 'unit': 'samples/s', 'cores': cores, 'kind': 'oracle',
+                         'sample': f'{args.steps} steps x {n} random samples (all {model.F} fields) of batch seed 7'},
+        'e2e': {'value': value, 'unit': 'samples/s', 'h2d_bytes_per_step': 0, 'd2h_bytes_per_step': 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------------- GPU arm
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument('--gpus', type=int, default=1)
+    ap.add_argument('--steps', type=int, default=20)
+    ap.add_argument('--warmup', type=int, default=5)
+    ap.add_argument('--impl', default='ours', choices=['ours', 'reference'])
+    ap.add_argument('--config', default='sharded1000')
+    ap.add_argument('--mode', default='float', choices=['float', 'int'])
+    ap.add_argument('--batches', type=int, default=3)
+    ap.add_argument('--plan', default='auto', help="tuned plan JSON, 'auto' (configs/tuned/) or 'none'")
+    ap.add_argument('--tune', action='store_true', help='run the two-stage tuner before timing')
+    ap.add_argument('--occupancy', type=int, default=0)
+    ap.add_argument('--no-e2e', action='store_true')
+    ap.add_argument('--no-cpu-baseline', action='store_true')
+    ap.add_argument('--ref-samples', type=int, default=256)
+    ap.add_argument('--cpu-samples', type=int, default=256)
+    ap.add_argument('--profile-only', action='store_true', help='short run for ncu (no e2e / cpu / clocks)')
+    args = ap.parse_args()
+
+    world = int(os.environ.get('WORLD_SIZE', '1'))
+    rank = int(os.environ.get('RANK', '0'))
+    local_rank = int(os.environ.get('LOCAL_RANK', '0'))
+
+    if args.impl == 'reference':
+        return run_reference(args, rank, world)
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_panzzxwslr0d24_b200 import synth
+    from paper_conf_sc_panzzxwslr0d24_b200.shard import ShardedEmbedding, partition_model, shard_batch
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device('cuda', local_rank)
+    if world > 1:
+        dist.init_process_group('nccl', device_id=dev)
+
+    model = synth.make_model(args.config)
+    B = model.batch
+    parts = partition_model(model, world)
+    sh = ShardedEmbedding(model, rank, world, device=local_rank, parts=parts)
+    plan = sh.plan
+    feats = sh.features
+
+    # tables of my features (physical tables generated once, aliased per feature)
+    phys = {}
+    for f in feats:
+        t = model.features[f].table
+        if t not in phys:
+            rows, dim = model.tables[t]
+            phys[t] = synth.make_table(t, rows, dim, args.mode, device=dev, seed=model.seed)
+    tables = [phys[model.features[f].table] for f in feats]
+
+    # batches: the global batch for my features, resident in HBM
+    batches, host_batches, alg_bytes = [], [], []
+    dims_local = np.asarray([model.dims[f] for f in feats], np.int64)
+    for i in range(args.batches):
+        full = synth.make_batch(model, 7 + i)
+        idx, off = shard_batch(full, feats)
+        host_batches.append((idx, off))
+        batches.append((torch.from_numpy(idx).to(dev), torch.from_numpy(off).to(dev)))
+        o = off.astype(np.int64)
+        nnz_f = o[np.arange(1, len(feats) + 1) * B] - o[np.arange(0, len(feats)) * B]
+        alg_bytes.append(4 * int(nnz_f.sum()) + 4 * int((dims_local * nnz_f).sum()) + 4 * B * int(dims_local.sum()))
+    alg_local = float(np.mean(alg_bytes))
+    ws = alg_local + sum(t.numel() * 4 for t in tables)
+    flush_between = (alg_local < 4 * L2_BYTES)
+
+    # tuned plan (stage-1/2 result exported by tools/tune_plan.py) or live tuning
+    plan_src = 'default (untuned heuristic)'
+    if args.tune:
+        hist = [(bi, bo, B) for (bi, bo) in batches[:2]]
+        st = plan.tune(hist, tables, verbose=(rank == 0))
+        plan_src = f"tuned live ({st['tune_seconds']:.0f}s, k={st['best_occupancy']})"
+    elif args.plan != 'none':
+        path = args.plan
+        if path == 'auto':
+            path = os.path.join(ROOT, 'configs', 'tuned', f'{args.config}_w{world}_r{rank}.json')
+        if os.path.exists(path):
+            with open(path) as fh:
+                plan.import_(json.load(fh))
+            plan_src = os.path.relpath(path, ROOT)
+    if args.occupancy:
+        plan.occupancy = args.occupancy
+
+    out_local = torch.empty((B, sh.d_local), dtype=torch.float32, device=dev)
+    out_x = torch.empty((B // world, sh.d_tot), dtype=torch.float32, device=dev) if world > 1 else None
+    flush_buf = torch.empty(2 * L2_BYTES // 4, dtype=torch.float32, device=dev) if flush_between else None
+    stream = torch.cuda.current_stream()
+
+    def step(i):
+        bi, bo = batches[i % len(batches)]
+        return sh.forward(bi, bo, B, tables, out_local=out_local, out=out_x)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    from paper_conf_sc_panzzxwslr0d24_b200.plan import l2_flush
+
+    for i in range(args.warmup):
+        step(i)
+    torch.cuda.synchronize()
+
+    clocks = ClockSampler(local_rank) if not args.profile_only else None
+    if clocks:
+        clocks.start()
+        time.sleep(0.3)
+    barrier()
+    torch.cuda.synchronize()
+    if flush_between:
+        evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+        for i in range(args.steps):
+            l2_flush(flush_buf)
+            evs[i][0].record(stream)
+            step(i)
+            evs[i][1].record(stream)
+        torch.cuda.synchronize()
+        elapsed_ms = sum(a.elapsed_time(b) for a, b in evs)
+    else:
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for i in range(args.steps):
+            step(i)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        elapsed_ms = e0.elapsed_time(e1)
+    barrier()
+    clk = clocks.stop() if clocks else None
+
+    if world > 1:
+        t = torch.tensor([elapsed_ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        elapsed_ms = float(t.item())
+    ms_per_step = elapsed_ms / args.steps
+    value = B * args.steps / (elapsed_ms / 1e3)
+
+    # per-kernel device time (events on the launch stream; PDL off in this pass)
+    plan.set_profiling(True)
+    plan.kernel_times(reset=True)
+    for i in range(args.steps):
+        if flush_between:
+            l2_flush(flush_buf)
+        bi, bo = batches[i % len(batches)]
+        plan.forward(bi, bo, B, tables, out=out_local)
+    kt = plan.kernel_times(reset=True)
+    plan.set_profiling(False)
+    fused_ms = kt['fused_ms'] / max(1, kt['forwards'])
+    map_ms = kt['map_ms'] / max(1, kt['forwards'])
+    peak, peak_src = _peaks()
+    achieved = alg_local / (fused_ms / 1e3) / 1e9
+    eff_gbs_step = alg_local / (ms_per_step / 1e3) / 1e9
+
+    traffic = None
+    tp = os.path.join(ROOT, 'profiles', f'ncu_traffic_{args.config}.json')
+    if os.path.exists(tp):
+        try:
+            with open(tp) as fh:
+                traffic = json.load(fh).get('dram_bytes_per_launch')
+        except Exception:
+            traffic = None
+
+    # end-to-end through the public API from pinned host buffers
+    e2e = None
+    if not args.no_e2e and not args.profile_only:
+        hb = [(torch.from_numpy(i).pin_memory(), torch.from_numpy(o).pin_memory()) for i, o in host_batches]
+        if world == 1:
+            hout = torch.empty((B, sh.d_local), dtype=torch.float32).pin_memory()
+            plan.forward_host(hb[0][0], hb[0][1], B, tables, hout)
+            torch.cuda.synchronize()
+            ke = max(3, min(args.steps, 10))
+            t0 = time.perf_counter()
+            for i in range(ke):
+                hi, ho = hb[i % len(hb)]
+                plan.forward_host(hi, ho, B, tables, hout)
+            dt = time.perf_counter() - t0
+            h2d = float(np.mean([hi.numel() * 4 + ho.numel() * 4 for hi, ho in hb]))
+            d2h = hout.numel() * 4
+        else:
+            hout = torch.empty((B // world, sh.d_tot), dtype=torch.float32).pin_memory()
+            di = [torch.empty_like(b[0], device=dev) for b in hb]
+            do = [torch.empty_like(b[1], device=dev) for b in hb]
+            ke = max(3, min(args.steps, 10))
+            barrier()
+            t0 = time.perf_counter()
+            for i in range(ke):
+                j = i % len(hb)
+                di[j].copy_(hb[j][0], non_blocking=True)
+                do[j].copy_(hb[j][1], non_blocking=True)
+                o = sh.forward(di[j], do[j], B, tables, out_local=out_local, out=out_x)
+                hout.copy_(o, non_blocking=True)
+                torch.cuda.current_stream().synchronize()
+            dt = time.perf_counter() - t0
+            t = torch.tensor([dt], dtype=torch.float64, device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            dt = float(t.item())
+            h2d = float(np.mean([hi.numel() * 4 + ho.numel() * 4 for hi, ho in hb]))
+            d2h = hout.numel() * 4
+        e2e = {'value': B * ke / dt, 'unit': 'samples/s', 'h2d_bytes_per_step': int(h2d),
+               'd2h_bytes_per_step': int(d2h), 'steps': ke, 'timing': 'wall clock per rank, max over ranks'}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline and not args.profile_only:
+        try:
+            from paper_conf_sc_panzzxwslr0d24_b200 import synth as _s
+            full = _s.make_batch(model, 7)
+            cores = len(os.sched_getaffinity(0))
+            S, dt, alg = oracle_sample_rate(model, full, args.cpu_samples, seed=0, nthreads=cores)
+            cpu = {'value': S / dt, 'unit': 'samples/s', 'cores': cores, 'kind': 'oracle',
+                   'sample': f'{S} random samples x all {model.F} fields of batch seed 7 (fp64 C oracle, OpenMP)',
+                   'effective_gbs': alg / dt / 1e9, 'seconds': dt}
+        except Exception as ex:  # never fail the bench line on the baseline leg
+            cpu = {'value': None, 'unit': 'samples/s', 'cores': None, 'kind': 'oracle', 'sample': f'failed: {ex}'}
+
+    launches_per_step = 2 + (1 if plan.export() and any(s[1] == 1 for s in plan.export()['schedules']) else 0)
+    launches_per_step += 1 if world > 1 else 0   # relayout kernel
+    if rank == 0:
+        line = {
+            'metric': _baseline_metric(),
+            'value': value,
+            'unit': 'samples/s',
+            'n_gpus': world,
+            'steps': args.steps,
+            'warmup': args.warmup,
+            'ms_per_step': ms_per_step,
+            'higher_is_better': True,
+            'scaling': 'strong' if world > 1 else 'weak',
+            'vs_baseline': None,
+            'dtype': 'f32',
+            'data': 'synthetic (seeded generator, SURVEY §8d recipe; tables: counter-based hash U[-1,1))',
+            'config': {'workload': args.config, 'global_batch': B, 'fields': model.F,
+                       'parallelism': f'tablewise{world}', 'plan': plan_src, 'occupancy': plan.occupancy,
+                       'l2': 'flushed between steps' if flush_between else
+                             f'inputs > L2 ({alg_local / 1e9:.2f} GB algorithmic per step per rank, '
+                             f'{args.batches} rotating batches)'},
+            'effective_hbm_gbs': eff_gbs_step * (world if world > 1 else 1),
+            'pct_of_8tbs': 100.0 * eff_gbs_step / 8000.0,
+            'roofline': {'bound': 'hbm', 'achieved': achieved, 'peak': peak, 'unit': 'GB/s',
+                         'frac': achieved / peak, 'traffic': traffic, 'kernel': 'recflex_fused_kernel',
+                         'peak_source': peak_src, 'fused_ms': fused_ms, 'map_ms': map_ms,
+                         'algorithmic_bytes_per_launch': alg_local},
+            'e2e': e2e,
+            'gpu_launches': launches_per_step * args.steps,
+            'clocks': clk,
+            'cpu_baseline': cpu,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == '__main__':
+    sys.exit(main())

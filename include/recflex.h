@@ -1,0 +1,248 @@
+/*
+ * recflex.h -- C ABI of the B200-native RecFlex hot path (librecflex.so).
+ *
+ * The operation (PAPER.md "P:n" = line n of the paper text):
+ *   For every feature field f and sample s, gather the rows of table T_f named
+ *   by the lookup IDs of bag (f, s) and pool them by elementwise reduction
+ *   (§II-A, Fig. 1); per-feature results are concatenated.
+ *   Each field runs its own schedule inside ONE fused kernel (§IV-B, Fig. 8,
+ *   P:168-234); schedules are chosen by the two-stage interference-simulated
+ *   tuner (§IV-A, Eq. 1-5); the block-to-feature map is computed
+ *   per batch from the offsets -- here by a device-side scan, with
+ *   no host round trip.
+ *
+ * Conventions for every entry point:
+ *   - Pointers named d_* / documented "device" are CUDA device pointers on the
+ *     plan's device; "host" pointers are ordinary (ideally pinned) host memory.
+ *   - A stream argument is a cudaStream_t passed as void* (NULL = legacy
+ *     default stream).
+ *   - Every call returns a recflex_status_t.  Host-checkable misuse returns
+ *     RECFLEX_ERR_INVALID_ARG before any launch; launch failures return
+ *     RECFLEX_ERR_CUDA.  Device-data errors (out-of-range IDs, non-monotone
+ *     offsets) are undefined behaviour in recflex_forward; recflex_validate
+ *     detects them (reading C3).
+ *   - The caller owns tables, indices, offsets, out and streams.  The plan
+ *     owns its descriptors and scratch.
+ *   - A plan is not thread-safe; one plan must not have two forwards in
+ *     flight on different streams (they share scratch).
+ *
+ * Data layout (readings C4, C6, C7 in DESIGN.md):
+ *   indices : int32 [nnz]          lookup IDs, feature-major KJT
+ *   offsets : int32 [F*B + 1]      bag (f,s) = indices[offsets[f*B+s] .. offsets[f*B+s+1])
+ *                                  offsets[0] == 0, non-decreasing, nnz < 2^31
+ *   tables  : F float32 row-major [rows_f][d_f], 32-byte aligned base
+ *   out     : float32 row-major [B][D_tot], D_tot = sum d_f, feature f at
+ *             columns [col_f, col_f + d_f), col_f = sum_{g<f} d_g; 16-byte
+ *             aligned base
+ */
+#ifndef RECFLEX_H_
+#define RECFLEX_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define RECFLEX_ABI_VERSION 1
+#define RECFLEX_MAX_OCCUPANCY 8          /* CTAs of 256 threads per SM: K = 8 (reading C14) */
+
+typedef struct recflex_plan_s *recflex_plan_t; /* opaque, library-owned */
+
+typedef enum { RECFLEX_POOL_SUM = 0, RECFLEX_POOL_MEAN = 1 } recflex_pool_t;
+
+typedef enum {
+    RECFLEX_OK = 0,
+    RECFLEX_ERR_INVALID_ARG = 1,
+    RECFLEX_ERR_CUDA = 2,
+    RECFLEX_ERR_OOM = 3,
+    RECFLEX_ERR_NOT_SUPPORTED = 4,
+    RECFLEX_ERR_INDEX_OOB = 5
+} recflex_status_t;
+
+/* Per-feature table spec plus hotness statistics from historical data
+ * ("embedding table specifications"; P:160 historical inputs). */
+typedef struct {
+    int64_t num_rows; /* rows_f, 1 <= rows_f < 2^31                              */
+    int32_t dim;      /* d_f >= 1; vector paths need d_f % 4 == 0 (else scalar)   */
+    int32_t pool;     /* recflex_pool_t; MEAN of an empty bag is 0 (reading C1)   */
+    float mean_len;   /* E[L | L > 0]   (pooling factor)                    */
+    float max_len;    /* observed max L (sizes scratch for nnz-partitioned tasks) */
+    float coverage;   /* P(L > 0)                                    */
+} recflex_feature_spec_t;
+
+/* A feature's schedule: catalog entry + its runtime thread-mapping parameters
+ * ("tunable parameters").  part 0: a task (CTA work unit) covers
+ * per_block consecutive samples; part 1: a task covers the bags whose first
+ * lookup falls in a window of per_block lookups (adaptive to the batch). */
+typedef struct {
+    int32_t sched_id;  /* index into the catalog (recflex_catalog_info)         */
+    int32_t part;      /* 0 = sample-partitioned, 1 = lookup(nnz)-partitioned    */
+    int32_t per_block; /* samples per task (part 0) or lookups per task (part 1) */
+} recflex_schedule_t;
+
+/* Catalog entry description (hand-written sm_100a schedule templates). */
+typedef enum {
+    RECFLEX_FAMILY_GROUP = 0, /* G lanes per bag; 256/G bags in flight per CTA (G=32: warp per sample) */
+    RECFLEX_FAMILY_BLOCK = 1  /* all 256 threads on one bag; smem partials + fixed-order reduction    */
+} recflex_family_t;
+
+typedef struct {
+    int32_t family; /* recflex_family_t                                        */
+    int32_t group;  /* G: lanes cooperating on one row (power of two, 1..32)   */
+    int32_t vec;    /* floats per lane per load: 1, 4 (128-bit) or 8 (256-bit) */
+    int32_t cols;   /* C: column chunks per lane (row span = G*vec*C floats)   */
+    int32_t unroll; /* U: rows in flight per lane                              */
+} recflex_catalog_info_t;
+
+/* ---- plan lifecycle --------------------------------------------------- */
+
+/* Validates specs, computes col_f (prefix sum of dims), picks heuristic
+ * default schedules (an untuned plan is valid), allocates plan scratch sized
+ * for max_batch on `device`.  No device data is read.  *out receives the plan. */
+recflex_status_t recflex_plan_create(const recflex_feature_spec_t *specs, int32_t num_features,
+                                     int32_t max_batch, int32_t device, recflex_plan_t *out);
+
+/* Frees all plan-owned memory.  NULL is a no-op. */
+void recflex_destroy(recflex_plan_t plan);
+
+const char *recflex_status_string(recflex_status_t status);
+
+/* ---- the hot path ----------------------------------------------------- */
+
+/* Fused multi-feature embedding-bag forward (async, stream-ordered, no host
+ * synchronisation and no allocation: CUDA-graph capturable).
+ *   indices, offsets : device, layout above; batch_size = B (0 <= B <= max_batch;
+ *                      B == 0 is a no-op)
+ *   tables           : HOST array of F device pointers (cached; re-uploaded
+ *                      only when a pointer changes)
+ *   out              : device float32 [B][D_tot], fully overwritten
+ * Launches: map kernel (device-side workload scan), optional task-range fill
+ * kernel (only if some feature is lookup-partitioned), fused kernel (PDL). */
+recflex_status_t recflex_forward(recflex_plan_t plan, const int32_t *indices, const int32_t *offsets,
+                                 int32_t batch_size, const float *const *tables, float *out,
+                                 void *stream);
+
+/* Same operation from HOST buffers (end-to-end path): copies h_indices[nnz] and
+ * h_offsets[F*B+1] to plan-owned device staging, runs recflex_forward, copies
+ * the pooled output back to h_out [B][D_tot]; blocks until h_out is written.
+ * Staging grows on demand (this entry point may allocate). */
+recflex_status_t recflex_forward_host(recflex_plan_t plan, const int32_t *h_indices, int64_t nnz,
+                                      const int32_t *h_offsets, int32_t batch_size,
+                                      const float *const *tables, float *h_out, void *stream);
+
+/* ---- tuner (§IV-A) ------------------------------------------------------ */
+
+typedef struct {
+    int32_t num_occupancies; /* how many entries of occupancies[] to try (0 = all 1..8)    */
+    int32_t occupancies[RECFLEX_MAX_OCCUPANCY];
+    int32_t reps;            /* stage-2 timed forwards per batch (median), default 7       */
+    int32_t pad_waves;       /* padding tasks = pad_waves * #SM * k, default 4     */
+    int32_t max_candidates;  /* per feature, 0 = all valid catalog candidates              */
+    int32_t verbose;         /* 1: print per-stage summaries to stderr                     */
+} recflex_tune_options_t;
+
+typedef struct {
+    int64_t local_launches;   /* stage 1 co-execution launches  (= F*K*N)           */
+    int64_t global_launches;  /* stage 2 timed fused launches    (= K*N*reps)        */
+    int64_t local_evals;      /* stage-1 cost evaluations (one per (k, f)) = F*K     */
+    int64_t global_evals;     /* stage-2 cost evaluations (one per k)      = K       */
+    int32_t best_occupancy;
+    double best_ms;           /* summed median forward time over tuning batches    */
+    double tune_seconds;
+} recflex_tune_stats_t;
+
+/* Two-stage interference-simulated tuning over num_batches historical batches
+ * (Eq. 5).  indices[i] / offsets[i] are DEVICE pointers of batch i with
+ * batch_sizes[i] samples; tables as in recflex_forward.  Blocking; may
+ * allocate.  Leaves the plan with the selected occupancy and schedules. */
+recflex_status_t recflex_tune(recflex_plan_t plan, int32_t num_batches, const int32_t *const *indices,
+                              const int32_t *const *offsets, const int32_t *batch_sizes,
+                              const float *const *tables, void *stream);
+recflex_status_t recflex_tune_ex(recflex_plan_t plan, int32_t num_batches, const int32_t *const *indices,
+                                 const int32_t *const *offsets, const int32_t *batch_sizes,
+                                 const float *const *tables, void *stream,
+                                 const recflex_tune_options_t *options, recflex_tune_stats_t *stats);
+
+/* The selection logic of the two-stage tuner, on caller-supplied costs
+ * (Eq. 3 per-feature local objective, Eq. 4 global objective).
+ *   local_cost(user, k_index, f, costs_out[num_candidates[f]]): one call = one
+ *     co-execution launch; fills the summed block times of every candidate.
+ *   global_cost(user, k_index, choice[F]) -> fused-kernel latency at O_k.
+ * Writes choice_out[F] and *best_k_index; tie -> lowest candidate index (local),
+ * larger k index (global).  Returns call counts through *local_calls and *global_calls. */
+typedef void (*recflex_local_cost_fn)(void *user, int32_t k_index, int32_t f, double *costs_out);
+typedef double (*recflex_global_cost_fn)(void *user, int32_t k_index, const int32_t *choice);
+recflex_status_t recflex_two_stage_select(int32_t num_features, int32_t num_k, const int32_t *num_candidates,
+                                          recflex_local_cost_fn local_cost, recflex_global_cost_fn global_cost,
+                                          void *user, int32_t *choice_out, int32_t *best_k_index,
+                                          int64_t *local_calls, int64_t *global_calls);
+
+/* ---- schedules / occupancy / catalog ------------------------------------ */
+
+recflex_status_t recflex_get_schedule(recflex_plan_t plan, int32_t f, recflex_schedule_t *sched,
+                                      int32_t *blocks_per_sm);
+/* Validates the schedule against d_f (vector width divides d_f, ...). */
+recflex_status_t recflex_set_schedule(recflex_plan_t plan, int32_t f, const recflex_schedule_t *sched);
+/* k CTAs (of 256 threads) per SM, 1..8: register cap __launch_bounds__(256,k)
+ * + shared-memory padding (reading C15). */
+recflex_status_t recflex_set_occupancy(recflex_plan_t plan, int32_t k);
+recflex_status_t recflex_get_occupancy(recflex_plan_t plan, int32_t *k);
+
+int32_t recflex_catalog_size(void);
+recflex_status_t recflex_catalog_info(int32_t sched_id, recflex_catalog_info_t *info);
+/* 1 if catalog entry sched_id can run a feature of dimension dim. */
+int32_t recflex_catalog_valid(int32_t sched_id, int32_t dim);
+
+/* cudaOccupancyMaxActiveBlocksPerMultiprocessor of the fused-kernel variant
+ * for occupancy k with its padded shared memory (should equal k). */
+recflex_status_t recflex_occupancy_check(int32_t device, int32_t k, int32_t *active_blocks_per_sm,
+                                         int32_t *registers_per_thread, int32_t *spill_bytes);
+
+/* ---- introspection / validation / persistence ---------------------------- */
+
+/* Runs the map (+ fill) kernels for offsets (device) and copies the task map
+ * to the host: host_block_start[F+1] (exclusive scan of feature_blocks, Fig. 8
+ * d_task_map in compressed form); host_task_range (nullable) receives, for
+ * lookup-partitioned features, [s0, s1) of every task as 2*total ints
+ * (-1 for sample-partitioned tasks).  Blocking. */
+recflex_status_t recflex_debug_task_map(recflex_plan_t plan, const int32_t *offsets, int32_t batch_size,
+                                        int32_t *host_block_start, int32_t *host_task_range,
+                                        int64_t task_range_capacity, void *stream);
+
+/* Checks offsets (offsets[0]==0, monotone, F*B+1 entries) and that every ID of
+ * feature f is in [0, rows_f).  Blocking.  RECFLEX_ERR_INDEX_OOB / INVALID_ARG. */
+recflex_status_t recflex_validate(recflex_plan_t plan, const int32_t *indices, const int32_t *offsets,
+                                  int32_t batch_size, void *stream);
+
+/* JSON export/import of the tuned state (occupancy + per-feature schedules),
+ * P:164 "re-tune periodically".  export: writes up to cap bytes incl. NUL,
+ * *len = required size. */
+recflex_status_t recflex_plan_export(recflex_plan_t plan, char *buf, size_t cap, size_t *len);
+recflex_status_t recflex_plan_import(recflex_plan_t plan, const char *json);
+
+/* Profiling: when enabled, recflex_forward brackets its kernels with CUDA
+ * events on the launch stream; recflex_get_kernel_times returns the summed
+ * device milliseconds of the map(+fill) and fused kernels since the last reset
+ * and the number of forwards.  Blocking (synchronises the events). */
+recflex_status_t recflex_set_profiling(recflex_plan_t plan, int32_t enable);
+recflex_status_t recflex_get_kernel_times(recflex_plan_t plan, double *map_ms, double *fused_ms,
+                                          int64_t *forwards, int32_t reset);
+
+/* ---- multi-GPU exchange helper ------------------------------------------- */
+
+/* Relayout after the table-wise pooled-output all-to-all:
+ * recv holds W chunks, chunk i = [rows][dims[i]] (row-major, contiguous, in
+ * rank order); out = [rows][sum dims] with chunk i at column offset
+ * sum_{j<i} dims[j].  Device pointers, async on stream. */
+recflex_status_t recflex_shard_concat(const float *recv, int32_t num_ranks, int32_t rows,
+                                      const int32_t *host_dims, float *out, void *stream);
+
+/* Writes `bytes` of a device scratch buffer to evict L2 (timing hygiene). */
+recflex_status_t recflex_l2_flush(void *d_scratch, size_t bytes, void *stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* RECFLEX_H_ */

@@ -1,0 +1,117 @@
+"""ctypes binding of include/recflex.h (librecflex.so).
+
+Argument marshalling only: every step of the hot path runs in the library's
+CUDA kernels.  There is no fallback -- if librecflex.so is missing or fails to
+load, importing this module raises (build it with ``python -m
+paper_conf_sc_panzzxwslr0d24_b200.build`` or ``__graft_entry__.build()``).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(HERE, 'lib', 'librecflex.so')
+
+c_int32 = ctypes.c_int32
+c_int64 = ctypes.c_int64
+c_void_p = ctypes.c_void_p
+P = ctypes.POINTER
+
+
+class FeatureSpec(ctypes.Structure):
+    _fields_ = [('num_rows', ctypes.c_int64), ('dim', ctypes.c_int32), ('pool', ctypes.c_int32),
+                ('mean_len', ctypes.c_float), ('max_len', ctypes.c_float), ('coverage', ctypes.c_float)]
+
+
+class Schedule(ctypes.Structure):
+    _fields_ = [('sched_id', ctypes.c_int32), ('part', ctypes.c_int32), ('per_block', ctypes.c_int32)]
+
+
+class CatalogInfo(ctypes.Structure):
+    _fields_ = [('family', ctypes.c_int32), ('group', ctypes.c_int32), ('vec', ctypes.c_int32),
+                ('cols', ctypes.c_int32), ('unroll', ctypes.c_int32)]
+
+
+class TuneOptions(ctypes.Structure):
+    _fields_ = [('num_occupancies', ctypes.c_int32), ('occupancies', ctypes.c_int32 * 8),
+                ('reps', ctypes.c_int32), ('pad_waves', ctypes.c_int32), ('max_candidates', ctypes.c_int32),
+                ('verbose', ctypes.c_int32)]
+
+
+class TuneStats(ctypes.Structure):
+    _fields_ = [('local_launches', ctypes.c_int64), ('global_launches', ctypes.c_int64),
+                ('local_evals', ctypes.c_int64), ('global_evals', ctypes.c_int64),
+                ('best_occupancy', ctypes.c_int32), ('best_ms', ctypes.c_double), ('tune_seconds', ctypes.c_double)]
+
+
+LOCAL_COST_FN = ctypes.CFUNCTYPE(None, c_void_p, c_int32, c_int32, P(ctypes.c_double))
+GLOBAL_COST_FN = ctypes.CFUNCTYPE(ctypes.c_double, c_void_p, c_int32, P(c_int32))
+
+OK = 0
+STATUS = {0: 'RECFLEX_OK', 1: 'RECFLEX_ERR_INVALID_ARG', 2: 'RECFLEX_ERR_CUDA', 3: 'RECFLEX_ERR_OOM',
+          4: 'RECFLEX_ERR_NOT_SUPPORTED', 5: 'RECFLEX_ERR_INDEX_OOB'}
+
+# name -> (restype, argtypes); the same names as include/recflex.h
+SIGNATURES = {
+    'recflex_plan_create': (c_int32, [P(FeatureSpec), c_int32, c_int32, c_int32, P(c_void_p)]),
+    'recflex_destroy': (None, [c_void_p]),
+    'recflex_status_string': (ctypes.c_char_p, [c_int32]),
+    'recflex_forward': (c_int32, [c_void_p, c_void_p, c_void_p, c_int32, P(c_void_p), c_void_p, c_void_p]),
+    'recflex_forward_host': (c_int32, [c_void_p, c_void_p, c_int64, c_void_p, c_int32, P(c_void_p), c_void_p,
+                                       c_void_p]),
+    'recflex_tune': (c_int32, [c_void_p, c_int32, P(c_void_p), P(c_void_p), P(c_int32), P(c_void_p), c_void_p]),
+    'recflex_tune_ex': (c_int32, [c_void_p, c_int32, P(c_void_p), P(c_void_p), P(c_int32), P(c_void_p), c_void_p,
+                                  P(TuneOptions), P(TuneStats)]),
+    'recflex_two_stage_select': (c_int32, [c_int32, c_int32, P(c_int32), LOCAL_COST_FN, GLOBAL_COST_FN, c_void_p,
+                                           P(c_int32), P(c_int32), P(c_int64), P(c_int64)]),
+    'recflex_get_schedule': (c_int32, [c_void_p, c_int32, P(Schedule), P(c_int32)]),
+    'recflex_set_schedule': (c_int32, [c_void_p, c_int32, P(Schedule)]),
+    'recflex_set_occupancy': (c_int32, [c_void_p, c_int32]),
+    'recflex_get_occupancy': (c_int32, [c_void_p, P(c_int32)]),
+    'recflex_catalog_size': (c_int32, []),
+    'recflex_catalog_info': (c_int32, [c_int32, P(CatalogInfo)]),
+    'recflex_catalog_valid': (c_int32, [c_int32, c_int32]),
+    'recflex_occupancy_check': (c_int32, [c_int32, c_int32, P(c_int32), P(c_int32), P(c_int32)]),
+    'recflex_debug_task_map': (c_int32, [c_void_p, c_void_p, c_int32, P(c_int32), P(c_int32), c_int64, c_void_p]),
+    'recflex_validate': (c_int32, [c_void_p, c_void_p, c_void_p, c_int32, c_void_p]),
+    'recflex_plan_export': (c_int32, [c_void_p, ctypes.c_char_p, ctypes.c_size_t, P(ctypes.c_size_t)]),
+    'recflex_plan_import': (c_int32, [c_void_p, ctypes.c_char_p]),
+    'recflex_set_profiling': (c_int32, [c_void_p, c_int32]),
+    'recflex_get_kernel_times': (c_int32, [c_void_p, P(ctypes.c_double), P(ctypes.c_double), P(c_int64), c_int32]),
+    'recflex_shard_concat': (c_int32, [c_void_p, c_int32, c_int32, P(c_int32), c_void_p, c_void_p]),
+    'recflex_l2_flush': (c_int32, [c_void_p, ctypes.c_size_t, c_void_p]),
+}
+
+
+class RecflexError(RuntimeError):
+    def __init__(self, code, where=''):
+        self.code = code
+        super().__init__(f'{where}: {STATUS.get(code, code)}')
+
+
+def _load():
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f'{LIB_PATH} is missing: build the CUDA library first '
+                          '(python -m paper_conf_sc_panzzxwslr0d24_b200.build); there is no fallback path')
+    lib = ctypes.CDLL(LIB_PATH)
+    for name, (res, args) in SIGNATURES.items():
+        fn = getattr(lib, name)
+        fn.restype = res
+        fn.argtypes = args
+    return lib
+
+
+lib = _load()
+
+
+def check(code, where=''):
+    if code != OK:
+        raise RecflexError(code, where)
+
+
+# thin same-name wrappers -------------------------------------------------------
+def __getattr__(name):
+    if name in SIGNATURES:
+        return getattr(lib, name)
+    raise AttributeError(name)

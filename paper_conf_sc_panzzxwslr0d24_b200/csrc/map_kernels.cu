@@ -1,0 +1,275 @@
+// map_kernels.cu -- runtime thread mapping on the device (Fig. 8
+// d_task_map / d_blocks_map) plus small helper kernels.
+//
+// The paper computes the map on the host ("host-side workload analysis",
+// P:170); here one CTA reads the batch's offsets and scans, so the forward has
+// no host round trip (reading C13).  Same integers as the oracle's formula:
+//   part 0 (sample-partitioned): feature_blocks = ceil(B / per_block)
+//   part 1 (lookup-partitioned): npb = max(per_block, ceil(nnz_f/(slots-2)))
+//                                feature_blocks = floor(nnz_f / npb) + 1
+//   cap > 0: feature_blocks = min(feature_blocks, cap)
+//   block_start = exclusive scan of feature_blocks in feature order.
+#include <cuda_runtime.h>
+
+#include "recflex_internal.h"
+
+namespace recflex {
+
+int fused_launch_k1(const FusedArgs &, const LaunchCfg &, void *);
+int fused_launch_k2(const FusedArgs &, const LaunchCfg &, void *);
+int fused_launch_k3(const FusedArgs &, const LaunchCfg &, void *);
+int fused_launch_k4(const FusedArgs &, const LaunchCfg &, void *);
+int fused_launch_k5(const FusedArgs &, const LaunchCfg &, void *);
+int fused_launch_k6(const FusedArgs &, const LaunchCfg &, void *);
+int fused_launch_k7(const FusedArgs &, const LaunchCfg &, void *);
+int fused_launch_k8(const FusedArgs &, const LaunchCfg &, void *);
+int fused_prepare_k1(int);
+int fused_prepare_k2(int);
+int fused_prepare_k3(int);
+int fused_prepare_k4(int);
+int fused_prepare_k5(int);
+int fused_prepare_k6(int);
+int fused_prepare_k7(int);
+int fused_prepare_k8(int);
+int fused_occupancy_k1(int, int *, int *, int *);
+int fused_occupancy_k2(int, int *, int *, int *);
+int fused_occupancy_k3(int, int *, int *, int *);
+int fused_occupancy_k4(int, int *, int *, int *);
+int fused_occupancy_k5(int, int *, int *, int *);
+int fused_occupancy_k6(int, int *, int *, int *);
+int fused_occupancy_k7(int, int *, int *, int *);
+int fused_occupancy_k8(int, int *, int *, int *);
+
+int fused_launch(int k, const FusedArgs &a, const LaunchCfg &cfg, void *stream) {
+    switch (k) {
+        case 1: return fused_launch_k1(a, cfg, stream);
+        case 2: return fused_launch_k2(a, cfg, stream);
+        case 3: return fused_launch_k3(a, cfg, stream);
+        case 4: return fused_launch_k4(a, cfg, stream);
+        case 5: return fused_launch_k5(a, cfg, stream);
+        case 6: return fused_launch_k6(a, cfg, stream);
+        case 7: return fused_launch_k7(a, cfg, stream);
+        case 8: return fused_launch_k8(a, cfg, stream);
+        default: return (int)cudaErrorInvalidValue;
+    }
+}
+
+int fused_prepare(int k, int device, int smem) {
+    cudaError_t e = cudaSetDevice(device);
+    if (e != cudaSuccess) return (int)e;
+    switch (k) {
+        case 1: return fused_prepare_k1(smem);
+        case 2: return fused_prepare_k2(smem);
+        case 3: return fused_prepare_k3(smem);
+        case 4: return fused_prepare_k4(smem);
+        case 5: return fused_prepare_k5(smem);
+        case 6: return fused_prepare_k6(smem);
+        case 7: return fused_prepare_k7(smem);
+        case 8: return fused_prepare_k8(smem);
+        default: return (int)cudaErrorInvalidValue;
+    }
+}
+
+int fused_occupancy(int k, int smem, int *blocks, int *regs, int *spill) {
+    switch (k) {
+        case 1: return fused_occupancy_k1(smem, blocks, regs, spill);
+        case 2: return fused_occupancy_k2(smem, blocks, regs, spill);
+        case 3: return fused_occupancy_k3(smem, blocks, regs, spill);
+        case 4: return fused_occupancy_k4(smem, blocks, regs, spill);
+        case 5: return fused_occupancy_k5(smem, blocks, regs, spill);
+        case 6: return fused_occupancy_k6(smem, blocks, regs, spill);
+        case 7: return fused_occupancy_k7(smem, blocks, regs, spill);
+        case 8: return fused_occupancy_k8(smem, blocks, regs, spill);
+        default: return (int)cudaErrorInvalidValue;
+    }
+}
+
+// ---------------------------------------------------------------------------
+// Map kernel: one CTA of 1024 threads, features in chunks of 1024 with a carry.
+// ---------------------------------------------------------------------------
+constexpr int kMapThreads = 1024;
+
+__global__ void __launch_bounds__(kMapThreads) recflex_map_kernel(MapArgs a) {
+    __shared__ int warp_tot[kMapThreads / 32];
+    __shared__ int s_carry;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    if (tid == 0) {
+        s_carry = 0;
+        *a.counter = 0;  // the fused kernel's task counter
+    }
+    __syncthreads();
+    for (int base = 0; base < a.F; base += kMapThreads) {
+        const int f = base + tid;
+        int blocks = 0;
+        if (f < a.F && a.B > 0) {
+            const FeatureDesc &fd = a.desc[f];
+            if (fd.part == 0) {
+                blocks = (a.B + fd.per_block - 1) / fd.per_block;
+            } else {
+                const int64_t fi = fd.in_feature;
+                const int nnz = a.offsets[(fi + 1) * a.B] - a.offsets[fi * a.B];
+                int npb = fd.per_block;
+                const int room = fd.slots - 2;  // slots hold blocks+1 entries (sentinel)
+                const int need = (nnz + room - 1) / room;
+                if (need > npb) npb = need;
+                a.npb_eff[f] = npb;
+                blocks = nnz / npb + 1;
+            }
+            if (fd.cap > 0 && blocks > fd.cap) blocks = fd.cap;
+        }
+        // block-wide exclusive scan
+        int incl = blocks;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int v = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o) incl += v;
+        }
+        if (lane == 31) warp_tot[warp] = incl;
+        __syncthreads();
+        if (warp == 0) {
+            int w = warp_tot[lane];
+            int wi = w;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const int v = __shfl_up_sync(0xffffffffu, wi, o);
+                if (lane >= o) wi += v;
+            }
+            warp_tot[lane] = wi - w;  // exclusive warp prefix
+        }
+        __syncthreads();
+        const int excl = s_carry + warp_tot[warp] + incl - blocks;
+        if (f < a.F) a.block_start[f] = excl;
+        __syncthreads();
+        if (tid == kMapThreads - 1) s_carry = excl + blocks;
+        __syncthreads();
+    }
+    if (tid == 0) a.block_start[a.F] = s_carry;
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+
+int map_launch(const MapArgs &a, void *stream) {
+    recflex_map_kernel<<<1, kMapThreads, 0, (cudaStream_t)stream>>>(a);
+    return (int)cudaGetLastError();
+}
+
+// ---------------------------------------------------------------------------
+// Fill kernel (only for lookup-partitioned features): task_start[q] = first
+// sample whose bag starts in lookup window q (Fig. 8's d_task_map payload for
+// adaptive tasks).  Thread per (feature, sample); disjoint writes.
+// ---------------------------------------------------------------------------
+__global__ void __launch_bounds__(256) recflex_fill_kernel(FillArgs a) {
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    const int k = blockIdx.y;
+    const int f = a.part1_features[k];
+    const FeatureDesc &fd = a.desc[f];
+    const int s = blockIdx.x * blockDim.x + threadIdx.x;
+    if (s < a.B) {
+        const int32_t *offs = a.offsets + (size_t)fd.in_feature * a.B;
+        const int base = offs[0];
+        const int npb = a.npb_eff[f];
+        const int blocks = a.block_start[f + 1] - a.block_start[f];
+        int32_t *ts = a.task_start + fd.slot_base;
+        const int q_hi = (offs[s] - base) / npb;
+        const int q_lo = (s == 0) ? -1 : (offs[s - 1] - base) / npb;
+        for (int q = q_lo + 1; q <= q_hi && q <= blocks; ++q) ts[q] = s;
+        if (s == a.B - 1)
+            for (int q = q_hi + 1; q <= blocks; ++q) ts[q] = a.B;
+    }
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+
+int fill_launch(const FillArgs &a, int grid_x, bool pdl, void *stream) {
+    cudaLaunchConfig_t lc = {};
+    lc.gridDim = dim3(grid_x, a.num_part1);
+    lc.blockDim = dim3(256);
+    lc.stream = (cudaStream_t)stream;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = pdl ? 1 : 0;
+    lc.attrs = attr;
+    lc.numAttrs = 1;
+    return (int)cudaLaunchKernelEx(&lc, recflex_fill_kernel, a);
+}
+
+// ---------------------------------------------------------------------------
+// Validation: flag bit 1 = bad offsets, bit 2 = index out of range.
+// ---------------------------------------------------------------------------
+__global__ void recflex_validate_kernel(const FeatureDesc *desc, int F, int in_F, const int32_t *indices,
+                                        const int32_t *offsets, int B, int32_t *flag) {
+    const int64_t n_off = (int64_t)in_F * B;
+    const int64_t gtid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    if (blockIdx.y == 0) {
+        for (int64_t k = gtid; k < n_off; k += stride)
+            if (offsets[k + 1] < offsets[k]) atomicOr(flag, 1);
+        if (gtid == 0 && offsets[0] != 0) atomicOr(flag, 1);
+        return;
+    }
+    const int f = blockIdx.y - 1;
+    if (f >= F) return;
+    const FeatureDesc &fd = desc[f];
+    const int64_t a = offsets[(int64_t)fd.in_feature * B], b = offsets[(int64_t)(fd.in_feature + 1) * B];
+    for (int64_t j = a + gtid; j < b; j += stride) {
+        const int v = indices[j];
+        if (v < 0 || (int64_t)v >= fd.rows) atomicOr(flag, 2);
+    }
+}
+
+int validate_launch(const FeatureDesc *desc, int F, int in_F, const int32_t *indices, const int32_t *offsets, int B,
+                    int32_t *flag, void *stream) {
+    dim3 grid(64, F + 1);
+    recflex_validate_kernel<<<grid, 256, 0, (cudaStream_t)stream>>>(desc, F, in_F, indices, offsets, B, flag);
+    return (int)cudaGetLastError();
+}
+
+// dst[i] = (src[i] + shift) mod rows  -- the tuner's duplicated input (reading C17)
+__global__ void recflex_remap_kernel(const int32_t *src, int32_t *dst, int64_t n, int64_t shift, int64_t rows) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        dst[i] = (int32_t)(((int64_t)src[i] + shift) % rows);
+}
+
+int remap_launch(const int32_t *src, int32_t *dst, int64_t n, int64_t shift, int64_t rows, void *stream) {
+    if (n <= 0) return 0;
+    int grid = (int)((n + 255) / 256);
+    if (grid > 4096) grid = 4096;
+    recflex_remap_kernel<<<grid, 256, 0, (cudaStream_t)stream>>>(src, dst, n, shift, rows);
+    return (int)cudaGetLastError();
+}
+
+// Relayout after the pooled-output all-to-all: chunk i [rows][dims[i]] -> columns
+__global__ void recflex_concat_kernel(const float *recv, int W, int rows, const int32_t *dims, const int32_t *cols,
+                                      int d_tot, float *out) {
+    const int64_t n = (int64_t)rows * d_tot;
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x) {
+        const int r = (int)(e / d_tot);
+        const int q = (int)(e % d_tot);
+        int i = 0;
+        while (i + 1 < W && cols[i + 1] <= q) ++i;
+        const int64_t chunk_base = (int64_t)rows * cols[i];  // chunks are contiguous in rank order
+        out[e] = recv[chunk_base + (int64_t)r * dims[i] + (q - cols[i])];
+    }
+}
+
+int concat_launch(const float *recv, int W, int rows, const int32_t *d_dims, const int32_t *d_cols, int d_tot,
+                  float *out, void *stream) {
+    const int64_t n = (int64_t)rows * d_tot;
+    if (n == 0) return 0;
+    int grid = (int)((n + 255) / 256);
+    if (grid > 148 * 16) grid = 148 * 16;
+    recflex_concat_kernel<<<grid, 256, 0, (cudaStream_t)stream>>>(recv, W, rows, d_dims, d_cols, d_tot, out);
+    return (int)cudaGetLastError();
+}
+
+__global__ void recflex_flush_kernel(float4 *buf, int64_t n4, float v) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += (int64_t)gridDim.x * blockDim.x)
+        buf[i] = make_float4(v, v, v, v);
+}
+
+int flush_launch(void *buf, size_t bytes, void *stream) {
+    const int64_t n4 = (int64_t)(bytes / 16);
+    if (n4 == 0) return 0;
+    recflex_flush_kernel<<<148 * 8, 256, 0, (cudaStream_t)stream>>>((float4 *)buf, n4, 0.f);
+    return (int)cudaGetLastError();
+}
+
+}  // namespace recflex

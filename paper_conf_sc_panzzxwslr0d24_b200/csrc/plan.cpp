@@ -1,0 +1,734 @@
+// plan.cpp -- C ABI: plan lifecycle, forward, schedules, occupancy, validation,
+// introspection, persistence.  (Tuner in tuner.cpp.)
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "plan_internal.h"
+
+using namespace recflex;
+
+namespace recflex {
+
+recflex_status_t cuda_status(cudaError_t e) {
+    if (e == cudaSuccess) return RECFLEX_OK;
+    if (e == cudaErrorMemoryAllocation) return RECFLEX_ERR_OOM;
+    return RECFLEX_ERR_CUDA;
+}
+
+static int next_pow2(int v) {
+    int p = 1;
+    while (p < v) p <<= 1;
+    return p;
+}
+
+int find_catalog(int family, int G, int VEC, int C, int U) {
+    for (int i = 0; i < kCatalogSize; ++i) {
+        const CatalogEntry &e = kCatalog[i];
+        if (e.family == family && e.G == G && e.VEC == VEC && e.C == C && e.U == U) return i;
+    }
+    return -1;
+}
+
+// samples per task for sample-partitioned tasks: ~4096 expected lookups per
+// task (enough work to amortise the task fetch), between 1 and 32 rounds of
+// the CTA's bag slots.
+int samples_per_task_default(int sched_id, float mean_len, float coverage) {
+    const CatalogEntry &e = kCatalog[sched_id];
+    const int slots = (e.family == RECFLEX_FAMILY_GROUP) ? kBlockThreads / e.G : 1;
+    double el = std::max(0.25, (double)mean_len * std::max(0.05, (double)coverage));
+    int R = (int)std::lround(4096.0 / (slots * el));
+    R = std::min(32, std::max(1, R));
+    if (e.family == RECFLEX_FAMILY_BLOCK) R = std::min(64, std::max(1, (int)std::lround(2048.0 / el)));
+    return slots * R;
+}
+
+recflex_schedule_t default_schedule(const recflex_feature_spec_t &spec) {
+    recflex_schedule_t s = {0, 0, 1};
+    const int d = spec.dim;
+    int id = -1;
+    if (d % 4 == 0) {
+        int lanes = d / 4;
+        int G = std::min(32, next_pow2(lanes));
+        int C = (lanes > 32) ? 2 : 1;
+        int U = spec.mean_len >= 6.f ? 8 : (spec.mean_len >= 2.5f ? 4 : 2);
+        if (C == 2 && U > 4) U = 4;
+        id = find_catalog(RECFLEX_FAMILY_GROUP, G, 4, C, U);
+    }
+    if (id < 0) id = find_catalog(RECFLEX_FAMILY_GROUP, std::min(32, next_pow2(d)), 1, 1, 4);
+    s.sched_id = id;
+    s.part = 0;
+    s.per_block = samples_per_task_default(id, spec.mean_len, spec.coverage);
+    return s;
+}
+
+int slots_for(int max_batch, float max_len) {
+    // reserved task-range entries for a lookup-partitioned feature: tasks of
+    // >= 128 lookups at the planned maximum, + sentinel; the map kernel raises
+    // the per-task lookups if a batch would need more (always correct).
+    double ml = std::max(1.0, (double)max_len);
+    double need = (double)max_batch * ml / 128.0 + 3.0;
+    need = std::min(need, (double)(1 << 20));
+    return (int)std::max(64.0, need);
+}
+
+bool schedule_valid_for(const recflex_schedule_t &s, int dim, int col, int d_tot) {
+    if (s.sched_id < 0 || s.sched_id >= kCatalogSize) return false;
+    if (s.part != 0 && s.part != 1) return false;
+    if (s.per_block < 1) return false;
+    const CatalogEntry &e = kCatalog[s.sched_id];
+    if (!catalog_valid(e, dim)) return false;
+    // vector stores need 16-byte aligned output columns
+    if (e.VEC > 1 && ((col % 4) != 0 || (d_tot % 4) != 0)) return false;
+    return true;
+}
+
+int min_dyn_smem(int F) {
+    int m = 8 * 256 * 4;  // BLOCK-family reduction scratch
+    if (F + 1 <= kSmemBlockStartCap) m += 4 * (F + 1);
+    return (m + 127) / 128 * 128;
+}
+
+// Shared-memory padding so that exactly k CTAs fit per SM (C15).
+recflex_status_t prepare_occupancy(recflex_plan_s *p, int k) {
+    if (k < 1 || k > kMaxOcc) return RECFLEX_ERR_INVALID_ARG;
+    if (p->prepared[k]) return RECFLEX_OK;
+    cudaError_t e = cudaSetDevice(p->device);
+    if (e != cudaSuccess) return cuda_status(e);
+    const int sm_total = 233472;  // 228 KB per SM
+    int dyn = ((sm_total / k - 1152) / 128) * 128;
+    dyn = std::max(dyn, min_dyn_smem(p->F));
+    dyn = std::min(dyn, 232448 - 128);
+    int rc = fused_prepare(k, p->device, 232448 - 128);
+    if (rc) return cuda_status((cudaError_t)rc);
+    int blocks = 0, regs = 0, spill = 0;
+    // walk the padding until the occupancy API reports exactly k (or as close as possible)
+    for (int it = 0; it < 64; ++it) {
+        rc = fused_occupancy(k, dyn, &blocks, &regs, &spill);
+        if (rc) return cuda_status((cudaError_t)rc);
+        if (blocks > k) {
+            dyn += 128;
+        } else if (blocks < k && dyn - 128 >= min_dyn_smem(p->F)) {
+            int b2 = 0;
+            fused_occupancy(k, dyn - 128, &b2, &regs, &spill);
+            if (b2 <= k) dyn -= 128;
+            else break;
+            if (b2 == k) break;
+        } else {
+            break;
+        }
+    }
+    rc = fused_occupancy(k, dyn, &blocks, &regs, &spill);
+    if (rc) return cuda_status((cudaError_t)rc);
+    p->smem[k] = dyn;
+    p->occ[k] = std::max(1, std::min(blocks, k));
+    p->prepared[k] = true;
+    return RECFLEX_OK;
+}
+
+recflex_status_t upload_desc(recflex_plan_s *p, cudaStream_t stream) {
+    for (int f = 0; f < p->F; ++f) p->desc[f].table = p->tables[f];
+    p->part1.clear();
+    for (int f = 0; f < p->F; ++f)
+        if (p->desc[f].part == 1) p->part1.push_back(f);
+    cudaError_t e = cudaMemcpyAsync(p->ex.d_desc, p->desc.data(), sizeof(FeatureDesc) * p->F,
+                                    cudaMemcpyHostToDevice, stream);
+    if (e != cudaSuccess) return cuda_status(e);
+    if (!p->part1.empty()) {
+        e = cudaMemcpyAsync(p->ex.d_part1, p->part1.data(), sizeof(int32_t) * p->part1.size(), cudaMemcpyHostToDevice,
+                            stream);
+        if (e != cudaSuccess) return cuda_status(e);
+    }
+    p->ex.num_part1 = (int)p->part1.size();
+    p->desc_dirty = false;
+    return RECFLEX_OK;
+}
+
+recflex_status_t run_pipeline(recflex_plan_s *p, const Exec &ex, const int32_t *indices, const int32_t *offsets,
+                              int B, float *out, int out_stride, int k, cudaStream_t stream, EventTriple *ev) {
+    recflex_status_t st = prepare_occupancy(p, k);
+    if (st != RECFLEX_OK) return st;
+    if (ev) cudaEventRecord(ev->e0, stream);
+    MapArgs ma;
+    ma.desc = ex.d_desc;
+    ma.offsets = offsets;
+    ma.F = ex.F;
+    ma.B = B;
+    ma.in_F = ex.in_F;
+    ma.block_start = ex.d_block_start;
+    ma.npb_eff = ex.d_npb_eff;
+    ma.counter = ex.d_counter;
+    int rc = map_launch(ma, stream);
+    if (rc) return cuda_status((cudaError_t)rc);
+    if (ex.num_part1 > 0) {
+        FillArgs fa;
+        fa.desc = ex.d_desc;
+        fa.offsets = offsets;
+        fa.block_start = ex.d_block_start;
+        fa.npb_eff = ex.d_npb_eff;
+        fa.part1_features = ex.d_part1;
+        fa.num_part1 = ex.num_part1;
+        fa.B = B;
+        fa.task_start = ex.d_task_start;
+        rc = fill_launch(fa, (B + 255) / 256, p->pdl, stream);
+        if (rc) return cuda_status((cudaError_t)rc);
+    }
+    if (ev) cudaEventRecord(ev->e1, stream);
+    FusedArgs a;
+    a.desc = ex.d_desc;
+    a.block_start = ex.d_block_start;
+    a.task_start = ex.d_task_start;
+    a.indices = indices;
+    a.offsets = offsets;
+    a.out = out;
+    a.counter = ex.d_counter;
+    a.timers = ex.d_timers;
+    a.timers_cap = ex.timers_cap;
+    a.F = ex.F;
+    a.B = B;
+    a.out_stride = out_stride;
+    LaunchCfg cfg;
+    cfg.grid = p->num_sms * p->occ[k];
+    cfg.smem = p->smem[k];
+    // With events between the kernels, PDL overlap is disabled (the event is a
+    // stream dependency point anyway).
+    cfg.pdl = p->pdl && ev == nullptr;
+    rc = fused_launch(k, a, cfg, stream);
+    if (rc) return cuda_status((cudaError_t)rc);
+    if (ev) cudaEventRecord(ev->e2, stream);
+    return RECFLEX_OK;
+}
+
+}  // namespace recflex
+
+// ===========================================================================
+// C ABI
+// ===========================================================================
+extern "C" {
+
+const char *recflex_status_string(recflex_status_t s) {
+    switch (s) {
+        case RECFLEX_OK: return "ok";
+        case RECFLEX_ERR_INVALID_ARG: return "invalid argument";
+        case RECFLEX_ERR_CUDA: return "CUDA error";
+        case RECFLEX_ERR_OOM: return "out of device memory";
+        case RECFLEX_ERR_NOT_SUPPORTED: return "not supported";
+        case RECFLEX_ERR_INDEX_OOB: return "lookup ID out of range";
+    }
+    return "unknown status";
+}
+
+int32_t recflex_catalog_size(void) { return kCatalogSize; }
+
+recflex_status_t recflex_catalog_info(int32_t id, recflex_catalog_info_t *info) {
+    if (id < 0 || id >= kCatalogSize || !info) return RECFLEX_ERR_INVALID_ARG;
+    const CatalogEntry &e = kCatalog[id];
+    info->family = e.family;
+    info->group = e.G;
+    info->vec = e.VEC;
+    info->cols = e.C;
+    info->unroll = e.U;
+    return RECFLEX_OK;
+}
+
+int32_t recflex_catalog_valid(int32_t id, int32_t dim) {
+    if (id < 0 || id >= kCatalogSize) return 0;
+    return catalog_valid(kCatalog[id], dim) ? 1 : 0;
+}
+
+static void plan_free_device(recflex_plan_s *p) {
+    cudaFree(p->ex.d_desc);
+    cudaFree(p->ex.d_block_start);
+    cudaFree(p->ex.d_npb_eff);
+    cudaFree(p->ex.d_counter);
+    cudaFree(p->ex.d_task_start);
+    cudaFree(p->ex.d_part1);
+    cudaFree(p->d_stage_idx);
+    cudaFree(p->d_stage_off);
+    cudaFree(p->d_stage_out);
+    for (auto &t : p->ev_pending) {
+        cudaEventDestroy(t.e0);
+        cudaEventDestroy(t.e1);
+        cudaEventDestroy(t.e2);
+    }
+    for (auto &t : p->ev_free) {
+        cudaEventDestroy(t.e0);
+        cudaEventDestroy(t.e1);
+        cudaEventDestroy(t.e2);
+    }
+}
+
+recflex_status_t recflex_plan_create(const recflex_feature_spec_t *specs, int32_t F, int32_t max_batch, int32_t device,
+                                     recflex_plan_t *out) {
+    if (!specs || !out || F <= 0 || max_batch <= 0) return RECFLEX_ERR_INVALID_ARG;
+    *out = nullptr;
+    int64_t d_tot = 0;
+    for (int f = 0; f < F; ++f) {
+        const recflex_feature_spec_t &s = specs[f];
+        if (s.num_rows <= 0 || s.num_rows >= (int64_t(1) << 31)) return RECFLEX_ERR_INVALID_ARG;
+        if (s.dim <= 0 || s.dim > 65536) return RECFLEX_ERR_INVALID_ARG;
+        if (s.pool != RECFLEX_POOL_SUM && s.pool != RECFLEX_POOL_MEAN) return RECFLEX_ERR_INVALID_ARG;
+        if (!(s.mean_len >= 0.f) || !(s.max_len >= 0.f) || !(s.coverage >= 0.f) || s.coverage > 1.f)
+            return RECFLEX_ERR_INVALID_ARG;
+        d_tot += s.dim;
+    }
+    if (d_tot >= (int64_t(1) << 31) || (int64_t)max_batch * d_tot >= (int64_t(1) << 40)) return RECFLEX_ERR_INVALID_ARG;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) return RECFLEX_ERR_INVALID_ARG;
+    if (cudaSetDevice(device) != cudaSuccess) return RECFLEX_ERR_CUDA;
+
+    recflex_plan_s *p = new recflex_plan_s();
+    p->device = device;
+    p->F = F;
+    p->max_batch = max_batch;
+    p->d_tot = d_tot;
+    p->specs.assign(specs, specs + F);
+    cudaDeviceGetAttribute(&p->num_sms, cudaDevAttrMultiProcessorCount, device);
+    p->desc.resize(F);
+    p->tables.assign(F, nullptr);
+    int64_t col = 0, slot = 0;
+    for (int f = 0; f < F; ++f) {
+        FeatureDesc &d = p->desc[f];
+        std::memset(&d, 0, sizeof(d));
+        d.rows = specs[f].num_rows;
+        d.dim = specs[f].dim;
+        d.col = (int32_t)col;
+        d.pool = specs[f].pool;
+        d.in_feature = f;
+        d.cap = 0;
+        d.slots = slots_for(max_batch, specs[f].max_len);
+        d.slot_base = (int32_t)slot;
+        slot += d.slots;
+        col += specs[f].dim;
+    }
+    if (slot >= (int64_t(1) << 31)) {
+        delete p;
+        return RECFLEX_ERR_INVALID_ARG;
+    }
+    p->slots_total = slot;
+    for (int f = 0; f < F; ++f) {
+        recflex_schedule_t s = default_schedule(specs[f]);
+        if (!schedule_valid_for(s, p->desc[f].dim, p->desc[f].col, (int)d_tot)) {
+            s.sched_id = find_catalog(RECFLEX_FAMILY_GROUP, std::min(32, next_pow2(specs[f].dim)), 1, 1, 4);
+            s.per_block = samples_per_task_default(s.sched_id, specs[f].mean_len, specs[f].coverage);
+        }
+        p->desc[f].sched = s.sched_id;
+        p->desc[f].part = s.part;
+        p->desc[f].per_block = s.per_block;
+    }
+    cudaError_t e = cudaSuccess;
+    p->ex.F = F;
+    p->ex.in_F = F;
+    if (e == cudaSuccess) e = cudaMalloc(&p->ex.d_desc, sizeof(FeatureDesc) * F);
+    if (e == cudaSuccess) e = cudaMalloc(&p->ex.d_block_start, sizeof(int32_t) * (F + 1));
+    if (e == cudaSuccess) e = cudaMalloc(&p->ex.d_npb_eff, sizeof(int32_t) * F);
+    if (e == cudaSuccess) e = cudaMalloc(&p->ex.d_counter, sizeof(int32_t) * 4);
+    if (e == cudaSuccess) e = cudaMalloc(&p->ex.d_task_start, sizeof(int32_t) * std::max<int64_t>(1, slot));
+    if (e == cudaSuccess) e = cudaMalloc(&p->ex.d_part1, sizeof(int32_t) * F);
+    if (e == cudaSuccess) e = cudaMemset(p->ex.d_npb_eff, 0, sizeof(int32_t) * F);
+    if (e != cudaSuccess) {
+        plan_free_device(p);
+        delete p;
+        return cuda_status(e);
+    }
+    if (const char *env = std::getenv("RECFLEX_OCCUPANCY")) {
+        int k = std::atoi(env);
+        if (k >= 1 && k <= kMaxOcc) p->k = k;
+    }
+    if (const char *env = std::getenv("RECFLEX_NO_PDL")) p->pdl = !(env[0] == '1');
+    *out = p;
+    return RECFLEX_OK;
+}
+
+void recflex_destroy(recflex_plan_t p) {
+    if (!p) return;
+    cudaSetDevice(p->device);
+    plan_free_device(p);
+    delete p;
+}
+
+static recflex_status_t sync_tables(recflex_plan_s *p, const float *const *tables, cudaStream_t stream) {
+    bool changed = false;
+    for (int f = 0; f < p->F; ++f) {
+        const float *t = tables[f];
+        if (!t) return RECFLEX_ERR_INVALID_ARG;
+        if (t != p->tables[f]) {
+            const CatalogEntry &e = kCatalog[p->desc[f].sched];
+            (void)e;
+            if (((uintptr_t)t) % 32 != 0) return RECFLEX_ERR_INVALID_ARG;
+            p->tables[f] = t;
+            changed = true;
+        }
+    }
+    if (changed || p->desc_dirty) return upload_desc(p, stream);
+    return RECFLEX_OK;
+}
+
+recflex_status_t recflex_forward(recflex_plan_t p, const int32_t *indices, const int32_t *offsets, int32_t B,
+                                 const float *const *tables, float *out, void *stream_) {
+    if (!p || !tables) return RECFLEX_ERR_INVALID_ARG;
+    if (B < 0 || B > p->max_batch) return RECFLEX_ERR_INVALID_ARG;
+    if (B == 0) return RECFLEX_OK;
+    if (!indices || !offsets || !out) return RECFLEX_ERR_INVALID_ARG;
+    if (((uintptr_t)out) % 16 != 0) return RECFLEX_ERR_INVALID_ARG;
+    cudaStream_t stream = (cudaStream_t)stream_;
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (cur != p->device) cudaSetDevice(p->device);
+    recflex_status_t st = sync_tables(p, tables, stream);
+    if (st != RECFLEX_OK) return st;
+    EventTriple *ev = nullptr;
+    EventTriple trip;
+    if (p->profiling) {
+        if (!p->ev_free.empty()) {
+            trip = p->ev_free.back();
+            p->ev_free.pop_back();
+        } else {
+            cudaEventCreate(&trip.e0);
+            cudaEventCreate(&trip.e1);
+            cudaEventCreate(&trip.e2);
+        }
+        ev = &trip;
+    }
+    st = run_pipeline(p, p->ex, indices, offsets, B, out, (int)p->d_tot, p->k, stream, ev);
+    if (ev) p->ev_pending.push_back(trip);
+    return st;
+}
+
+recflex_status_t recflex_forward_host(recflex_plan_t p, const int32_t *h_indices, int64_t nnz, const int32_t *h_offsets,
+                                      int32_t B, const float *const *tables, float *h_out, void *stream_) {
+    if (!p || !tables || B < 0 || B > p->max_batch || nnz < 0) return RECFLEX_ERR_INVALID_ARG;
+    if (B == 0) return RECFLEX_OK;
+    if (!h_offsets || !h_out || (nnz > 0 && !h_indices)) return RECFLEX_ERR_INVALID_ARG;
+    cudaStream_t stream = (cudaStream_t)stream_;
+    cudaSetDevice(p->device);
+    const int64_t n_off = (int64_t)p->F * B + 1;
+    const int64_t n_out = (int64_t)B * p->d_tot;
+    cudaError_t e = cudaSuccess;
+    if (nnz > p->stage_idx_cap) {
+        cudaFree(p->d_stage_idx);
+        p->d_stage_idx = nullptr;
+        e = cudaMalloc(&p->d_stage_idx, sizeof(int32_t) * std::max<int64_t>(nnz, 1));
+        if (e != cudaSuccess) return cuda_status(e);
+        p->stage_idx_cap = nnz;
+    }
+    if (!p->d_stage_idx) {
+        e = cudaMalloc(&p->d_stage_idx, sizeof(int32_t));
+        if (e != cudaSuccess) return cuda_status(e);
+    }
+    if (n_off > p->stage_off_cap) {
+        cudaFree(p->d_stage_off);
+        e = cudaMalloc(&p->d_stage_off, sizeof(int32_t) * n_off);
+        if (e != cudaSuccess) return cuda_status(e);
+        p->stage_off_cap = n_off;
+    }
+    if (n_out > p->stage_out_cap) {
+        cudaFree(p->d_stage_out);
+        e = cudaMalloc(&p->d_stage_out, sizeof(float) * n_out);
+        if (e != cudaSuccess) return cuda_status(e);
+        p->stage_out_cap = n_out;
+    }
+    if (nnz > 0) e = cudaMemcpyAsync(p->d_stage_idx, h_indices, sizeof(int32_t) * nnz, cudaMemcpyHostToDevice, stream);
+    if (e == cudaSuccess)
+        e = cudaMemcpyAsync(p->d_stage_off, h_offsets, sizeof(int32_t) * n_off, cudaMemcpyHostToDevice, stream);
+    if (e != cudaSuccess) return cuda_status(e);
+    recflex_status_t st = recflex_forward(p, p->d_stage_idx, p->d_stage_off, B, tables, p->d_stage_out, stream);
+    if (st != RECFLEX_OK) return st;
+    e = cudaMemcpyAsync(h_out, p->d_stage_out, sizeof(float) * n_out, cudaMemcpyDeviceToHost, stream);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(stream);
+    return cuda_status(e);
+}
+
+recflex_status_t recflex_get_schedule(recflex_plan_t p, int32_t f, recflex_schedule_t *s, int32_t *blocks_per_sm) {
+    if (!p || f < 0 || f >= p->F) return RECFLEX_ERR_INVALID_ARG;
+    if (s) {
+        s->sched_id = p->desc[f].sched;
+        s->part = p->desc[f].part;
+        s->per_block = p->desc[f].per_block;
+    }
+    if (blocks_per_sm) *blocks_per_sm = p->k;
+    return RECFLEX_OK;
+}
+
+recflex_status_t recflex_set_schedule(recflex_plan_t p, int32_t f, const recflex_schedule_t *s) {
+    if (!p || !s || f < 0 || f >= p->F) return RECFLEX_ERR_INVALID_ARG;
+    if (!schedule_valid_for(*s, p->desc[f].dim, p->desc[f].col, (int)p->d_tot)) return RECFLEX_ERR_INVALID_ARG;
+    p->desc[f].sched = s->sched_id;
+    p->desc[f].part = s->part;
+    p->desc[f].per_block = s->per_block;
+    p->desc_dirty = true;
+    return RECFLEX_OK;
+}
+
+recflex_status_t recflex_set_occupancy(recflex_plan_t p, int32_t k) {
+    if (!p || k < 1 || k > kMaxOcc) return RECFLEX_ERR_INVALID_ARG;
+    p->k = k;
+    return RECFLEX_OK;
+}
+
+recflex_status_t recflex_get_occupancy(recflex_plan_t p, int32_t *k) {
+    if (!p || !k) return RECFLEX_ERR_INVALID_ARG;
+    *k = p->k;
+    return RECFLEX_OK;
+}
+
+recflex_status_t recflex_occupancy_check(int32_t device, int32_t k, int32_t *active, int32_t *regs, int32_t *spill) {
+    if (k < 1 || k > kMaxOcc) return RECFLEX_ERR_INVALID_ARG;
+    recflex_feature_spec_t spec = {1000, 16, 0, 1.f, 1.f, 1.f};
+    recflex_plan_t p = nullptr;
+    recflex_status_t st = recflex_plan_create(&spec, 1, 1, device, &p);
+    if (st != RECFLEX_OK) return st;
+    st = prepare_occupancy(p, k);
+    if (st == RECFLEX_OK) {
+        int b = 0, r = 0, s = 0;
+        int rc = fused_occupancy(k, p->smem[k], &b, &r, &s);
+        if (rc) st = cuda_status((cudaError_t)rc);
+        if (active) *active = b;
+        if (regs) *regs = r;
+        if (spill) *spill = s;
+    }
+    recflex_destroy(p);
+    return st;
+}
+
+recflex_status_t recflex_debug_task_map(recflex_plan_t p, const int32_t *offsets, int32_t B, int32_t *h_bs,
+                                        int32_t *h_ranges, int64_t cap, void *stream_) {
+    if (!p || !offsets || !h_bs || B < 0 || B > p->max_batch) return RECFLEX_ERR_INVALID_ARG;
+    cudaStream_t stream = (cudaStream_t)stream_;
+    cudaSetDevice(p->device);
+    if (p->desc_dirty || p->ex.num_part1 != 0 || true) {
+        // descriptors may be stale if no forward ran yet (tables not known): upload with null tables
+        for (int f = 0; f < p->F; ++f) p->desc[f].table = p->tables[f];
+        recflex_status_t st = upload_desc(p, stream);
+        if (st != RECFLEX_OK) return st;
+    }
+    MapArgs ma;
+    ma.desc = p->ex.d_desc;
+    ma.offsets = offsets;
+    ma.F = p->F;
+    ma.B = B;
+    ma.in_F = p->F;
+    ma.block_start = p->ex.d_block_start;
+    ma.npb_eff = p->ex.d_npb_eff;
+    ma.counter = p->ex.d_counter;
+    int rc = map_launch(ma, stream);
+    if (rc) return cuda_status((cudaError_t)rc);
+    if (p->ex.num_part1 > 0 && B > 0) {
+        FillArgs fa;
+        fa.desc = p->ex.d_desc;
+        fa.offsets = offsets;
+        fa.block_start = p->ex.d_block_start;
+        fa.npb_eff = p->ex.d_npb_eff;
+        fa.part1_features = p->ex.d_part1;
+        fa.num_part1 = p->ex.num_part1;
+        fa.B = B;
+        fa.task_start = p->ex.d_task_start;
+        rc = fill_launch(fa, (B + 255) / 256, false, stream);
+        if (rc) return cuda_status((cudaError_t)rc);
+    }
+    cudaError_t e = cudaMemcpyAsync(h_bs, p->ex.d_block_start, sizeof(int32_t) * (p->F + 1), cudaMemcpyDeviceToHost,
+                                    stream);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(stream);
+    if (e != cudaSuccess) return cuda_status(e);
+    if (h_ranges) {
+        const int64_t total = h_bs[p->F];
+        if (cap < 2 * total) return RECFLEX_ERR_INVALID_ARG;
+        std::vector<int32_t> ts;
+        if (p->slots_total > 0) {
+            ts.resize(p->slots_total);
+            e = cudaMemcpy(ts.data(), p->ex.d_task_start, sizeof(int32_t) * p->slots_total, cudaMemcpyDeviceToHost);
+            if (e != cudaSuccess) return cuda_status(e);
+        }
+        for (int f = 0; f < p->F; ++f) {
+            for (int64_t t = h_bs[f]; t < h_bs[f + 1]; ++t) {
+                const int rel = (int)(t - h_bs[f]);
+                if (p->desc[f].part == 1) {
+                    h_ranges[2 * t] = ts[p->desc[f].slot_base + rel];
+                    h_ranges[2 * t + 1] = ts[p->desc[f].slot_base + rel + 1];
+                } else {
+                    h_ranges[2 * t] = -1;
+                    h_ranges[2 * t + 1] = -1;
+                }
+            }
+        }
+    }
+    return RECFLEX_OK;
+}
+
+recflex_status_t recflex_validate(recflex_plan_t p, const int32_t *indices, const int32_t *offsets, int32_t B,
+                                  void *stream_) {
+    if (!p || !offsets || B < 0 || B > p->max_batch) return RECFLEX_ERR_INVALID_ARG;
+    if (B == 0) return RECFLEX_OK;
+    cudaStream_t stream = (cudaStream_t)stream_;
+    cudaSetDevice(p->device);
+    recflex_status_t st = upload_desc(p, stream);
+    if (st != RECFLEX_OK) return st;
+    int32_t *d_flag = nullptr;
+    cudaError_t e = cudaMalloc(&d_flag, sizeof(int32_t));
+    if (e != cudaSuccess) return cuda_status(e);
+    cudaMemsetAsync(d_flag, 0, sizeof(int32_t), stream);
+    // offsets first (a broken CSR would make the index ranges meaningless)
+    int rc = validate_launch(p->ex.d_desc, 0, p->F, indices, offsets, B, d_flag, stream);
+    int32_t flag = 0;
+    if (!rc) e = cudaMemcpyAsync(&flag, d_flag, sizeof(int32_t), cudaMemcpyDeviceToHost, stream);
+    if (!rc && e == cudaSuccess) e = cudaStreamSynchronize(stream);
+    if (rc || e != cudaSuccess) {
+        cudaFree(d_flag);
+        return rc ? cuda_status((cudaError_t)rc) : cuda_status(e);
+    }
+    if (flag & 1) {
+        cudaFree(d_flag);
+        return RECFLEX_ERR_INVALID_ARG;
+    }
+    if (!indices) {
+        cudaFree(d_flag);
+        return RECFLEX_ERR_INVALID_ARG;
+    }
+    rc = validate_launch(p->ex.d_desc, p->F, p->F, indices, offsets, B, d_flag, stream);
+    if (!rc) e = cudaMemcpyAsync(&flag, d_flag, sizeof(int32_t), cudaMemcpyDeviceToHost, stream);
+    if (!rc && e == cudaSuccess) e = cudaStreamSynchronize(stream);
+    cudaFree(d_flag);
+    if (rc) return cuda_status((cudaError_t)rc);
+    if (e != cudaSuccess) return cuda_status(e);
+    if (flag & 1) return RECFLEX_ERR_INVALID_ARG;
+    if (flag & 2) return RECFLEX_ERR_INDEX_OOB;
+    return RECFLEX_OK;
+}
+
+recflex_status_t recflex_set_profiling(recflex_plan_t p, int32_t enable) {
+    if (!p) return RECFLEX_ERR_INVALID_ARG;
+    p->profiling = enable != 0;
+    return RECFLEX_OK;
+}
+
+recflex_status_t recflex_get_kernel_times(recflex_plan_t p, double *map_ms, double *fused_ms, int64_t *forwards,
+                                          int32_t reset) {
+    if (!p) return RECFLEX_ERR_INVALID_ARG;
+    for (auto &t : p->ev_pending) {
+        cudaError_t e = cudaEventSynchronize(t.e2);
+        if (e != cudaSuccess) return cuda_status(e);
+        float a = 0, b = 0;
+        cudaEventElapsedTime(&a, t.e0, t.e1);
+        cudaEventElapsedTime(&b, t.e1, t.e2);
+        p->map_ms += a;
+        p->fused_ms += b;
+        p->forwards += 1;
+        p->ev_free.push_back(t);
+    }
+    p->ev_pending.clear();
+    if (map_ms) *map_ms = p->map_ms;
+    if (fused_ms) *fused_ms = p->fused_ms;
+    if (forwards) *forwards = p->forwards;
+    if (reset) {
+        p->map_ms = p->fused_ms = 0;
+        p->forwards = 0;
+    }
+    return RECFLEX_OK;
+}
+
+recflex_status_t recflex_plan_export(recflex_plan_t p, char *buf, size_t cap, size_t *len) {
+    if (!p) return RECFLEX_ERR_INVALID_ARG;
+    std::string s = "{\"abi\": " + std::to_string(RECFLEX_ABI_VERSION) + ", \"catalog_size\": " +
+                    std::to_string(kCatalogSize) + ", \"num_features\": " + std::to_string(p->F) +
+                    ", \"occupancy\": " + std::to_string(p->k) + ", \"schedules\": [";
+    for (int f = 0; f < p->F; ++f) {
+        if (f) s += ", ";
+        s += "[" + std::to_string(p->desc[f].sched) + ", " + std::to_string(p->desc[f].part) + ", " +
+             std::to_string(p->desc[f].per_block) + "]";
+    }
+    s += "]}";
+    if (len) *len = s.size() + 1;
+    if (buf && cap > 0) {
+        size_t n = std::min(cap - 1, s.size());
+        std::memcpy(buf, s.data(), n);
+        buf[n] = '\0';
+        if (cap < s.size() + 1) return RECFLEX_ERR_INVALID_ARG;
+    }
+    return RECFLEX_OK;
+}
+
+static bool parse_int_after(const char *&c, long *v) {
+    while (*c && !(*c == '-' || (*c >= '0' && *c <= '9'))) {
+        if (*c == ']' || *c == '}') return false;
+        ++c;
+    }
+    if (!*c) return false;
+    char *end = nullptr;
+    *v = std::strtol(c, &end, 10);
+    c = end;
+    return true;
+}
+
+recflex_status_t recflex_plan_import(recflex_plan_t p, const char *json) {
+    if (!p || !json) return RECFLEX_ERR_INVALID_ARG;
+    const char *c = std::strstr(json, "\"catalog_size\"");
+    long v = 0;
+    if (!c) return RECFLEX_ERR_INVALID_ARG;
+    c += 14;
+    if (!parse_int_after(c, &v) || v != kCatalogSize) return RECFLEX_ERR_NOT_SUPPORTED;
+    c = std::strstr(json, "\"num_features\"");
+    if (!c) return RECFLEX_ERR_INVALID_ARG;
+    c += 14;
+    if (!parse_int_after(c, &v) || v != p->F) return RECFLEX_ERR_INVALID_ARG;
+    c = std::strstr(json, "\"occupancy\"");
+    if (!c) return RECFLEX_ERR_INVALID_ARG;
+    c += 11;
+    if (!parse_int_after(c, &v) || v < 1 || v > kMaxOcc) return RECFLEX_ERR_INVALID_ARG;
+    const int k = (int)v;
+    c = std::strstr(json, "\"schedules\"");
+    if (!c) return RECFLEX_ERR_INVALID_ARG;
+    c = std::strchr(c, '[');
+    if (!c) return RECFLEX_ERR_INVALID_ARG;
+    ++c;
+    std::vector<recflex_schedule_t> ss(p->F);
+    for (int f = 0; f < p->F; ++f) {
+        c = std::strchr(c, '[');
+        if (!c) return RECFLEX_ERR_INVALID_ARG;
+        ++c;
+        long a = 0, b = 0, d = 0;
+        if (!parse_int_after(c, &a) || !parse_int_after(c, &b) || !parse_int_after(c, &d))
+            return RECFLEX_ERR_INVALID_ARG;
+        ss[f] = {(int32_t)a, (int32_t)b, (int32_t)d};
+        if (!schedule_valid_for(ss[f], p->desc[f].dim, p->desc[f].col, (int)p->d_tot)) return RECFLEX_ERR_INVALID_ARG;
+    }
+    for (int f = 0; f < p->F; ++f) recflex_set_schedule(p, f, &ss[f]);
+    p->k = k;
+    return RECFLEX_OK;
+}
+
+recflex_status_t recflex_shard_concat(const float *recv, int32_t W, int32_t rows, const int32_t *host_dims, float *out,
+                                      void *stream_) {
+    if (!recv || !out || !host_dims || W <= 0 || rows < 0) return RECFLEX_ERR_INVALID_ARG;
+    cudaStream_t stream = (cudaStream_t)stream_;
+    std::vector<int32_t> h(2 * W);
+    int32_t tot = 0;
+    for (int i = 0; i < W; ++i) {
+        if (host_dims[i] < 0) return RECFLEX_ERR_INVALID_ARG;
+        h[i] = host_dims[i];
+        h[W + i] = tot;
+        tot += host_dims[i];
+    }
+    int32_t *d = nullptr;
+    cudaError_t e = cudaMallocAsync(&d, sizeof(int32_t) * 2 * W, stream);
+    if (e != cudaSuccess) return cuda_status(e);
+    e = cudaMemcpyAsync(d, h.data(), sizeof(int32_t) * 2 * W, cudaMemcpyHostToDevice, stream);
+    if (e != cudaSuccess) return cuda_status(e);
+    int rc = concat_launch(recv, W, rows, d, d + W, tot, out, stream);
+    cudaFreeAsync(d, stream);
+    if (rc) return cuda_status((cudaError_t)rc);
+    return RECFLEX_OK;
+}
+
+recflex_status_t recflex_l2_flush(void *buf, size_t bytes, void *stream_) {
+    if (!buf) return RECFLEX_ERR_INVALID_ARG;
+    int rc = flush_launch(buf, bytes, stream_);
+    return rc ? cuda_status((cudaError_t)rc) : RECFLEX_OK;
+}
+
+}  // extern "C"

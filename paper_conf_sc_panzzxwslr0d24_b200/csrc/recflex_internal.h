@@ -1,0 +1,142 @@
+// recflex_internal.h -- shared between host plan code and device kernels of
+// librecflex.so (NOT shared with oracle/).
+#pragma once
+#include <stdint.h>
+
+#include "../../include/recflex.h"
+
+namespace recflex {
+
+constexpr int kBlockThreads = 256;   // one CTA = the thread-mapping unit
+constexpr int kMaxOcc = RECFLEX_MAX_OCCUPANCY;
+constexpr int kSmemBlockStartCap = 4096;   // features whose block_start fits in smem (ints)
+
+// Per-feature device descriptor: the paper's `args + arg_offsets[f]` and
+// `schedule_map[f]` (Fig. 8) folded into one record.
+struct __align__(16) FeatureDesc {
+    const float *table;   // T_f, [rows][dim]
+    int64_t rows;
+    int32_t dim;
+    int32_t col;          // col_f
+    int32_t pool;         // 0 sum, 1 mean
+    int32_t sched;        // catalog id
+    int32_t part;         // 0 sample-partitioned, 1 lookup-partitioned
+    int32_t per_block;    // spb or npb
+    int32_t cap;          // max tasks (tuning padding), 0 = none
+    int32_t slots;        // reserved task-range slots (part 1), incl. sentinel
+    int32_t slot_base;    // first slot of this feature in task_range scratch (part 1)
+    int32_t in_feature;   // which KJT feature slot this descriptor reads (identity for plans)
+};
+static_assert(sizeof(FeatureDesc) == 64, "FeatureDesc layout");
+
+struct MapArgs {
+    const FeatureDesc *desc;
+    const int32_t *offsets;
+    int32_t F;
+    int32_t B;
+    int32_t in_F;          // number of KJT features in offsets (F_in), offsets has in_F*B+1 entries
+    int32_t *block_start;  // [F+1]
+    int32_t *npb_eff;      // [F] effective lookups per task (part 1)
+    int32_t *counter;      // task counter for the persistent fused kernel
+};
+
+struct FillArgs {
+    const FeatureDesc *desc;
+    const int32_t *offsets;
+    const int32_t *block_start;
+    const int32_t *npb_eff;
+    const int32_t *part1_features;  // list of part-1 feature ids
+    int32_t num_part1;
+    int32_t B;
+    int32_t *task_start;            // slots
+};
+
+struct FusedArgs {
+    const FeatureDesc *desc;
+    const int32_t *block_start;   // [F+1]
+    const int32_t *task_start;    // part-1 slots
+    const int32_t *indices;
+    const int32_t *offsets;
+    float *out;
+    int32_t *counter;
+    long long *timers;            // per task cycles (tuning), or nullptr
+    int32_t F;
+    int32_t B;
+    int32_t out_stride;           // D_tot
+    int32_t timers_cap;
+};
+
+// ---------------------------------------------------------------------------
+// Schedule catalog: X(family, G, VEC, C, U).  The id of an entry is its
+// position.  Hand-written templates ("schedule templates").
+// ---------------------------------------------------------------------------
+#define RECFLEX_CATALOG(X)                                                      \
+    /* GROUP, 128-bit rows, one column chunk per lane */                        \
+    X(0, 1, 4, 1, 2) X(0, 1, 4, 1, 4) X(0, 1, 4, 1, 8)                          \
+    X(0, 2, 4, 1, 2) X(0, 2, 4, 1, 4) X(0, 2, 4, 1, 8)                          \
+    X(0, 4, 4, 1, 2) X(0, 4, 4, 1, 4) X(0, 4, 4, 1, 8)                          \
+    X(0, 8, 4, 1, 2) X(0, 8, 4, 1, 4) X(0, 8, 4, 1, 8)                          \
+    X(0, 16, 4, 1, 2) X(0, 16, 4, 1, 4) X(0, 16, 4, 1, 8)                       \
+    X(0, 32, 4, 1, 2) X(0, 32, 4, 1, 4) X(0, 32, 4, 1, 8)                       \
+    /* GROUP, 128-bit rows, two column chunks per lane */                       \
+    X(0, 1, 4, 2, 2) X(0, 1, 4, 2, 4)                                           \
+    X(0, 2, 4, 2, 2) X(0, 2, 4, 2, 4)                                           \
+    X(0, 4, 4, 2, 2) X(0, 4, 4, 2, 4)                                           \
+    X(0, 8, 4, 2, 2) X(0, 8, 4, 2, 4)                                           \
+    X(0, 16, 4, 2, 2) X(0, 16, 4, 2, 4)                                         \
+    X(0, 32, 4, 2, 2) X(0, 32, 4, 2, 4)                                         \
+    /* GROUP, 256-bit rows (LDG.256) */                                         \
+    X(0, 1, 8, 1, 2) X(0, 1, 8, 1, 4)                                           \
+    X(0, 2, 8, 1, 2) X(0, 2, 8, 1, 4)                                           \
+    X(0, 4, 8, 1, 2) X(0, 4, 8, 1, 4)                                           \
+    X(0, 8, 8, 1, 2) X(0, 8, 8, 1, 4)                                           \
+    X(0, 16, 8, 1, 2) X(0, 16, 8, 1, 4)                                         \
+    X(0, 32, 8, 1, 2) X(0, 32, 8, 1, 4)                                         \
+    /* GROUP, scalar rows (any dim / alignment) */                              \
+    X(0, 1, 1, 1, 4) X(0, 2, 1, 1, 4) X(0, 4, 1, 1, 4)                          \
+    X(0, 8, 1, 1, 4) X(0, 16, 1, 1, 4) X(0, 32, 1, 1, 4)                        \
+    /* BLOCK: whole CTA on one bag, 128-bit rows */                             \
+    X(1, 1, 4, 1, 4) X(1, 2, 4, 1, 4) X(1, 4, 4, 1, 4)                          \
+    X(1, 8, 4, 1, 4) X(1, 16, 4, 1, 4) X(1, 32, 4, 1, 2) X(1, 32, 4, 1, 4)     \
+    /* BLOCK, 256-bit rows */                                                   \
+    X(1, 16, 8, 1, 2) X(1, 16, 8, 1, 4)
+
+struct CatalogEntry {
+    int family, G, VEC, C, U;
+};
+
+#define RECFLEX_CAT_ENTRY(fam, g, v, c, u) {fam, g, v, c, u},
+static constexpr CatalogEntry kCatalog[] = {RECFLEX_CATALOG(RECFLEX_CAT_ENTRY)};
+#undef RECFLEX_CAT_ENTRY
+constexpr int kCatalogSize = sizeof(kCatalog) / sizeof(kCatalog[0]);
+
+// Can entry e run a feature of dimension d?  (vector width divides d; at least
+// a quarter of the lanes hold real columns; wide rows take several passes)
+inline bool catalog_valid(const CatalogEntry &e, int d) {
+    if (d <= 0) return false;
+    if (d % e.VEC != 0) return false;
+    int span = e.G * e.VEC * e.C;
+    if (4 * d < span) return false;
+    return true;
+}
+
+// ---- kernel launchers (device code in .cu files) ----------------------------
+struct LaunchCfg {
+    int grid;
+    int smem;     // dynamic shared memory bytes (padding for occupancy control)
+    bool pdl;
+};
+
+int fused_launch(int k, const FusedArgs &a, const LaunchCfg &cfg, void *stream);  // returns cudaError_t
+int fused_prepare(int k, int device, int smem_bytes);                              // cudaFuncSetAttribute
+int fused_occupancy(int k, int smem_bytes, int *blocks, int *regs, int *spill);
+int map_launch(const MapArgs &a, void *stream);
+int fill_launch(const FillArgs &a, int grid_x, bool pdl, void *stream);
+int validate_launch(const FeatureDesc *desc, int F, int in_F, const int32_t *indices, const int32_t *offsets, int B,
+                    int32_t *flag, void *stream);
+int remap_launch(const int32_t *src, int32_t *dst, int64_t n, int64_t shift, int64_t rows, void *stream);
+int concat_launch(const float *recv, int W, int rows, const int32_t *d_dims, const int32_t *d_cols, int d_tot,
+                  float *out, void *stream);
+int flush_launch(void *buf, size_t bytes, void *stream);
+
+}  // namespace recflex

@@ -1,0 +1,290 @@
+// schedules.cuh -- the hand-written schedule catalog (sm_100a).
+//
+// The paper's schedule templates are device functions that do
+// one feature's gather+pool for the CTA's slice of work ("Schedule1 ..
+// ScheduleN", Fig. 8 line 1).  Two families here, each a template over
+//   G   lanes cooperating on one table row (power of two, <= 32),
+//   VEC floats per lane per load (1: 32-bit, 4: LDG.128, 8: LDG.256),
+//   C   column chunks held per lane (row span G*VEC*C floats per pass),
+//   U   rows in flight per lane (unroll of the bag loop).
+// GROUP: 256/G groups per CTA, each group pools whole bags (G = 32 is the
+//        TorchRec-style warp-per-sample mapping, G < 32 packs several samples
+//        per warp for small dims / one-hot fields).
+// BLOCK: the whole CTA pools one bag (HugeCTR-style block-per-sample),
+//        warp-shuffle + shared-memory fixed-order reduction, for long bags.
+//
+// Accumulation is fp32 in registers in a fixed order per (plan, batch):
+// GROUP adds a bag's rows strictly in ascending lookup order, so its result is
+// the sequential fp32 sum; BLOCK uses a fixed strided split + fixed tree.  No
+// floating-point atomics anywhere -> bitwise run-to-run determinism (C22).
+#pragma once
+#include <cuda_runtime.h>
+
+#include "recflex_internal.h"
+
+namespace recflex {
+
+// ---- loads ---------------------------------------------------------------
+// Rows are gathered once and never reused by the CTA: bypass L1 allocation so
+// the (reused) index lines stay resident.  `.nc` = read-only path.
+template <int VEC>
+__device__ __forceinline__ void ld_row(const float *p, float (&v)[VEC]);
+
+template <>
+__device__ __forceinline__ void ld_row<1>(const float *p, float (&v)[1]) {
+    asm("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(v[0]) : "l"(p));
+}
+template <>
+__device__ __forceinline__ void ld_row<4>(const float *p, float (&v)[4]) {
+    asm("ld.global.nc.L1::no_allocate.v4.f32 {%0, %1, %2, %3}, [%4];"
+        : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3])
+        : "l"(p));
+}
+template <>
+__device__ __forceinline__ void ld_row<8>(const float *p, float (&v)[8]) {
+    asm("ld.global.nc.L1::no_allocate.v8.f32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
+        : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3]), "=f"(v[4]), "=f"(v[5]), "=f"(v[6]), "=f"(v[7])
+        : "l"(p));
+}
+
+__device__ __forceinline__ int ld_idx(const int32_t *p) { return __ldg(p); }
+
+template <int VEC>
+__device__ __forceinline__ void st_out(float *p, const float (&v)[VEC]) {
+    if constexpr (VEC == 1) {
+        p[0] = v[0];
+    } else if constexpr (VEC == 4) {
+        *reinterpret_cast<float4 *>(p) = make_float4(v[0], v[1], v[2], v[3]);
+    } else {
+        reinterpret_cast<float4 *>(p)[0] = make_float4(v[0], v[1], v[2], v[3]);
+        reinterpret_cast<float4 *>(p)[1] = make_float4(v[4], v[5], v[6], v[7]);
+    }
+}
+
+// Pool epilogue: MEAN = SUM / L, correctly rounded to fp32; an empty bag stays
+// 0 for both pools (readings C1, C21).  The quotient is formed in fp64 with a
+// Newton-refined reciprocal (relative error < 2^-51) and rounded once to fp32:
+// a/L for a 24-bit-mantissa a and integer 1 <= L < 2^24 is never an fp32
+// rounding midpoint and lies >= ~2^-49 (relative) away from one, so this
+// equals IEEE div.rn -- without div.rn's out-of-line slow-path CALL, whose
+// caller-saved spills would otherwise inflate every inlined schedule.
+__device__ __forceinline__ float div_by_len(float a, int L) {
+    const double b = (double)L;
+    double y;
+    asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(b));
+#pragma unroll
+    for (int it = 0; it < 3; ++it) {
+        const double e = fma(-b, y, 1.0);
+        y = fma(y, e, y);
+    }
+    return (float)((double)a * y);
+}
+
+template <int VEC>
+__device__ __forceinline__ void pool_finish(float (&acc)[VEC], int pool, int L) {
+    if (pool == RECFLEX_POOL_MEAN && L > 0) {
+#pragma unroll
+        for (int e = 0; e < VEC; ++e) acc[e] = div_by_len(acc[e], L);
+    }
+}
+
+// Everything a schedule needs for one task, passed by value (registers): the
+// paper's `args + arg_offsets[feature_idx]` (Fig. 8 line 17) resolved.
+struct TaskCtx {
+    const float *table;     // T_f
+    const int32_t *offs;    // this feature's B+1 offsets
+    const int32_t *idx;     // all lookup IDs
+    float *out;             // out + col_f
+    int dim;
+    int pool;
+    int out_stride;
+    int s0, s1;             // samples of this task
+};
+
+// ---- GROUP family --------------------------------------------------------
+// Samples [s0, s1) of the task; group g takes samples s0+g, s0+g+NG, ...
+template <int G, int VEC, int C, int U>
+__device__ __noinline__ void sched_group(const float *__restrict__ T, const int32_t *__restrict__ offs,
+                                        const int32_t *__restrict__ idx, float *__restrict__ out, int d, int pool,
+                                        int out_stride, int s0, int s1) {
+    constexpr int NG = kBlockThreads / G;
+    constexpr int SPAN = G * VEC * C;
+    const int tid = threadIdx.x;
+    const int gid = tid / G;
+    const int lg = tid % G;
+    const int passes = (d + SPAN - 1) / SPAN;
+
+    for (int s = s0 + gid; s < s1; s += NG) {
+        const int lo = ld_idx(offs + s);
+        const int hi = ld_idx(offs + s + 1);
+        float *__restrict__ orow = out + (size_t)s * out_stride;
+        for (int p = 0; p < passes; ++p) {
+            int colv[C];
+            bool ok[C];
+#pragma unroll
+            for (int c = 0; c < C; ++c) {
+                colv[c] = p * SPAN + c * G * VEC + lg * VEC;
+                ok[c] = colv[c] < d;
+            }
+            float acc[C][VEC];
+#pragma unroll
+            for (int c = 0; c < C; ++c)
+#pragma unroll
+                for (int e = 0; e < VEC; ++e) acc[c][e] = 0.f;
+
+            int j = lo;
+            for (; j + U <= hi; j += U) {
+                int id[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u) id[u] = ld_idx(idx + j + u);
+                float v[U][C][VEC];
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+#pragma unroll
+                    for (int c = 0; c < C; ++c)
+                        if (ok[c]) ld_row<VEC>(T + (size_t)id[u] * d + colv[c], v[u][c]);
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+#pragma unroll
+                    for (int c = 0; c < C; ++c)
+                        if (ok[c])
+#pragma unroll
+                            for (int e = 0; e < VEC; ++e) acc[c][e] += v[u][c][e];
+            }
+            if (j < hi) {  // ragged tail of the bag: n < U rows
+                const int n = hi - j;
+                int id[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u) id[u] = (u < n) ? ld_idx(idx + j + u) : 0;
+                float v[U][C][VEC];
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+#pragma unroll
+                    for (int c = 0; c < C; ++c)
+                        if (u < n && ok[c]) ld_row<VEC>(T + (size_t)id[u] * d + colv[c], v[u][c]);
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+                    if (u < n)
+#pragma unroll
+                        for (int c = 0; c < C; ++c)
+                            if (ok[c])
+#pragma unroll
+                                for (int e = 0; e < VEC; ++e) acc[c][e] += v[u][c][e];
+            }
+#pragma unroll
+            for (int c = 0; c < C; ++c) {
+                if (ok[c]) {
+                    pool_finish<VEC>(acc[c], pool, hi - lo);
+                    st_out<VEC>(orow + colv[c], acc[c]);
+                }
+            }
+        }
+    }
+}
+
+// ---- BLOCK family ----------------------------------------------------------
+// One bag at a time for the whole CTA.  Group g takes lookups lo+g, lo+g+NG, ...
+// (adjacent groups read adjacent IDs: coalesced index loads).  Partials:
+// xor-butterfly across the groups of a warp (every lane gets bit-identical
+// sums), then the 8 warp partials are summed in warp order from shared memory.
+template <int G, int VEC, int C, int U>
+__device__ __noinline__ void sched_block(const float *__restrict__ T, const int32_t *__restrict__ offs,
+                                        const int32_t *__restrict__ idx, float *__restrict__ out, int d, int pool,
+                                        int out_stride, int s0, int s1, float *red /* [8][SPAN] */) {
+    constexpr int NG = kBlockThreads / G;
+    constexpr int SPAN = G * VEC * C;
+    constexpr int NW = kBlockThreads / 32;
+    const int tid = threadIdx.x;
+    const int gid = tid / G;
+    const int lg = tid % G;
+    const int warp = tid >> 5;
+    const int lane = tid & 31;
+    const int passes = (d + SPAN - 1) / SPAN;
+
+    for (int s = s0; s < s1; ++s) {
+        const int lo = ld_idx(offs + s);
+        const int hi = ld_idx(offs + s + 1);
+        float *__restrict__ orow = out + (size_t)s * out_stride;
+        for (int p = 0; p < passes; ++p) {
+            int colv[C];
+            bool ok[C];
+#pragma unroll
+            for (int c = 0; c < C; ++c) {
+                colv[c] = p * SPAN + c * G * VEC + lg * VEC;
+                ok[c] = colv[c] < d;
+            }
+            float acc[C][VEC];
+#pragma unroll
+            for (int c = 0; c < C; ++c)
+#pragma unroll
+                for (int e = 0; e < VEC; ++e) acc[c][e] = 0.f;
+
+            int j = lo + gid;
+            for (; j + (U - 1) * NG < hi; j += U * NG) {
+                int id[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u) id[u] = ld_idx(idx + j + u * NG);
+                float v[U][C][VEC];
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+#pragma unroll
+                    for (int c = 0; c < C; ++c)
+                        if (ok[c]) ld_row<VEC>(T + (size_t)id[u] * d + colv[c], v[u][c]);
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+#pragma unroll
+                    for (int c = 0; c < C; ++c)
+                        if (ok[c])
+#pragma unroll
+                            for (int e = 0; e < VEC; ++e) acc[c][e] += v[u][c][e];
+            }
+            {
+                int id[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u) id[u] = (j + u * NG < hi) ? ld_idx(idx + j + u * NG) : 0;
+                float v[U][C][VEC];
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+#pragma unroll
+                    for (int c = 0; c < C; ++c)
+                        if (j + u * NG < hi && ok[c]) ld_row<VEC>(T + (size_t)id[u] * d + colv[c], v[u][c]);
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+                    if (j + u * NG < hi)
+#pragma unroll
+                        for (int c = 0; c < C; ++c)
+                            if (ok[c])
+#pragma unroll
+                                for (int e = 0; e < VEC; ++e) acc[c][e] += v[u][c][e];
+            }
+            // groups of one warp -> one partial (butterfly: identical on all lanes)
+#pragma unroll
+            for (int o = G; o < 32; o <<= 1)
+#pragma unroll
+                for (int c = 0; c < C; ++c)
+#pragma unroll
+                    for (int e = 0; e < VEC; ++e) acc[c][e] += __shfl_xor_sync(0xffffffffu, acc[c][e], o);
+            if (lane < G) {
+#pragma unroll
+                for (int c = 0; c < C; ++c)
+#pragma unroll
+                    for (int e = 0; e < VEC; ++e) red[warp * SPAN + c * G * VEC + lg * VEC + e] = acc[c][e];
+            }
+            __syncthreads();
+            const int L = hi - lo;
+            for (int q = tid; q < SPAN; q += kBlockThreads) {
+                const int col = p * SPAN + q;
+                if (col < d) {
+                    float v[1] = {0.f};
+#pragma unroll
+                    for (int w = 0; w < NW; ++w) v[0] += red[w * SPAN + q];
+                    pool_finish<1>(v, pool, L);
+                    orow[col] = v[0];
+                }
+            }
+            __syncthreads();
+        }
+    }
+}
+
+}  // namespace recflex

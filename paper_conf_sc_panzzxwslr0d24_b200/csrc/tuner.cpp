@@ -1,0 +1,536 @@
+// tuner.cpp -- the interference-aware two-stage schedule tuner (§IV-A).
+//
+//   Eq. 2: L(s; xi) ~ sum_f sum_b l_b^(f)(s^(f); xi^(f)) / (#SM * O/W)
+//   Eq. 3: per feature, min over s^(f) of sum_b l_b^(f), under a fixed O
+//   Eq. 4: min over O_k of the fused latency with the stage-1 choice s_k
+//   Eq. 5: objectives summed over sampled historical batches xi_i
+//
+// Local stage (Fig. 6/7): for every occupancy k and feature f, ONE
+// launch of the fused kernel whose task list is
+//   [padding tasks: #SM*k] [every candidate of f, each on its own copy of
+//   xi^(f)] [padding tasks: (pad_waves-1)*#SM*k]
+// with per-task clock64 timers; each candidate's score is the sum of
+// its tasks' cycles (Eq. 3), lowest wins (tie -> lower candidate index).
+// Padding tasks are the batch's other features on their current schedules
+// ("redundant embedding operations") and keep every SM at k CTAs while
+// the candidates run.  The duplicated input of candidate c remaps every ID by
+// i -> (i + c*floor(rows/N)) mod rows (reading C17): same statistics, no
+// cross-candidate L2 reuse.
+// Global stage: for each k, time the real fused forward with s_k at
+// occupancy k (median of R event-timed runs after an L2 flush, per batch,
+// summed over batches); argmin, tie -> larger k (reading C20).
+// Complexity: F*K local evaluations + K global evaluations.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <limits>
+#include <vector>
+
+#include "plan_internal.h"
+
+using namespace recflex;
+
+// ---------------------------------------------------------------------------
+// Selection core (testable with a mock cost function)
+// ---------------------------------------------------------------------------
+extern "C" recflex_status_t recflex_two_stage_select(int32_t F, int32_t K, const int32_t *ncand,
+                                                     recflex_local_cost_fn local_cost,
+                                                     recflex_global_cost_fn global_cost, void *user,
+                                                     int32_t *choice_out, int32_t *best_k, int64_t *local_calls,
+                                                     int64_t *global_calls) {
+    if (F <= 0 || K <= 0 || !ncand || !local_cost || !global_cost || !choice_out || !best_k)
+        return RECFLEX_ERR_INVALID_ARG;
+    for (int f = 0; f < F; ++f)
+        if (ncand[f] <= 0) return RECFLEX_ERR_INVALID_ARG;
+    std::vector<std::vector<int32_t>> choice(K, std::vector<int32_t>(F, 0));
+    int64_t lc = 0, gc = 0;
+    // Local stage: one co-execution per (f, k); f outer so a feature's
+    // duplicated input is built once and reused for every k.
+    for (int f = 0; f < F; ++f) {
+        std::vector<double> costs(ncand[f]);
+        for (int k = 0; k < K; ++k) {
+            std::fill(costs.begin(), costs.end(), std::numeric_limits<double>::infinity());
+            local_cost(user, k, f, costs.data());
+            ++lc;
+            int best = 0;
+            for (int c = 1; c < ncand[f]; ++c)
+                if (costs[c] < costs[best]) best = c;
+            choice[k][f] = best;
+        }
+    }
+    // Global stage
+    int bk = 0;
+    double bcost = std::numeric_limits<double>::infinity();
+    for (int k = 0; k < K; ++k) {
+        double c = global_cost(user, k, choice[k].data());
+        ++gc;
+        if (c <= bcost) {  // tie -> larger k
+            bcost = c;
+            bk = k;
+        }
+    }
+    std::memcpy(choice_out, choice[bk].data(), sizeof(int32_t) * F);
+    *best_k = bk;
+    if (local_calls) *local_calls = lc;
+    if (global_calls) *global_calls = gc;
+    return RECFLEX_OK;
+}
+
+namespace {
+
+struct Batch {
+    const int32_t *d_idx;
+    const int32_t *d_off;
+    int B;
+    std::vector<int32_t> h_off;  // F*B+1
+    int64_t nnz(int f) const { return (int64_t)h_off[(size_t)(f + 1) * B] - h_off[(size_t)f * B]; }
+    int64_t begin(int f) const { return h_off[(size_t)f * B]; }
+};
+
+template <typename T>
+struct DevBuf {
+    T *p = nullptr;
+    int64_t cap = 0;
+    cudaError_t ensure(int64_t n) {
+        if (n <= cap) return cudaSuccess;
+        cudaFree(p);
+        p = nullptr;
+        cap = 0;
+        cudaError_t e = cudaMalloc(&p, sizeof(T) * std::max<int64_t>(n, 1));
+        if (e == cudaSuccess) cap = n;
+        return e;
+    }
+    ~DevBuf() { cudaFree(p); }
+};
+
+int64_t task_count(const FeatureDesc &d, int B, int64_t nnz) {
+    int64_t blocks;
+    if (B == 0) return 0;
+    if (d.part == 0) {
+        blocks = (B + d.per_block - 1) / d.per_block;
+    } else {
+        int64_t npb = d.per_block;
+        const int64_t room = d.slots - 2;
+        const int64_t need = (nnz + room - 1) / room;
+        if (need > npb) npb = need;
+        blocks = nnz / npb + 1;
+    }
+    if (d.cap > 0 && blocks > d.cap) blocks = d.cap;
+    return blocks;
+}
+
+struct Tuner {
+    recflex_plan_s *p;
+    cudaStream_t stream;
+    std::vector<Batch> batches;
+    std::vector<int> ks;
+    int reps = 7;
+    int pad_waves = 4;
+    int verbose = 0;
+    std::vector<std::vector<recflex_schedule_t>> cands;  // per feature
+    recflex_status_t err = RECFLEX_OK;
+    int64_t local_launches = 0, global_launches = 0;
+
+    // per-feature tuning inputs (rebuilt when f changes), one per batch
+    int cur_f = -1;
+    struct TP {
+        DevBuf<int32_t> idx, off;
+        std::vector<int32_t> h_off;
+        std::vector<int> pad_slots;   // KJT slot -> original feature (padding)
+        int n_cand = 0;
+        int in_F = 0;
+    };
+    std::vector<TP> tps;
+
+    DevBuf<FeatureDesc> d_desc;
+    DevBuf<int32_t> d_bs, d_npb, d_counter, d_ts, d_part1;
+    DevBuf<long long> d_timers;
+    DevBuf<float> d_out;
+    DevBuf<float> d_flush;
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+
+    void fail(recflex_status_t s) {
+        if (err == RECFLEX_OK) err = s;
+    }
+    void check(cudaError_t e) {
+        if (e != cudaSuccess) fail(cuda_status(e));
+    }
+
+    void build_inputs(int f) {
+        cur_f = f;
+        tps.clear();
+        tps.resize(batches.size());
+        const int n = (int)cands[f].size();
+        const int64_t rows = p->desc[f].rows;
+        const int kmax = *std::max_element(ks.begin(), ks.end());
+        const int64_t pad_target = (int64_t)pad_waves * p->num_sms * kmax;
+        for (size_t i = 0; i < batches.size(); ++i) {
+            const Batch &bt = batches[i];
+            TP &tp = tps[i];
+            const int B = bt.B;
+            tp.n_cand = n;
+            // padding slots: other features, cyclically from f+1, until pad_target tasks
+            int64_t ptasks = 0;
+            for (int step = 1; ptasks < pad_target && step <= 4 * p->F + 4; ++step) {
+                const int g = (p->F == 1) ? f : (f + step) % p->F;
+                if (g == f && p->F > 1) continue;
+                const int64_t t = task_count(p->desc[g], B, bt.nnz(g));
+                if (t <= 0) continue;
+                tp.pad_slots.push_back(g);
+                ptasks += t;
+            }
+            tp.in_F = n + (int)tp.pad_slots.size();
+            // offsets of the tuning KJT
+            tp.h_off.assign((size_t)tp.in_F * B + 1, 0);
+            int64_t pos = 0;
+            auto put_feature = [&](int slot, int g) {
+                const int32_t base = bt.h_off[(size_t)g * B];
+                for (int s = 0; s < B; ++s) tp.h_off[(size_t)slot * B + s] = (int32_t)(pos + bt.h_off[(size_t)g * B + s] - base);
+                pos += bt.nnz(g);
+            };
+            for (int c = 0; c < n; ++c) put_feature(c, f);
+            for (size_t j = 0; j < tp.pad_slots.size(); ++j) put_feature(n + (int)j, tp.pad_slots[j]);
+            tp.h_off[(size_t)tp.in_F * B] = (int32_t)pos;
+            if (pos >= (int64_t(1) << 31)) {
+                fail(RECFLEX_ERR_NOT_SUPPORTED);
+                return;
+            }
+            check(tp.idx.ensure(pos));
+            check(tp.off.ensure((int64_t)tp.in_F * B + 1));
+            if (err) return;
+            check(cudaMemcpyAsync(tp.off.p, tp.h_off.data(), sizeof(int32_t) * tp.h_off.size(), cudaMemcpyHostToDevice,
+                                  stream));
+            const int64_t nnz_f = bt.nnz(f);
+            for (int c = 0; c < n; ++c) {
+                const int64_t shift = (int64_t)c * (rows / std::max(1, n));
+                int rc = remap_launch(bt.d_idx + bt.begin(f), tp.idx.p + (int64_t)c * nnz_f, nnz_f, shift, rows, stream);
+                if (rc) fail(cuda_status((cudaError_t)rc));
+            }
+            int64_t at = (int64_t)n * nnz_f;
+            for (int g : tp.pad_slots) {
+                const int64_t m = bt.nnz(g);
+                if (m > 0)
+                    check(cudaMemcpyAsync(tp.idx.p + at, bt.d_idx + bt.begin(g), sizeof(int32_t) * m,
+                                          cudaMemcpyDeviceToDevice, stream));
+                at += m;
+            }
+            check(cudaStreamSynchronize(stream));
+        }
+    }
+
+    // Eq. 3 costs of all candidates of f at occupancy ks[ki], summed over batches.
+    void local_cost(int ki, int f, double *costs) {
+        if (err) return;
+        if (cur_f != f) build_inputs(f);
+        if (err) return;
+        const int k = ks[ki];
+        const int n = (int)cands[f].size();
+        std::vector<double> sum(n, 0.0);
+        const FeatureDesc &base = p->desc[f];
+        for (size_t i = 0; i < batches.size(); ++i) {
+            const Batch &bt = batches[i];
+            TP &tp = tps[i];
+            const int B = bt.B;
+            // descriptor list: [pre padding][candidates][post padding]
+            std::vector<FeatureDesc> ds;
+            const int64_t pre_target = (int64_t)p->num_sms * k;
+            const int64_t post_target = (int64_t)(pad_waves - 1) * p->num_sms * k;
+            int dim_max = 4;
+            for (int g : tp.pad_slots) dim_max = std::max(dim_max, p->desc[g].dim);
+            const int dump_col = ((n * base.dim + 3) / 4) * 4;
+            const int d_tp = ((dump_col + dim_max + 3) / 4) * 4;
+            size_t ps = 0;
+            auto add_pad = [&](int64_t target) {
+                int64_t got = 0;
+                while (got < target && ps < tp.pad_slots.size()) {
+                    const int g = tp.pad_slots[ps];
+                    FeatureDesc d = p->desc[g];
+                    d.in_feature = n + (int)ps;
+                    d.col = dump_col;
+                    const int64_t nnz = bt.nnz(g);
+                    if (d.part == 1) d.slots = (int32_t)(nnz / d.per_block + 3);
+                    int64_t t = task_count(d, B, nnz);
+                    if (got + t > target) {
+                        d.cap = (int32_t)(target - got);
+                        t = d.cap;
+                    }
+                    got += t;
+                    ds.push_back(d);
+                    ++ps;
+                }
+            };
+            add_pad(pre_target);
+            const int cand_first = (int)ds.size();
+            for (int c = 0; c < n; ++c) {
+                FeatureDesc d = base;
+                d.sched = cands[f][c].sched_id;
+                d.part = cands[f][c].part;
+                d.per_block = cands[f][c].per_block;
+                d.cap = 0;
+                d.in_feature = c;
+                d.col = c * base.dim;
+                d.rows = base.rows;
+                if (d.part == 1) d.slots = (int32_t)(bt.nnz(f) / d.per_block + 3);
+                ds.push_back(d);
+            }
+            add_pad(post_target);
+            // slots for part-1 descriptors
+            int64_t slot = 0;
+            std::vector<int32_t> part1;
+            int64_t total = 0;
+            std::vector<int64_t> first(ds.size() + 1, 0);
+            for (size_t v = 0; v < ds.size(); ++v) {
+                FeatureDesc &d = ds[v];
+                d.table = p->tables[d.in_feature < n ? f : tp.pad_slots[d.in_feature - n]];
+                if (d.part == 1) {
+                    d.slot_base = (int32_t)slot;
+                    slot += d.slots;
+                    part1.push_back((int32_t)v);
+                }
+                first[v] = total;
+                const int g = d.in_feature < n ? f : tp.pad_slots[d.in_feature - n];
+                total += task_count(d, B, bt.nnz(g));
+            }
+            first[ds.size()] = total;
+            const int V = (int)ds.size();
+            check(d_desc.ensure(V));
+            check(d_bs.ensure(V + 1));
+            check(d_npb.ensure(V));
+            check(d_counter.ensure(4));
+            check(d_ts.ensure(std::max<int64_t>(slot, 1)));
+            check(d_part1.ensure(std::max<int64_t>((int64_t)part1.size(), 1)));
+            check(d_timers.ensure(std::max<int64_t>(total, 1)));
+            check(d_out.ensure((int64_t)B * d_tp));
+            if (err) return;
+            check(cudaMemcpyAsync(d_desc.p, ds.data(), sizeof(FeatureDesc) * V, cudaMemcpyHostToDevice, stream));
+            if (!part1.empty())
+                check(cudaMemcpyAsync(d_part1.p, part1.data(), sizeof(int32_t) * part1.size(), cudaMemcpyHostToDevice,
+                                      stream));
+            check(cudaMemsetAsync(d_timers.p, 0, sizeof(long long) * std::max<int64_t>(total, 1), stream));
+            Exec ex;
+            ex.F = V;
+            ex.in_F = tp.in_F;
+            ex.d_desc = d_desc.p;
+            ex.d_block_start = d_bs.p;
+            ex.d_npb_eff = d_npb.p;
+            ex.d_counter = d_counter.p;
+            ex.d_task_start = d_ts.p;
+            ex.d_part1 = d_part1.p;
+            ex.num_part1 = (int)part1.size();
+            ex.d_timers = d_timers.p;
+            ex.timers_cap = (int)total;
+            recflex_status_t st = run_pipeline(p, ex, tp.idx.p, tp.off.p, B, d_out.p, d_tp, k, stream, nullptr);
+            if (st != RECFLEX_OK) {
+                fail(st);
+                return;
+            }
+            ++local_launches;
+            std::vector<long long> tm(total);
+            std::vector<int32_t> bs(V + 1);
+            check(cudaMemcpyAsync(tm.data(), d_timers.p, sizeof(long long) * total, cudaMemcpyDeviceToHost, stream));
+            check(cudaMemcpyAsync(bs.data(), d_bs.p, sizeof(int32_t) * (V + 1), cudaMemcpyDeviceToHost, stream));
+            check(cudaStreamSynchronize(stream));
+            if (err) return;
+            for (int c = 0; c < n; ++c) {
+                const int v = cand_first + c;
+                double s = 0;
+                for (int64_t t = bs[v]; t < bs[v + 1]; ++t) s += (double)tm[t];
+                sum[c] += s;
+            }
+        }
+        for (int c = 0; c < n; ++c) costs[c] = sum[c];
+    }
+
+    void apply(const int32_t *choice) {
+        for (int f = 0; f < p->F; ++f) {
+            const recflex_schedule_t &s = cands[f][choice[f]];
+            p->desc[f].sched = s.sched_id;
+            p->desc[f].part = s.part;
+            p->desc[f].per_block = s.per_block;
+        }
+        p->desc_dirty = true;
+    }
+
+    // Eq. 4 latency of the fused forward with `choice` at occupancy ks[ki] (ms, Eq. 5 sum).
+    double global_cost(int ki, const int32_t *choice) {
+        if (err) return std::numeric_limits<double>::infinity();
+        apply(choice);
+        const int k = ks[ki];
+        p->k = k;
+        recflex_status_t st = upload_desc(p, stream);
+        if (st != RECFLEX_OK) {
+            fail(st);
+            return 1e30;
+        }
+        double total = 0;
+        for (const Batch &bt : batches) {
+            check(d_out.ensure((int64_t)bt.B * p->d_tot));
+            if (err) return 1e30;
+            std::vector<float> ms;
+            for (int r = 0; r < reps + 1; ++r) {
+                int rc = flush_launch(d_flush.p, sizeof(float) * d_flush.cap, stream);
+                if (rc) fail(cuda_status((cudaError_t)rc));
+                check(cudaEventRecord(e0, stream));
+                st = run_pipeline(p, p->ex, bt.d_idx, bt.d_off, bt.B, d_out.p, (int)p->d_tot, k, stream, nullptr);
+                if (st != RECFLEX_OK) {
+                    fail(st);
+                    return 1e30;
+                }
+                check(cudaEventRecord(e1, stream));
+                check(cudaEventSynchronize(e1));
+                float t = 0;
+                cudaEventElapsedTime(&t, e0, e1);
+                ++global_launches;
+                if (r > 0) ms.push_back(t);  // first run = warm-up
+            }
+            std::sort(ms.begin(), ms.end());
+            total += ms[ms.size() / 2];
+        }
+        if (verbose) std::fprintf(stderr, "[recflex tune] global k=%d: %.4f ms\n", k, total);
+        return total;
+    }
+};
+
+void cb_local(void *u, int32_t ki, int32_t f, double *costs) { static_cast<Tuner *>(u)->local_cost(ki, f, costs); }
+double cb_global(void *u, int32_t ki, const int32_t *choice) { return static_cast<Tuner *>(u)->global_cost(ki, choice); }
+
+std::vector<recflex_schedule_t> candidates_for(const recflex_plan_s *p, int f, int max_c) {
+    std::vector<recflex_schedule_t> out;
+    const recflex_feature_spec_t &sp = p->specs[f];
+    const FeatureDesc &d = p->desc[f];
+    // the plan's current schedule is always candidate 0 (tie -> keep it)
+    out.push_back({d.sched, d.part, d.per_block});
+    const bool multi_hot = sp.max_len > 1.5f;
+    for (int id = 0; id < kCatalogSize; ++id) {
+        const CatalogEntry &e = kCatalog[id];
+        recflex_schedule_t s = {id, 0, 1};
+        s.per_block = samples_per_task_default(id, sp.mean_len, sp.coverage);
+        if (!schedule_valid_for(s, d.dim, d.col, (int)p->d_tot)) continue;
+        const int span = e.G * e.VEC * e.C;
+        const int passes = (d.dim + span - 1) / span;
+        if (passes > 2) continue;
+        if (e.VEC == 1 && d.dim % 4 == 0) continue;  // scalar only where vectors cannot run
+        if (!multi_hot && e.family == RECFLEX_FAMILY_BLOCK) continue;
+        if (!multi_hot && e.U > 2) continue;  // one-hot bags: unroll is irrelevant
+        auto same = [&](const recflex_schedule_t &o) {
+            return o.sched_id == s.sched_id && o.part == s.part && o.per_block == s.per_block;
+        };
+        if (std::none_of(out.begin(), out.end(), same)) out.push_back(s);
+        if (multi_hot && e.family == RECFLEX_FAMILY_GROUP) {
+            recflex_schedule_t s1 = {id, 1, 4096};
+            if (std::none_of(out.begin(), out.end(), same) || true) {
+                bool dup = false;
+                for (auto &o : out)
+                    if (o.sched_id == s1.sched_id && o.part == 1 && o.per_block == s1.per_block) dup = true;
+                if (!dup) out.push_back(s1);
+            }
+        }
+    }
+    if (max_c > 0 && (int)out.size() > max_c) out.resize(max_c);
+    return out;
+}
+
+}  // namespace
+
+extern "C" recflex_status_t recflex_tune_ex(recflex_plan_t p, int32_t N, const int32_t *const *indices,
+                                            const int32_t *const *offsets, const int32_t *batch_sizes,
+                                            const float *const *tables, void *stream_,
+                                            const recflex_tune_options_t *opt, recflex_tune_stats_t *stats) {
+    if (!p || N <= 0 || !indices || !offsets || !batch_sizes || !tables) return RECFLEX_ERR_INVALID_ARG;
+    auto t_start = std::chrono::steady_clock::now();
+    cudaStream_t stream = (cudaStream_t)stream_;
+    cudaSetDevice(p->device);
+    Tuner T;
+    T.p = p;
+    T.stream = stream;
+    if (opt && opt->num_occupancies > 0) {
+        for (int i = 0; i < opt->num_occupancies && i < kMaxOcc; ++i) {
+            if (opt->occupancies[i] < 1 || opt->occupancies[i] > kMaxOcc) return RECFLEX_ERR_INVALID_ARG;
+            T.ks.push_back(opt->occupancies[i]);
+        }
+        std::sort(T.ks.begin(), T.ks.end());
+        T.ks.erase(std::unique(T.ks.begin(), T.ks.end()), T.ks.end());
+    } else {
+        for (int k = 1; k <= kMaxOcc; ++k) T.ks.push_back(k);
+    }
+    if (opt && opt->reps > 0) T.reps = opt->reps;
+    if (opt && opt->pad_waves > 0) T.pad_waves = opt->pad_waves;
+    if (opt) T.verbose = opt->verbose;
+    const int max_c = opt ? opt->max_candidates : 0;
+    for (int i = 0; i < N; ++i) {
+        if (batch_sizes[i] <= 0 || batch_sizes[i] > p->max_batch || !indices[i] || !offsets[i])
+            return RECFLEX_ERR_INVALID_ARG;
+    }
+    // tables -> descriptors
+    for (int f = 0; f < p->F; ++f) {
+        if (!tables[f] || ((uintptr_t)tables[f]) % 32) return RECFLEX_ERR_INVALID_ARG;
+        p->tables[f] = tables[f];
+    }
+    p->desc_dirty = true;
+    for (int k : T.ks) {
+        recflex_status_t st = prepare_occupancy(p, k);
+        if (st != RECFLEX_OK) return st;
+    }
+    T.batches.resize(N);
+    for (int i = 0; i < N; ++i) {
+        Batch &b = T.batches[i];
+        b.d_idx = indices[i];
+        b.d_off = offsets[i];
+        b.B = batch_sizes[i];
+        b.h_off.resize((size_t)p->F * b.B + 1);
+        cudaError_t e = cudaMemcpy(b.h_off.data(), offsets[i], sizeof(int32_t) * b.h_off.size(), cudaMemcpyDeviceToHost);
+        if (e != cudaSuccess) return cuda_status(e);
+    }
+    T.cands.resize(p->F);
+    std::vector<int32_t> ncand(p->F);
+    for (int f = 0; f < p->F; ++f) {
+        T.cands[f] = candidates_for(p, f, max_c);
+        ncand[f] = (int32_t)T.cands[f].size();
+    }
+    if (T.d_flush.ensure(64 << 20) != cudaSuccess) return RECFLEX_ERR_OOM;  // 256 MB = 2x L2
+    cudaEventCreate(&T.e0);
+    cudaEventCreate(&T.e1);
+    std::vector<int32_t> choice(p->F);
+    int32_t best_k = 0;
+    int64_t lc = 0, gc = 0;
+    recflex_status_t st = recflex_two_stage_select(p->F, (int32_t)T.ks.size(), ncand.data(), cb_local, cb_global, &T,
+                                                   choice.data(), &best_k, &lc, &gc);
+    cudaEventDestroy(T.e0);
+    cudaEventDestroy(T.e1);
+    if (st == RECFLEX_OK) st = T.err;
+    if (st != RECFLEX_OK) return st;
+    T.apply(choice.data());
+    p->k = T.ks[best_k];
+    st = upload_desc(p, stream);
+    if (st != RECFLEX_OK) return st;
+    double best_ms = 0;
+    {
+        // re-measure the selected configuration for the stats
+        best_ms = T.global_cost(best_k, choice.data());
+    }
+    recflex_tune_stats_t s = {};
+    s.local_launches = T.local_launches;
+    s.global_launches = T.global_launches;
+    s.local_evals = lc;
+    s.global_evals = gc;
+    s.best_occupancy = p->k;
+    s.best_ms = best_ms;
+    s.tune_seconds = std::chrono::duration<double>(std::chrono::steady_clock::now() - t_start).count();
+    p->last_stats = s;
+    if (stats) *stats = s;
+    if (T.verbose) {
+        std::fprintf(stderr, "[recflex tune] best k=%d, %.4f ms, %lld local + %lld global launches, %.1f s\n", p->k,
+                     best_ms, (long long)s.local_launches, (long long)s.global_launches, s.tune_seconds);
+    }
+    return T.err;
+}
+
+extern "C" recflex_status_t recflex_tune(recflex_plan_t p, int32_t N, const int32_t *const *indices,
+                                         const int32_t *const *offsets, const int32_t *batch_sizes,
+                                         const float *const *tables, void *stream) {
+    return recflex_tune_ex(p, N, indices, offsets, batch_sizes, tables, stream, nullptr, nullptr);
+}

@@ -1,0 +1,243 @@
+"""Python face of the C ABI: a Plan object over torch tensors.
+
+torch supplies device memory and streams only; every call below marshals
+pointers into librecflex.so (include/recflex.h) and the work runs in its CUDA
+kernels.  Names follow the C entry points (recflex_forward -> Plan.forward, ...).
+"""
+from __future__ import annotations
+
+import ctypes
+import json
+from typing import List, Optional, Sequence
+
+import torch
+
+from . import _lib
+from ._lib import check, lib
+
+POOL_SUM = 0
+POOL_MEAN = 1
+
+
+def catalog():
+    """List of dicts describing every catalog entry (schedule templates)."""
+    out = []
+    for i in range(lib.recflex_catalog_size()):
+        ci = _lib.CatalogInfo()
+        check(lib.recflex_catalog_info(i, ctypes.byref(ci)), 'recflex_catalog_info')
+        out.append(dict(id=i, family=('group', 'block')[ci.family], G=ci.group, VEC=ci.vec, C=ci.cols,
+                        U=ci.unroll))
+    return out
+
+
+def occupancy_check(k: int, device: int = 0):
+    a, r, s = ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int32()
+    check(lib.recflex_occupancy_check(device, k, ctypes.byref(a), ctypes.byref(r), ctypes.byref(s)),
+          'recflex_occupancy_check')
+    return dict(active_blocks=a.value, registers=r.value, local_bytes=s.value)
+
+
+def _stream_ptr(stream):
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return ctypes.c_void_p(stream.cuda_stream)
+
+
+def _dptr(t: torch.Tensor, dtype, name):
+    if not t.is_cuda:
+        raise ValueError(f'{name} must be a CUDA tensor')
+    if t.dtype != dtype:
+        raise TypeError(f'{name} must be {dtype}, got {t.dtype}')
+    if not t.is_contiguous():
+        raise ValueError(f'{name} must be contiguous')
+    return ctypes.c_void_p(t.data_ptr())
+
+
+class Plan:
+    """recflex_plan_create / recflex_destroy around a list of feature specs.
+
+    specs: sequence of dicts with keys rows, dim, pool, mean_len, max_len, coverage.
+    """
+
+    def __init__(self, specs: Sequence[dict], max_batch: int, device: int = 0):
+        F = len(specs)
+        arr = (_lib.FeatureSpec * F)()
+        for i, s in enumerate(specs):
+            arr[i].num_rows = int(s['rows'])
+            arr[i].dim = int(s['dim'])
+            arr[i].pool = int(s.get('pool', POOL_SUM))
+            arr[i].mean_len = float(s.get('mean_len', 1.0))
+            arr[i].max_len = float(s.get('max_len', 1.0))
+            arr[i].coverage = float(s.get('coverage', 1.0))
+        self._h = ctypes.c_void_p()
+        check(lib.recflex_plan_create(arr, F, int(max_batch), int(device), ctypes.byref(self._h)),
+              'recflex_plan_create')
+        self.F = F
+        self.dims = [int(s['dim']) for s in specs]
+        self.d_tot = sum(self.dims)
+        self.max_batch = int(max_batch)
+        self.device = int(device)
+        self._tables_key = None
+        self._tables_arr = None
+
+    @classmethod
+    def from_model(cls, model, max_batch: Optional[int] = None, device: int = 0) -> 'Plan':
+        specs = [dict(rows=f.rows, dim=f.dim, pool=f.pool, mean_len=f.mean_len(), max_len=f.max_len(),
+                      coverage=f.coverage) for f in model.features]
+        return cls(specs, max_batch or model.batch, device)
+
+    # -------------------------------------------------------------- lifecycle
+    def close(self):
+        if getattr(self, '_h', None) and self._h.value:
+            lib.recflex_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # -------------------------------------------------------------- helpers
+    def _tables(self, tables: Sequence[torch.Tensor]):
+        if len(tables) != self.F:
+            raise ValueError(f'expected {self.F} tables, got {len(tables)}')
+        key = tuple(t.data_ptr() for t in tables)
+        if key != self._tables_key:
+            for f, t in enumerate(tables):
+                if not (t.is_cuda and t.dtype == torch.float32 and t.is_contiguous() and t.dim() == 2
+                        and t.shape[1] == self.dims[f]):
+                    raise ValueError(f'table {f}: need contiguous CUDA float32 [rows, {self.dims[f]}]')
+            self._tables_arr = (ctypes.c_void_p * self.F)(*key)
+            self._tables_key = key
+        return self._tables_arr
+
+    # -------------------------------------------------------------- hot path
+    def forward(self, indices: torch.Tensor, offsets: torch.Tensor, B: int, tables: Sequence[torch.Tensor],
+                out: Optional[torch.Tensor] = None, stream=None) -> torch.Tensor:
+        """recflex_forward: pooled [B, D_tot] float32 (async on `stream`)."""
+        if out is None:
+            out = torch.empty((B, self.d_tot), dtype=torch.float32, device=offsets.device)
+        if out.shape != (B, self.d_tot) or out.dtype != torch.float32 or not out.is_contiguous():
+            raise ValueError('out must be contiguous float32 [B, D_tot]')
+        if offsets.numel() != self.F * B + 1:
+            raise ValueError('offsets must have F*B+1 entries')
+        tarr = self._tables(tables)
+        idx_ptr = _dptr(indices, torch.int32, 'indices') if indices.numel() else ctypes.c_void_p(offsets.data_ptr())
+        check(lib.recflex_forward(self._h, idx_ptr, _dptr(offsets, torch.int32, 'offsets'), int(B),
+                                  tarr, _dptr(out, torch.float32, 'out'), _stream_ptr(stream)),
+              'recflex_forward')
+        return out
+
+    def forward_host(self, indices: torch.Tensor, offsets: torch.Tensor, B: int, tables: Sequence[torch.Tensor],
+                     out: torch.Tensor, stream=None) -> torch.Tensor:
+        """recflex_forward_host: host (pinned) int32 inputs -> host float32 out [B, D_tot]; blocking."""
+        for name, t, dt in (('indices', indices, torch.int32), ('offsets', offsets, torch.int32),
+                            ('out', out, torch.float32)):
+            if t.is_cuda or t.dtype != dt or not t.is_contiguous():
+                raise ValueError(f'{name} must be a contiguous host {dt} tensor')
+        tarr = self._tables(tables)
+        check(lib.recflex_forward_host(self._h, ctypes.c_void_p(indices.data_ptr()), int(indices.numel()),
+                                       ctypes.c_void_p(offsets.data_ptr()), int(B), tarr,
+                                       ctypes.c_void_p(out.data_ptr()), _stream_ptr(stream)),
+              'recflex_forward_host')
+        return out
+
+    # -------------------------------------------------------------- tuner
+    def tune(self, batches: Sequence[tuple], tables: Sequence[torch.Tensor], occupancies: Optional[List[int]] = None,
+             reps: int = 7, pad_waves: int = 4, max_candidates: int = 0, verbose: bool = False, stream=None) -> dict:
+        """recflex_tune_ex over historical batches [(indices, offsets, B), ...]."""
+        N = len(batches)
+        idx_arr = (ctypes.c_void_p * N)(*[b[0].data_ptr() for b in batches])
+        off_arr = (ctypes.c_void_p * N)(*[b[1].data_ptr() for b in batches])
+        bs_arr = (ctypes.c_int32 * N)(*[int(b[2]) for b in batches])
+        opt = _lib.TuneOptions()
+        if occupancies:
+            opt.num_occupancies = len(occupancies)
+            for i, k in enumerate(occupancies):
+                opt.occupancies[i] = int(k)
+        opt.reps = reps
+        opt.pad_waves = pad_waves
+        opt.max_candidates = max_candidates
+        opt.verbose = 1 if verbose else 0
+        st = _lib.TuneStats()
+        check(lib.recflex_tune_ex(self._h, N, idx_arr, off_arr, bs_arr, self._tables(tables), _stream_ptr(stream),
+                                  ctypes.byref(opt), ctypes.byref(st)), 'recflex_tune_ex')
+        return dict(local_launches=st.local_launches, global_launches=st.global_launches,
+                    local_evals=st.local_evals, global_evals=st.global_evals,
+                    best_occupancy=st.best_occupancy, best_ms=st.best_ms, tune_seconds=st.tune_seconds)
+
+    # -------------------------------------------------------------- schedules
+    def get_schedule(self, f: int) -> dict:
+        s = _lib.Schedule()
+        k = ctypes.c_int32()
+        check(lib.recflex_get_schedule(self._h, f, ctypes.byref(s), ctypes.byref(k)), 'recflex_get_schedule')
+        return dict(sched_id=s.sched_id, part=s.part, per_block=s.per_block)
+
+    def set_schedule(self, f: int, sched_id: int, part: int = 0, per_block: int = 256):
+        s = _lib.Schedule(int(sched_id), int(part), int(per_block))
+        check(lib.recflex_set_schedule(self._h, f, ctypes.byref(s)), 'recflex_set_schedule')
+
+    @property
+    def occupancy(self) -> int:
+        k = ctypes.c_int32()
+        check(lib.recflex_get_occupancy(self._h, ctypes.byref(k)), 'recflex_get_occupancy')
+        return k.value
+
+    @occupancy.setter
+    def occupancy(self, k: int):
+        check(lib.recflex_set_occupancy(self._h, int(k)), 'recflex_set_occupancy')
+
+    # -------------------------------------------------------------- introspection
+    def debug_task_map(self, offsets: torch.Tensor, B: int, ranges: bool = False, stream=None):
+        bs = (ctypes.c_int32 * (self.F + 1))()
+        if not ranges:
+            check(lib.recflex_debug_task_map(self._h, _dptr(offsets, torch.int32, 'offsets'), int(B), bs, None, 0,
+                                             _stream_ptr(stream)), 'recflex_debug_task_map')
+            return list(bs), None
+        check(lib.recflex_debug_task_map(self._h, _dptr(offsets, torch.int32, 'offsets'), int(B), bs, None, 0,
+                                         _stream_ptr(stream)), 'recflex_debug_task_map')
+        total = bs[self.F]
+        rg = (ctypes.c_int32 * max(2, 2 * total))()
+        check(lib.recflex_debug_task_map(self._h, _dptr(offsets, torch.int32, 'offsets'), int(B), bs, rg,
+                                         max(2, 2 * total), _stream_ptr(stream)), 'recflex_debug_task_map')
+        return list(bs), [(rg[2 * t], rg[2 * t + 1]) for t in range(total)]
+
+    def validate(self, indices: torch.Tensor, offsets: torch.Tensor, B: int, stream=None) -> int:
+        """Returns the raw status (0 ok, 1 invalid offsets, 5 index out of range)."""
+        ip = ctypes.c_void_p(indices.data_ptr()) if indices.numel() else ctypes.c_void_p(offsets.data_ptr())
+        return int(lib.recflex_validate(self._h, ip, _dptr(offsets, torch.int32, 'offsets'), int(B),
+                                        _stream_ptr(stream)))
+
+    def export(self) -> dict:
+        n = ctypes.c_size_t()
+        check(lib.recflex_plan_export(self._h, None, 0, ctypes.byref(n)), 'recflex_plan_export')
+        buf = ctypes.create_string_buffer(n.value)
+        check(lib.recflex_plan_export(self._h, buf, n.value, ctypes.byref(n)), 'recflex_plan_export')
+        return json.loads(buf.value.decode())
+
+    def import_(self, state: dict):
+        check(lib.recflex_plan_import(self._h, json.dumps(state).encode()), 'recflex_plan_import')
+
+    def set_profiling(self, enable: bool):
+        check(lib.recflex_set_profiling(self._h, 1 if enable else 0), 'recflex_set_profiling')
+
+    def kernel_times(self, reset: bool = True) -> dict:
+        a, b, n = ctypes.c_double(), ctypes.c_double(), ctypes.c_int64()
+        check(lib.recflex_get_kernel_times(self._h, ctypes.byref(a), ctypes.byref(b), ctypes.byref(n),
+                                           1 if reset else 0), 'recflex_get_kernel_times')
+        return dict(map_ms=a.value, fused_ms=b.value, forwards=n.value)
+
+
+def shard_concat(recv: torch.Tensor, dims_per_rank: Sequence[int], rows: int, out: torch.Tensor, stream=None):
+    """recflex_shard_concat: [W chunks of rows x d_i] -> [rows, sum d_i]."""
+    W = len(dims_per_rank)
+    dims = (ctypes.c_int32 * W)(*[int(d) for d in dims_per_rank])
+    check(lib.recflex_shard_concat(_dptr(recv, torch.float32, 'recv'), W, int(rows), dims,
+                                   _dptr(out, torch.float32, 'out'), _stream_ptr(stream)), 'recflex_shard_concat')
+    return out
+
+
+def l2_flush(buf: torch.Tensor, stream=None):
+    check(lib.recflex_l2_flush(ctypes.c_void_p(buf.data_ptr()), buf.numel() * buf.element_size(),
+                               _stream_ptr(stream)), 'recflex_l2_flush')

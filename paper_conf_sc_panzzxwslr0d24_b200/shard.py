@@ -1,0 +1,125 @@
+"""Table-wise sharding across GPUs (§VII: "place different
+embedding tables on multiple GPUs through heuristics ... and then use RecFlex to
+optimize the embedding operations on each GPU") with the pooled-output
+exchange TorchRec-style table-wise sharding needs.
+
+  * partition: greedy LPT over features by estimated bytes per batch
+    (reading C24): E[L]*cov*(4d+4)*B + 4*d*B, largest first, to the least
+    loaded rank (ties: lower feature id first, lower rank).
+  * each rank runs its own fused RecFlex plan over ALL B samples of its
+    features -> out_r [B][D_r] (row-major, so rank j's B/W-sample block is
+    contiguous: no pre-permutation before the all-to-all);
+  * alltoallv over NCCL: rank r sends block j (B/W x D_r) to rank j and
+    receives B/W x D_i from every rank i;
+  * relayout [W][B/W][D_i] -> [B/W][D_tot'] with the library's CUDA kernel
+    (recflex_shard_concat).  Columns are grouped by rank (rank 0's features
+    first, in their global order), i.e. a fixed permutation of the 1-GPU
+    layout given by `column_order()`.
+"""
+from __future__ import annotations
+
+from typing import List, Sequence
+
+import numpy as np
+
+
+def feature_cost(feat, B: int) -> float:
+    el = feat.mean_len() * feat.coverage
+    return el * (4 * feat.dim + 4) * B + 4.0 * feat.dim * B
+
+
+def lpt_partition(costs: Sequence[float], W: int) -> List[List[int]]:
+    """Greedy longest-processing-time partition; each part sorted by feature id."""
+    if W <= 0:
+        raise ValueError('W must be positive')
+    order = sorted(range(len(costs)), key=lambda f: (-float(costs[f]), f))
+    load = [0.0] * W
+    parts: List[List[int]] = [[] for _ in range(W)]
+    for f in order:
+        r = min(range(W), key=lambda i: (load[i], i))
+        parts[r].append(f)
+        load[r] += float(costs[f])
+    return [sorted(p) for p in parts]
+
+
+def partition_model(model, W: int) -> List[List[int]]:
+    return lpt_partition([feature_cost(f, model.batch) for f in model.features], W)
+
+
+def column_order(model, parts: List[List[int]]) -> np.ndarray:
+    """Global column index of every column of the exchanged [B/W][D_tot'] output."""
+    col = np.cumsum([0] + model.dims)
+    order = []
+    for part in parts:
+        for f in part:
+            order.extend(range(col[f], col[f + 1]))
+    return np.asarray(order, np.int64)
+
+
+def shard_batch(batch, features: Sequence[int]):
+    """KJT restricted to `features` (feature-major, rebased): indices, offsets."""
+    B = batch.B
+    offs = batch.offsets.astype(np.int64)
+    idx_parts, off_parts = [], []
+    pos = 0
+    for f in features:
+        a, b = offs[f * B], offs[(f + 1) * B]
+        idx_parts.append(batch.indices[a:b])
+        off_parts.append(offs[f * B:(f + 1) * B] - a + pos)
+        pos += b - a
+    off_parts.append(np.asarray([pos], np.int64))
+    idx = np.concatenate(idx_parts) if idx_parts else np.zeros(0, np.int32)
+    return idx.astype(np.int32), np.concatenate(off_parts).astype(np.int32)
+
+
+def split_sizes(B: int, W: int, dims_per_rank: Sequence[int], rank: int):
+    """alltoallv element counts for rank `rank`: (input_splits, output_splits)."""
+    if B % W:
+        raise ValueError('table-wise exchange needs B % W == 0 (reading C23)')
+    rows = B // W
+    inp = [rows * dims_per_rank[rank]] * W
+    out = [rows * d for d in dims_per_rank]
+    return inp, out
+
+
+def exchange(send, dims_per_rank: Sequence[int], B: int, group=None):
+    """Pooled-output alltoallv: send [B][D_r] -> recv [sum_i B/W*D_i] (chunks in rank order)."""
+    import torch
+    import torch.distributed as dist
+    W = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    inp, out = split_sizes(B, W, dims_per_rank, rank)
+    recv = torch.empty(sum(out), dtype=send.dtype, device=send.device)
+    dist.all_to_all_single(recv, send.reshape(-1), output_split_sizes=out, input_split_sizes=inp, group=group)
+    return recv
+
+
+class ShardedEmbedding:
+    """One rank's slice of a table-wise sharded model: plan + exchange + relayout."""
+
+    def __init__(self, model, rank: int, world: int, device: int = 0, parts=None):
+        from .plan import Plan
+        self.model = model
+        self.rank, self.world = rank, world
+        self.parts = parts if parts is not None else partition_model(model, world)
+        self.features = self.parts[rank]
+        self.dims_per_rank = [sum(model.dims[f] for f in p) for p in self.parts]
+        specs = [dict(rows=model.features[f].rows, dim=model.features[f].dim, pool=model.features[f].pool,
+                      mean_len=model.features[f].mean_len(), max_len=model.features[f].max_len(),
+                      coverage=model.features[f].coverage) for f in self.features]
+        self.plan = Plan(specs, model.batch, device)
+        self.d_local = self.dims_per_rank[rank]
+        self.d_tot = sum(self.dims_per_rank)
+
+    def forward(self, indices, offsets, B, tables, out_local=None, out=None, group=None, stream=None):
+        import torch
+        from .plan import shard_concat
+        out_local = self.plan.forward(indices, offsets, B, tables, out=out_local, stream=stream)
+        if self.world == 1:
+            return out_local
+        recv = exchange(out_local, self.dims_per_rank, B, group)
+        rows = B // self.world
+        if out is None:
+            out = torch.empty((rows, self.d_tot), dtype=torch.float32, device=out_local.device)
+        shard_concat(recv, self.dims_per_rank, rows, out, stream=stream)
+        return out

@@ -291,13 +291,22 @@ def table_rows(table_id: int, row_start: int, row_end: int, dim: int, mode: str 
                device='cpu', seed: int = MODEL_SEED):
     """Rows [row_start, row_end) of physical table ``table_id`` as a float32 torch tensor."""
     import torch
-    r = torch.arange(row_start, row_end, dtype=torch.int64, device=device)
+    return table_rows_at(table_id, torch.arange(row_start, row_end, dtype=torch.int64, device=device), dim, mode,
+                         device, seed)
+
+
+def table_rows_at(table_id: int, row_ids, dim: int, mode: str = 'float', device='cpu',
+                  seed: int = MODEL_SEED):
+    """Selected rows (any order, repeats allowed) of a physical table -- the same
+    values make_table produces at those rows."""
+    import torch
+    r = torch.as_tensor(row_ids, dtype=torch.int64, device=device).reshape(-1)
     h0 = _mix32(torch.tensor(((table_id * 0x27D4EB2F) + (seed * 0x165667B1)) & M32, dtype=torch.int64,
                              device=device))
-    h1 = _mix32((h0 ^ (r & M32)) & M32)                      # [rows]
+    h1 = _mix32((h0 ^ (r & M32)) & M32)
     c = torch.arange(dim, dtype=torch.int64, device=device)
-    ck = (c * 0x61C88647) & M32                               # [dim]
-    h2 = _mix32((h1[:, None] + ck[None, :]) & M32)            # [rows, dim]
+    ck = (c * 0x61C88647) & M32
+    h2 = _mix32((h1[:, None] + ck[None, :]) & M32)
     if mode == 'float':
         out = (h2 >> 8).to(torch.float64) * (2.0 ** -23) - 1.0
     elif mode == 'int':

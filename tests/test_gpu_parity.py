@@ -1,0 +1,357 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Bars:
+  * integer-valued tables (reading C11): every fp32 partial sum is exact, so the
+    pooled output must match the oracle BIT-FOR-BIT regardless of reduction
+    order -- this pins the gathered index sets;
+  * U[-1,1) tables: |gpu - oracle| <= 1e-5 * (1 + |oracle|) * sqrt(L) per element
+    (north-star tolerance), empty bags exactly 0;
+  * thread map: bit-exact against the oracle's Fig. 8 task map.
+"""
+import math
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from paper_conf_sc_panzzxwslr0d24_b200 import synth
+
+pytestmark = pytest.mark.gpu
+
+
+def _plan_mod():
+    from paper_conf_sc_panzzxwslr0d24_b200 import plan
+    return plan
+
+
+class Case:
+    """A model + batch + tables resident on cuda:0, oracle on demand."""
+
+    def __init__(self, model, batch, mode='float'):
+        self.model, self.batch, self.mode = model, batch, mode
+        dev = torch.device('cuda', 0)
+        self.phys = [synth.make_table(t, rows, dim, mode, device=dev, seed=model.seed)
+                     for t, (rows, dim) in enumerate(model.tables)]
+        self.tables = [self.phys[f.table] for f in model.features]
+        self.idx = torch.from_numpy(batch.indices).to(dev)
+        self.off = torch.from_numpy(batch.offsets).to(dev)
+        self.B = batch.B
+
+    def getter(self, f, rows):
+        feat = self.model.features[f]
+        return synth.table_rows_at(feat.table, rows, feat.dim, self.mode, seed=self.model.seed).numpy()
+
+    def oracle(self, samples=None):
+        if samples is None:
+            samples = np.arange(self.B)
+        return oracle.sampled_forward(self.model, self.batch, samples, self.getter)
+
+
+def check_tol(gpu, ref, lens, dims):
+    """Per-element north-star tolerance; lens [S][F] bag lengths."""
+    L = np.repeat(lens, dims, axis=1).astype(np.float64)
+    tol = 1e-5 * (1.0 + np.abs(ref)) * np.sqrt(np.maximum(L, 1.0))
+    err = np.abs(gpu.astype(np.float64) - ref)
+    assert np.all(gpu[L == 0] == 0.0), 'empty bags must be exactly 0'
+    bad = err > tol
+    assert not bad.any(), f'{bad.sum()} elements out of tolerance; max err/tol {np.max(err / tol):.3g}'
+    return float(np.max(err / tol)) if err.size else 0.0
+
+
+def run_plan(case, plan=None, stream=None):
+    P = _plan_mod()
+    if plan is None:
+        plan = P.Plan.from_model(case.model, max_batch=case.B)
+    out = plan.forward(case.idx, case.off, case.B, case.tables, stream=stream)
+    torch.cuda.synchronize()
+    return plan, out.cpu().numpy()
+
+
+# ---------------------------------------------------------------------------- configs
+
+@pytest.mark.parametrize('mode', ['int', 'float'])
+def test_tiny_full(mode):
+    m = synth.make_model('tiny')
+    case = Case(m, synth.make_batch(m, 7), mode)
+    _, out = run_plan(case)
+    ref, lens = case.oracle()
+    if mode == 'int':
+        assert np.array_equal(out.astype(np.float64), ref)
+    else:
+        check_tol(out, ref, lens, m.dims)
+
+
+@pytest.mark.parametrize('name', ['medium', 'fig3'])
+def test_medium_full_int_and_float(name):
+    m = synth.make_model(name)
+    b = synth.make_batch(m, 7)
+    for mode in ('int', 'float'):
+        case = Case(m, b, mode)
+        _, out = run_plan(case)
+        ref, lens = case.oracle()
+        if mode == 'int':
+            assert np.array_equal(out.astype(np.float64), ref)
+        else:
+            check_tol(out, ref, lens, m.dims)
+
+
+def test_industrial_sampled():
+    m = synth.make_model('industrial')
+    b = synth.make_batch(m, 7)
+    case = Case(m, b, 'float')
+    _, out = run_plan(case)
+    rng = np.random.default_rng(0)
+    samples = np.unique(np.concatenate([[0, b.B - 1], rng.integers(0, b.B, 200)]))
+    ref, lens = case.oracle(samples)
+    check_tol(out[samples], ref, lens, m.dims)
+
+
+@pytest.mark.parametrize('name', ['heavy', 'sharded1000'])
+def test_full_size_sampled(name):
+    """BASELINE.json full sizes, default (untuned) launch configuration; sampled rows."""
+    m = synth.make_model(name)
+    b = synth.make_batch(m, 7)
+    case = Case(m, b, 'int')
+    _, out = run_plan(case)
+    rng = np.random.default_rng(1)
+    samples = np.unique(np.concatenate([[0, b.B - 1], rng.integers(0, b.B, 48)]))
+    ref, lens = case.oracle(samples)
+    assert np.array_equal(out[samples].astype(np.float64), ref)
+    del case
+    torch.cuda.empty_cache()
+
+
+# ---------------------------------------------------------------------------- every catalog entry
+
+def _mixed_model():
+    feats = []
+    dims = [4, 8, 12, 16, 24, 32, 64, 96, 128, 256, 3, 1]
+    for i, d in enumerate(dims):
+        kind = 'onehot' if i % 3 == 0 else 'uniform'
+        feats.append(synth.Feature(rows=997 + 13 * i, dim=d, pool=i % 2, kind=kind,
+                                   coverage=0.7 if kind == 'onehot' else 1.0, lo=0, hi=37 + 5 * i,
+                                   lmax=1 if kind == 'onehot' else 37 + 5 * i, table=i))
+    return synth.custom_model('mixed', feats, 301)
+
+
+@pytest.mark.parametrize('part', [0, 1])
+def test_every_catalog_entry_int_bitexact(part):
+    P = _plan_mod()
+    m = _mixed_model()
+    b = synth.make_batch(m, 3)
+    case = Case(m, b, 'int')
+    ref, lens = case.oracle()
+    plan = P.Plan.from_model(m, max_batch=b.B)
+    cat = P.catalog()
+    col = np.cumsum([0] + m.dims)
+    tested = 0
+    for e in cat:
+        for per_block in ((7, 64) if part == 0 else (5, 300)):
+            used = []
+            for f, feat in enumerate(m.features):
+                try:
+                    plan.set_schedule(f, e['id'], part, per_block)
+                    used.append(f)
+                except Exception:
+                    pass  # entry not valid for this dim
+            if not used:
+                continue
+            _, out = run_plan(case, plan)
+            for f in used:
+                a, z = col[f], col[f + 1]
+                assert np.array_equal(out[:, a:z].astype(np.float64), ref[:, a:z]), (e, f, per_block)
+            tested += 1
+            # restore defaults for the next entry
+            plan = P.Plan.from_model(m, max_batch=b.B)
+    assert tested >= 40
+
+
+@pytest.mark.parametrize('k', range(1, 9))
+def test_each_occupancy_variant_parity(k):
+    P = _plan_mod()
+    m = _mixed_model()
+    b = synth.make_batch(m, 5)
+    case = Case(m, b, 'int')
+    plan = P.Plan.from_model(m, max_batch=b.B)
+    plan.occupancy = k
+    _, out = run_plan(case, plan)
+    ref, _ = case.oracle()
+    assert np.array_equal(out.astype(np.float64), ref)
+
+
+@pytest.mark.parametrize('k', range(1, 9))
+def test_occupancy_api_matches_k(k):
+    """P:129 occupancy control: padded smem + __launch_bounds__ give exactly k CTAs/SM."""
+    P = _plan_mod()
+    r = P.occupancy_check(k)
+    assert r['active_blocks'] == k, r
+
+
+# ---------------------------------------------------------------------------- thread map
+
+@pytest.mark.parametrize('seed', range(3))
+def test_task_map_bitexact_vs_oracle(seed):
+    P = _plan_mod()
+    rng = np.random.default_rng(seed)
+    m = _mixed_model()
+    b = synth.make_batch(m, 11 + seed)
+    plan = P.Plan.from_model(m, max_batch=b.B)
+    mode, pb = [], []
+    for f, feat in enumerate(m.features):
+        s = plan.get_schedule(f)
+        if rng.random() < 0.5:
+            s['part'] = 1
+            s['per_block'] = int(rng.integers(1, 200))
+        else:
+            s['part'] = 0
+            s['per_block'] = int(rng.integers(1, 300))
+        plan.set_schedule(f, s['sched_id'], s['part'], s['per_block'])
+        mode.append(s['part'])
+        pb.append(s['per_block'])
+    off = torch.from_numpy(b.offsets).cuda()
+    bs, ranges = plan.debug_task_map(off, b.B, ranges=True)
+    blocks, tf, tr = oracle.task_map(b.B, mode, pb, b.offsets)
+    exp_bs = oracle.block_start_from_task_map(m.F, tf)
+    assert bs == exp_bs.tolist()
+    for f in range(m.F):
+        if mode[f] != 1:
+            continue
+        s0, s1 = oracle.nnz_task_ranges(b.B, pb[f], b.offsets[f * b.B:(f + 1) * b.B + 1], int(blocks[f]))
+        got = ranges[bs[f]:bs[f + 1]]
+        assert [g[0] for g in got] == s0.tolist()
+        assert [g[1] for g in got] == s1.tolist()
+
+
+# ---------------------------------------------------------------------------- edge cases
+
+def test_all_empty_and_ragged_batches():
+    P = _plan_mod()
+    m = _mixed_model()
+    lens = np.zeros((m.F, 33), np.int64)
+    lens[1, 5] = 700   # one very long bag
+    lens[4, 32] = 1    # last sample only
+    b = synth.batch_from_lengths(lens, [f.rows for f in m.features], seed=3)
+    case = Case(m, b, 'int')
+    plan = P.Plan.from_model(m, max_batch=64)
+    _, out = run_plan(case, plan)
+    ref, _ = case.oracle()
+    assert np.array_equal(out.astype(np.float64), ref)
+    assert np.count_nonzero(out) > 0
+
+
+def test_batch_zero_is_noop_and_bad_args():
+    P = _plan_mod()
+    m = synth.make_model('tiny')
+    b = synth.make_batch(m, 7)
+    case = Case(m, b, 'int')
+    plan = P.Plan.from_model(m, max_batch=b.B)
+    off0 = torch.zeros(1, dtype=torch.int32, device='cuda')
+    out0 = torch.empty((0, m.d_tot), dtype=torch.float32, device='cuda')
+    plan.forward(case.idx, off0, 0, case.tables, out=out0)
+    with pytest.raises(Exception):
+        plan.forward(case.idx, case.off, b.B + 1, case.tables)       # B > max_batch
+    with pytest.raises(Exception):
+        P.Plan([dict(rows=0, dim=4)], 8)                               # bad spec
+    with pytest.raises(Exception):
+        P.Plan([dict(rows=10, dim=4)], 8, device=99)                   # bad device
+
+
+def test_validate_detects_bad_inputs():
+    P = _plan_mod()
+    m = synth.make_model('tiny')
+    b = synth.make_batch(m, 7)
+    case = Case(m, b, 'int')
+    plan = P.Plan.from_model(m, max_batch=b.B)
+    assert plan.validate(case.idx, case.off, b.B) == 0
+    bad = case.idx.clone()
+    bad[-1] = m.features[-1].rows
+    assert plan.validate(bad, case.off, b.B) == 5
+    neg = case.idx.clone()
+    neg[0] = -1
+    assert plan.validate(neg, case.off, b.B) == 5
+    boff = case.off.clone()
+    boff[3] = boff[4] + 1
+    assert plan.validate(case.idx, boff, b.B) == 1
+
+
+def test_determinism_ten_runs():
+    m = synth.make_model('medium')
+    case = Case(m, synth.make_batch(m, 7), 'float')
+    plan, first = run_plan(case)
+    for _ in range(9):
+        _, o = run_plan(case, plan)
+        assert np.array_equal(o, first)
+
+
+def test_forward_host_matches_device_path():
+    P = _plan_mod()
+    m = synth.make_model('medium')
+    b = synth.make_batch(m, 8)
+    case = Case(m, b, 'float')
+    plan, dev_out = run_plan(case)
+    hi = torch.from_numpy(b.indices).pin_memory()
+    ho = torch.from_numpy(b.offsets).pin_memory()
+    hout = torch.empty((b.B, m.d_tot), dtype=torch.float32).pin_memory()
+    plan.forward_host(hi, ho, b.B, case.tables, hout)
+    assert np.array_equal(hout.numpy(), dev_out)
+
+
+def test_cuda_graph_capture_replay():
+    m = synth.make_model('medium')
+    case = Case(m, synth.make_batch(m, 7), 'int')
+    plan, ref = run_plan(case)
+    out = torch.empty((case.B, m.d_tot), dtype=torch.float32, device='cuda')
+    s = torch.cuda.Stream()
+    s.wait_stream(torch.cuda.current_stream())
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        plan.forward(case.idx, case.off, case.B, case.tables, out=out, stream=s)
+    out.zero_()
+    g.replay()
+    torch.cuda.synchronize()
+    assert np.array_equal(out.cpu().numpy(), ref)
+
+
+def test_export_import_roundtrip():
+    P = _plan_mod()
+    m = _mixed_model()
+    plan = P.Plan.from_model(m, max_batch=64)
+    plan.set_schedule(2, plan.get_schedule(2)['sched_id'], 1, 123)
+    plan.occupancy = 6
+    st = plan.export()
+    p2 = P.Plan.from_model(m, max_batch=64)
+    p2.import_(st)
+    assert p2.export() == st
+
+
+def test_shard_concat():
+    P = _plan_mod()
+    rows, dims = 37, [4, 12, 8]
+    chunks = [torch.randn(rows, d, device='cuda') for d in dims]
+    recv = torch.cat([c.reshape(-1) for c in chunks])
+    out = torch.empty(rows, sum(dims), device='cuda')
+    P.shard_concat(recv, dims, rows, out)
+    torch.cuda.synchronize()
+    assert torch.equal(out, torch.cat(chunks, dim=1))
+
+
+# ---------------------------------------------------------------------------- tuner
+
+def test_tuner_runs_counts_and_keeps_parity():
+    P = _plan_mod()
+    m = synth.make_model('fig3')
+    bts = [synth.make_batch(m, 7 + i) for i in range(2)]
+    case = Case(m, bts[0], 'int')
+    plan = P.Plan.from_model(m)
+    hist = [(torch.from_numpy(b.indices).cuda(), torch.from_numpy(b.offsets).cuda(), b.B) for b in bts]
+    ks = [2, 4, 8]
+    st = plan.tune(hist, case.tables, occupancies=ks, reps=3)
+    F, K, N = m.F, len(ks), len(hist)
+    assert st['local_evals'] == F * K            # P:144 O(F*K + K)
+    assert st['global_evals'] == K
+    assert st['local_launches'] == F * K * N
+    assert st['best_occupancy'] in ks
+    _, out = run_plan(case, plan)
+    ref, _ = case.oracle()
+    assert np.array_equal(out.astype(np.float64), ref)
