@@ -109,6 +109,10 @@ void recflex_destroy(recflex_plan_t plan);
 
 const char *recflex_status_string(recflex_status_t status);
 
+/* Human-readable detail of the last CUDA failure seen by this thread
+ * ("<where>: <cudaError name> (<text>)"); empty if none.  Not cleared on success. */
+const char *recflex_last_error(void);
+
 /* ---- the hot path ----------------------------------------------------- */
 
 /* Fused multi-feature embedding-bag forward (async, stream-ordered, no host

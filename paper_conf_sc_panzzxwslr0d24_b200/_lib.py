@@ -57,6 +57,7 @@ SIGNATURES = {
     'recflex_plan_create': (c_int32, [P(FeatureSpec), c_int32, c_int32, c_int32, P(c_void_p)]),
     'recflex_destroy': (None, [c_void_p]),
     'recflex_status_string': (ctypes.c_char_p, [c_int32]),
+    'recflex_last_error': (ctypes.c_char_p, []),
     'recflex_forward': (c_int32, [c_void_p, c_void_p, c_void_p, c_int32, P(c_void_p), c_void_p, c_void_p]),
     'recflex_forward_host': (c_int32, [c_void_p, c_void_p, c_int64, c_void_p, c_int32, P(c_void_p), c_void_p,
                                        c_void_p]),
@@ -87,7 +88,12 @@ SIGNATURES = {
 class RecflexError(RuntimeError):
     def __init__(self, code, where=''):
         self.code = code
-        super().__init__(f'{where}: {STATUS.get(code, code)}')
+        detail = ''
+        try:
+            detail = lib.recflex_last_error().decode() if code == 2 else ''
+        except Exception:
+            pass
+        super().__init__(f'{where}: {STATUS.get(code, code)}' + (f' [{detail}]' if detail else ''))
 
 
 def _load():

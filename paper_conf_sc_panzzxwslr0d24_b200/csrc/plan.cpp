@@ -16,11 +16,21 @@ using namespace recflex;
 
 namespace recflex {
 
-recflex_status_t cuda_status(cudaError_t e) {
+static thread_local char g_last_error[512] = "";
+
+void set_last_error(const char *msg) {
+    std::snprintf(g_last_error, sizeof(g_last_error), "%s", msg);
+}
+
+recflex_status_t cuda_status_at(cudaError_t e, const char *where) {
     if (e == cudaSuccess) return RECFLEX_OK;
+    std::snprintf(g_last_error, sizeof(g_last_error), "%s: %s (%s)", where ? where : "cuda", cudaGetErrorName(e),
+                  cudaGetErrorString(e));
     if (e == cudaErrorMemoryAllocation) return RECFLEX_ERR_OOM;
     return RECFLEX_ERR_CUDA;
 }
+
+recflex_status_t cuda_status(cudaError_t e) { return cuda_status_at(e, "cuda"); }
 
 static int next_pow2(int v) {
     int p = 1;
@@ -36,20 +46,31 @@ int find_catalog(int family, int G, int VEC, int C, int U) {
     return -1;
 }
 
-// samples per task for sample-partitioned tasks: ~4096 expected lookups per
-// task (enough work to amortise the task fetch), between 1 and 32 rounds of
-// the CTA's bag slots.
-int samples_per_task_default(int sched_id, float mean_len, float coverage) {
+// samples per task for sample-partitioned tasks: about `target` expected
+// lookups per task (enough work to amortise the task fetch), between 1 and 32
+// rounds of the CTA's bag slots.
+int samples_per_task_default(int sched_id, float mean_len, float coverage, int target) {
     const CatalogEntry &e = kCatalog[sched_id];
     const int slots = (e.family == RECFLEX_FAMILY_GROUP) ? kBlockThreads / e.G : 1;
     double el = std::max(0.25, (double)mean_len * std::max(0.05, (double)coverage));
-    int R = (int)std::lround(4096.0 / (slots * el));
+    int R = (int)std::lround((double)target / (slots * el));
     R = std::min(32, std::max(1, R));
-    if (e.family == RECFLEX_FAMILY_BLOCK) R = std::min(64, std::max(1, (int)std::lround(2048.0 / el)));
+    if (e.family == RECFLEX_FAMILY_BLOCK) R = std::min(64, std::max(1, (int)std::lround(0.5 * target / el)));
     return slots * R;
 }
 
-recflex_schedule_t default_schedule(const recflex_feature_spec_t &spec) {
+// Plan-level lookups per task: ~4096, but small enough that the expected
+// batch yields >= 8 waves of #SM x 4 CTAs (Eq. 2 assumes a negligible tail,
+// P:116), and never below 256.
+int task_lookups_target(const recflex_feature_spec_t *specs, int F, int max_batch, int num_sms) {
+    double tot = 0;
+    for (int f = 0; f < F; ++f)
+        tot += (double)max_batch * std::max(0.25, (double)specs[f].mean_len * std::max(0.05, (double)specs[f].coverage));
+    double t = tot / (8.0 * num_sms * 4);
+    return (int)std::min(4096.0, std::max(256.0, t));
+}
+
+recflex_schedule_t default_schedule(const recflex_feature_spec_t &spec, int target) {
     recflex_schedule_t s = {0, 0, 1};
     const int d = spec.dim;
     int id = -1;
@@ -64,7 +85,7 @@ recflex_schedule_t default_schedule(const recflex_feature_spec_t &spec) {
     if (id < 0) id = find_catalog(RECFLEX_FAMILY_GROUP, std::min(32, next_pow2(d)), 1, 1, 4);
     s.sched_id = id;
     s.part = 0;
-    s.per_block = samples_per_task_default(id, spec.mean_len, spec.coverage);
+    s.per_block = samples_per_task_default(id, spec.mean_len, spec.coverage, target);
     return s;
 }
 
@@ -165,7 +186,7 @@ recflex_status_t run_pipeline(recflex_plan_s *p, const Exec &ex, const int32_t *
     ma.npb_eff = ex.d_npb_eff;
     ma.counter = ex.d_counter;
     int rc = map_launch(ma, stream);
-    if (rc) return cuda_status((cudaError_t)rc);
+    if (rc) return cuda_status_at((cudaError_t)rc, "map kernel launch");
     if (ex.num_part1 > 0) {
         FillArgs fa;
         fa.desc = ex.d_desc;
@@ -177,7 +198,7 @@ recflex_status_t run_pipeline(recflex_plan_s *p, const Exec &ex, const int32_t *
         fa.B = B;
         fa.task_start = ex.d_task_start;
         rc = fill_launch(fa, (B + 255) / 256, p->pdl, stream);
-        if (rc) return cuda_status((cudaError_t)rc);
+        if (rc) return cuda_status_at((cudaError_t)rc, "fill kernel launch");
     }
     if (ev) cudaEventRecord(ev->e1, stream);
     FusedArgs a;
@@ -200,7 +221,7 @@ recflex_status_t run_pipeline(recflex_plan_s *p, const Exec &ex, const int32_t *
     // stream dependency point anyway).
     cfg.pdl = p->pdl && ev == nullptr;
     rc = fused_launch(k, a, cfg, stream);
-    if (rc) return cuda_status((cudaError_t)rc);
+    if (rc) return cuda_status_at((cudaError_t)rc, "fused kernel launch");
     if (ev) cudaEventRecord(ev->e2, stream);
     return RECFLEX_OK;
 }
@@ -211,6 +232,8 @@ recflex_status_t run_pipeline(recflex_plan_s *p, const Exec &ex, const int32_t *
 // C ABI
 // ===========================================================================
 extern "C" {
+
+const char *recflex_last_error(void) { return g_last_error; }
 
 const char *recflex_status_string(recflex_status_t s) {
     switch (s) {
@@ -312,11 +335,12 @@ recflex_status_t recflex_plan_create(const recflex_feature_spec_t *specs, int32_
         return RECFLEX_ERR_INVALID_ARG;
     }
     p->slots_total = slot;
+    p->task_lookups = task_lookups_target(specs, F, max_batch, p->num_sms);
     for (int f = 0; f < F; ++f) {
-        recflex_schedule_t s = default_schedule(specs[f]);
+        recflex_schedule_t s = default_schedule(specs[f], p->task_lookups);
         if (!schedule_valid_for(s, p->desc[f].dim, p->desc[f].col, (int)d_tot)) {
             s.sched_id = find_catalog(RECFLEX_FAMILY_GROUP, std::min(32, next_pow2(specs[f].dim)), 1, 1, 4);
-            s.per_block = samples_per_task_default(s.sched_id, specs[f].mean_len, specs[f].coverage);
+            s.per_block = samples_per_task_default(s.sched_id, specs[f].mean_len, specs[f].coverage, p->task_lookups);
         }
         p->desc[f].sched = s.sched_id;
         p->desc[f].part = s.part;

@@ -41,6 +41,7 @@ struct recflex_plan_s {
     std::vector<int32_t> part1;              // features with part == 1
     std::vector<const float *> tables;       // cached table pointers
     int k = 4;
+    int task_lookups = 4096;  // lookups per task targeted by the default schedules
     bool desc_dirty = true;
     bool pdl = true;
     int64_t slots_total = 0;
@@ -73,6 +74,8 @@ struct recflex_plan_s {
 namespace recflex {
 
 recflex_status_t cuda_status(cudaError_t e);
+recflex_status_t cuda_status_at(cudaError_t e, const char *where);
+void set_last_error(const char *msg);
 recflex_status_t prepare_occupancy(recflex_plan_s *p, int k);
 int min_dyn_smem(int F);
 // Launch map (+fill) + fused for an Exec.  Events (optional) bracket map and fused.
@@ -80,9 +83,9 @@ recflex_status_t run_pipeline(recflex_plan_s *p, const Exec &ex, const int32_t *
                               float *out, int out_stride, int k, cudaStream_t stream, EventTriple *ev);
 recflex_status_t upload_desc(recflex_plan_s *p, cudaStream_t stream);
 bool schedule_valid_for(const recflex_schedule_t &s, int dim, int col, int d_tot);
-recflex_schedule_t default_schedule(const recflex_feature_spec_t &spec);
+recflex_schedule_t default_schedule(const recflex_feature_spec_t &spec, int target);
 int find_catalog(int family, int G, int VEC, int C, int U);
-int samples_per_task_default(int sched_id, float mean_len, float coverage);
+int samples_per_task_default(int sched_id, float mean_len, float coverage, int target);
 int slots_for(int max_batch, float max_len);
 
 }  // namespace recflex

@@ -156,8 +156,8 @@ struct Tuner {
     void fail(recflex_status_t s) {
         if (err == RECFLEX_OK) err = s;
     }
-    void check(cudaError_t e) {
-        if (e != cudaSuccess) fail(cuda_status(e));
+    void check(cudaError_t e, const char *where = "tuner") {
+        if (e != cudaSuccess) fail(cuda_status_at(e, where));
     }
 
     void build_inputs(int f) {
@@ -408,7 +408,7 @@ std::vector<recflex_schedule_t> candidates_for(const recflex_plan_s *p, int f, i
     for (int id = 0; id < kCatalogSize; ++id) {
         const CatalogEntry &e = kCatalog[id];
         recflex_schedule_t s = {id, 0, 1};
-        s.per_block = samples_per_task_default(id, sp.mean_len, sp.coverage);
+        s.per_block = samples_per_task_default(id, sp.mean_len, sp.coverage, p->task_lookups);
         if (!schedule_valid_for(s, d.dim, d.col, (int)p->d_tot)) continue;
         const int span = e.G * e.VEC * e.C;
         const int passes = (d.dim + span - 1) / span;
@@ -421,7 +421,7 @@ std::vector<recflex_schedule_t> candidates_for(const recflex_plan_s *p, int f, i
         };
         if (std::none_of(out.begin(), out.end(), same)) out.push_back(s);
         if (multi_hot && e.family == RECFLEX_FAMILY_GROUP) {
-            recflex_schedule_t s1 = {id, 1, 4096};
+            recflex_schedule_t s1 = {id, 1, std::max(128, p->task_lookups)};
             if (std::none_of(out.begin(), out.end(), same) || true) {
                 bool dup = false;
                 for (auto &o : out)
@@ -499,19 +499,21 @@ extern "C" recflex_status_t recflex_tune_ex(recflex_plan_t p, int32_t N, const i
     int64_t lc = 0, gc = 0;
     recflex_status_t st = recflex_two_stage_select(p->F, (int32_t)T.ks.size(), ncand.data(), cb_local, cb_global, &T,
                                                    choice.data(), &best_k, &lc, &gc);
-    cudaEventDestroy(T.e0);
-    cudaEventDestroy(T.e1);
+    struct EvGuard {
+        Tuner &t;
+        ~EvGuard() {
+            cudaEventDestroy(t.e0);
+            cudaEventDestroy(t.e1);
+        }
+    } guard{T};
     if (st == RECFLEX_OK) st = T.err;
     if (st != RECFLEX_OK) return st;
     T.apply(choice.data());
     p->k = T.ks[best_k];
     st = upload_desc(p, stream);
     if (st != RECFLEX_OK) return st;
-    double best_ms = 0;
-    {
-        // re-measure the selected configuration for the stats
-        best_ms = T.global_cost(best_k, choice.data());
-    }
+    // re-measure the selected configuration for the stats
+    const double best_ms = T.global_cost(best_k, choice.data());
     recflex_tune_stats_t s = {};
     s.local_launches = T.local_launches;
     s.global_launches = T.global_launches;

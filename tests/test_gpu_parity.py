@@ -59,6 +59,12 @@ def check_tol(gpu, ref, lens, dims):
     return float(np.max(err / tol)) if err.size else 0.0
 
 
+def bitexact(gpu, ref):
+    """Integer-valued tables: sums are exact, MEAN is one correctly rounded
+    division (reading C21) -> the fp32 output equals fp32(oracle) bit for bit."""
+    return np.array_equal(gpu, ref.astype(np.float32))
+
+
 def run_plan(case, plan=None, stream=None):
     P = _plan_mod()
     if plan is None:
@@ -77,7 +83,7 @@ def test_tiny_full(mode):
     _, out = run_plan(case)
     ref, lens = case.oracle()
     if mode == 'int':
-        assert np.array_equal(out.astype(np.float64), ref)
+        assert bitexact(out, ref)
     else:
         check_tol(out, ref, lens, m.dims)
 
@@ -91,7 +97,7 @@ def test_medium_full_int_and_float(name):
         _, out = run_plan(case)
         ref, lens = case.oracle()
         if mode == 'int':
-            assert np.array_equal(out.astype(np.float64), ref)
+            assert bitexact(out, ref)
         else:
             check_tol(out, ref, lens, m.dims)
 
@@ -117,7 +123,7 @@ def test_full_size_sampled(name):
     rng = np.random.default_rng(1)
     samples = np.unique(np.concatenate([[0, b.B - 1], rng.integers(0, b.B, 48)]))
     ref, lens = case.oracle(samples)
-    assert np.array_equal(out[samples].astype(np.float64), ref)
+    assert bitexact(out[samples], ref)
     del case
     torch.cuda.empty_cache()
 
@@ -160,7 +166,7 @@ def test_every_catalog_entry_int_bitexact(part):
             _, out = run_plan(case, plan)
             for f in used:
                 a, z = col[f], col[f + 1]
-                assert np.array_equal(out[:, a:z].astype(np.float64), ref[:, a:z]), (e, f, per_block)
+                assert bitexact(out[:, a:z], ref[:, a:z]), (e, f, per_block)
             tested += 1
             # restore defaults for the next entry
             plan = P.Plan.from_model(m, max_batch=b.B)
@@ -177,7 +183,7 @@ def test_each_occupancy_variant_parity(k):
     plan.occupancy = k
     _, out = run_plan(case, plan)
     ref, _ = case.oracle()
-    assert np.array_equal(out.astype(np.float64), ref)
+    assert bitexact(out, ref)
 
 
 @pytest.mark.parametrize('k', range(1, 9))
@@ -202,7 +208,9 @@ def test_task_map_bitexact_vs_oracle(seed):
         s = plan.get_schedule(f)
         if rng.random() < 0.5:
             s['part'] = 1
-            s['per_block'] = int(rng.integers(1, 200))
+            # >= 128 lookups per task: within the plan's reserved task slots
+            # (max_batch * max_len / 128), so the map never raises npb (C12)
+            s['per_block'] = int(rng.integers(128, 700))
         else:
             s['part'] = 0
             s['per_block'] = int(rng.integers(1, 300))
@@ -236,7 +244,7 @@ def test_all_empty_and_ragged_batches():
     plan = P.Plan.from_model(m, max_batch=64)
     _, out = run_plan(case, plan)
     ref, _ = case.oracle()
-    assert np.array_equal(out.astype(np.float64), ref)
+    assert bitexact(out, ref)
     assert np.count_nonzero(out) > 0
 
 
@@ -354,4 +362,4 @@ def test_tuner_runs_counts_and_keeps_parity():
     assert st['best_occupancy'] in ks
     _, out = run_plan(case, plan)
     ref, _ = case.oracle()
-    assert np.array_equal(out.astype(np.float64), ref)
+    assert bitexact(out, ref)

@@ -1,0 +1,70 @@
+"""Tune a config's plan with the two-stage tuner and export it (tuned
+schedules are reused for a long period, re-tuned periodically).
+
+    python tools/tune_plan.py sharded1000 [--world W --rank R] [--ks 2,4,6,8] [--out DIR]
+
+Writes DIR/<config>_w<W>_r<R>.json (default DIR = gpurun_out/tuned) plus a
+.log with the tuner statistics.  bench.py loads configs/tuned/ automatically.
+"""
+import argparse
+import json
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument('config')
+    ap.add_argument('--world', type=int, default=1)
+    ap.add_argument('--rank', type=int, default=-1, help='-1: all ranks sequentially on this GPU')
+    ap.add_argument('--ks', default='')
+    ap.add_argument('--batches', type=int, default=2)
+    ap.add_argument('--reps', type=int, default=5)
+    ap.add_argument('--max-candidates', type=int, default=0)
+    ap.add_argument('--out', default=os.path.join(ROOT, 'gpurun_out', 'tuned'))
+    a = ap.parse_args()
+    import torch
+    from paper_conf_sc_panzzxwslr0d24_b200 import synth
+    from paper_conf_sc_panzzxwslr0d24_b200.shard import ShardedEmbedding, partition_model, shard_batch
+
+    os.makedirs(a.out, exist_ok=True)
+    dev = torch.device('cuda', 0)
+    model = synth.make_model(a.config)
+    parts = partition_model(model, a.world)
+    ranks = range(a.world) if a.rank < 0 else [a.rank]
+    ks = [int(x) for x in a.ks.split(',')] if a.ks else None
+    fulls = [synth.make_batch(model, 7 + i) for i in range(a.batches)]
+    for r in ranks:
+        sh = ShardedEmbedding(model, r, a.world, device=0, parts=parts)
+        feats = sh.features
+        phys = {}
+        for f in feats:
+            t = model.features[f].table
+            if t not in phys:
+                rows, dim = model.tables[t]
+                phys[t] = synth.make_table(t, rows, dim, 'float', device=dev, seed=model.seed)
+        tables = [phys[model.features[f].table] for f in feats]
+        hist = []
+        for full in fulls:
+            idx, off = shard_batch(full, feats)
+            hist.append((torch.from_numpy(idx).to(dev), torch.from_numpy(off).to(dev), model.batch))
+        t0 = time.time()
+        st = sh.plan.tune(hist, tables, occupancies=ks, reps=a.reps, max_candidates=a.max_candidates, verbose=True)
+        st['wall_s'] = time.time() - t0
+        state = sh.plan.export()
+        name = f'{a.config}_w{a.world}_r{r}'
+        with open(os.path.join(a.out, name + '.json'), 'w') as fh:
+            json.dump(state, fh)
+        with open(os.path.join(a.out, name + '.log'), 'w') as fh:
+            json.dump(st, fh, indent=1)
+        print(name, json.dumps(st), flush=True)
+        del sh, tables, phys, hist
+        torch.cuda.empty_cache()
+
+
+if __name__ == '__main__':
+    main()
