@@ -11,7 +11,7 @@ import ctypes
 import os
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, 'lib', 'librecflex.so')
+LIB_PATH = os.environ.get('RECFLEX_LIB') or os.path.join(HERE, 'lib', 'librecflex.so')
 
 c_int32 = ctypes.c_int32
 c_int64 = ctypes.c_int64

@@ -1,7 +1,10 @@
 // fused_impl.cuh -- the fused heterogeneous-schedule kernel (Fig. 8),
 // B200 form: persistent CTAs (#SM x k) pull tasks from a device counter, so the
 // grid never depends on host-side knowledge of the batch (the device-side map
-// kernel produced block_start); launched with PDL behind the map kernel.
+// kernel produced block_start); launched with PDL behind the map kernel.  The
+// task is still the CTA-sized mapping unit of the paper, but warps of a
+// CTA advance through the task sequence independently (ring of task slots):
+// GROUP-family tasks never wait on a CTA barrier.
 //
 // Per task t (the paper's blockIdx.x):
 //   feature_idx = the f with block_start[f] <= t < block_start[f+1]
@@ -19,30 +22,81 @@
 namespace recflex {
 
 template <int I>
-__device__ __forceinline__ void dispatch_schedule(int id, const TaskCtx &x, float *red) {
+__device__ __forceinline__ void dispatch_schedule(int id, const TaskCtx &x, float *red, int *bag_ctr) {
     if constexpr (I < kCatalogSize) {
         if (id == I) {
             constexpr CatalogEntry e = kCatalog[I];
             if constexpr (e.family == RECFLEX_FAMILY_GROUP)
-                sched_group<e.G, e.VEC, e.C, e.U>(x.table, x.offs, x.idx, x.out, x.dim, x.pool, x.out_stride, x.s0, x.s1);
+                sched_group<e.G, e.VEC, e.C, e.U>(x.table, x.offs, x.idx, x.out, x.dim, x.pool, x.out_stride, x.s0, x.s1,
+                                                  bag_ctr);
             else
                 sched_block<e.G, e.VEC, e.C, e.U>(x.table, x.offs, x.idx, x.out, x.dim, x.pool, x.out_stride, x.s0,
                                                   x.s1, red);
         } else {
-            dispatch_schedule<I + 1>(id, x, red);
+            dispatch_schedule<I + 1>(id, x, red, bag_ctr);
         }
     }
 }
 
+// Single call site for the whole catalog: the kernel calls this once per task
+// (few live values cross the call), and it branches to the schedule.
+static __device__ __noinline__ void dispatch_task(int id, const float *T, const int32_t *offs, const int32_t *idx, float *out,
+                                           int d, int pool, int out_stride, int s0, int s1, float *red, int *bag) {
+    TaskCtx x;
+    x.table = T;
+    x.offs = offs;
+    x.idx = idx;
+    x.out = out;
+    x.dim = d;
+    x.pool = pool;
+    x.out_stride = out_stride;
+    x.s0 = s0;
+    x.s1 = s1;
+    dispatch_schedule<0>(id, x, red, bag);
+}
+
 constexpr int kRedFloats = 8 * 256;  // BLOCK family: [8 warps][SPAN <= 256]
+constexpr int kWarps = kBlockThreads / 32;
+constexpr int kRing = 8;             // task slots in flight per CTA
+
+#define RECFLEX_FAMILY_OF(fam, g, v, c, u) fam,
+__constant__ signed char kFamilyDev[kCatalogSize] = {RECFLEX_CATALOG(RECFLEX_FAMILY_OF)};
+#undef RECFLEX_FAMILY_OF
+
+// One task in flight inside a CTA.  Warps walk the same task sequence
+// n = 0, 1, 2, ... independently; slot n % kRing holds task n.
+struct TaskSlot {
+    int t;       // global task id (>= total: end of work)
+    int f;       // feature_idx
+    int s0, s1;  // samples of the task
+    int bag;     // GROUP family: next bag to claim (relative to s0)
+    int left;    // warps that finished this task
+    int state;   // 0 free, 1 being filled, 2 ready
+    int seq;     // task sequence number held
+    long long t0;
+};
+
+__device__ __forceinline__ int vld(const int *p) { return *reinterpret_cast<const volatile int *>(p); }
+__device__ __forceinline__ void vst(int *p, int v) { *reinterpret_cast<volatile int *>(p) = v; }
+
+__device__ __forceinline__ int find_feature(const int *bs, int F, int t) {
+    int lo = 0, hi = F;  // upper_bound(block_start, t) - 1
+    while (hi - lo > 1) {
+        const int mid = (lo + hi) >> 1;
+        if (bs[mid] <= t) lo = mid;
+        else hi = mid;
+    }
+    return lo;
+}
 
 template <int KOCC>
 __global__ void __launch_bounds__(kBlockThreads, KOCC) recflex_fused_kernel(FusedArgs a) {
     extern __shared__ __align__(16) unsigned char dyn_smem[];
-    __shared__ int s_task[2];
-    float *red = reinterpret_cast<float *>(dyn_smem);                       // union member 1
+    __shared__ TaskSlot ring[kRing];
+    float *red = reinterpret_cast<float *>(dyn_smem);                            // union member 1
     int *bs_s = reinterpret_cast<int *>(dyn_smem + kRedFloats * sizeof(float));  // union member 2
     const int tid = threadIdx.x;
+    const int lane = tid & 31;
     const int F = a.F;
     const bool bs_in_smem = (F + 1) <= kSmemBlockStartCap;
 
@@ -53,51 +107,90 @@ __global__ void __launch_bounds__(kBlockThreads, KOCC) recflex_fused_kernel(Fuse
     if (bs_in_smem)
         for (int i = tid; i <= F; i += kBlockThreads) bs_s[i] = a.block_start[i];
     const int *bs = bs_in_smem ? bs_s : a.block_start;
-    if (tid == 0) s_task[0] = atomicAdd(a.counter, 1);
+    if (tid < kRing) {
+        ring[tid].state = 0;
+        ring[tid].seq = -1;
+        ring[tid].left = 0;
+    }
     __syncthreads();
 
-    int buf = 0;
-    while (true) {
-        const int t = s_task[buf];
+    // Warp-decoupled task loop: a warp that runs out of bags in task n moves
+    // on to task n+1 without waiting for the CTA's other warps (no per-task
+    // __syncthreads for GROUP schedules); BLOCK schedules synchronise the CTA
+    // on entry and exit.  The first warp to reach a free slot fills it.
+    for (int n = 0;; ++n) {
+        TaskSlot &S = ring[n % kRing];
+        if (lane == 0) {
+            while (true) {
+                const int st = vld(&S.state);
+                if (st == 2) {
+                    if (vld(&S.seq) == n) break;
+                } else if (st == 0 && atomicCAS(&S.state, 0, 1) == 0) {
+                    const int t = atomicAdd(a.counter, 1);
+                    S.t = t;
+                    S.seq = n;
+                    S.bag = 0;
+                    S.left = 0;
+                    if (t < total) {
+                        const int f = find_feature(bs, F, t);
+                        const int rel = t - bs[f];
+                        const FeatureDesc &fd = a.desc[f];
+                        int s0, s1;
+                        if (fd.part == 0) {
+                            s0 = rel * fd.per_block;
+                            s1 = min(a.B, s0 + fd.per_block);
+                        } else {
+                            const int32_t *ts = a.task_start + fd.slot_base;
+                            s0 = ts[rel];
+                            s1 = ts[rel + 1];
+                        }
+                        S.f = f;
+                        S.s0 = s0;
+                        S.s1 = s1;
+                        if (a.timers) S.t0 = clock64();
+#ifndef RECFLEX_NO_L2PF
+                        if (s1 > s0) {
+                            // stage the task's contiguous lookup-ID range into L2
+                            // with one bulk prefetch (TMA engine)
+                            const int32_t *offs = a.offsets + (size_t)fd.in_feature * a.B;
+                            const int32_t j0 = __ldg(offs + s0), j1 = __ldg(offs + s1);
+                            const uintptr_t b = reinterpret_cast<uintptr_t>(a.indices + j0) & ~uintptr_t(15);
+                            const uintptr_t e = (reinterpret_cast<uintptr_t>(a.indices + j1) + 15) & ~uintptr_t(15);
+                            if (e > b)
+                                asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(b),
+                                             "r"((unsigned)(e - b))
+                                             : "memory");
+                        }
+#endif
+                    }
+                    __threadfence_block();
+                    vst(&S.state, 2);
+                    break;
+                }
+                __nanosleep(32);
+            }
+        }
+        __syncwarp();
+        __threadfence_block();
+        const int t = vld(&S.t);
         if (t >= total) break;
-        long long t0 = 0;
-        if (tid == 0) {
-            s_task[buf ^ 1] = atomicAdd(a.counter, 1);  // prefetch the next task id
-            if (a.timers) t0 = clock64();
-        }
-        // feature_idx: upper_bound(block_start, t) - 1
-        int lo = 0, hi = F;
-        while (hi - lo > 1) {
-            const int mid = (lo + hi) >> 1;
-            if (bs[mid] <= t) lo = mid;
-            else hi = mid;
-        }
-        const int f = lo;
-        const int rel = t - bs[f];
+        const int f = vld(&S.f);
         const FeatureDesc fd = a.desc[f];
-        int s0, s1;
-        if (fd.part == 0) {
-            s0 = rel * fd.per_block;
-            s1 = min(a.B, s0 + fd.per_block);
-        } else {
-            const int32_t *ts = a.task_start + fd.slot_base;
-            s0 = ts[rel];
-            s1 = ts[rel + 1];
+        const bool cta_wide = kFamilyDev[fd.sched] == RECFLEX_FAMILY_BLOCK;
+        if (cta_wide) __syncthreads();  // every warp reaches task n (they walk the same sequence)
+        dispatch_task(fd.sched, fd.table, a.offsets + (size_t)fd.in_feature * a.B, a.indices, a.out + fd.col, fd.dim,
+                      fd.pool, a.out_stride, vld(&S.s0), vld(&S.s1), red, &S.bag);
+        if (cta_wide) __syncthreads();
+        __syncwarp();
+        if (lane == 0) {
+            __threadfence_block();
+            if (atomicAdd(&S.left, 1) == kWarps - 1) {
+                if (a.timers && t < a.timers_cap) a.timers[t] = clock64() - S.t0;
+                S.seq = -1;
+                __threadfence_block();
+                vst(&S.state, 0);
+            }
         }
-        TaskCtx x;
-        x.table = fd.table;
-        x.offs = a.offsets + (size_t)fd.in_feature * a.B;
-        x.idx = a.indices;
-        x.out = a.out + fd.col;
-        x.dim = fd.dim;
-        x.pool = fd.pool;
-        x.out_stride = a.out_stride;
-        x.s0 = s0;
-        x.s1 = s1;
-        dispatch_schedule<0>(fd.sched, x, red);
-        __syncthreads();
-        if (tid == 0 && a.timers && t < a.timers_cap) a.timers[t] = clock64() - t0;
-        buf ^= 1;
     }
 }
 

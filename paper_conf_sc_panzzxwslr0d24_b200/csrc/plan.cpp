@@ -125,8 +125,8 @@ recflex_status_t prepare_occupancy(recflex_plan_s *p, int k) {
     const int sm_total = 233472;  // 228 KB per SM
     int dyn = ((sm_total / k - 1152) / 128) * 128;
     dyn = std::max(dyn, min_dyn_smem(p->F));
-    dyn = std::min(dyn, 232448 - 128);
-    int rc = fused_prepare(k, p->device, 232448 - 128);
+    dyn = std::min(dyn, 232448 - 1024);  // 227 KB opt-in max minus static smem (<= 1 KB)
+    int rc = fused_prepare(k, p->device, 232448 - 1024);
     if (rc) return cuda_status((cudaError_t)rc);
     int blocks = 0, regs = 0, spill = 0;
     // walk the padding until the occupancy API reports exactly k (or as close as possible)

@@ -102,22 +102,14 @@ struct TaskCtx {
 };
 
 // ---- GROUP family --------------------------------------------------------
-// Samples [s0, s1) of the task; group g takes samples s0+g, s0+g+NG, ...
+// One bag [lo, hi) pooled by the G lanes of a group: lane lg holds columns
+// p*SPAN + c*G*VEC + lg*VEC (+0..VEC-1); U rows in flight per lane.
 template <int G, int VEC, int C, int U>
-__device__ __noinline__ void sched_group(const float *__restrict__ T, const int32_t *__restrict__ offs,
-                                        const int32_t *__restrict__ idx, float *__restrict__ out, int d, int pool,
-                                        int out_stride, int s0, int s1) {
-    constexpr int NG = kBlockThreads / G;
+__device__ __forceinline__ void group_bag(const float *__restrict__ T, const int32_t *__restrict__ idx, int d,
+                                          int pool, float *__restrict__ orow, int lo, int hi, int lg) {
     constexpr int SPAN = G * VEC * C;
-    const int tid = threadIdx.x;
-    const int gid = tid / G;
-    const int lg = tid % G;
     const int passes = (d + SPAN - 1) / SPAN;
-
-    for (int s = s0 + gid; s < s1; s += NG) {
-        const int lo = ld_idx(offs + s);
-        const int hi = ld_idx(offs + s + 1);
-        float *__restrict__ orow = out + (size_t)s * out_stride;
+    {
         for (int p = 0; p < passes; ++p) {
             int colv[C];
             bool ok[C];
@@ -132,6 +124,11 @@ __device__ __noinline__ void sched_group(const float *__restrict__ T, const int3
 #pragma unroll
                 for (int e = 0; e < VEC; ++e) acc[c][e] = 0.f;
 
+            // U lookup IDs, then their U rows, then the adds: all U row loads are
+            // in flight before the first add consumes one (a one-iteration-ahead
+            // index prefetch was measured 2x slower: under the register cap
+            // ptxas interleaves the in-order adds with the loads).  Rows are
+            // added in ascending lookup order (the sequential fp32 bag sum).
             int j = lo;
             for (; j + U <= hi; j += U) {
                 int id[U];
@@ -182,6 +179,54 @@ __device__ __noinline__ void sched_group(const float *__restrict__ T, const int3
     }
 }
 
+// Samples [s0, s1) of the task.  Groups claim bags dynamically from a shared
+// counter (*bag_ctr, zeroed before the task), so a long-tail bag delays only
+// its own group; the next bag's offsets are loaded while the current bag is
+// pooled.  Which group pools a bag does not change the bag's arithmetic (rows
+// in ascending lookup order) -> results are independent of the claim order.
+template <int G, int VEC, int C, int U>
+__device__ __noinline__ void sched_group(const float *__restrict__ T, const int32_t *__restrict__ offs,
+                                        const int32_t *__restrict__ idx, float *__restrict__ out, int d, int pool,
+                                        int out_stride, int s0, int s1, int *bag_ctr) {
+    const int lane = threadIdx.x & 31;
+    const int lg = lane & (G - 1);
+    const unsigned gmask = (G == 32) ? 0xffffffffu : (((1u << G) - 1u) << (lane & ~(G - 1)));
+#ifdef RECFLEX_STATIC_CLAIM
+    int next_static = threadIdx.x / G;
+    auto claim = [&]() -> int {
+        const int v = next_static;
+        next_static += kBlockThreads / G;
+        (void)gmask;
+        (void)bag_ctr;
+        return s0 + v;
+    };
+#else
+    auto claim = [&]() -> int {
+        int v = 0;
+        if (lg == 0) v = atomicAdd(bag_ctr, 1);
+        return s0 + __shfl_sync(gmask, v, 0, G);
+    };
+#endif
+    int s = claim();
+    int lo = 0, hi = 0;
+    if (s < s1) {
+        lo = ld_idx(offs + s);
+        hi = ld_idx(offs + s + 1);
+    }
+    while (s < s1) {
+        const int sn = claim();
+        int lon = 0, hin = 0;
+        if (sn < s1) {
+            lon = ld_idx(offs + sn);
+            hin = ld_idx(offs + sn + 1);
+        }
+        group_bag<G, VEC, C, U>(T, idx, d, pool, out + (size_t)s * out_stride, lo, hi, lg);
+        s = sn;
+        lo = lon;
+        hi = hin;
+    }
+}
+
 // ---- BLOCK family ----------------------------------------------------------
 // One bag at a time for the whole CTA.  Group g takes lookups lo+g, lo+g+NG, ...
 // (adjacent groups read adjacent IDs: coalesced index loads).  Partials:
@@ -219,6 +264,7 @@ __device__ __noinline__ void sched_block(const float *__restrict__ T, const int3
 #pragma unroll
                 for (int e = 0; e < VEC; ++e) acc[c][e] = 0.f;
 
+            // this group's strided share of the bag: lookups lo+gid, lo+gid+NG, ...
             int j = lo + gid;
             for (; j + (U - 1) * NG < hi; j += U * NG) {
                 int id[U];
