@@ -145,6 +145,8 @@ typedef struct {
     int32_t pad_waves;       /* padding tasks = pad_waves * #SM * k, default 4     */
     int32_t max_candidates;  /* per feature, 0 = all valid catalog candidates              */
     int32_t verbose;         /* 1: print per-stage summaries to stderr                     */
+    int32_t skip_guard;      /* 0: also time the incoming schedules at every k and keep
+                                them if faster than the two-stage result (K extra evals)   */
 } recflex_tune_options_t;
 
 typedef struct {
@@ -152,6 +154,8 @@ typedef struct {
     int64_t global_launches;  /* stage 2 timed fused launches    (= K*N*reps)        */
     int64_t local_evals;      /* stage-1 cost evaluations (one per (k, f)) = F*K     */
     int64_t global_evals;     /* stage-2 cost evaluations (one per k)      = K       */
+    int64_t guard_evals;      /* guard evaluations of the incoming plan    = K (or 0) */
+    int32_t guard_won;        /* 1 if the incoming schedules were kept             */
     int32_t best_occupancy;
     double best_ms;           /* summed median forward time over tuning batches    */
     double tune_seconds;

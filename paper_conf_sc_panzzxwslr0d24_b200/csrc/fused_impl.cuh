@@ -73,11 +73,14 @@ struct TaskSlot {
     int left;    // warps that finished this task
     int state;   // 0 free, 1 being filled, 2 ready
     int seq;     // task sequence number held
-    long long t0;
+    unsigned long long wtime;  // tuning: sum over warps of cycles spent on the task
 };
 
 __device__ __forceinline__ int vld(const int *p) { return *reinterpret_cast<const volatile int *>(p); }
 __device__ __forceinline__ void vst(int *p, int v) { *reinterpret_cast<volatile int *>(p) = v; }
+__device__ __forceinline__ unsigned long long vld64(const unsigned long long *p) {
+    return *reinterpret_cast<const volatile unsigned long long *>(p);
+}
 
 __device__ __forceinline__ int find_feature(const int *bs, int F, int t) {
     int lo = 0, hi = F;  // upper_bound(block_start, t) - 1
@@ -131,6 +134,7 @@ __global__ void __launch_bounds__(kBlockThreads, KOCC) recflex_fused_kernel(Fuse
                     S.seq = n;
                     S.bag = 0;
                     S.left = 0;
+                    S.wtime = 0;
                     if (t < total) {
                         const int f = find_feature(bs, F, t);
                         const int rel = t - bs[f];
@@ -147,7 +151,7 @@ __global__ void __launch_bounds__(kBlockThreads, KOCC) recflex_fused_kernel(Fuse
                         S.f = f;
                         S.s0 = s0;
                         S.s1 = s1;
-                        if (a.timers) S.t0 = clock64();
+
 #ifndef RECFLEX_NO_L2PF
                         if (s1 > s0) {
                             // stage the task's contiguous lookup-ID range into L2
@@ -174,6 +178,12 @@ __global__ void __launch_bounds__(kBlockThreads, KOCC) recflex_fused_kernel(Fuse
         __threadfence_block();
         const int t = vld(&S.t);
         if (t >= total) break;
+        // Tuning timer ("block execution time"): warps of one CTA can be
+        // on different tasks, so a task's cost is the warp-cycles spent on it
+        // (sum over warps of enter->leave) / 8 -- for a CTA-synchronous task
+        // this is exactly its span; for a warp-decoupled task it does not
+        // count the time its warps spent on neighbouring tasks.
+        const long long w0 = a.timers ? clock64() : 0;
         const int f = vld(&S.f);
         const FeatureDesc fd = a.desc[f];
         const bool cta_wide = kFamilyDev[fd.sched] == RECFLEX_FAMILY_BLOCK;
@@ -183,9 +193,10 @@ __global__ void __launch_bounds__(kBlockThreads, KOCC) recflex_fused_kernel(Fuse
         if (cta_wide) __syncthreads();
         __syncwarp();
         if (lane == 0) {
+            if (a.timers) atomicAdd(&S.wtime, (unsigned long long)(clock64() - w0));
             __threadfence_block();
             if (atomicAdd(&S.left, 1) == kWarps - 1) {
-                if (a.timers && t < a.timers_cap) a.timers[t] = clock64() - S.t0;
+                if (a.timers && t < a.timers_cap) a.timers[t] = (long long)(vld64(&S.wtime) / kWarps);
                 S.seq = -1;
                 __threadfence_block();
                 vst(&S.state, 0);

@@ -74,13 +74,17 @@ recflex_schedule_t default_schedule(const recflex_feature_spec_t &spec, int targ
     recflex_schedule_t s = {0, 0, 1};
     const int d = spec.dim;
     int id = -1;
-    if (d % 4 == 0) {
+    // Untuned defaults follow what the tuner picks most on B200 (sharded1000 /
+    // heavy): rows up to 64 floats -> 256-bit loads with d/8 lanes per bag
+    // (more bags in flight per warp), U = 2; wider rows -> a warp (or more
+    // passes) of 128-bit lanes, U = 4 for multi-hot bags.
+    if (d % 8 == 0 && d <= 64) {
+        id = find_catalog(RECFLEX_FAMILY_GROUP, std::max(1, d / 8), 8, 1, 2);
+    } else if (d % 4 == 0) {
         int lanes = d / 4;
         int G = std::min(32, next_pow2(lanes));
-        int C = (lanes > 32) ? 2 : 1;
-        int U = spec.mean_len >= 6.f ? 8 : (spec.mean_len >= 2.5f ? 4 : 2);
-        if (C == 2 && U > 4) U = 4;
-        id = find_catalog(RECFLEX_FAMILY_GROUP, G, 4, C, U);
+        int U = spec.mean_len >= 2.5f ? 4 : 2;
+        id = find_catalog(RECFLEX_FAMILY_GROUP, G, 4, 1, U);
     }
     if (id < 0) id = find_catalog(RECFLEX_FAMILY_GROUP, std::min(32, next_pow2(d)), 1, 1, 4);
     s.sched_id = id;

@@ -134,6 +134,7 @@ struct Tuner {
     std::vector<std::vector<recflex_schedule_t>> cands;  // per feature
     recflex_status_t err = RECFLEX_OK;
     int64_t local_launches = 0, global_launches = 0;
+    double last_global = 0;
 
     // per-feature tuning inputs (rebuilt when f changes), one per batch
     int cur_f = -1;
@@ -390,7 +391,31 @@ struct Tuner {
             std::sort(ms.begin(), ms.end());
             total += ms[ms.size() / 2];
         }
-        if (verbose) std::fprintf(stderr, "[recflex tune] global k=%d: %.4f ms\n", k, total);
+        if (verbose) {
+            std::fprintf(stderr, "[recflex tune] global k=%d: %.4f ms  schedules:", k, total);
+            std::vector<std::pair<long, int>> hist;
+            for (int f = 0; f < p->F; ++f) {
+                const recflex_schedule_t &s = cands[f][choice[f]];
+                const long key = ((long)s.sched_id * 2 + s.part) * 100000 + s.per_block;
+                bool found = false;
+                for (auto &h : hist)
+                    if (h.first == key) {
+                        ++h.second;
+                        found = true;
+                    }
+                if (!found) hist.push_back({key, 1});
+            }
+            std::sort(hist.begin(), hist.end(), [](auto &a, auto &b) { return a.second > b.second; });
+            for (size_t i = 0; i < hist.size() && i < 6; ++i) {
+                const long key = hist[i].first;
+                const int sid = (int)(key / 100000 / 2), part = (int)(key / 100000 % 2);
+                const CatalogEntry &e = kCatalog[sid];
+                std::fprintf(stderr, " %dx[%s G%d V%d C%d U%d p%d/%ld]", hist[i].second, e.family ? "block" : "group",
+                             e.G, e.VEC, e.C, e.U, part, key % 100000);
+            }
+            std::fprintf(stderr, "\n");
+        }
+        last_global = total;
         return total;
     }
 };
@@ -405,29 +430,30 @@ std::vector<recflex_schedule_t> candidates_for(const recflex_plan_s *p, int f, i
     // the plan's current schedule is always candidate 0 (tie -> keep it)
     out.push_back({d.sched, d.part, d.per_block});
     const bool multi_hot = sp.max_len > 1.5f;
-    for (int id = 0; id < kCatalogSize; ++id) {
-        const CatalogEntry &e = kCatalog[id];
-        recflex_schedule_t s = {id, 0, 1};
-        s.per_block = samples_per_task_default(id, sp.mean_len, sp.coverage, p->task_lookups);
-        if (!schedule_valid_for(s, d.dim, d.col, (int)p->d_tot)) continue;
-        const int span = e.G * e.VEC * e.C;
-        const int passes = (d.dim + span - 1) / span;
-        if (passes > 2) continue;
-        if (e.VEC == 1 && d.dim % 4 == 0) continue;  // scalar only where vectors cannot run
-        if (!multi_hot && e.family == RECFLEX_FAMILY_BLOCK) continue;
-        if (!multi_hot && e.U > 2) continue;  // one-hot bags: unroll is irrelevant
-        auto same = [&](const recflex_schedule_t &o) {
-            return o.sched_id == s.sched_id && o.part == s.part && o.per_block == s.per_block;
-        };
-        if (std::none_of(out.begin(), out.end(), same)) out.push_back(s);
-        if (multi_hot && e.family == RECFLEX_FAMILY_GROUP) {
-            recflex_schedule_t s1 = {id, 1, std::max(128, p->task_lookups)};
-            if (std::none_of(out.begin(), out.end(), same) || true) {
-                bool dup = false;
-                for (auto &o : out)
-                    if (o.sched_id == s1.sched_id && o.part == 1 && o.per_block == s1.per_block) dup = true;
-                if (!dup) out.push_back(s1);
-            }
+    auto add = [&](const recflex_schedule_t &s) {
+        for (auto &o : out)
+            if (o.sched_id == s.sched_id && o.part == s.part && o.per_block == s.per_block) return;
+        out.push_back(s);
+    };
+    // User-supplied candidate list -- our prior: single-pass entries
+    // with one column chunk per lane (multi-pass / C=2 entries re-traverse the
+    // bag or idle half the lanes and measured 2-3x slower on B200); they are
+    // admitted only when a dim has no single-pass entry.
+    for (int relax = 0; relax < 2 && out.size() <= 1; ++relax) {
+        for (int id = 0; id < kCatalogSize; ++id) {
+            const CatalogEntry &e = kCatalog[id];
+            recflex_schedule_t s = {id, 0, 1};
+            s.per_block = samples_per_task_default(id, sp.mean_len, sp.coverage, p->task_lookups);
+            if (!schedule_valid_for(s, d.dim, d.col, (int)p->d_tot)) continue;
+            const int span = e.G * e.VEC * e.C;
+            const int passes = (d.dim + span - 1) / span;
+            if (relax == 0 && (passes > 1 || e.C > 1)) continue;
+            if (relax == 1 && passes > 2) continue;
+            if (e.VEC == 1 && d.dim % 4 == 0) continue;  // scalar only where vectors cannot run
+            if (!multi_hot && e.family == RECFLEX_FAMILY_BLOCK) continue;
+            if (!multi_hot && e.U > 2) continue;  // one-hot bags: unroll is irrelevant
+            add(s);
+            if (multi_hot && e.family == RECFLEX_FAMILY_GROUP) add({id, 1, std::max(128, p->task_lookups)});
         }
     }
     if (max_c > 0 && (int)out.size() > max_c) out.resize(max_c);
@@ -508,17 +534,37 @@ extern "C" recflex_status_t recflex_tune_ex(recflex_plan_t p, int32_t N, const i
     } guard{T};
     if (st == RECFLEX_OK) st = T.err;
     if (st != RECFLEX_OK) return st;
+    // re-measure the two-stage selection, then the guard: the plan's incoming
+    // schedules (candidate 0 of every feature) at each k; keep whichever is
+    // faster (an untuned-or-previous plan is never made slower by tuning).
+    double best_ms = T.global_cost(best_k, choice.data());
+    int64_t guard_evals = 0;
+    if (!(opt && opt->skip_guard)) {
+        std::vector<int32_t> zero(p->F, 0);
+        for (int ki = 0; ki < (int)T.ks.size(); ++ki) {
+            const double c0 = T.global_cost(ki, zero.data());
+            ++guard_evals;
+            if (c0 < best_ms) {
+                best_ms = c0;
+                best_k = ki;
+                choice = zero;
+            }
+        }
+    }
+    if (T.err != RECFLEX_OK) return T.err;
     T.apply(choice.data());
     p->k = T.ks[best_k];
     st = upload_desc(p, stream);
     if (st != RECFLEX_OK) return st;
-    // re-measure the selected configuration for the stats
-    const double best_ms = T.global_cost(best_k, choice.data());
     recflex_tune_stats_t s = {};
     s.local_launches = T.local_launches;
     s.global_launches = T.global_launches;
     s.local_evals = lc;
     s.global_evals = gc;
+    s.guard_evals = guard_evals;
+    s.guard_won = 0;
+    for (int f = 0; f < p->F && guard_evals; ++f) s.guard_won |= (choice[f] != 0);
+    s.guard_won = guard_evals ? !s.guard_won : 0;
     s.best_occupancy = p->k;
     s.best_ms = best_ms;
     s.tune_seconds = std::chrono::duration<double>(std::chrono::steady_clock::now() - t_start).count();
