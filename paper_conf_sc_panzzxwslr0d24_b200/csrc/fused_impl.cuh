@@ -29,6 +29,9 @@ __device__ __forceinline__ void dispatch_schedule(int id, const TaskCtx &x, floa
             if constexpr (e.family == RECFLEX_FAMILY_GROUP)
                 sched_group<e.G, e.VEC, e.C, e.U>(x.table, x.offs, x.idx, x.out, x.dim, x.pool, x.out_stride, x.s0, x.s1,
                                                   bag_ctr);
+            else if constexpr (e.family == RECFLEX_FAMILY_FLAT)
+                sched_flat<e.G, e.VEC, e.U>(x.table, x.offs, x.idx, x.out, x.dim, x.pool, x.out_stride, x.s0, x.s1,
+                                            bag_ctr);
             else
                 sched_block<e.G, e.VEC, e.C, e.U>(x.table, x.offs, x.idx, x.out, x.dim, x.pool, x.out_stride, x.s0,
                                                   x.s1, red);

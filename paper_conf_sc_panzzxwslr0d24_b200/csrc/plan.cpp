@@ -51,7 +51,8 @@ int find_catalog(int family, int G, int VEC, int C, int U) {
 // rounds of the CTA's bag slots.
 int samples_per_task_default(int sched_id, float mean_len, float coverage, int target) {
     const CatalogEntry &e = kCatalog[sched_id];
-    const int slots = (e.family == RECFLEX_FAMILY_GROUP) ? kBlockThreads / e.G : 1;
+    const int slots = (e.family == RECFLEX_FAMILY_GROUP) ? kBlockThreads / e.G
+                      : (e.family == RECFLEX_FAMILY_FLAT) ? (kBlockThreads / e.G) * 8 : 1;
     double el = std::max(0.25, (double)mean_len * std::max(0.05, (double)coverage));
     int R = (int)std::lround((double)target / (slots * el));
     R = std::min(32, std::max(1, R));

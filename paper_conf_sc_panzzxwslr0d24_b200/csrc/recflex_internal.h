@@ -99,7 +99,15 @@ struct FusedArgs {
     X(1, 1, 4, 1, 4) X(1, 2, 4, 1, 4) X(1, 4, 4, 1, 4)                          \
     X(1, 8, 4, 1, 4) X(1, 16, 4, 1, 4) X(1, 32, 4, 1, 2) X(1, 32, 4, 1, 4)     \
     /* BLOCK, 256-bit rows */                                                   \
-    X(1, 16, 8, 1, 2) X(1, 16, 8, 1, 4)
+    X(1, 16, 8, 1, 2) X(1, 16, 8, 1, 4)                                         \
+    /* FLAT: runs of bags walked as one lookup range, 128-bit rows */           \
+    X(2, 1, 4, 1, 2) X(2, 1, 4, 1, 4) X(2, 2, 4, 1, 2) X(2, 2, 4, 1, 4)         \
+    X(2, 4, 4, 1, 2) X(2, 4, 4, 1, 4) X(2, 8, 4, 1, 2) X(2, 8, 4, 1, 4)         \
+    X(2, 16, 4, 1, 2) X(2, 16, 4, 1, 4) X(2, 32, 4, 1, 2) X(2, 32, 4, 1, 4)     \
+    /* FLAT, 256-bit rows */                                                    \
+    X(2, 1, 8, 1, 2) X(2, 1, 8, 1, 4) X(2, 2, 8, 1, 2) X(2, 2, 8, 1, 4)         \
+    X(2, 4, 8, 1, 2) X(2, 4, 8, 1, 4) X(2, 8, 8, 1, 2) X(2, 8, 8, 1, 4)         \
+    X(2, 16, 8, 1, 2) X(2, 16, 8, 1, 4)
 
 struct CatalogEntry {
     int family, G, VEC, C, U;

@@ -124,6 +124,77 @@ __device__ __forceinline__ void group_bag(const float *__restrict__ T, const int
 #pragma unroll
                 for (int e = 0; e < VEC; ++e) acc[c][e] = 0.f;
 
+#ifndef RECFLEX_NO_SHFL_IDX
+            if constexpr (U <= G && G >= 4) {
+                // Lookup IDs through registers: lane lg holds ID cb+lg of the
+                // current chunk of G IDs (one coalesced load per chunk) and the
+                // next chunk is already in flight; each iteration broadcasts its
+                // U IDs with shuffles.  This takes the per-iteration index load
+                // (20% of heavy's stall samples as a dependent L1 load) off the
+                // row loads' critical path.
+                const int lane = threadIdx.x & 31;
+                const unsigned gmask = (G == 32) ? 0xffffffffu : (((1u << G) - 1u) << (lane & ~(G - 1)));
+                int cb = lo;
+                int cur = (lo + lg < hi) ? ld_idx(idx + lo + lg) : 0;
+                int nxt = (lo + G + lg < hi) ? ld_idx(idx + lo + G + lg) : 0;
+                int j = lo;
+                for (; j + U <= hi; j += U) {
+                    if (j - cb >= G) {
+                        cb += G;
+                        cur = nxt;
+                        nxt = (cb + G + lg < hi) ? ld_idx(idx + cb + G + lg) : 0;
+                    }
+                    unsigned id[U];
+#pragma unroll
+                    for (int u = 0; u < U; ++u) id[u] = (unsigned)__shfl_sync(gmask, cur, (j - cb) + u, G);
+                    float v[U][C][VEC];
+#pragma unroll
+                    for (int u = 0; u < U; ++u)
+#pragma unroll
+                        for (int c = 0; c < C; ++c)
+                            if (ok[c]) ld_row<VEC>(T + (size_t)id[u] * (unsigned)d + colv[c], v[u][c]);
+#pragma unroll
+                    for (int u = 0; u < U; ++u)
+#pragma unroll
+                        for (int c = 0; c < C; ++c)
+                            if (ok[c])
+#pragma unroll
+                                for (int e = 0; e < VEC; ++e) acc[c][e] += v[u][c][e];
+                }
+                if (j < hi) {
+                    if (j - cb >= G) {
+                        cb += G;
+                        cur = nxt;
+                    }
+                    const int n = hi - j;
+                    unsigned id[U];
+#pragma unroll
+                    for (int u = 0; u < U; ++u) id[u] = (unsigned)__shfl_sync(gmask, cur, (j - cb) + u, G);
+                    float v[U][C][VEC];
+#pragma unroll
+                    for (int u = 0; u < U; ++u)
+#pragma unroll
+                        for (int c = 0; c < C; ++c)
+                            if (u < n && ok[c]) ld_row<VEC>(T + (size_t)id[u] * (unsigned)d + colv[c], v[u][c]);
+#pragma unroll
+                    for (int u = 0; u < U; ++u)
+                        if (u < n)
+#pragma unroll
+                            for (int c = 0; c < C; ++c)
+                                if (ok[c])
+#pragma unroll
+                                    for (int e = 0; e < VEC; ++e) acc[c][e] += v[u][c][e];
+                }
+#pragma unroll
+                for (int c = 0; c < C; ++c) {
+                    if (ok[c]) {
+                        pool_finish<VEC>(acc[c], pool, hi - lo);
+                        st_out<VEC>(orow + colv[c], acc[c]);
+                    }
+                }
+                continue;
+            }
+#endif
             // U lookup IDs, then their U rows, then the adds: all U row loads are
             // in flight before the first add consumes one (a one-iteration-ahead
             // index prefetch was measured 2x slower: under the register cap
@@ -224,6 +295,75 @@ __device__ __noinline__ void sched_group(const float *__restrict__ T, const int3
         s = sn;
         lo = lon;
         hi = hin;
+    }
+}
+
+// ---- FLAT family -----------------------------------------------------------
+// A group claims a run of kFlatRun consecutive bags and walks their lookups as
+// one contiguous range (the KJT stores a run's bags back to back): every
+// iteration keeps U rows in flight whatever the bag lengths, so one-hot and
+// short bags no longer pay a dependent offsets -> IDs -> rows chain per bag.
+// When a row crosses the current bag's end, the finished bag is pooled and
+// stored and its accumulator reset; rows of a bag are still added in
+// ascending lookup order (same arithmetic as GROUP).
+constexpr int kFlatRun = 8;
+
+template <int G, int VEC, int U>
+__device__ __noinline__ void sched_flat(const float *__restrict__ T, const int32_t *__restrict__ offs,
+                                       const int32_t *__restrict__ idx, float *__restrict__ out, int d, int pool,
+                                       int out_stride, int s0, int s1, int *bag_ctr) {
+    const int lane = threadIdx.x & 31;
+    const int lg = lane & (G - 1);
+    const unsigned gmask = (G == 32) ? 0xffffffffu : (((1u << G) - 1u) << (lane & ~(G - 1)));
+    constexpr int SPAN = G * VEC;
+    const int passes = (d + SPAN - 1) / SPAN;
+    while (true) {
+        int v = 0;
+        if (lg == 0) v = atomicAdd(bag_ctr, kFlatRun);
+        const int s = s0 + __shfl_sync(gmask, v, 0, G);
+        if (s >= s1) break;
+        const int se = min(s1, s + kFlatRun);
+        const int A = ld_idx(offs + s);
+        const int Z = ld_idx(offs + se);
+        for (int p = 0; p < passes; ++p) {
+            const int col = p * SPAN + lg * VEC;
+            const bool ok = col < d;
+            float acc[VEC];
+#pragma unroll
+            for (int e = 0; e < VEC; ++e) acc[e] = 0.f;
+            int b = s;               // bag being accumulated
+            int bstart = A;          // its first lookup
+            int bend = ld_idx(offs + s + 1);
+            auto finish_bag = [&]() {
+                if (ok) {
+                    pool_finish<VEC>(acc, pool, bend - bstart);
+                    st_out<VEC>(out + (size_t)b * out_stride + col, acc);
+                }
+#pragma unroll
+                for (int e = 0; e < VEC; ++e) acc[e] = 0.f;
+                ++b;
+                bstart = bend;
+                if (b < se) bend = ld_idx(offs + b + 1);
+            };
+            for (int j = A; j < Z; j += U) {
+                unsigned id[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u) id[u] = (j + u < Z) ? (unsigned)ld_idx(idx + j + u) : 0u;
+                float r[U][VEC];
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+                    if (j + u < Z && ok) ld_row<VEC>(T + (size_t)id[u] * (unsigned)d + col, r[u]);
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    if (j + u < Z) {
+                        while (j + u >= bend) finish_bag();
+#pragma unroll
+                        for (int e = 0; e < VEC; ++e) acc[e] += r[u][e];
+                    }
+                }
+            }
+            while (b < se) finish_bag();  // the last bag(s) of the run, incl. trailing empty bags
+        }
     }
 }
 
