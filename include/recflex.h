@@ -148,6 +148,9 @@ typedef struct {
     int32_t verbose;         /* 1: print per-stage summaries to stderr                     */
     int32_t skip_guard;      /* 0: also time the incoming schedules at every k and keep
                                 them if faster than the two-stage result (K extra evals)   */
+    int32_t skip_refine;     /* 0: after selection, try every candidate per cluster of
+                                same-dim / same-length-class features in the real fused
+                                forward at the chosen k; keep if > 0.5% faster     */
 } recflex_tune_options_t;
 
 typedef struct {
@@ -160,6 +163,8 @@ typedef struct {
     int32_t best_occupancy;
     double best_ms;           /* summed median forward time over tuning batches    */
     double tune_seconds;
+    int64_t refine_evals;     /* cluster-refinement forwards timed                 */
+    double refine_gain;       /* latency before refinement / after (>= 1)          */
 } recflex_tune_stats_t;
 
 /* Two-stage interference-simulated tuning over num_batches historical batches

@@ -36,14 +36,15 @@ class CatalogInfo(ctypes.Structure):
 class TuneOptions(ctypes.Structure):
     _fields_ = [('num_occupancies', ctypes.c_int32), ('occupancies', ctypes.c_int32 * 8),
                 ('reps', ctypes.c_int32), ('pad_waves', ctypes.c_int32), ('max_candidates', ctypes.c_int32),
-                ('verbose', ctypes.c_int32), ('skip_guard', ctypes.c_int32)]
+                ('verbose', ctypes.c_int32), ('skip_guard', ctypes.c_int32), ('skip_refine', ctypes.c_int32)]
 
 
 class TuneStats(ctypes.Structure):
     _fields_ = [('local_launches', ctypes.c_int64), ('global_launches', ctypes.c_int64),
                 ('local_evals', ctypes.c_int64), ('global_evals', ctypes.c_int64),
                 ('guard_evals', ctypes.c_int64), ('guard_won', ctypes.c_int32),
-                ('best_occupancy', ctypes.c_int32), ('best_ms', ctypes.c_double), ('tune_seconds', ctypes.c_double)]
+                ('best_occupancy', ctypes.c_int32), ('best_ms', ctypes.c_double), ('tune_seconds', ctypes.c_double),
+                ('refine_evals', ctypes.c_int64), ('refine_gain', ctypes.c_double)]
 
 
 LOCAL_COST_FN = ctypes.CFUNCTYPE(None, c_void_p, c_int32, c_int32, P(ctypes.c_double))

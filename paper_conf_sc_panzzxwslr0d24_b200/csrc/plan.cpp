@@ -129,6 +129,7 @@ recflex_status_t prepare_occupancy(recflex_plan_s *p, int k) {
     if (e != cudaSuccess) return cuda_status(e);
     const int sm_total = 233472;  // 228 KB per SM
     int dyn = ((sm_total / k - 1152) / 128) * 128;
+    if (p->no_smem_pad) dyn = min_dyn_smem(p->F);  // experiment: leave L1 its capacity
     dyn = std::max(dyn, min_dyn_smem(p->F));
     dyn = std::min(dyn, 232448 - 1024);  // 227 KB opt-in max minus static smem (<= 1 KB)
     int rc = fused_prepare(k, p->device, 232448 - 1024);
@@ -371,6 +372,7 @@ recflex_status_t recflex_plan_create(const recflex_feature_spec_t *specs, int32_
         if (k >= 1 && k <= kMaxOcc) p->k = k;
     }
     if (const char *env = std::getenv("RECFLEX_NO_PDL")) p->pdl = !(env[0] == '1');
+    if (const char *env = std::getenv("RECFLEX_NO_SMEM_PAD")) p->no_smem_pad = (env[0] == '1');
     *out = p;
     return RECFLEX_OK;
 }

@@ -44,6 +44,7 @@ struct recflex_plan_s {
     int task_lookups = 4096;  // lookups per task targeted by the default schedules
     bool desc_dirty = true;
     bool pdl = true;
+    bool no_smem_pad = false;  // RECFLEX_NO_SMEM_PAD=1: occupancy by grid size + registers only
     int64_t slots_total = 0;
 
     recflex::Exec ex;  // plan-owned device scratch

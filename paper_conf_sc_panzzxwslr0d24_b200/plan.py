@@ -146,7 +146,7 @@ class Plan:
     # -------------------------------------------------------------- tuner
     def tune(self, batches: Sequence[tuple], tables: Sequence[torch.Tensor], occupancies: Optional[List[int]] = None,
              reps: int = 7, pad_waves: int = 4, max_candidates: int = 0, verbose: bool = False, guard: bool = True,
-             stream=None) -> dict:
+             refine: bool = True, stream=None) -> dict:
         """recflex_tune_ex over historical batches [(indices, offsets, B), ...]."""
         N = len(batches)
         idx_arr = (ctypes.c_void_p * N)(*[b[0].data_ptr() for b in batches])
@@ -162,12 +162,13 @@ class Plan:
         opt.max_candidates = max_candidates
         opt.verbose = 1 if verbose else 0
         opt.skip_guard = 0 if guard else 1
+        opt.skip_refine = 0 if refine else 1
         st = _lib.TuneStats()
         check(lib.recflex_tune_ex(self._h, N, idx_arr, off_arr, bs_arr, self._tables(tables), _stream_ptr(stream),
                                   ctypes.byref(opt), ctypes.byref(st)), 'recflex_tune_ex')
         return dict(local_launches=st.local_launches, global_launches=st.global_launches,
                     local_evals=st.local_evals, global_evals=st.global_evals, guard_evals=st.guard_evals,
-                    guard_won=bool(st.guard_won),
+                    guard_won=bool(st.guard_won), refine_evals=st.refine_evals, refine_gain=st.refine_gain,
                     best_occupancy=st.best_occupancy, best_ms=st.best_ms, tune_seconds=st.tune_seconds)
 
     # -------------------------------------------------------------- schedules

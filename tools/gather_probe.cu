@@ -39,6 +39,60 @@ __global__ void probe(const float4 *__restrict__ table, const int *__restrict__ 
     if (acc == 123.456f) out[0] = acc;
 }
 
+// Bag mode (512 B rows only): warp-per-bag over fixed-length bags of L lookups,
+// warps claim bags from a global counter, pooled row stored per bag.
+template <int U>
+__global__ void probe_bags(const float4 *__restrict__ table, const int *__restrict__ idx, int nbags, int L,
+                           float4 *out, int *counter) {
+    const int lane = threadIdx.x & 31;
+    while (true) {
+        int b = 0;
+        if (lane == 0) b = atomicAdd(counter, 1);
+        b = __shfl_sync(0xffffffffu, b, 0);
+        if (b >= nbags) break;
+        float4 acc = make_float4(0, 0, 0, 0);
+        const int lo = b * L, hi = lo + L;
+        for (int j = lo; j < hi; j += U) {
+            float4 v[U];
+            int id[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u) id[u] = __ldg(idx + j + u);
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                const float4 *p = table + (long long)id[u] * 32 + lane;
+                asm volatile("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
+                             : "=f"(v[u].x), "=f"(v[u].y), "=f"(v[u].z), "=f"(v[u].w) : "l"(p));
+            }
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                acc.x += v[u].x; acc.y += v[u].y; acc.z += v[u].z; acc.w += v[u].w;
+            }
+        }
+        out[(long long)b * 32 + lane] = acc;
+    }
+}
+
+template <int U>
+void run_bags(const float4 *table, const int *idx, long long n, int L, float4 *out, int *counter, int ctas, int sms) {
+    cudaEvent_t a, b;
+    cudaEventCreate(&a);
+    cudaEventCreate(&b);
+    const int nbags = (int)(n / L);
+    float best = 1e9;
+    for (int r = 0; r < 6; ++r) {
+        cudaMemset(counter, 0, 4);
+        cudaEventRecord(a);
+        probe_bags<U><<<sms * ctas, 256>>>(table, idx, nbags, L, out, counter);
+        cudaEventRecord(b);
+        CK(cudaEventSynchronize(b));
+        float ms;
+        cudaEventElapsedTime(&ms, a, b);
+        if (r && ms < best) best = ms;
+    }
+    double bytes = (double)nbags * L * 516 + (double)nbags * 512;
+    printf("bags L=%4d U=%d ctas/SM=%d : %8.3f ms  %7.0f GB/s (rows+idx+out)\n", L, U, ctas, best, bytes / best / 1e6);
+}
+
 template <int G, int U>
 void run(const float4 *table, long long table_rows, const int *idx, long long n, float *out, int ctas_per_sm, int sms) {
     cudaEvent_t a, b;
@@ -68,14 +122,17 @@ __global__ void init_idx(int *idx, long long n, long long rows, unsigned long lo
         z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
         z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
         z ^= z >> 31;
-        idx[i] = (int)(z % (unsigned long long)rows);
+        idx[i] = (int)(z % (unsigned long long)(rows < 2147483647ll ? rows : 2147483647ll));
     }
 }
 
-int main() {
+int main(int argc, char **argv) {
     int sms;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
-    const long long table_bytes = 40ll << 30;  // 40 GiB table (>> L2)
+    const long long table_gib = argc > 1 ? atoll(argv[1]) : 40;
+    const int only512 = argc > 2 ? atoi(argv[2]) : 0;
+    const long long table_bytes = table_gib << 30;  // table (>> L2)
+    printf("table %lld GiB\n", table_gib);
     float4 *table;
     CK(cudaMalloc(&table, table_bytes));
     CK(cudaMemset(table, 0, table_bytes));
@@ -96,8 +153,26 @@ int main() {
         run<G, 8>(table, rows, idx, n, out, ctas, sms);
         cudaFree(idx);
     };
-    for (int ctas : {4, 8}) {
+    if (only512 == 2) {  // bag mode
+        long long rows = table_bytes / 512;
+        long long n = total_row_bytes / 512;
+        int *idx, *counter;
+        float4 *outb;
+        CK(cudaMalloc(&idx, n * 4));
+        CK(cudaMalloc(&counter, 4));
+        CK(cudaMalloc(&outb, (n / 1) * 16 * 32 / 50 + 4096));
+        init_idx<<<4096, 256>>>(idx, n, rows, 12345);
+        CK(cudaDeviceSynchronize());
+        for (int ctas : {4, 6})
+            for (int L : {100, 1000}) {
+                run_bags<2>(table, idx, n, L, outb, counter, ctas, sms);
+                run_bags<4>(table, idx, n, L, outb, counter, ctas, sms);
+            }
+        return 0;
+    }
+    for (int ctas : {4, 6, 8}) {
         go(std::integral_constant<int, 32>{}, ctas);
+        if (only512) continue;
         go(std::integral_constant<int, 16>{}, ctas);
         go(std::integral_constant<int, 8>{}, ctas);
         go(std::integral_constant<int, 4>{}, ctas);
