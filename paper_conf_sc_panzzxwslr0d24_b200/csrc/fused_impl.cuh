@@ -81,6 +81,20 @@ struct TaskSlot {
 
 __device__ __forceinline__ int vld(const int *p) { return *reinterpret_cast<const volatile int *>(p); }
 __device__ __forceinline__ void vst(int *p, int v) { *reinterpret_cast<volatile int *>(p) = v; }
+// Slot hand-off flags: release store by the filling / last-leaving warp,
+// acquire load by the waiting warps (CTA scope, shared memory).
+__device__ __forceinline__ int ld_acquire(const int *p) {
+    int v;
+    asm volatile("ld.acquire.cta.shared::cta.b32 %0, [%1];"
+                 : "=r"(v)
+                 : "r"((unsigned)__cvta_generic_to_shared(p))
+                 : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release(int *p, int v) {
+    asm volatile("st.release.cta.shared::cta.b32 [%0], %1;" ::"r"((unsigned)__cvta_generic_to_shared(p)), "r"(v)
+                 : "memory");
+}
 __device__ __forceinline__ unsigned long long vld64(const unsigned long long *p) {
     return *reinterpret_cast<const volatile unsigned long long *>(p);
 }
@@ -128,7 +142,7 @@ __global__ void __launch_bounds__(kBlockThreads, KOCC) recflex_fused_kernel(Fuse
         TaskSlot &S = ring[n % kRing];
         if (lane == 0) {
             while (true) {
-                const int st = vld(&S.state);
+                const int st = ld_acquire(&S.state);
                 if (st == 2) {
                     if (vld(&S.seq) == n) break;
                 } else if (st == 0 && atomicCAS(&S.state, 0, 1) == 0) {
@@ -170,8 +184,7 @@ __global__ void __launch_bounds__(kBlockThreads, KOCC) recflex_fused_kernel(Fuse
                         }
 #endif
                     }
-                    __threadfence_block();
-                    vst(&S.state, 2);
+                    st_release(&S.state, 2);
                     break;
                 }
                 __nanosleep(32);
@@ -201,8 +214,7 @@ __global__ void __launch_bounds__(kBlockThreads, KOCC) recflex_fused_kernel(Fuse
             if (atomicAdd(&S.left, 1) == kWarps - 1) {
                 if (a.timers && t < a.timers_cap) a.timers[t] = (long long)(vld64(&S.wtime) / kWarps);
                 S.seq = -1;
-                __threadfence_block();
-                vst(&S.state, 0);
+                st_release(&S.state, 0);
             }
         }
     }
