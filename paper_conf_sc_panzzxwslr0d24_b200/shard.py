@@ -90,6 +90,14 @@ def exchange(send, dims_per_rank: Sequence[int], B: int, group=None):
     rank = dist.get_rank(group)
     inp, out = split_sizes(B, W, dims_per_rank, rank)
     recv = torch.empty(sum(out), dtype=send.dtype, device=send.device)
+    if send.is_cuda and dist.get_backend(group) == 'gloo':
+        # test plumbing only (several ranks sharing one GPU, where NCCL refuses):
+        # gloo has no CUDA all-to-all, so the exchange is staged through host memory
+        r_cpu = torch.empty(sum(out), dtype=send.dtype)
+        dist.all_to_all_single(r_cpu, send.reshape(-1).cpu(), output_split_sizes=out, input_split_sizes=inp,
+                               group=group)
+        recv.copy_(r_cpu)
+        return recv
     dist.all_to_all_single(recv, send.reshape(-1), output_split_sizes=out, input_split_sizes=inp, group=group)
     return recv
 
