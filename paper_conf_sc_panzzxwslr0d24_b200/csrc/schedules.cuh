@@ -124,6 +124,76 @@ __device__ __forceinline__ void group_bag(const float *__restrict__ T, const int
 #pragma unroll
                 for (int e = 0; e < VEC; ++e) acc[c][e] = 0.f;
 
+#ifdef RECFLEX_FASTLOOP
+            if constexpr (U <= G && G >= 4 && C == 1) {
+                if ((p + 1) * SPAN <= d) {
+                    // EXPERIMENT, off by default (measured 16% SLOWER on heavy,
+                    // 7% on sharded1000): the row addresses of iteration i+1
+                    // (shuffle + one IMAD.WIDE each) are formed while the rows of
+                    // iteration i are in flight.  The shuffles issued behind the
+                    // outstanding row loads appear to complete in order behind
+                    // them, so nothing is gained and the loop gets longer.
+                    const int lane = threadIdx.x & 31;
+                    const unsigned gmask = (G == 32) ? 0xffffffffu : (((1u << G) - 1u) << (lane & ~(G - 1)));
+                    const char *base = reinterpret_cast<const char *>(T + colv[0]);
+                    const unsigned rowb = (unsigned)d * 4u;
+                    int cb = lo;
+                    int cur = (lo + lg < hi) ? ld_idx(idx + lo + lg) : 0;
+                    int nxt = (lo + G + lg < hi) ? ld_idx(idx + lo + G + lg) : 0;
+                    int j = lo;
+                    const float *pa[U];
+                    if (j + U <= hi) {
+#pragma unroll
+                        for (int u = 0; u < U; ++u)
+                            pa[u] = reinterpret_cast<const float *>(
+                                base + (size_t)(unsigned)__shfl_sync(gmask, cur, u, G) * rowb);
+                    }
+                    while (j + U <= hi) {
+                        float v[U][VEC];
+#pragma unroll
+                        for (int u = 0; u < U; ++u) ld_row<VEC>(pa[u], v[u]);
+                        const int jn = j + U;
+                        if (jn + U <= hi) {
+                            if (jn - cb >= G) {
+                                cb += G;
+                                cur = nxt;
+                                nxt = (cb + G + lg < hi) ? ld_idx(idx + cb + G + lg) : 0;
+                            }
+#pragma unroll
+                            for (int u = 0; u < U; ++u)
+                                pa[u] = reinterpret_cast<const float *>(
+                                    base + (size_t)(unsigned)__shfl_sync(gmask, cur, (jn - cb) + u, G) * rowb);
+                        }
+#pragma unroll
+                        for (int u = 0; u < U; ++u)
+#pragma unroll
+                            for (int e = 0; e < VEC; ++e) acc[0][e] += v[u][e];
+                        j = jn;
+                    }
+                    if (j < hi) {  // ragged tail: n < U rows
+                        if (j - cb >= G) {
+                            cb += G;
+                            cur = nxt;
+                        }
+                        const int n = hi - j;
+                        float v[U][VEC];
+#pragma unroll
+                        for (int u = 0; u < U; ++u) {
+                            const unsigned id = (unsigned)__shfl_sync(gmask, cur, (j - cb) + u, G);
+                            if (u < n) ld_row<VEC>(reinterpret_cast<const float *>(base + (size_t)id * rowb), v[u]);
+                        }
+#pragma unroll
+                        for (int u = 0; u < U; ++u)
+                            if (u < n)
+#pragma unroll
+                                for (int e = 0; e < VEC; ++e) acc[0][e] += v[u][e];
+                    }
+                    pool_finish<VEC>(acc[0], pool, hi - lo);
+                    st_out<VEC>(orow + colv[0], acc[0]);
+                    continue;
+                }
+            }
+#endif
 #ifndef RECFLEX_NO_SHFL_IDX
             if constexpr (U <= G && G >= 4) {
                 // Lookup IDs through registers: lane lg holds ID cb+lg of the
