@@ -86,7 +86,9 @@ typedef struct {
 typedef enum {
     RECFLEX_FAMILY_GROUP = 0, /* G lanes per bag; 256/G bags in flight per CTA (G=32: warp per sample) */
     RECFLEX_FAMILY_BLOCK = 1, /* all 256 threads on one bag; smem partials + fixed-order reduction    */
-    RECFLEX_FAMILY_FLAT = 2   /* G lanes walk a run of 8 consecutive bags as one lookup range       */
+    RECFLEX_FAMILY_FLAT = 2,  /* G lanes walk a run of 8 consecutive bags as one lookup range       */
+    RECFLEX_FAMILY_BULK = 3   /* warp per run of bags; rows by TMA bulk copies into smem stages
+                                 (only in experimental builds; not in the default catalog)         */
 } recflex_family_t;
 
 typedef struct {

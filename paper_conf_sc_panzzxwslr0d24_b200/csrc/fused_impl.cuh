@@ -32,6 +32,9 @@ __device__ __forceinline__ void dispatch_schedule(int id, const TaskCtx &x, floa
             else if constexpr (e.family == RECFLEX_FAMILY_FLAT)
                 sched_flat<e.G, e.VEC, e.U>(x.table, x.offs, x.idx, x.out, x.dim, x.pool, x.out_stride, x.s0, x.s1,
                                             bag_ctr);
+            else if constexpr (e.family == RECFLEX_FAMILY_BULK)
+                sched_bulk<e.U>(x.table, x.offs, x.idx, x.out, x.dim, x.pool, x.out_stride, x.s0, x.s1, bag_ctr,
+                                x.wsmem, x.wbytes);
             else
                 sched_block<e.G, e.VEC, e.C, e.U>(x.table, x.offs, x.idx, x.out, x.dim, x.pool, x.out_stride, x.s0,
                                                   x.s1, red);
@@ -44,8 +47,11 @@ __device__ __forceinline__ void dispatch_schedule(int id, const TaskCtx &x, floa
 // Single call site for the whole catalog: the kernel calls this once per task
 // (few live values cross the call), and it branches to the schedule.
 static __device__ __noinline__ void dispatch_task(int id, const float *T, const int32_t *offs, const int32_t *idx, float *out,
-                                           int d, int pool, int out_stride, int s0, int s1, float *red, int *bag) {
+                                           int d, int pool, int out_stride, int s0, int s1, float *red, int *bag,
+                                           unsigned char *wsmem, int wbytes) {
     TaskCtx x;
+    x.wsmem = wsmem;
+    x.wbytes = wbytes;
     x.table = T;
     x.offs = offs;
     x.idx = idx;
@@ -119,6 +125,11 @@ __global__ void __launch_bounds__(kBlockThreads, KOCC) recflex_fused_kernel(Fuse
     const int lane = tid & 31;
     const int F = a.F;
     const bool bs_in_smem = (F + 1) <= kSmemBlockStartCap;
+    // BULK-family stage slices: whatever dynamic smem the occupancy padding
+    // leaves after the reduction scratch and the block_start cache, split 8 ways
+    const int bulk_off = (kRedFloats * 4 + (bs_in_smem ? 4 * (F + 1) : 0) + 127) & ~127;
+    const int wbytes = ((a.smem_bytes - bulk_off) / kWarps) & ~127;
+    unsigned char *wsmem = dyn_smem + bulk_off + (tid >> 5) * (wbytes > 0 ? wbytes : 0);
 
     // PDL: everything above overlapped the map kernel; wait for its results.
     asm volatile("griddepcontrol.wait;" ::: "memory");
@@ -205,7 +216,7 @@ __global__ void __launch_bounds__(kBlockThreads, KOCC) recflex_fused_kernel(Fuse
         const bool cta_wide = kFamilyDev[fd.sched] == RECFLEX_FAMILY_BLOCK;
         if (cta_wide) __syncthreads();  // every warp reaches task n (they walk the same sequence)
         dispatch_task(fd.sched, fd.table, a.offsets + (size_t)fd.in_feature * a.B, a.indices, a.out + fd.col, fd.dim,
-                      fd.pool, a.out_stride, vld(&S.s0), vld(&S.s1), red, &S.bag);
+                      fd.pool, a.out_stride, vld(&S.s0), vld(&S.s1), red, &S.bag, wsmem, wbytes);
         if (cta_wide) __syncthreads();
         __syncwarp();
         if (lane == 0) {

@@ -52,7 +52,9 @@ int find_catalog(int family, int G, int VEC, int C, int U) {
 int samples_per_task_default(int sched_id, float mean_len, float coverage, int target) {
     const CatalogEntry &e = kCatalog[sched_id];
     const int slots = (e.family == RECFLEX_FAMILY_GROUP) ? kBlockThreads / e.G
-                      : (e.family == RECFLEX_FAMILY_FLAT) ? (kBlockThreads / e.G) * 8 : 1;
+                      : (e.family == RECFLEX_FAMILY_FLAT || e.family == RECFLEX_FAMILY_BULK)
+                          ? (kBlockThreads / e.G) * 8
+                          : 1;
     double el = std::max(0.25, (double)mean_len * std::max(0.05, (double)coverage));
     int R = (int)std::lround((double)target / (slots * el));
     R = std::min(32, std::max(1, R));
@@ -220,6 +222,7 @@ recflex_status_t run_pipeline(recflex_plan_s *p, const Exec &ex, const int32_t *
     a.F = ex.F;
     a.B = B;
     a.out_stride = out_stride;
+    a.smem_bytes = p->smem[k];
     LaunchCfg cfg;
     cfg.grid = p->num_sms * p->occ[k];
     cfg.smem = p->smem[k];

@@ -64,6 +64,7 @@ struct FusedArgs {
     int32_t B;
     int32_t out_stride;           // D_tot
     int32_t timers_cap;
+    int32_t smem_bytes;           // dynamic shared memory of the launch (BULK stages live in it)
 };
 
 // ---------------------------------------------------------------------------
@@ -107,7 +108,17 @@ struct FusedArgs {
     /* FLAT, 256-bit rows */                                                    \
     X(2, 1, 8, 1, 2) X(2, 1, 8, 1, 4) X(2, 2, 8, 1, 2) X(2, 2, 8, 1, 4)         \
     X(2, 4, 8, 1, 2) X(2, 4, 8, 1, 4) X(2, 8, 8, 1, 2) X(2, 8, 8, 1, 4)         \
-    X(2, 16, 8, 1, 2) X(2, 16, 8, 1, 4)
+    X(2, 16, 8, 1, 2) X(2, 16, 8, 1, 4) RECFLEX_CATALOG_EXPERIMENTAL(X)
+
+// BULK (rows by TMA bulk copy into smem stages) is built only on request:
+// per-row cp.async.bulk of random rows from multi-GB tables measured 10-100x
+// slower than register loads on B200 (the copy engine's address translation
+// thrashes), see DESIGN.md §6.
+#ifdef RECFLEX_EXPERIMENTAL_BULK
+#define RECFLEX_CATALOG_EXPERIMENTAL(X) X(3, 32, 4, 1, 2) X(3, 32, 4, 1, 4) X(3, 32, 4, 1, 8)
+#else
+#define RECFLEX_CATALOG_EXPERIMENTAL(X)
+#endif
 
 struct CatalogEntry {
     int family, G, VEC, C, U;
@@ -125,6 +136,7 @@ inline bool catalog_valid(const CatalogEntry &e, int d) {
     if (d % e.VEC != 0) return false;
     int span = e.G * e.VEC * e.C;
     if (4 * d < span) return false;
+    if (e.family == 3 && (d < 32 || d > 128)) return false;  // BULK: 128..512-byte rows, one pass
     return true;
 }
 

@@ -410,7 +410,8 @@ struct Tuner {
                 const long key = hist[i].first;
                 const int sid = (int)(key / 100000 / 2), part = (int)(key / 100000 % 2);
                 const CatalogEntry &e = kCatalog[sid];
-                std::fprintf(stderr, " %dx[%s G%d V%d C%d U%d p%d/%ld]", hist[i].second, e.family == 2 ? "flat" : (e.family ? "block" : "group"),
+                std::fprintf(stderr, " %dx[%s G%d V%d C%d U%d p%d/%ld]", hist[i].second,
+                             e.family == 3 ? "bulk" : (e.family == 2 ? "flat" : (e.family ? "block" : "group")),
                              e.G, e.VEC, e.C, e.U, part, key % 100000);
             }
             std::fprintf(stderr, "\n");
@@ -450,7 +451,7 @@ std::vector<recflex_schedule_t> candidates_for(const recflex_plan_s *p, int f, i
             if (relax == 0 && (passes > 1 || e.C > 1)) continue;
             if (relax == 1 && passes > 2) continue;
             if (e.VEC == 1 && d.dim % 4 == 0) continue;  // scalar only where vectors cannot run
-            if (!multi_hot && e.family == RECFLEX_FAMILY_BLOCK) continue;
+            if (!multi_hot && (e.family == RECFLEX_FAMILY_BLOCK || e.family == RECFLEX_FAMILY_BULK)) continue;
             if (!multi_hot && e.family == RECFLEX_FAMILY_GROUP && e.U > 2) continue;  // one bag = one row
             add(s);
             if (multi_hot && e.family != RECFLEX_FAMILY_BLOCK) add({id, 1, std::max(128, p->task_lookups)});
