@@ -75,11 +75,14 @@ typedef struct {
 /* A feature's schedule: catalog entry + its runtime thread-mapping parameters
  * ("tunable parameters").  part 0: a task (CTA work unit) covers
  * per_block consecutive samples; part 1: a task covers the bags whose first
- * lookup falls in a window of per_block lookups (adaptive to the batch). */
+ * lookup falls in a window of per_block lookups (adaptive to the batch);
+ * part 2: STATIC mapping -- exactly per_block tasks whatever the batch, each
+ * covering ceil(B/per_block) samples (the paper's ablation straw man, P:81,
+ * P:328-338; for experiments, never chosen by the tuner). */
 typedef struct {
     int32_t sched_id;  /* index into the catalog (recflex_catalog_info)         */
-    int32_t part;      /* 0 = sample-partitioned, 1 = lookup(nnz)-partitioned    */
-    int32_t per_block; /* samples per task (part 0) or lookups per task (part 1) */
+    int32_t part;      /* 0 sample-, 1 lookup(nnz)-partitioned, 2 static         */
+    int32_t per_block; /* samples per task (0), lookups per task (1), tasks (2)  */
 } recflex_schedule_t;
 
 /* Catalog entry description (hand-written sm_100a schedule templates). */

@@ -123,6 +123,8 @@ def task_map(B, mode, per_block, offsets, cap=None):
     for f in range(F):
         if mode[f] == 0:
             ub += (B + pb[f] - 1) // pb[f]
+        elif mode[f] == 2:
+            ub += int(pb[f])
         else:
             ub += (int(off[(f + 1) * B]) - int(off[f * B])) // pb[f] + 1
     ub = max(ub, 1)

@@ -127,6 +127,7 @@ int oracle_embedding_bag(int F, int B, const int *dims, const int *pools,
  * Task map of Fig. 8.
  *   mode[f]: 0 = sample-partitioned (per_block[f] = samples per block)
  *            1 = nnz-partitioned    (per_block[f] = lookups per block)
+ *            2 = static             (per_block[f] = fixed block count)
  *   cap[f]:  0 = none, else feature_blocks = min(feature_blocks, cap[f])
  * Outputs blocks_map[F] (d_blocks_map), task_feature/task_rel[max_tasks]
  * (d_task_map .x/.y), *num_tasks.  Returns ORACLE_ERR_ARG if max_tasks is short.
@@ -139,6 +140,10 @@ int oracle_task_map(int F, int B, const int *mode, const int *per_block, const i
         int64_t blocks;
         if (mode[f] == 0) {
             blocks = ((int64_t)B + per_block[f] - 1) / per_block[f];
+        } else if (mode[f] == 2) {
+            /* static thread mapping (P:328-338 ablation): a fixed block count */
+            blocks = per_block[f];
+            if (B == 0) blocks = 0;
         } else {
             int64_t nnz_f = (int64_t)offsets[(int64_t)(f + 1) * B] - offsets[(int64_t)f * B];
             blocks = nnz_f / per_block[f] + 1;

@@ -171,6 +171,10 @@ __global__ void __launch_bounds__(kBlockThreads, KOCC) recflex_fused_kernel(Fuse
                         if (fd.part == 0) {
                             s0 = rel * fd.per_block;
                             s1 = min(a.B, s0 + fd.per_block);
+                        } else if (fd.part == 2) {
+                            const int per = (a.B + fd.per_block - 1) / fd.per_block;
+                            s0 = min(a.B, rel * per);
+                            s1 = min(a.B, s0 + per);
                         } else {
                             const int32_t *ts = a.task_start + fd.slot_base;
                             s0 = ts[rel];

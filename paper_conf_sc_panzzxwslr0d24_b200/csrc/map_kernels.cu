@@ -105,6 +105,10 @@ __global__ void __launch_bounds__(kMapThreads) recflex_map_kernel(MapArgs a) {
             const FeatureDesc &fd = a.desc[f];
             if (fd.part == 0) {
                 blocks = (a.B + fd.per_block - 1) / fd.per_block;
+            } else if (fd.part == 2) {
+                // static mapping (paper's ablation straw man): a fixed
+                // number of blocks whatever the batch; each takes ceil(B/blocks)
+                blocks = fd.per_block;
             } else {
                 const int64_t fi = fd.in_feature;
                 const int nnz = a.offsets[(fi + 1) * a.B] - a.offsets[fi * a.B];

@@ -108,7 +108,7 @@ int slots_for(int max_batch, float max_len) {
 
 bool schedule_valid_for(const recflex_schedule_t &s, int dim, int col, int d_tot) {
     if (s.sched_id < 0 || s.sched_id >= kCatalogSize) return false;
-    if (s.part != 0 && s.part != 1) return false;
+    if (s.part < 0 || s.part > 2) return false;
     if (s.per_block < 1) return false;
     const CatalogEntry &e = kCatalog[s.sched_id];
     if (!catalog_valid(e, dim)) return false;

@@ -112,6 +112,8 @@ int64_t task_count(const FeatureDesc &d, int B, int64_t nnz) {
     if (B == 0) return 0;
     if (d.part == 0) {
         blocks = (B + d.per_block - 1) / d.per_block;
+    } else if (d.part == 2) {
+        blocks = d.per_block;
     } else {
         int64_t npb = d.per_block;
         const int64_t room = d.slots - 2;

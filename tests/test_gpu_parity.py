@@ -141,7 +141,7 @@ def _mixed_model():
     return synth.custom_model('mixed', feats, 301)
 
 
-@pytest.mark.parametrize('part', [0, 1])
+@pytest.mark.parametrize('part', [0, 1, 2])
 def test_every_catalog_entry_int_bitexact(part):
     P = _plan_mod()
     m = _mixed_model()
@@ -153,7 +153,7 @@ def test_every_catalog_entry_int_bitexact(part):
     col = np.cumsum([0] + m.dims)
     tested = 0
     for e in cat:
-        for per_block in ((7, 64) if part == 0 else (5, 300)):
+        for per_block in {0: (7, 64), 1: (5, 300), 2: (3, 17)}[part]:
             used = []
             for f, feat in enumerate(m.features):
                 try:
@@ -206,11 +206,15 @@ def test_task_map_bitexact_vs_oracle(seed):
     mode, pb = [], []
     for f, feat in enumerate(m.features):
         s = plan.get_schedule(f)
-        if rng.random() < 0.5:
+        r = rng.random()
+        if r < 0.4:
             s['part'] = 1
             # >= 128 lookups per task: within the plan's reserved task slots
             # (max_batch * max_len / 128), so the map never raises npb (C12)
             s['per_block'] = int(rng.integers(128, 700))
+        elif r < 0.6:
+            s['part'] = 2  # static mapping: fixed task count
+            s['per_block'] = int(rng.integers(1, 40))
         else:
             s['part'] = 0
             s['per_block'] = int(rng.integers(1, 300))

@@ -251,6 +251,8 @@ def _brute_task_map(B, mode, pb, off, cap):
     for f in range(F):
         if mode[f] == 0:
             n = -(-B // pb[f])
+        elif mode[f] == 2:  # static mapping: fixed block count
+            n = pb[f]
         else:
             nnz = int(off[(f + 1) * B]) - int(off[f * B])
             n = nnz // pb[f] + 1
@@ -267,7 +269,7 @@ def test_task_map_vs_brute_force(seed):
     F, B = int(rng.integers(1, 9)), int(rng.integers(1, 70))
     lens = rng.integers(0, 30, size=(F, B))
     b = synth.batch_from_lengths(lens, [100] * F, seed=seed)
-    mode = rng.integers(0, 2, size=F).tolist()
+    mode = rng.integers(0, 3, size=F).tolist()
     pb = [int(rng.integers(1, 40)) for _ in range(F)]
     cap = [int(rng.integers(0, 4)) if rng.random() < 0.3 else 0 for _ in range(F)]
     blocks, tf, tr = oracle.task_map(B, mode, pb, b.offsets, cap)
