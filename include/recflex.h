@@ -156,6 +156,10 @@ typedef struct {
     int32_t skip_refine;     /* 0: after selection, try every candidate per cluster of
                                 same-dim / same-length-class features in the real fused
                                 forward at the chosen k; keep if > 0.5% faster     */
+    int32_t local_mode;      /* 0: interference-simulated co-execution with padding (the
+                                paper's method); 1: separate-combine straw man -- each
+                                candidate timed alone in a non-padded launch (P:73, P:324,
+                                for the Fig. 11 ablation)                                   */
 } recflex_tune_options_t;
 
 typedef struct {

@@ -36,7 +36,8 @@ class CatalogInfo(ctypes.Structure):
 class TuneOptions(ctypes.Structure):
     _fields_ = [('num_occupancies', ctypes.c_int32), ('occupancies', ctypes.c_int32 * 8),
                 ('reps', ctypes.c_int32), ('pad_waves', ctypes.c_int32), ('max_candidates', ctypes.c_int32),
-                ('verbose', ctypes.c_int32), ('skip_guard', ctypes.c_int32), ('skip_refine', ctypes.c_int32)]
+                ('verbose', ctypes.c_int32), ('skip_guard', ctypes.c_int32), ('skip_refine', ctypes.c_int32),
+                ('local_mode', ctypes.c_int32)]
 
 
 class TuneStats(ctypes.Structure):

@@ -132,6 +132,7 @@ struct Tuner {
     std::vector<int> ks;
     int reps = 7;
     int pad_waves = 4;
+    bool separate = false;  // local_mode 1: separate-combine straw man (ablation)
     int verbose = 0;
     std::vector<std::vector<recflex_schedule_t>> cands;  // per feature
     recflex_status_t err = RECFLEX_OK;
@@ -226,10 +227,79 @@ struct Tuner {
     }
 
     // Eq. 3 costs of all candidates of f at occupancy ks[ki], summed over batches.
+    // Straw man 1 of the paper (ablation P:324 / Fig. 11): every
+    // candidate in its OWN non-padded launch, cost = its measured latency.
+    void local_cost_separate(int ki, int f, double *costs) {
+        const int k = ks[ki];
+        const int n = (int)cands[f].size();
+        const FeatureDesc &base = p->desc[f];
+        for (int c = 0; c < n; ++c) costs[c] = 0;
+        for (size_t i = 0; i < batches.size(); ++i) {
+            const Batch &bt = batches[i];
+            TP &tp = tps[i];
+            const int B = bt.B;
+            for (int c = 0; c < n; ++c) {
+                FeatureDesc d = base;
+                d.sched = cands[f][c].sched_id;
+                d.part = cands[f][c].part;
+                d.per_block = cands[f][c].per_block;
+                d.cap = 0;
+                d.in_feature = c;
+                d.col = 0;
+                d.slot_base = 0;
+                if (d.part == 1) d.slots = (int32_t)(bt.nnz(f) / d.per_block + 3);
+                d.table = p->tables[f];
+                const int32_t p1 = 0;
+                check(d_desc.ensure(1));
+                check(d_bs.ensure(2));
+                check(d_npb.ensure(1));
+                check(d_counter.ensure(4));
+                check(d_ts.ensure(std::max<int64_t>(d.part == 1 ? d.slots : 1, 1)));
+                check(d_part1.ensure(1));
+                check(d_out.ensure((int64_t)B * ((base.dim + 3) / 4 * 4)));
+                if (err) return;
+                check(cudaMemcpyAsync(d_desc.p, &d, sizeof(FeatureDesc), cudaMemcpyHostToDevice, stream));
+                check(cudaMemcpyAsync(d_part1.p, &p1, sizeof(int32_t), cudaMemcpyHostToDevice, stream));
+                Exec ex;
+                ex.F = 1;
+                ex.in_F = tp.in_F;
+                ex.d_desc = d_desc.p;
+                ex.d_block_start = d_bs.p;
+                ex.d_npb_eff = d_npb.p;
+                ex.d_counter = d_counter.p;
+                ex.d_task_start = d_ts.p;
+                ex.d_part1 = d_part1.p;
+                ex.num_part1 = d.part == 1 ? 1 : 0;
+                std::vector<float> ms;
+                for (int r = 0; r < 4; ++r) {
+                    check(cudaEventRecord(e0, stream));
+                    recflex_status_t st = run_pipeline(p, ex, tp.idx.p, tp.off.p, B, d_out.p,
+                                                       (base.dim + 3) / 4 * 4, k, stream, nullptr);
+                    if (st != RECFLEX_OK) {
+                        fail(st);
+                        return;
+                    }
+                    check(cudaEventRecord(e1, stream));
+                    check(cudaEventSynchronize(e1));
+                    float t = 0;
+                    cudaEventElapsedTime(&t, e0, e1);
+                    if (r) ms.push_back(t);
+                    ++local_launches;
+                }
+                std::sort(ms.begin(), ms.end());
+                costs[c] += ms[ms.size() / 2];
+            }
+        }
+    }
+
     void local_cost(int ki, int f, double *costs) {
         if (err) return;
         if (cur_f != f) build_inputs(f);
         if (err) return;
+        if (separate) {
+            local_cost_separate(ki, f, costs);
+            return;
+        }
         const int k = ks[ki];
         const int n = (int)cands[f].size();
         std::vector<double> sum(n, 0.0);
@@ -489,6 +559,7 @@ extern "C" recflex_status_t recflex_tune_ex(recflex_plan_t p, int32_t N, const i
     if (opt && opt->reps > 0) T.reps = opt->reps;
     if (opt && opt->pad_waves > 0) T.pad_waves = opt->pad_waves;
     if (opt) T.verbose = opt->verbose;
+    if (opt) T.separate = opt->local_mode == 1;
     const int max_c = opt ? opt->max_candidates : 0;
     for (int i = 0; i < N; ++i) {
         if (batch_sizes[i] <= 0 || batch_sizes[i] > p->max_batch || !indices[i] || !offsets[i])

@@ -146,7 +146,7 @@ class Plan:
     # -------------------------------------------------------------- tuner
     def tune(self, batches: Sequence[tuple], tables: Sequence[torch.Tensor], occupancies: Optional[List[int]] = None,
              reps: int = 7, pad_waves: int = 4, max_candidates: int = 0, verbose: bool = False, guard: bool = True,
-             refine: bool = True, stream=None) -> dict:
+             refine: bool = True, separate: bool = False, stream=None) -> dict:
         """recflex_tune_ex over historical batches [(indices, offsets, B), ...]."""
         N = len(batches)
         idx_arr = (ctypes.c_void_p * N)(*[b[0].data_ptr() for b in batches])
@@ -163,6 +163,7 @@ class Plan:
         opt.verbose = 1 if verbose else 0
         opt.skip_guard = 0 if guard else 1
         opt.skip_refine = 0 if refine else 1
+        opt.local_mode = 1 if separate else 0
         st = _lib.TuneStats()
         check(lib.recflex_tune_ex(self._h, N, idx_arr, off_arr, bs_arr, self._tables(tables), _stream_ptr(stream),
                                   ctypes.byref(opt), ctypes.byref(st)), 'recflex_tune_ex')

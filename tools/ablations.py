@@ -142,15 +142,49 @@ def ablation_swap(config, lines, nfeat=3, seed=0):
     lines.append('')
 
 
+def ablation_tuning(config, lines, ks=(4,)):
+    """Fig. 11 / P:324: two-stage interference-simulated tuning vs the
+    separate-combine straw man (each candidate timed alone, non-padded)."""
+    import time
+    from paper_conf_sc_panzzxwslr0d24_b200 import synth
+    from paper_conf_sc_panzzxwslr0d24_b200.plan import Plan
+    m, tables, out, flush = setup(config, synth.make_model(config).batch)
+    hist = [synth.make_batch(m, 7 + i) for i in range(2)]
+    hist_dev = [(*dev_batch(b), m.batch) for b in hist]
+    test = dev_batch(synth.make_batch(m, 50))
+    rows = []
+    for label, kw in (('default heuristic (untuned)', None),
+                      ('separate-combine (straw man 1)', dict(separate=True, guard=False, refine=False)),
+                      ('two-stage co-execution (paper)', dict(separate=False, guard=False, refine=False)),
+                      ('two-stage + guard + cluster refinement (ours)', dict(separate=False, guard=True, refine=True))):
+        plan = Plan.from_model(m)
+        plan.occupancy = ks[0]
+        t0 = time.time()
+        st = plan.tune(hist_dev, tables, occupancies=list(ks), reps=5, **kw) if kw is not None else {}
+        tt = time.time() - t0
+        ms = timer(plan, test, m.batch, tables, out, flush)
+        rows.append((label, ms, tt, st.get('local_launches', 0)))
+        print(label, ms, tt, flush=True)
+    base = rows[0][1]
+    lines += [f'## Tuning strategies ({config}, k in {list(ks)}; Fig. 11 / P:324)', '',
+              'Each plan is tuned on 2 historical batches and timed on a held-out batch (median of 7, L2 flushed).',
+              '', '| tuner | fused forward (ms) | vs untuned | tuning time (s) | local launches |', '|---|---|---|---|---|']
+    for label, ms, tt, ll in rows:
+        lines.append(f'| {label} | {ms:.3f} | {base / ms:.2f}x | {tt:.0f} | {ll} |')
+    lines.append('')
+
+
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument('which', choices=['mapping', 'swap'])
+    ap.add_argument('which', choices=['mapping', 'swap', 'tuning'])
     ap.add_argument('--config', default='industrial')
     ap.add_argument('--out', default='')
     a = ap.parse_args()
     lines = []
     if a.which == 'mapping':
         ablation_mapping(a.config, lines)
+    elif a.which == 'tuning':
+        ablation_tuning(a.config, lines)
     else:
         ablation_swap(a.config, lines)
     out = a.out or os.path.join(ROOT, 'gpurun_out', f'ablation_{a.which}_{a.config}.md')
