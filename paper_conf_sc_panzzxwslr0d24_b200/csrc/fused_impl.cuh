@@ -115,6 +115,52 @@ __device__ __forceinline__ int find_feature(const int *bs, int F, int t) {
     return lo;
 }
 
+// Claim the next task from the device counter and decode it into slot S
+// (called by one lane that won the slot's 0 -> 1 CAS); publishes with a
+// release store of state = 2.
+__device__ __forceinline__ void fill_slot(TaskSlot &S, int n, const FusedArgs &a, const int *bs, int F, int total) {
+    const int t = atomicAdd(a.counter, 1);
+    S.t = t;
+    S.seq = n;
+    S.bag = 0;
+    S.left = 0;
+    S.wtime = 0;
+    if (t < total) {
+        const int f = find_feature(bs, F, t);
+        const int rel = t - bs[f];
+        const FeatureDesc &fd = a.desc[f];
+        int s0, s1;
+        if (fd.part == 0) {
+            s0 = rel * fd.per_block;
+            s1 = min(a.B, s0 + fd.per_block);
+        } else if (fd.part == 2) {
+            const int per = (a.B + fd.per_block - 1) / fd.per_block;
+            s0 = min(a.B, rel * per);
+            s1 = min(a.B, s0 + per);
+        } else {
+            const int32_t *ts = a.task_start + fd.slot_base;
+            s0 = ts[rel];
+            s1 = ts[rel + 1];
+        }
+        S.f = f;
+        S.s0 = s0;
+        S.s1 = s1;
+#ifndef RECFLEX_NO_L2PF
+        if (s1 > s0) {
+            // stage the task's contiguous lookup-ID range into L2 with one bulk
+            // prefetch (TMA engine)
+            const int32_t *offs = a.offsets + (size_t)fd.in_feature * a.B;
+            const int32_t j0 = __ldg(offs + s0), j1 = __ldg(offs + s1);
+            const uintptr_t b = reinterpret_cast<uintptr_t>(a.indices + j0) & ~uintptr_t(15);
+            const uintptr_t e = (reinterpret_cast<uintptr_t>(a.indices + j1) + 15) & ~uintptr_t(15);
+            if (e > b)
+                asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(b), "r"((unsigned)(e - b)) : "memory");
+        }
+#endif
+    }
+    st_release(&S.state, 2);
+}
+
 template <int KOCC>
 __global__ void __launch_bounds__(kBlockThreads, KOCC) recflex_fused_kernel(FusedArgs a) {
     extern __shared__ __align__(16) unsigned char dyn_smem[];
@@ -157,53 +203,18 @@ __global__ void __launch_bounds__(kBlockThreads, KOCC) recflex_fused_kernel(Fuse
                 if (st == 2) {
                     if (vld(&S.seq) == n) break;
                 } else if (st == 0 && atomicCAS(&S.state, 0, 1) == 0) {
-                    const int t = atomicAdd(a.counter, 1);
-                    S.t = t;
-                    S.seq = n;
-                    S.bag = 0;
-                    S.left = 0;
-                    S.wtime = 0;
-                    if (t < total) {
-                        const int f = find_feature(bs, F, t);
-                        const int rel = t - bs[f];
-                        const FeatureDesc &fd = a.desc[f];
-                        int s0, s1;
-                        if (fd.part == 0) {
-                            s0 = rel * fd.per_block;
-                            s1 = min(a.B, s0 + fd.per_block);
-                        } else if (fd.part == 2) {
-                            const int per = (a.B + fd.per_block - 1) / fd.per_block;
-                            s0 = min(a.B, rel * per);
-                            s1 = min(a.B, s0 + per);
-                        } else {
-                            const int32_t *ts = a.task_start + fd.slot_base;
-                            s0 = ts[rel];
-                            s1 = ts[rel + 1];
-                        }
-                        S.f = f;
-                        S.s0 = s0;
-                        S.s1 = s1;
-
-#ifndef RECFLEX_NO_L2PF
-                        if (s1 > s0) {
-                            // stage the task's contiguous lookup-ID range into L2
-                            // with one bulk prefetch (TMA engine)
-                            const int32_t *offs = a.offsets + (size_t)fd.in_feature * a.B;
-                            const int32_t j0 = __ldg(offs + s0), j1 = __ldg(offs + s1);
-                            const uintptr_t b = reinterpret_cast<uintptr_t>(a.indices + j0) & ~uintptr_t(15);
-                            const uintptr_t e = (reinterpret_cast<uintptr_t>(a.indices + j1) + 15) & ~uintptr_t(15);
-                            if (e > b)
-                                asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(b),
-                                             "r"((unsigned)(e - b))
-                                             : "memory");
-                        }
-#endif
-                    }
-                    st_release(&S.state, 2);
+                    fill_slot(S, n, a, bs, F, total);
                     break;
                 }
                 __nanosleep(32);
             }
+#ifdef RECFLEX_FILL_AHEAD
+            // EXPERIMENT, off by default (heavy unchanged, sharded1000 9% slower):
+            // claim and decode task n+1 now, so the warps that reach it later
+            // find it ready instead of waiting on its fill
+            TaskSlot &N = ring[(n + 1) % kRing];
+            if (ld_acquire(&N.state) == 0 && atomicCAS(&N.state, 0, 1) == 0) fill_slot(N, n + 1, a, bs, F, total);
+#endif
         }
         __syncwarp();
         __threadfence_block();
