@@ -253,6 +253,32 @@ recflex_status_t recflex_set_profiling(recflex_plan_t plan, int32_t enable);
 recflex_status_t recflex_get_kernel_times(recflex_plan_t plan, double *map_ms, double *fused_ms,
                                           int64_t *forwards, int32_t reset);
 
+/* ---- fused pooled-output exchange ------------------------ */
+
+/* recflex_forward with the table-wise all-to-all folded into the fused
+ * kernel's store epilogue: the pooled row of sample s (of this plan's
+ * features) is written straight into destination j = s / rows_per_dst,
+ * buffer host_dst[j] (a DEVICE pointer valid on this plan's device: local,
+ * NVLink peer-enabled, or CUDA-IPC mapped), at row s - j*rows_per_dst and
+ * columns [col_base + col_f, col_base + col_f + d_f) of a [rows][dst_stride]
+ * float32 layout.  Requires B == num_dst * rows_per_dst, 16-byte aligned
+ * buffers, col_base and dst_stride multiples of 4, col_base + D_tot <= stride.
+ * Async on `stream`; the caller orders the destination's reads after every
+ * writer's kernel (e.g. a collective barrier on the same streams). */
+recflex_status_t recflex_forward_routed(recflex_plan_t plan, const int32_t *indices, const int32_t *offsets,
+                                        int32_t batch_size, const float *const *tables, float *const *host_dst,
+                                        int32_t num_dst, int32_t rows_per_dst, int32_t dst_stride,
+                                        int32_t col_base, void *stream);
+
+/* CUDA IPC helpers for the routed forward across processes: 64-byte handle of
+ * a device allocation, map a peer process's handle, unmap. */
+recflex_status_t recflex_ipc_get_handle(const void *d_ptr, void *handle64);
+recflex_status_t recflex_ipc_open_handle(const void *handle64, void **d_ptr);
+recflex_status_t recflex_ipc_close(void *d_ptr);
+/* Own cudaMalloc allocation (so its IPC handle maps at offset 0) / free. */
+recflex_status_t recflex_device_alloc(size_t bytes, int32_t device, void **d_ptr);
+recflex_status_t recflex_device_free(void *d_ptr);
+
 /* ---- multi-GPU exchange helper ------------------------------------------- */
 
 /* Relayout after the table-wise pooled-output all-to-all:

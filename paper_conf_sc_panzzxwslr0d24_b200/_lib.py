@@ -85,6 +85,13 @@ SIGNATURES = {
     'recflex_get_kernel_times': (c_int32, [c_void_p, P(ctypes.c_double), P(ctypes.c_double), P(c_int64), c_int32]),
     'recflex_shard_concat': (c_int32, [c_void_p, c_int32, c_int32, P(c_int32), c_void_p, c_void_p]),
     'recflex_l2_flush': (c_int32, [c_void_p, ctypes.c_size_t, c_void_p]),
+    'recflex_forward_routed': (c_int32, [c_void_p, c_void_p, c_void_p, c_int32, P(c_void_p), P(c_void_p), c_int32,
+                                         c_int32, c_int32, c_int32, c_void_p]),
+    'recflex_ipc_get_handle': (c_int32, [c_void_p, c_void_p]),
+    'recflex_ipc_open_handle': (c_int32, [c_void_p, P(c_void_p)]),
+    'recflex_ipc_close': (c_int32, [c_void_p]),
+    'recflex_device_alloc': (c_int32, [ctypes.c_size_t, c_int32, P(c_void_p)]),
+    'recflex_device_free': (c_int32, [c_void_p]),
 }
 
 

@@ -27,16 +27,16 @@ __device__ __forceinline__ void dispatch_schedule(int id, const TaskCtx &x, floa
         if (id == I) {
             constexpr CatalogEntry e = kCatalog[I];
             if constexpr (e.family == RECFLEX_FAMILY_GROUP)
-                sched_group<e.G, e.VEC, e.C, e.U>(x.table, x.offs, x.idx, x.out, x.dim, x.pool, x.out_stride, x.s0, x.s1,
+                sched_group<e.G, e.VEC, e.C, e.U>(x.table, x.offs, x.idx, x.out, x.dim, x.pool, x.ro, x.s0, x.s1,
                                                   bag_ctr);
             else if constexpr (e.family == RECFLEX_FAMILY_FLAT)
-                sched_flat<e.G, e.VEC, e.U>(x.table, x.offs, x.idx, x.out, x.dim, x.pool, x.out_stride, x.s0, x.s1,
+                sched_flat<e.G, e.VEC, e.U>(x.table, x.offs, x.idx, x.out, x.dim, x.pool, x.ro, x.s0, x.s1,
                                             bag_ctr);
             else if constexpr (e.family == RECFLEX_FAMILY_BULK)
-                sched_bulk<e.U>(x.table, x.offs, x.idx, x.out, x.dim, x.pool, x.out_stride, x.s0, x.s1, bag_ctr,
+                sched_bulk<e.U>(x.table, x.offs, x.idx, x.out, x.dim, x.pool, x.ro, x.s0, x.s1, bag_ctr,
                                 x.wsmem, x.wbytes);
             else
-                sched_block<e.G, e.VEC, e.C, e.U>(x.table, x.offs, x.idx, x.out, x.dim, x.pool, x.out_stride, x.s0,
+                sched_block<e.G, e.VEC, e.C, e.U>(x.table, x.offs, x.idx, x.out, x.dim, x.pool, x.ro, x.s0,
                                                   x.s1, red);
         } else {
             dispatch_schedule<I + 1>(id, x, red, bag_ctr);
@@ -47,7 +47,7 @@ __device__ __forceinline__ void dispatch_schedule(int id, const TaskCtx &x, floa
 // Single call site for the whole catalog: the kernel calls this once per task
 // (few live values cross the call), and it branches to the schedule.
 static __device__ __noinline__ void dispatch_task(int id, const float *T, const int32_t *offs, const int32_t *idx, float *out,
-                                           int d, int pool, int out_stride, int s0, int s1, float *red, int *bag,
+                                           int d, int pool, const OutRoute ro, int s0, int s1, float *red, int *bag,
                                            unsigned char *wsmem, int wbytes) {
     TaskCtx x;
     x.wsmem = wsmem;
@@ -58,7 +58,7 @@ static __device__ __noinline__ void dispatch_task(int id, const float *T, const 
     x.out = out;
     x.dim = d;
     x.pool = pool;
-    x.out_stride = out_stride;
+    x.ro = ro;
     x.s0 = s0;
     x.s1 = s1;
     dispatch_schedule<0>(id, x, red, bag);
@@ -230,8 +230,13 @@ __global__ void __launch_bounds__(kBlockThreads, KOCC) recflex_fused_kernel(Fuse
         const FeatureDesc fd = a.desc[f];
         const bool cta_wide = kFamilyDev[fd.sched] == RECFLEX_FAMILY_BLOCK;
         if (cta_wide) __syncthreads();  // every warp reaches task n (they walk the same sequence)
+        OutRoute ro;
+        ro.ptrs = a.out_ptrs;
+        ro.rows = a.route_rows;
+        ro.colofs = a.col_base + fd.col;
+        ro.stride = a.out_stride;
         dispatch_task(fd.sched, fd.table, a.offsets + (size_t)fd.in_feature * a.B, a.indices, a.out + fd.col, fd.dim,
-                      fd.pool, a.out_stride, vld(&S.s0), vld(&S.s1), red, &S.bag, wsmem, wbytes);
+                      fd.pool, ro, vld(&S.s0), vld(&S.s1), red, &S.bag, wsmem, wbytes);
         if (cta_wide) __syncthreads();
         __syncwarp();
         if (lane == 0) {

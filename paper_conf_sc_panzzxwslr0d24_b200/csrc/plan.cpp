@@ -223,6 +223,9 @@ recflex_status_t run_pipeline(recflex_plan_s *p, const Exec &ex, const int32_t *
     a.B = B;
     a.out_stride = out_stride;
     a.smem_bytes = p->smem[k];
+    a.out_ptrs = ex.out_ptrs;
+    a.route_rows = ex.route_rows;
+    a.col_base = ex.col_base;
     LaunchCfg cfg;
     cfg.grid = p->num_sms * p->occ[k];
     cfg.smem = p->smem[k];
@@ -275,6 +278,7 @@ int32_t recflex_catalog_valid(int32_t id, int32_t dim) {
 }
 
 static void plan_free_device(recflex_plan_s *p) {
+    cudaFree(p->d_route);
     cudaFree(p->ex.d_desc);
     cudaFree(p->ex.d_block_start);
     cudaFree(p->ex.d_npb_eff);
@@ -433,6 +437,79 @@ recflex_status_t recflex_forward(recflex_plan_t p, const int32_t *indices, const
     st = run_pipeline(p, p->ex, indices, offsets, B, out, (int)p->d_tot, p->k, stream, ev);
     if (ev) p->ev_pending.push_back(trip);
     return st;
+}
+
+recflex_status_t recflex_forward_routed(recflex_plan_t p, const int32_t *indices, const int32_t *offsets, int32_t B,
+                                        const float *const *tables, float *const *host_dst, int32_t num_dst,
+                                        int32_t rows_per_dst, int32_t dst_stride, int32_t col_base, void *stream_) {
+    if (!p || !tables || !host_dst || num_dst <= 0 || num_dst > 1024 || rows_per_dst <= 0 || dst_stride <= 0 ||
+        col_base < 0 || col_base + p->d_tot > dst_stride)
+        return RECFLEX_ERR_INVALID_ARG;
+    if (B < 0 || B > p->max_batch || (int64_t)num_dst * rows_per_dst != B) return RECFLEX_ERR_INVALID_ARG;
+    if (B == 0) return RECFLEX_OK;
+    if (!indices || !offsets) return RECFLEX_ERR_INVALID_ARG;
+    // vector stores need 16-byte aligned rows / columns
+    if ((dst_stride % 4) || (col_base % 4)) return RECFLEX_ERR_INVALID_ARG;
+    for (int j = 0; j < num_dst; ++j)
+        if (!host_dst[j] || ((uintptr_t)host_dst[j]) % 16) return RECFLEX_ERR_INVALID_ARG;
+    cudaStream_t stream = (cudaStream_t)stream_;
+    cudaSetDevice(p->device);
+    recflex_status_t st = sync_tables(p, tables, stream);
+    if (st != RECFLEX_OK) return st;
+    bool same = (int)p->route_cache.size() == num_dst;
+    for (int j = 0; same && j < num_dst; ++j) same = p->route_cache[j] == host_dst[j];
+    if (!same) {
+        if ((int)p->route_cache.size() < num_dst) {
+            cudaFree(p->d_route);
+            p->d_route = nullptr;
+            cudaError_t e = cudaMalloc(&p->d_route, sizeof(float *) * num_dst);
+            if (e != cudaSuccess) return cuda_status(e);
+        }
+        p->route_cache.assign(host_dst, host_dst + num_dst);
+        cudaError_t e = cudaMemcpyAsync(p->d_route, p->route_cache.data(), sizeof(float *) * num_dst,
+                                        cudaMemcpyHostToDevice, stream);
+        if (e != cudaSuccess) return cuda_status(e);
+    }
+    Exec ex = p->ex;
+    ex.out_ptrs = p->d_route;
+    ex.route_rows = rows_per_dst;
+    ex.col_base = col_base;
+    return run_pipeline(p, ex, indices, offsets, B, host_dst[0], dst_stride, p->k, stream, nullptr);
+}
+
+recflex_status_t recflex_ipc_get_handle(const void *d_ptr, void *handle64) {
+    if (!d_ptr || !handle64) return RECFLEX_ERR_INVALID_ARG;
+    cudaIpcMemHandle_t h;
+    cudaError_t e = cudaIpcGetMemHandle(&h, const_cast<void *>(d_ptr));
+    if (e != cudaSuccess) return cuda_status_at(e, "cudaIpcGetMemHandle");
+    static_assert(sizeof(h) == 64, "IPC handle size");
+    std::memcpy(handle64, &h, 64);
+    return RECFLEX_OK;
+}
+
+recflex_status_t recflex_ipc_open_handle(const void *handle64, void **d_ptr) {
+    if (!handle64 || !d_ptr) return RECFLEX_ERR_INVALID_ARG;
+    cudaIpcMemHandle_t h;
+    std::memcpy(&h, handle64, 64);
+    cudaError_t e = cudaIpcOpenMemHandle(d_ptr, h, cudaIpcMemLazyEnablePeerAccess);
+    return cuda_status_at(e, "cudaIpcOpenMemHandle");
+}
+
+recflex_status_t recflex_device_alloc(size_t bytes, int32_t device, void **d_ptr) {
+    if (!d_ptr || bytes == 0) return RECFLEX_ERR_INVALID_ARG;
+    cudaError_t e = cudaSetDevice(device);
+    if (e == cudaSuccess) e = cudaMalloc(d_ptr, bytes);
+    return cuda_status_at(e, "cudaMalloc");
+}
+
+recflex_status_t recflex_device_free(void *d_ptr) {
+    if (!d_ptr) return RECFLEX_ERR_INVALID_ARG;
+    return cuda_status_at(cudaFree(d_ptr), "cudaFree");
+}
+
+recflex_status_t recflex_ipc_close(void *d_ptr) {
+    if (!d_ptr) return RECFLEX_ERR_INVALID_ARG;
+    return cuda_status_at(cudaIpcCloseMemHandle(d_ptr), "cudaIpcCloseMemHandle");
 }
 
 recflex_status_t recflex_forward_host(recflex_plan_t p, const int32_t *h_indices, int64_t nnz, const int32_t *h_offsets,

@@ -22,6 +22,9 @@ struct Exec {
     int num_part1 = 0;
     long long *d_timers = nullptr;
     int timers_cap = 0;
+    float *const *out_ptrs = nullptr;  // routed mode: device array of destination buffers
+    int route_rows = 0;                // 0 = local output
+    int col_base = 0;
 };
 
 struct EventTriple {
@@ -62,6 +65,9 @@ struct recflex_plan_s {
     int64_t forwards = 0;
 
     // host-buffer entry point staging
+    // routed forward: destination pointer table (device) and its host copy
+    float **d_route = nullptr;
+    std::vector<float *> route_cache;
     int32_t *d_stage_idx = nullptr;
     int64_t stage_idx_cap = 0;
     int32_t *d_stage_off = nullptr;

@@ -65,6 +65,11 @@ struct FusedArgs {
     int32_t out_stride;           // D_tot
     int32_t timers_cap;
     int32_t smem_bytes;           // dynamic shared memory of the launch (BULK stages live in it)
+    // fused pooled-output exchange (routed mode): sample s is stored into
+    // out_ptrs[s / route_rows] at row s % route_rows, column col_base + col_f
+    float *const *out_ptrs;       // device array of destination pointers (peer / IPC-mapped)
+    int32_t route_rows;           // 0 = local mode (out + s * out_stride + col_f)
+    int32_t col_base;
 };
 
 // ---------------------------------------------------------------------------

@@ -88,6 +88,25 @@ __device__ __forceinline__ void pool_finish(float (&acc)[VEC], int pool, int L) 
     }
 }
 
+// Where the pooled row of sample s goes.  Local mode (rows == 0): out + s *
+// stride (out already offset by col_f).  Routed mode (fused pooled-output
+// exchange): sample s belongs to destination rank j = s / rows,
+// whose [rows][stride] buffer (a peer / IPC-mapped pointer) receives it at row
+// s - j*rows, column colofs (+ the lane's column): the all-to-all happens in
+// the store epilogue of the fused kernel itself.
+struct OutRoute {
+    float *const *ptrs;  // destination buffers (routed mode)
+    int rows;            // samples per destination, 0 = local mode
+    int colofs;          // col_base of this rank + col_f (routed mode)
+    int stride;          // row stride of the output (floats)
+};
+
+__device__ __forceinline__ float *out_row(float *out, int s, const OutRoute &r) {
+    if (r.rows == 0) return out + (size_t)s * r.stride;
+    const int j = s / r.rows;
+    return r.ptrs[j] + (size_t)(s - j * r.rows) * r.stride + r.colofs;
+}
+
 // Everything a schedule needs for one task, passed by value (registers): the
 // paper's `args + arg_offsets[feature_idx]` (Fig. 8 line 17) resolved.
 struct TaskCtx {
@@ -97,7 +116,7 @@ struct TaskCtx {
     float *out;             // out + col_f
     int dim;
     int pool;
-    int out_stride;
+    OutRoute ro;            // output placement (local or routed to peers)
     int s0, s1;             // samples of this task
     unsigned char *wsmem;   // this warp's private shared-memory slice (BULK stages)
     int wbytes;             // its size
@@ -330,7 +349,7 @@ __device__ __forceinline__ void group_bag(const float *__restrict__ T, const int
 template <int G, int VEC, int C, int U>
 __device__ __noinline__ void sched_group(const float *__restrict__ T, const int32_t *__restrict__ offs,
                                         const int32_t *__restrict__ idx, float *__restrict__ out, int d, int pool,
-                                        int out_stride, int s0, int s1, int *bag_ctr) {
+                                        const OutRoute ro, int s0, int s1, int *bag_ctr) {
     const int lane = threadIdx.x & 31;
     const int lg = lane & (G - 1);
     const unsigned gmask = (G == 32) ? 0xffffffffu : (((1u << G) - 1u) << (lane & ~(G - 1)));
@@ -363,7 +382,7 @@ __device__ __noinline__ void sched_group(const float *__restrict__ T, const int3
             lon = ld_idx(offs + sn);
             hin = ld_idx(offs + sn + 1);
         }
-        group_bag<G, VEC, C, U>(T, idx, d, pool, out + (size_t)s * out_stride, lo, hi, lg);
+        group_bag<G, VEC, C, U>(T, idx, d, pool, out_row(out, s, ro), lo, hi, lg);
         s = sn;
         lo = lon;
         hi = hin;
@@ -383,7 +402,7 @@ constexpr int kFlatRun = 8;
 template <int G, int VEC, int U>
 __device__ __noinline__ void sched_flat(const float *__restrict__ T, const int32_t *__restrict__ offs,
                                        const int32_t *__restrict__ idx, float *__restrict__ out, int d, int pool,
-                                       int out_stride, int s0, int s1, int *bag_ctr) {
+                                       const OutRoute ro, int s0, int s1, int *bag_ctr) {
     const int lane = threadIdx.x & 31;
     const int lg = lane & (G - 1);
     const unsigned gmask = (G == 32) ? 0xffffffffu : (((1u << G) - 1u) << (lane & ~(G - 1)));
@@ -409,7 +428,7 @@ __device__ __noinline__ void sched_flat(const float *__restrict__ T, const int32
             auto finish_bag = [&]() {
                 if (ok) {
                     pool_finish<VEC>(acc, pool, bend - bstart);
-                    st_out<VEC>(out + (size_t)b * out_stride + col, acc);
+                    st_out<VEC>(out_row(out, b, ro) + col, acc);
                 }
 #pragma unroll
                 for (int e = 0; e < VEC; ++e) acc[e] = 0.f;
@@ -478,7 +497,7 @@ constexpr int kBulkBarBytes = 8 * kBulkMaxStages;
 template <int U>
 __device__ __noinline__ void sched_bulk(const float *__restrict__ T, const int32_t *__restrict__ offs,
                                        const int32_t *__restrict__ idx, float *__restrict__ out, int d, int pool,
-                                       int out_stride, int s0, int s1, int *bag_ctr, unsigned char *wsmem,
+                                       const OutRoute ro, int s0, int s1, int *bag_ctr, unsigned char *wsmem,
                                        int wbytes) {
     const int lane = threadIdx.x & 31;
     const unsigned rowb = (unsigned)d * 4u;
@@ -499,7 +518,7 @@ __device__ __noinline__ void sched_bulk(const float *__restrict__ T, const int32
             if (s >= s1) return;
             const int se = min(s1, s + kFlatRun);
             for (int b = s; b < se; ++b)
-                group_bag<32, 4, 1, 4>(T, idx, d, pool, out + (size_t)b * out_stride, ld_idx(offs + b),
+                group_bag<32, 4, 1, 4>(T, idx, d, pool, out_row(out, b, ro), ld_idx(offs + b),
                                        ld_idx(offs + b + 1), lane);
         }
     }
@@ -539,7 +558,7 @@ __device__ __noinline__ void sched_bulk(const float *__restrict__ T, const int32
         auto finish_bag = [&]() {
             if (ok) {
                 pool_finish<4>(acc, pool, bend - bstart);
-                st_out<4>(out + (size_t)b * out_stride + lane * 4, acc);
+                st_out<4>(out_row(out, b, ro) + lane * 4, acc);
             }
             acc[0] = acc[1] = acc[2] = acc[3] = 0.f;
             ++b;
@@ -585,7 +604,7 @@ __device__ __noinline__ void sched_bulk(const float *__restrict__ T, const int32
 template <int G, int VEC, int C, int U>
 __device__ __noinline__ void sched_block(const float *__restrict__ T, const int32_t *__restrict__ offs,
                                         const int32_t *__restrict__ idx, float *__restrict__ out, int d, int pool,
-                                        int out_stride, int s0, int s1, float *red /* [8][SPAN] */) {
+                                        const OutRoute ro, int s0, int s1, float *red /* [8][SPAN] */) {
     constexpr int NG = kBlockThreads / G;
     constexpr int SPAN = G * VEC * C;
     constexpr int NW = kBlockThreads / 32;
@@ -599,7 +618,7 @@ __device__ __noinline__ void sched_block(const float *__restrict__ T, const int3
     for (int s = s0; s < s1; ++s) {
         const int lo = ld_idx(offs + s);
         const int hi = ld_idx(offs + s + 1);
-        float *__restrict__ orow = out + (size_t)s * out_stride;
+        float *__restrict__ orow = out_row(out, s, ro);
         for (int p = 0; p < passes; ++p) {
             int colv[C];
             bool ok[C];

@@ -129,6 +129,19 @@ class Plan:
               'recflex_forward')
         return out
 
+    def forward_routed(self, indices: torch.Tensor, offsets: torch.Tensor, B: int, tables: Sequence[torch.Tensor],
+                       dst_ptrs: Sequence[int], rows_per_dst: int, dst_stride: int, col_base: int, stream=None):
+        """recflex_forward_routed: pooled rows stored straight into destination buffers
+        (device pointers, e.g. IPC-mapped peers): the fused all-to-all epilogue."""
+        if offsets.numel() != self.F * B + 1:
+            raise ValueError('offsets must have F*B+1 entries')
+        tarr = self._tables(tables)
+        darr = (ctypes.c_void_p * len(dst_ptrs))(*[int(p) for p in dst_ptrs])
+        idx_ptr = _dptr(indices, torch.int32, 'indices') if indices.numel() else ctypes.c_void_p(offsets.data_ptr())
+        check(lib.recflex_forward_routed(self._h, idx_ptr, _dptr(offsets, torch.int32, 'offsets'), int(B), tarr, darr,
+                                         len(dst_ptrs), int(rows_per_dst), int(dst_stride), int(col_base),
+                                         _stream_ptr(stream)), 'recflex_forward_routed')
+
     def forward_host(self, indices: torch.Tensor, offsets: torch.Tensor, B: int, tables: Sequence[torch.Tensor],
                      out: torch.Tensor, stream=None) -> torch.Tensor:
         """recflex_forward_host: host (pinned) int32 inputs -> host float32 out [B, D_tot]; blocking."""
@@ -241,6 +254,43 @@ def shard_concat(recv: torch.Tensor, dims_per_rank: Sequence[int], rows: int, ou
     check(lib.recflex_shard_concat(_dptr(recv, torch.float32, 'recv'), W, int(rows), dims,
                                    _dptr(out, torch.float32, 'out'), _stream_ptr(stream)), 'recflex_shard_concat')
     return out
+
+
+class DeviceBuffer:
+    """A float32 [rows, cols] buffer from the library's own cudaMalloc (so its
+    CUDA-IPC handle maps at offset 0), viewed as a torch tensor."""
+
+    def __init__(self, rows: int, cols: int, device: int = 0):
+        self.ptr = ctypes.c_void_p()
+        nbytes = max(4, rows * cols * 4)
+        check(lib.recflex_device_alloc(nbytes, device, ctypes.byref(self.ptr)), 'recflex_device_alloc')
+        self.__cuda_array_interface__ = {'shape': (rows, cols), 'typestr': '<f4', 'data': (self.ptr.value, False),
+                                         'version': 3, 'strides': None}
+        self.tensor = torch.as_tensor(self, device=torch.device('cuda', device))
+
+    def close(self):
+        if self.ptr and self.ptr.value:
+            lib.recflex_device_free(self.ptr)
+            self.ptr = ctypes.c_void_p()
+
+
+def ipc_handle(t) -> bytes:
+    """64-byte CUDA IPC handle of a DeviceBuffer (or a tensor that starts its allocation)."""
+    ptr = t.ptr.value if isinstance(t, DeviceBuffer) else t.data_ptr()
+    buf = ctypes.create_string_buffer(64)
+    check(lib.recflex_ipc_get_handle(ctypes.c_void_p(ptr), buf), 'recflex_ipc_get_handle')
+    return buf.raw
+
+
+def ipc_open(handle: bytes) -> int:
+    p = ctypes.c_void_p()
+    check(lib.recflex_ipc_open_handle(ctypes.create_string_buffer(handle, 64), ctypes.byref(p)),
+          'recflex_ipc_open_handle')
+    return int(p.value)
+
+
+def ipc_close(ptr: int):
+    check(lib.recflex_ipc_close(ctypes.c_void_p(ptr)), 'recflex_ipc_close')
 
 
 def l2_flush(buf: torch.Tensor, stream=None):

@@ -131,3 +131,60 @@ class ShardedEmbedding:
             out = torch.empty((rows, self.d_tot), dtype=torch.float32, device=out_local.device)
         shard_concat(recv, self.dims_per_rank, rows, out, stream=stream)
         return out
+
+
+class FusedShardedEmbedding(ShardedEmbedding):
+    """Table-wise sharding with the pooled-output all-to-all FUSED into the
+    fused kernel's store epilogue: every rank's kernel writes
+    each pooled row straight into the owning rank's final [B/W][D_tot] buffer
+    through CUDA-IPC-mapped peer pointers (NVLink peer stores across GPUs of a
+    node; plain stores when ranks share a device), so there is no separate
+    all-to-all pass and no relayout.  A collective barrier after the kernel
+    orders the destination's reads after every writer (stream-ordered
+    all_reduce on NCCL; host barrier on gloo)."""
+
+    def __init__(self, model, rank: int, world: int, device: int = 0, parts=None, group=None):
+        import torch.distributed as dist
+        from .plan import DeviceBuffer, ipc_handle, ipc_open
+        super().__init__(model, rank, world, device, parts)
+        if model.batch % world:
+            raise ValueError('fused exchange needs B % W == 0 (reading C23)')
+        self.group = group
+        self.rows = model.batch // world
+        self.col_base = sum(self.dims_per_rank[:rank])
+        self.buf = DeviceBuffer(self.rows, self.d_tot, device)
+        handles = [None] * world
+        dist.all_gather_object(handles, (rank, ipc_handle(self.buf)), group=group)
+        self.dst = [0] * world
+        self._opened = []
+        for r, h in handles:
+            if r == rank:
+                self.dst[r] = self.buf.ptr.value
+            else:
+                p = ipc_open(h)
+                self.dst[r] = p
+                self._opened.append(p)
+        import torch
+        self._flag = torch.zeros(1, dtype=torch.float32, device=torch.device('cuda', device))
+
+    def forward(self, indices, offsets, B, tables, out_local=None, out=None, group=None, stream=None):
+        import torch
+        import torch.distributed as dist
+        if B != self.model.batch:
+            raise ValueError('the fused exchange buffers are sized for the model batch')
+        self.plan.forward_routed(indices, offsets, B, tables, self.dst, self.rows, self.d_tot, self.col_base,
+                                 stream=stream)
+        g = group if group is not None else self.group
+        if dist.get_backend(g) == 'nccl':
+            dist.all_reduce(self._flag, group=g)  # stream-ordered: every writer's kernel precedes it
+        else:
+            torch.cuda.current_stream().synchronize()
+            dist.barrier(group=g)
+        return self.buf.tensor
+
+    def close(self):
+        from .plan import ipc_close
+        for p in self._opened:
+            ipc_close(p)
+        self._opened = []
+        self.buf.close()
