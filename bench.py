@@ -206,6 +206,8 @@ def main():
     ap.add_argument('--cpu-samples', type=int, default=1024, help='cpu_baseline: samples in the bounded sample')
     ap.add_argument('--cpu-seconds', type=float, default=10.0, help='cpu_baseline: minimum timed CPU seconds')
     ap.add_argument('--profile-only', action='store_true', help='short run for ncu (no e2e / cpu / clocks)')
+    ap.add_argument('--exchange', default='nccl', choices=['nccl', 'fused'],
+                    help='N>1: NCCL alltoallv + relayout kernel, or peer stores fused into the kernel epilogue')
     args = ap.parse_args()
 
     world = int(os.environ.get('WORLD_SIZE', '1'))
@@ -228,7 +230,11 @@ def main():
     model = synth.make_model(args.config)
     B = model.batch
     parts = partition_model(model, world)
-    sh = ShardedEmbedding(model, rank, world, device=local_rank, parts=parts)
+    if world > 1 and args.exchange == 'fused':
+        from paper_conf_sc_panzzxwslr0d24_b200.shard import FusedShardedEmbedding
+        sh = FusedShardedEmbedding(model, rank, world, device=local_rank, parts=parts)
+    else:
+        sh = ShardedEmbedding(model, rank, world, device=local_rank, parts=parts)
     plan = sh.plan
     feats = sh.features
 
@@ -405,7 +411,7 @@ def main():
             cpu = {'value': None, 'unit': 'samples/s', 'cores': None, 'kind': 'oracle', 'sample': f'failed: {ex}'}
 
     launches_per_step = 2 + (1 if plan.export() and any(s[1] == 1 for s in plan.export()['schedules']) else 0)
-    launches_per_step += 1 if world > 1 else 0   # relayout kernel
+    launches_per_step += 1 if (world > 1 and args.exchange == 'nccl') else 0   # relayout kernel
     if rank == 0:
         line = {
             'metric': _baseline_metric(),
@@ -422,6 +428,7 @@ def main():
             'data': 'synthetic (seeded generator, SURVEY §8d recipe; tables: counter-based hash U[-1,1))',
             'config': {'workload': args.config, 'global_batch': B, 'fields': model.F,
                        'parallelism': f'tablewise{world}', 'plan': plan_src, 'occupancy': plan.occupancy,
+                       'exchange': (args.exchange if world > 1 else 'none'),
                        'l2': 'flushed between steps' if flush_between else
                              f'inputs > L2 ({alg_local / 1e9:.2f} GB algorithmic per step per rank, '
                              f'{args.batches} rotating batches)'},
