@@ -107,7 +107,7 @@ class ClockSampler:
 
 # ------------------------------------------------------------------------- CPU oracle arm
 def oracle_sample_rate(model, batch, n_samples: int, seed: int = 0, nthreads: int = 0, min_seconds: float = 0.0,
-                       max_reps: int = 1000):
+                       max_reps: int = 1000, dtype: str = 'f32'):
     """Time the oracle (as it stands) on a bounded sample of the workload.
 
     Input preparation (regenerating the referenced table rows from the seeded
@@ -129,7 +129,7 @@ def oracle_sample_rate(model, batch, n_samples: int, seed: int = 0, nthreads: in
         if uniq.size == 0:
             uniq = np.zeros(1, np.int64)
         feat = model.features[f]
-        tables.append(synth.table_rows_at(feat.table, uniq, feat.dim, 'float', seed=model.seed).numpy())
+        tables.append(synth.table_rows_stored(feat.table, uniq, feat.dim, dtype, 'float', seed=model.seed))
         pos = 0
         for bag in bags:
             sub_idx.append(inv[pos:pos + bag.size].astype(np.int32))
@@ -141,12 +141,13 @@ def oracle_sample_rate(model, batch, n_samples: int, seed: int = 0, nthreads: in
     # algorithmic bytes of the sample (C26)
     nnz_f = np.asarray([off[(f + 1) * S] - off[f * S] for f in range(F)], np.int64)
     dims = np.asarray(model.dims, np.int64)
-    alg = 4 * int(nnz_f.sum()) + 4 * int((dims * nnz_f).sum()) + 4 * S * int(dims.sum())
+    rowb = np.asarray([synth.row_bytes(d, dtype) for d in model.dims], np.int64)
+    alg = 4 * int(nnz_f.sum()) + int((rowb * nnz_f).sum()) + 4 * S * int(dims.sum())
     pools = [f.pool for f in model.features]
     reps, dt = 0, 0.0
     while reps == 0 or (dt < min_seconds and reps < max_reps):
         t0 = time.perf_counter()
-        oracle.embedding_bag(tables, model.dims, pools, idx, off, S, nthreads=nthreads)
+        oracle.embedding_bag(tables, model.dims, pools, idx, off, S, nthreads=nthreads, dtypes=[dtype] * F)
         dt += time.perf_counter() - t0
         reps += 1
     return S * reps, dt, alg * reps
@@ -196,6 +197,8 @@ def main():
     ap.add_argument('--impl', default='ours', choices=['ours', 'reference'])
     ap.add_argument('--config', default='sharded1000')
     ap.add_argument('--mode', default='float', choices=['float', 'int'])
+    ap.add_argument('--dtype', default='f32', choices=['f32', 'f16', 'bf16', 'i8'],
+                    help='table row storage (SURVEY NEXT #3); accumulation and output stay fp32')
     ap.add_argument('--batches', type=int, default=3)
     ap.add_argument('--plan', default='auto', help="tuned plan JSON, 'auto' (configs/tuned/) or 'none'")
     ap.add_argument('--tune', action='store_true', help='run the two-stage tuner before timing')
@@ -229,12 +232,12 @@ def main():
 
     model = synth.make_model(args.config)
     B = model.batch
-    parts = partition_model(model, world)
+    parts = partition_model(model, world, args.dtype)
     if world > 1 and args.exchange == 'fused':
         from paper_conf_sc_panzzxwslr0d24_b200.shard import FusedShardedEmbedding
-        sh = FusedShardedEmbedding(model, rank, world, device=local_rank, parts=parts)
+        sh = FusedShardedEmbedding(model, rank, world, device=local_rank, parts=parts, dtype=args.dtype)
     else:
-        sh = ShardedEmbedding(model, rank, world, device=local_rank, parts=parts)
+        sh = ShardedEmbedding(model, rank, world, device=local_rank, parts=parts, dtype=args.dtype)
     plan = sh.plan
     feats = sh.features
 
@@ -244,12 +247,13 @@ def main():
         t = model.features[f].table
         if t not in phys:
             rows, dim = model.tables[t]
-            phys[t] = synth.make_table(t, rows, dim, args.mode, device=dev, seed=model.seed)
+            phys[t] = synth.make_table_stored(t, rows, dim, args.dtype, args.mode, device=dev, seed=model.seed)
     tables = [phys[model.features[f].table] for f in feats]
 
     # batches: the global batch for my features, resident in HBM
     batches, host_batches, alg_bytes = [], [], []
     dims_local = np.asarray([model.dims[f] for f in feats], np.int64)
+    rowb_local = np.asarray([synth.row_bytes(model.dims[f], args.dtype) for f in feats], np.int64)
     for i in range(args.batches):
         full = synth.make_batch(model, 7 + i)
         idx, off = shard_batch(full, feats)
@@ -257,9 +261,10 @@ def main():
         batches.append((torch.from_numpy(idx).to(dev), torch.from_numpy(off).to(dev)))
         o = off.astype(np.int64)
         nnz_f = o[np.arange(1, len(feats) + 1) * B] - o[np.arange(0, len(feats)) * B]
-        alg_bytes.append(4 * int(nnz_f.sum()) + 4 * int((dims_local * nnz_f).sum()) + 4 * B * int(dims_local.sum()))
+        # C26: IDs + gathered rows (stored bytes) + pooled fp32 output
+        alg_bytes.append(4 * int(nnz_f.sum()) + int((rowb_local * nnz_f).sum()) + 4 * B * int(dims_local.sum()))
     alg_local = float(np.mean(alg_bytes))
-    ws = alg_local + sum(t.numel() * 4 for t in tables)
+    ws = alg_local + sum(t.numel() * t.element_size() for t in tables)
     flush_between = (alg_local < 4 * L2_BYTES)
 
     # tuned plan (stage-1/2 result exported by tools/tune_plan.py) or live tuning
@@ -272,6 +277,8 @@ def main():
         path = args.plan
         if path == 'auto':
             path = os.path.join(ROOT, 'configs', 'tuned', f'{args.config}_w{world}_r{rank}.json')
+        if args.dtype != 'f32' and args.plan == 'auto':
+            path = os.path.join(ROOT, 'configs', 'tuned', f'{args.config}_{args.dtype}_w{world}_r{rank}.json')
         if os.path.exists(path):
             with open(path) as fh:
                 plan.import_(json.load(fh))
@@ -348,7 +355,8 @@ def main():
     eff_gbs_step = alg_local / (ms_per_step / 1e3) / 1e9
 
     traffic = None
-    tp = os.path.join(ROOT, 'profiles', f'ncu_traffic_{args.config}.json')
+    tp = os.path.join(ROOT, 'profiles', f'ncu_traffic_{args.config}' + ('' if args.dtype == 'f32' else f'_{args.dtype}')
+                      + '.json')
     if os.path.exists(tp):
         try:
             with open(tp) as fh:
@@ -402,7 +410,7 @@ def main():
             full = _s.make_batch(model, 7)
             cores = len(os.sched_getaffinity(0))
             S, dt, alg = oracle_sample_rate(model, full, args.cpu_samples, seed=0, nthreads=cores,
-                                            min_seconds=args.cpu_seconds)
+                                            min_seconds=args.cpu_seconds, dtype=args.dtype)
             cpu = {'value': S / dt, 'unit': 'samples/s', 'cores': cores, 'kind': 'oracle',
                    'sample': f'{args.cpu_samples} random samples x all {model.F} fields of batch seed 7, '
                              f'oracle repeated to {dt:.1f} s ({S} samples total; fp64 C oracle, OpenMP)',
@@ -424,9 +432,9 @@ def main():
             'higher_is_better': True,
             'scaling': 'strong' if world > 1 else 'weak',
             'vs_baseline': None,
-            'dtype': 'f32',
+            'dtype': 'f32' if args.dtype == 'f32' else f'{args.dtype} rows, f32 accumulate/output',
             'data': 'synthetic (seeded generator, SURVEY §8d recipe; tables: counter-based hash U[-1,1))',
-            'config': {'workload': args.config, 'global_batch': B, 'fields': model.F,
+            'config': {'workload': args.config, 'global_batch': B, 'fields': model.F, 'table_dtype': args.dtype,
                        'parallelism': f'tablewise{world}', 'plan': plan_src, 'occupancy': plan.occupancy,
                        'exchange': (args.exchange if world > 1 else 'none'),
                        'l2': 'flushed between steps' if flush_between else

@@ -30,7 +30,17 @@
  *   indices : int32 [nnz]          lookup IDs, feature-major KJT
  *   offsets : int32 [F*B + 1]      bag (f,s) = indices[offsets[f*B+s] .. offsets[f*B+s+1])
  *                                  offsets[0] == 0, non-decreasing, nnz < 2^31
- *   tables  : F float32 row-major [rows_f][d_f], 32-byte aligned base
+ *   tables  : F row-major tables, 32-byte aligned base, in the feature's
+ *             storage type (recflex_dtype_t; the paper is
+ *             silent on precision, reading C5):
+ *               F32  float32  [rows_f][d_f]                      (default)
+ *               F16  binary16 [rows_f][d_f]
+ *               BF16 bfloat16 [rows_f][d_f]
+ *               I8   rowwise-quantised: row r is RECFLEX_I8_ROW_BYTES(d_f)
+ *                    bytes = d_f int8 codes q, then float32 scale, float32
+ *                    bias, zero padding to a multiple of 16 bytes; the row's
+ *                    value in column c is scale * q[c] + bias
+ *             Rows are always accumulated in fp32; the output is fp32.
  *   out     : float32 row-major [B][D_tot], D_tot = sum d_f, feature f at
  *             columns [col_f, col_f + d_f), col_f = sum_{g<f} d_g; 16-byte
  *             aligned base
@@ -45,12 +55,23 @@
 extern "C" {
 #endif
 
-#define RECFLEX_ABI_VERSION 1
+#define RECFLEX_ABI_VERSION 2
 #define RECFLEX_MAX_OCCUPANCY 8          /* CTAs of 256 threads per SM: K = 8 (reading C14) */
 
 typedef struct recflex_plan_s *recflex_plan_t; /* opaque, library-owned */
 
 typedef enum { RECFLEX_POOL_SUM = 0, RECFLEX_POOL_MEAN = 1 } recflex_pool_t;
+
+/* Storage type of a feature's table rows. */
+typedef enum {
+    RECFLEX_DTYPE_F32 = 0,  /* float32                                                   */
+    RECFLEX_DTYPE_F16 = 1,  /* IEEE binary16; needs d_f % 4 == 0                         */
+    RECFLEX_DTYPE_BF16 = 2, /* bfloat16 (upper half of a float32); needs d_f % 4 == 0    */
+    RECFLEX_DTYPE_I8 = 3    /* int8 codes + per-row float32 scale and bias; d_f % 8 == 0 */
+} recflex_dtype_t;
+
+/* Bytes per row of an I8 table: d codes + 8 bytes scale/bias, padded to 16. */
+#define RECFLEX_I8_ROW_BYTES(d) ((((int64_t)(d)) + 8 + 15) / 16 * 16)
 
 typedef enum {
     RECFLEX_OK = 0,
@@ -70,6 +91,7 @@ typedef struct {
     float mean_len;   /* E[L | L > 0]   (pooling factor)                    */
     float max_len;    /* observed max L (sizes scratch for nnz-partitioned tasks) */
     float coverage;   /* P(L > 0)                                    */
+    int32_t dtype;    /* recflex_dtype_t of the table rows (0 = F32)              */
 } recflex_feature_spec_t;
 
 /* A feature's schedule: catalog entry + its runtime thread-mapping parameters
@@ -100,11 +122,12 @@ typedef struct {
     int32_t vec;    /* floats per lane per load: 1, 4 (128-bit) or 8 (256-bit) */
     int32_t cols;   /* C: column chunks per lane (row span = G*vec*C floats)   */
     int32_t unroll; /* U: rows in flight per lane                              */
+    int32_t dtype;  /* recflex_dtype_t the entry gathers (vec counts elements)  */
 } recflex_catalog_info_t;
 
 /* ---- plan lifecycle --------------------------------------------------- */
 
-/* Validates specs, computes col_f (prefix sum of dims), picks heuristic
+/* Validates specs (incl. each dtype's dim constraint), computes col_f (prefix sum of dims), picks heuristic
  * default schedules (an untuned plan is valid), allocates plan scratch sized
  * for max_batch on `device`.  No device data is read.  *out receives the plan. */
 recflex_status_t recflex_plan_create(const recflex_feature_spec_t *specs, int32_t num_features,
@@ -131,7 +154,7 @@ const char *recflex_last_error(void);
  * Launches: map kernel (device-side workload scan), optional task-range fill
  * kernel (only if some feature is lookup-partitioned), fused kernel (PDL). */
 recflex_status_t recflex_forward(recflex_plan_t plan, const int32_t *indices, const int32_t *offsets,
-                                 int32_t batch_size, const float *const *tables, float *out,
+                                 int32_t batch_size, const void *const *tables, float *out,
                                  void *stream);
 
 /* Same operation from HOST buffers (end-to-end path): copies h_indices[nnz] and
@@ -140,7 +163,7 @@ recflex_status_t recflex_forward(recflex_plan_t plan, const int32_t *indices, co
  * Staging grows on demand (this entry point may allocate). */
 recflex_status_t recflex_forward_host(recflex_plan_t plan, const int32_t *h_indices, int64_t nnz,
                                       const int32_t *h_offsets, int32_t batch_size,
-                                      const float *const *tables, float *h_out, void *stream);
+                                      const void *const *tables, float *h_out, void *stream);
 
 /* ---- tuner (§IV-A) ------------------------------------------------------ */
 
@@ -182,10 +205,10 @@ typedef struct {
  * allocate.  Leaves the plan with the selected occupancy and schedules. */
 recflex_status_t recflex_tune(recflex_plan_t plan, int32_t num_batches, const int32_t *const *indices,
                               const int32_t *const *offsets, const int32_t *batch_sizes,
-                              const float *const *tables, void *stream);
+                              const void *const *tables, void *stream);
 recflex_status_t recflex_tune_ex(recflex_plan_t plan, int32_t num_batches, const int32_t *const *indices,
                                  const int32_t *const *offsets, const int32_t *batch_sizes,
-                                 const float *const *tables, void *stream,
+                                 const void *const *tables, void *stream,
                                  const recflex_tune_options_t *options, recflex_tune_stats_t *stats);
 
 /* The selection logic of the two-stage tuner, on caller-supplied costs
@@ -215,8 +238,10 @@ recflex_status_t recflex_get_occupancy(recflex_plan_t plan, int32_t *k);
 
 int32_t recflex_catalog_size(void);
 recflex_status_t recflex_catalog_info(int32_t sched_id, recflex_catalog_info_t *info);
-/* 1 if catalog entry sched_id can run a feature of dimension dim. */
+/* 1 if catalog entry sched_id can run a float32 feature of dimension dim. */
 int32_t recflex_catalog_valid(int32_t sched_id, int32_t dim);
+/* 1 if catalog entry sched_id can run a feature of dimension dim stored as dtype. */
+int32_t recflex_catalog_valid_dtype(int32_t sched_id, int32_t dim, int32_t dtype);
 
 /* cudaOccupancyMaxActiveBlocksPerMultiprocessor of the fused-kernel variant
  * for occupancy k with its padded shared memory (should equal k). */
@@ -266,7 +291,7 @@ recflex_status_t recflex_get_kernel_times(recflex_plan_t plan, double *map_ms, d
  * Async on `stream`; the caller orders the destination's reads after every
  * writer's kernel (e.g. a collective barrier on the same streams). */
 recflex_status_t recflex_forward_routed(recflex_plan_t plan, const int32_t *indices, const int32_t *offsets,
-                                        int32_t batch_size, const float *const *tables, float *const *host_dst,
+                                        int32_t batch_size, const void *const *tables, float *const *host_dst,
                                         int32_t num_dst, int32_t rows_per_dst, int32_t dst_stride,
                                         int32_t col_base, void *stream);
 

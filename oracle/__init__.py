@@ -13,6 +13,9 @@ Functions and the passages they follow (PAPER.md "P:n"):
   embedding_bag  -- P:41, P:51 (§II-A): gather the rows named by each sample's
                     lookup IDs, pool them by elementwise reduction, concatenate
                     per-feature outputs.  Readings C1, C2, C6.
+  decode_rows    -- the value of a stored row element per storage type (SURVEY
+                    NEXT #3: f16 / bf16 / rowwise int8); embedding_bag takes
+                    stored tables and decodes every element with it.
   task_map       -- Fig. 8: d_blocks_map and d_task_map, reading C12.
   nnz_task_ranges-- reading C12 for nnz-partitioned schedules.
 """
@@ -40,7 +43,7 @@ def build(force: bool = False) -> str:
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
         tmp = _LIB + f'.tmp{os.getpid()}'
         subprocess.check_call(['gcc', '-O2', '-fopenmp', '-fPIC', '-shared', '-std=c11', '-Wall',
-                               '-o', tmp, _SRC])
+                               '-o', tmp, _SRC, '-lm'])
         os.replace(tmp, _LIB)
     return _LIB
 
@@ -57,6 +60,16 @@ def lib():
                 ctypes.c_int, ctypes.c_int, P(ctypes.c_int), P(ctypes.c_int),
                 P(ctypes.c_void_p), P(ctypes.c_int64), P(ctypes.c_int32), P(ctypes.c_int32),
                 P(ctypes.c_double), ctypes.c_int]
+            L.oracle_embedding_bag_typed.restype = ctypes.c_int
+            L.oracle_embedding_bag_typed.argtypes = [
+                ctypes.c_int, ctypes.c_int, P(ctypes.c_int), P(ctypes.c_int), P(ctypes.c_int),
+                P(ctypes.c_void_p), P(ctypes.c_int64), P(ctypes.c_int32), P(ctypes.c_int32),
+                P(ctypes.c_double), ctypes.c_int]
+            L.oracle_decode_rows.restype = ctypes.c_int
+            L.oracle_decode_rows.argtypes = [ctypes.c_int, ctypes.c_void_p, ctypes.c_int64, ctypes.c_int,
+                                             P(ctypes.c_double)]
+            L.oracle_row_bytes.restype = ctypes.c_int64
+            L.oracle_row_bytes.argtypes = [ctypes.c_int, ctypes.c_int]
             L.oracle_task_map.restype = ctypes.c_int
             L.oracle_task_map.argtypes = [
                 ctypes.c_int, ctypes.c_int, P(ctypes.c_int), P(ctypes.c_int), P(ctypes.c_int),
@@ -82,16 +95,53 @@ def max_threads() -> int:
     return int(lib().oracle_max_threads())
 
 
-def embedding_bag(tables, dims, pools, indices, offsets, B, nthreads: int = 0) -> np.ndarray:
+DTYPES = {'f32': 0, 'f16': 1, 'bf16': 2, 'i8': 3}
+
+
+def row_bytes(dtype, dim: int) -> int:
+    return int(lib().oracle_row_bytes(DTYPES.get(dtype, dtype), int(dim)))
+
+
+def _stored(t, dtype, dim):
+    """A stored table (numpy array or CPU torch tensor) as contiguous raw bytes [rows][row_bytes]."""
+    code = DTYPES.get(dtype, dtype)
+    if code == 0:
+        a = np.ascontiguousarray(t.numpy() if hasattr(t, 'numpy') else t, dtype=np.float32)
+        if a.ndim != 2 or a.shape[1] != dim:
+            raise ValueError(f'table shape {a.shape} vs dim {dim}')
+        return a
+    if hasattr(t, 'view') and hasattr(t, 'dtype') and not isinstance(t, np.ndarray):  # torch (bf16 has no numpy)
+        import torch
+        t = t.contiguous().view(torch.uint8).numpy()
+    a = np.ascontiguousarray(t).view(np.uint8)
+    a = a.reshape(a.shape[0], -1)
+    if a.shape[1] != row_bytes(code, dim):
+        raise ValueError(f'stored row bytes {a.shape[1]} vs {row_bytes(code, dim)} for dim {dim} dtype {dtype}')
+    return a
+
+
+def decode_rows(rows, dim: int, dtype) -> np.ndarray:
+    """fp64 values of stored rows (oracle_decode), [n][dim]."""
+    a = _stored(rows, dtype, dim)
+    out = np.zeros((a.shape[0], dim), np.float64)
+    rc = lib().oracle_decode_rows(DTYPES.get(dtype, dtype), a.ctypes.data, a.shape[0], int(dim),
+                                  _ptr(out, ctypes.c_double))
+    if rc != 0:
+        raise OracleError(rc)
+    return out
+
+
+def embedding_bag(tables, dims, pools, indices, offsets, B, nthreads: int = 0, dtypes=None) -> np.ndarray:
     """fp64 pooled output [B][sum(dims)].
 
-    tables: list of F float32 arrays [rows_f][d_f] (one per feature; aliasing allowed)
+    tables: list of F stored tables (one per feature; aliasing allowed):
+    float32 arrays [rows_f][d_f] when dtypes is None, else per dtypes[f]
+    ('f32', 'f16', 'bf16', 'i8' -- numpy arrays or CPU torch tensors; an i8
+    row is d int8 codes, float32 scale, float32 bias, zero padding to 16 bytes).
     """
     F = len(dims)
-    tabs = [np.ascontiguousarray(t, dtype=np.float32) for t in tables]
-    for f in range(F):
-        if tabs[f].ndim != 2 or tabs[f].shape[1] != dims[f]:
-            raise ValueError(f'table {f} shape {tabs[f].shape} vs dim {dims[f]}')
+    dts = [DTYPES.get(d, d) for d in (dtypes if dtypes is not None else [0] * F)]
+    tabs = [_stored(t, dts[f], dims[f]) for f, t in enumerate(tables)]
     dims_a = np.asarray(dims, np.intc)
     pools_a = np.asarray(pools, np.intc)
     rows_a = np.asarray([t.shape[0] for t in tabs], np.int64)
@@ -103,9 +153,11 @@ def embedding_bag(tables, dims, pools, indices, offsets, B, nthreads: int = 0) -
     out = np.zeros((B, int(dims_a.sum())), np.float64)
     if idx.size == 0:
         idx = np.zeros(1, np.int32)
-    rc = lib().oracle_embedding_bag(F, B, _ptr(dims_a, ctypes.c_int), _ptr(pools_a, ctypes.c_int),
-                                    ptrs, _ptr(rows_a, ctypes.c_int64), _ptr(idx, ctypes.c_int32),
-                                    _ptr(off, ctypes.c_int32), _ptr(out, ctypes.c_double), int(nthreads))
+    dt_a = np.asarray(dts, np.intc)
+    rc = lib().oracle_embedding_bag_typed(F, B, _ptr(dims_a, ctypes.c_int), _ptr(pools_a, ctypes.c_int),
+                                          _ptr(dt_a, ctypes.c_int), ptrs, _ptr(rows_a, ctypes.c_int64),
+                                          _ptr(idx, ctypes.c_int32), _ptr(off, ctypes.c_int32),
+                                          _ptr(out, ctypes.c_double), int(nthreads))
     if rc != 0:
         raise OracleError({-1: 'index out of range', -2: 'bad offsets', -3: 'bad argument'}.get(rc, rc))
     return out
@@ -164,12 +216,12 @@ def nnz_task_ranges(B, npb, feature_offsets, blocks):
 # Full-size sampled checks: compute selected samples one by one.
 # ---------------------------------------------------------------------------
 
-def sampled_forward(model, batch, samples, table_getter):
+def sampled_forward(model, batch, samples, table_getter, dtype='f32'):
     """Oracle output rows for the given sample ids of a (possibly huge) batch.
 
-    table_getter(feature_index, unique_row_ids) -> float32 [n][d_f] rows of that
-    feature's table (from the seeded generator).  Returns fp64 [len(samples)][D_tot]
-    and the per-(sample, feature) bag lengths [len(samples)][F].
+    table_getter(feature_index, unique_row_ids) -> stored rows [n] of that
+    feature's table in `dtype` (from the seeded generator).  Returns fp64
+    [len(samples)][D_tot] and the per-(sample, feature) bag lengths [len(samples)][F].
     """
     F, B = batch.F, batch.B
     samples = np.asarray(samples, np.int64)
@@ -189,7 +241,10 @@ def sampled_forward(model, batch, samples, table_getter):
         uniq, inv = np.unique(allids, return_inverse=True)
         if uniq.size == 0:
             uniq = np.zeros(1, np.int64)
-        tables.append(np.asarray(table_getter(f, uniq), np.float32).reshape(uniq.size, model.features[f].dim))
+        rows_f = table_getter(f, uniq)
+        if DTYPES.get(dtype, dtype) == 0:
+            rows_f = np.asarray(rows_f, np.float32).reshape(uniq.size, model.features[f].dim)
+        tables.append(rows_f)
         pos = 0
         for bag in bags:
             sub_idx.append(inv[pos:pos + bag.size].astype(np.int32))
@@ -197,5 +252,6 @@ def sampled_forward(model, batch, samples, table_getter):
             sub_off.append(sub_off[-1] + bag.size)
     idx = np.concatenate(sub_idx) if sub_idx else np.zeros(0, np.int32)
     off = np.asarray(sub_off, np.int32)
-    out = embedding_bag(tables, model.dims, [f.pool for f in model.features], idx, off, S)
+    out = embedding_bag(tables, model.dims, [f.pool for f in model.features], idx, off, S,
+                        dtypes=[dtype] * F)
     return out, lens

@@ -23,6 +23,18 @@
  *       Pinned by tests/test_oracle.py (worked example in tests/golden,
  *       torch.nn.functional.embedding_bag, brute force, closed-form invariants).
  *
+ *   oracle_decode         -- the value of element c of a stored table row, per
+ *       storage type (the paper is silent on precision,
+ *       reading C5): F32 = the float; F16 = IEEE 754 binary16 written out
+ *       from its fields (sign, 5-bit exponent with bias 15, 10-bit fraction,
+ *       subnormals, inf/nan); BF16 = the 16 bits as the upper half of an IEEE
+ *       binary32; I8 = scale * q + bias with q the signed code and scale, bias
+ *       the row's two float32 after its d codes (rowwise-quantised row: d
+ *       codes, scale, bias, zero padding to a multiple of 16 bytes),
+ *       evaluated in fp64.
+ *       Pinned by tests/test_oracle.py: exhaustive over all 2^16 patterns
+ *       against numpy float16 and torch bfloat16, hand-decoded I8 rows.
+ *
  *   oracle_task_map       -- the runtime thread map of Fig. 8:
  *       d_blocks_map[f] = feature_blocks, and d_task_map[b] = (feature_idx,
  *       rel_bidx) enumerating, feature by feature, rel = 0..feature_blocks-1.
@@ -36,6 +48,7 @@
  *       task owns: {s : floor((off[s]-off[0]) / npb) == rel}, written out by
  *       brute force over s for every task (reading C12).
  */
+#include <math.h>
 #include <stdint.h>
 #include <stdlib.h>
 #include <string.h>
@@ -51,6 +64,60 @@
 #define POOL_SUM 0
 #define POOL_MEAN 1
 
+#define DT_F32 0
+#define DT_F16 1
+#define DT_BF16 2
+#define DT_I8 3
+
+/* bytes per stored row of dimension d */
+int64_t oracle_row_bytes(int dtype, int d) {
+    switch (dtype) {
+        case DT_F16:
+        case DT_BF16: return 2 * (int64_t)d;
+        case DT_I8: return ((int64_t)d + 8 + 15) / 16 * 16;
+        default: return 4 * (int64_t)d;
+    }
+}
+
+/* value of element c of the stored row at `row` (d elements) */
+double oracle_decode(int dtype, const unsigned char *row, int c, int d) {
+    if (dtype == DT_F16) {
+        unsigned h = (unsigned)row[2 * c] | ((unsigned)row[2 * c + 1] << 8);
+        int sign = (h >> 15) & 1, e = (h >> 10) & 31, m = h & 1023;
+        double v;
+        if (e == 0) v = ldexp((double)m, -24);                 /* subnormal: m * 2^-24 */
+        else if (e == 31) v = m ? NAN : INFINITY;
+        else v = ldexp((double)(1024 + m), e - 25);            /* (1 + m/1024) * 2^(e-15) */
+        return sign ? -v : v;
+    }
+    if (dtype == DT_BF16) {
+        uint32_t u = ((uint32_t)row[2 * c] | ((uint32_t)row[2 * c + 1] << 8)) << 16;
+        float f;
+        memcpy(&f, &u, 4);
+        return (double)f;
+    }
+    if (dtype == DT_I8) {
+        int q = (int)(signed char)row[c];
+        float scale, bias;
+        memcpy(&scale, row + d, 4);
+        memcpy(&bias, row + d + 4, 4);
+        return (double)scale * (double)q + (double)bias;
+    }
+    {
+        float f;
+        memcpy(&f, row + 4 * (int64_t)c, 4);
+        return (double)f;
+    }
+}
+
+/* decode n stored rows into out[n][d] (for pinning the decode) */
+int oracle_decode_rows(int dtype, const void *rows, int64_t n, int d, double *out) {
+    const int64_t rb = oracle_row_bytes(dtype, d);
+    for (int64_t r = 0; r < n; ++r)
+        for (int c = 0; c < d; ++c) out[r * d + c] = oracle_decode(dtype, (const unsigned char *)rows + r * rb, c, d);
+    return ORACLE_OK;
+}
+
 int oracle_version(void) { return 1; }
 
 int oracle_max_threads(void) {
@@ -63,15 +130,16 @@ int oracle_max_threads(void) {
 
 /*
  * F features, batch B.
- * dims[f], pools[f], rows[f]; tables[f] -> float32 [rows[f]][dims[f]] row-major.
+ * dims[f], pools[f], rows[f]; dtypes[f] (NULL = all float32); tables[f] ->
+ * [rows[f]] stored rows of oracle_row_bytes(dtypes[f], dims[f]) bytes.
  * indices int32[nnz], offsets int32[F*B+1] (feature-major KJT CSR).
  * out -> double [B][sum(dims)].
  * nthreads <= 0: library default.
  */
-int oracle_embedding_bag(int F, int B, const int *dims, const int *pools,
-                         const float *const *tables, const int64_t *rows,
-                         const int32_t *indices, const int32_t *offsets,
-                         double *out, int nthreads) {
+int oracle_embedding_bag_typed(int F, int B, const int *dims, const int *pools, const int *dtypes,
+                               const void *const *tables, const int64_t *rows,
+                               const int32_t *indices, const int32_t *offsets,
+                               double *out, int nthreads) {
     if (F <= 0 || B < 0) return ORACLE_ERR_ARG;
     int64_t d_tot = 0;
     int64_t *col = (int64_t *)malloc(sizeof(int64_t) * (size_t)F);
@@ -98,7 +166,9 @@ int oracle_embedding_bag(int F, int B, const int *dims, const int *pools,
 #pragma omp parallel for schedule(dynamic)
     for (int f = 0; f < F; ++f) {
         const int d = dims[f];
-        const float *T = tables[f];
+        const int dt = dtypes ? dtypes[f] : DT_F32;
+        const int64_t rb = oracle_row_bytes(dt, d);
+        const unsigned char *T = (const unsigned char *)tables[f];
         double *acc = (double *)malloc(sizeof(double) * (size_t)(d > 0 ? d : 1));
         for (int s = 0; s < B; ++s) {
             const int64_t lo = offsets[(int64_t)f * B + s];
@@ -106,8 +176,8 @@ int oracle_embedding_bag(int F, int B, const int *dims, const int *pools,
             const int64_t L = hi - lo;
             for (int c = 0; c < d; ++c) acc[c] = 0.0;
             for (int64_t j = lo; j < hi; ++j) {             /* ascending j */
-                const float *row = T + (int64_t)indices[j] * d;
-                for (int c = 0; c < d; ++c) acc[c] += (double)row[c];
+                const unsigned char *row = T + (int64_t)indices[j] * rb;
+                for (int c = 0; c < d; ++c) acc[c] += oracle_decode(dt, row, c, d);
             }
             double *o = out + (int64_t)s * d_tot + col[f];
             for (int c = 0; c < d; ++c) {
@@ -121,6 +191,14 @@ int oracle_embedding_bag(int F, int B, const int *dims, const int *pools,
     }
     free(col);
     return ORACLE_OK;
+}
+
+int oracle_embedding_bag(int F, int B, const int *dims, const int *pools,
+                         const float *const *tables, const int64_t *rows,
+                         const int32_t *indices, const int32_t *offsets,
+                         double *out, int nthreads) {
+    return oracle_embedding_bag_typed(F, B, dims, pools, NULL, (const void *const *)tables, rows, indices, offsets,
+                                      out, nthreads);
 }
 
 /*

@@ -21,7 +21,8 @@ P = ctypes.POINTER
 
 class FeatureSpec(ctypes.Structure):
     _fields_ = [('num_rows', ctypes.c_int64), ('dim', ctypes.c_int32), ('pool', ctypes.c_int32),
-                ('mean_len', ctypes.c_float), ('max_len', ctypes.c_float), ('coverage', ctypes.c_float)]
+                ('mean_len', ctypes.c_float), ('max_len', ctypes.c_float), ('coverage', ctypes.c_float),
+                ('dtype', ctypes.c_int32)]
 
 
 class Schedule(ctypes.Structure):
@@ -30,7 +31,7 @@ class Schedule(ctypes.Structure):
 
 class CatalogInfo(ctypes.Structure):
     _fields_ = [('family', ctypes.c_int32), ('group', ctypes.c_int32), ('vec', ctypes.c_int32),
-                ('cols', ctypes.c_int32), ('unroll', ctypes.c_int32)]
+                ('cols', ctypes.c_int32), ('unroll', ctypes.c_int32), ('dtype', ctypes.c_int32)]
 
 
 class TuneOptions(ctypes.Structure):
@@ -76,6 +77,7 @@ SIGNATURES = {
     'recflex_catalog_size': (c_int32, []),
     'recflex_catalog_info': (c_int32, [c_int32, P(CatalogInfo)]),
     'recflex_catalog_valid': (c_int32, [c_int32, c_int32]),
+    'recflex_catalog_valid_dtype': (c_int32, [c_int32, c_int32, c_int32]),
     'recflex_occupancy_check': (c_int32, [c_int32, c_int32, P(c_int32), P(c_int32), P(c_int32)]),
     'recflex_debug_task_map': (c_int32, [c_void_p, c_void_p, c_int32, P(c_int32), P(c_int32), c_int64, c_void_p]),
     'recflex_validate': (c_int32, [c_void_p, c_void_p, c_void_p, c_int32, c_void_p]),

@@ -26,18 +26,23 @@ __device__ __forceinline__ void dispatch_schedule(int id, const TaskCtx &x, floa
     if constexpr (I < kCatalogSize) {
         if (id == I) {
             constexpr CatalogEntry e = kCatalog[I];
+            // fp32 entries: G compiled in (the tuned path); reduced-precision
+            // entries share one instantiation per (family, ET, VEC, C, U) with
+            // G passed at run time -- ptxas time grows superlinearly with the
+            // number of functions in the kernel's call graph.
+            constexpr int GT = (e.ET == RECFLEX_DTYPE_F32) ? e.G : 0;
             if constexpr (e.family == RECFLEX_FAMILY_GROUP)
-                sched_group<e.G, e.VEC, e.C, e.U>(x.table, x.offs, x.idx, x.out, x.dim, x.pool, x.ro, x.s0, x.s1,
-                                                  bag_ctr);
+                sched_group<e.ET, GT, e.VEC, e.C, e.U>(x.table, x.rowb, e.G, x.offs, x.idx, x.out, x.dim, x.pool, x.ro,
+                                                        x.s0, x.s1, bag_ctr);
             else if constexpr (e.family == RECFLEX_FAMILY_FLAT)
-                sched_flat<e.G, e.VEC, e.U>(x.table, x.offs, x.idx, x.out, x.dim, x.pool, x.ro, x.s0, x.s1,
-                                            bag_ctr);
+                sched_flat<e.ET, GT, e.VEC, e.U>(x.table, x.rowb, e.G, x.offs, x.idx, x.out, x.dim, x.pool, x.ro, x.s0,
+                                                  x.s1, bag_ctr);
             else if constexpr (e.family == RECFLEX_FAMILY_BULK)
-                sched_bulk<e.U>(x.table, x.offs, x.idx, x.out, x.dim, x.pool, x.ro, x.s0, x.s1, bag_ctr,
-                                x.wsmem, x.wbytes);
+                sched_bulk<e.U>(reinterpret_cast<const float *>(x.table), x.offs, x.idx, x.out, x.dim, x.pool, x.ro,
+                                x.s0, x.s1, bag_ctr, x.wsmem, x.wbytes);
             else
-                sched_block<e.G, e.VEC, e.C, e.U>(x.table, x.offs, x.idx, x.out, x.dim, x.pool, x.ro, x.s0,
-                                                  x.s1, red);
+                sched_block<e.ET, GT, e.VEC, e.C, e.U>(x.table, x.rowb, e.G, x.offs, x.idx, x.out, x.dim, x.pool, x.ro,
+                                                        x.s0, x.s1, red);
         } else {
             dispatch_schedule<I + 1>(id, x, red, bag_ctr);
         }
@@ -46,13 +51,15 @@ __device__ __forceinline__ void dispatch_schedule(int id, const TaskCtx &x, floa
 
 // Single call site for the whole catalog: the kernel calls this once per task
 // (few live values cross the call), and it branches to the schedule.
-static __device__ __noinline__ void dispatch_task(int id, const float *T, const int32_t *offs, const int32_t *idx, float *out,
+static __device__ __noinline__ void dispatch_task(int id, const char *T, unsigned rowb, const int32_t *offs,
+                                                  const int32_t *idx, float *out,
                                            int d, int pool, const OutRoute ro, int s0, int s1, float *red, int *bag,
                                            unsigned char *wsmem, int wbytes) {
     TaskCtx x;
     x.wsmem = wsmem;
     x.wbytes = wbytes;
     x.table = T;
+    x.rowb = rowb;
     x.offs = offs;
     x.idx = idx;
     x.out = out;
@@ -68,7 +75,7 @@ constexpr int kRedFloats = 8 * 256;  // BLOCK family: [8 warps][SPAN <= 256]
 constexpr int kWarps = kBlockThreads / 32;
 constexpr int kRing = 8;             // task slots in flight per CTA
 
-#define RECFLEX_FAMILY_OF(fam, g, v, c, u) fam,
+#define RECFLEX_FAMILY_OF(fam, et, g, v, c, u) fam,
 __constant__ signed char kFamilyDev[kCatalogSize] = {RECFLEX_CATALOG(RECFLEX_FAMILY_OF)};
 #undef RECFLEX_FAMILY_OF
 
@@ -235,7 +242,7 @@ __global__ void __launch_bounds__(kBlockThreads, KOCC) recflex_fused_kernel(Fuse
         ro.rows = a.route_rows;
         ro.colofs = a.col_base + fd.col;
         ro.stride = a.out_stride;
-        dispatch_task(fd.sched, fd.table, a.offsets + (size_t)fd.in_feature * a.B, a.indices, a.out + fd.col, fd.dim,
+        dispatch_task(fd.sched, static_cast<const char *>(fd.table), (unsigned)fd.row_bytes, a.offsets + (size_t)fd.in_feature * a.B, a.indices, a.out + fd.col, fd.dim,
                       fd.pool, ro, vld(&S.s0), vld(&S.s1), red, &S.bag, wsmem, wbytes);
         if (cta_wide) __syncthreads();
         __syncwarp();

@@ -38,12 +38,21 @@ static int next_pow2(int v) {
     return p;
 }
 
-int find_catalog(int family, int G, int VEC, int C, int U) {
+int find_catalog(int family, int G, int VEC, int C, int U, int ET) {
     for (int i = 0; i < kCatalogSize; ++i) {
         const CatalogEntry &e = kCatalog[i];
-        if (e.family == family && e.G == G && e.VEC == VEC && e.C == C && e.U == U) return i;
+        if (e.family == family && e.ET == ET && e.G == G && e.VEC == VEC && e.C == C && e.U == U) return i;
     }
     return -1;
+}
+
+int row_bytes_of(int dim, int dtype) {
+    switch (dtype) {
+        case RECFLEX_DTYPE_F16:
+        case RECFLEX_DTYPE_BF16: return 2 * dim;
+        case RECFLEX_DTYPE_I8: return (int)RECFLEX_I8_ROW_BYTES(dim);
+        default: return 4 * dim;
+    }
 }
 
 // samples per task for sample-partitioned tasks: about `target` expected
@@ -77,6 +86,24 @@ recflex_schedule_t default_schedule(const recflex_feature_spec_t &spec, int targ
     recflex_schedule_t s = {0, 0, 1};
     const int d = spec.dim;
     int id = -1;
+    if (spec.dtype != RECFLEX_DTYPE_F32) {
+        // Reduced-precision rows: the same shapes in BYTES as the fp32 rule
+        // below -- 32-byte lanes for short rows (16-bit) / 16-byte lanes
+        // (int8), one lane group per row, U = 2 for one-hot bags.
+        const int et = spec.dtype;
+        const int U = spec.mean_len >= 2.5f ? 4 : 2;
+        if (et == RECFLEX_DTYPE_I8) {
+            if (d % 16 == 0) id = find_catalog(RECFLEX_FAMILY_GROUP, std::min(32, next_pow2(d / 16)), 16, 1, U, et);
+            if (id < 0) id = find_catalog(RECFLEX_FAMILY_GROUP, std::min(16, next_pow2(d / 8)), 8, 1, U, et);
+        } else {
+            if (d % 16 == 0 && d <= 128) id = find_catalog(RECFLEX_FAMILY_GROUP, d / 16, 16, 1, 2, et);
+            if (id < 0 && d % 8 == 0) id = find_catalog(RECFLEX_FAMILY_GROUP, std::min(32, next_pow2(d / 8)), 8, 1, U, et);
+            if (id < 0) id = find_catalog(RECFLEX_FAMILY_GROUP, std::min(8, next_pow2(d / 4)), 4, 1, 4, et);
+        }
+        s.sched_id = id;
+        s.per_block = id >= 0 ? samples_per_task_default(id, spec.mean_len, spec.coverage, target) : 1;
+        return s;
+    }
     // Untuned defaults follow what the tuner picks most on B200 (sharded1000 /
     // heavy): rows up to 64 floats -> 256-bit loads with d/8 lanes per bag
     // (more bags in flight per warp), U = 2; wider rows -> a warp (or more
@@ -106,12 +133,12 @@ int slots_for(int max_batch, float max_len) {
     return (int)std::max(64.0, need);
 }
 
-bool schedule_valid_for(const recflex_schedule_t &s, int dim, int col, int d_tot) {
+bool schedule_valid_for(const recflex_schedule_t &s, int dim, int dtype, int col, int d_tot) {
     if (s.sched_id < 0 || s.sched_id >= kCatalogSize) return false;
     if (s.part < 0 || s.part > 2) return false;
     if (s.per_block < 1) return false;
     const CatalogEntry &e = kCatalog[s.sched_id];
-    if (!catalog_valid(e, dim)) return false;
+    if (!catalog_valid(e, dim, dtype)) return false;
     // vector stores need 16-byte aligned output columns
     if (e.VEC > 1 && ((col % 4) != 0 || (d_tot % 4) != 0)) return false;
     return true;
@@ -269,12 +296,18 @@ recflex_status_t recflex_catalog_info(int32_t id, recflex_catalog_info_t *info) 
     info->vec = e.VEC;
     info->cols = e.C;
     info->unroll = e.U;
+    info->dtype = e.ET;
     return RECFLEX_OK;
 }
 
 int32_t recflex_catalog_valid(int32_t id, int32_t dim) {
     if (id < 0 || id >= kCatalogSize) return 0;
     return catalog_valid(kCatalog[id], dim) ? 1 : 0;
+}
+
+int32_t recflex_catalog_valid_dtype(int32_t id, int32_t dim, int32_t dtype) {
+    if (id < 0 || id >= kCatalogSize) return 0;
+    return catalog_valid(kCatalog[id], dim, dtype) ? 1 : 0;
 }
 
 static void plan_free_device(recflex_plan_s *p) {
@@ -312,6 +345,10 @@ recflex_status_t recflex_plan_create(const recflex_feature_spec_t *specs, int32_
         if (s.pool != RECFLEX_POOL_SUM && s.pool != RECFLEX_POOL_MEAN) return RECFLEX_ERR_INVALID_ARG;
         if (!(s.mean_len >= 0.f) || !(s.max_len >= 0.f) || !(s.coverage >= 0.f) || s.coverage > 1.f)
             return RECFLEX_ERR_INVALID_ARG;
+        if (s.dtype < RECFLEX_DTYPE_F32 || s.dtype > RECFLEX_DTYPE_I8) return RECFLEX_ERR_INVALID_ARG;
+        if ((s.dtype == RECFLEX_DTYPE_F16 || s.dtype == RECFLEX_DTYPE_BF16) && s.dim % 4 != 0)
+            return RECFLEX_ERR_INVALID_ARG;
+        if (s.dtype == RECFLEX_DTYPE_I8 && s.dim % 8 != 0) return RECFLEX_ERR_INVALID_ARG;
         d_tot += s.dim;
     }
     if (d_tot >= (int64_t(1) << 31) || (int64_t)max_batch * d_tot >= (int64_t(1) << 40)) return RECFLEX_ERR_INVALID_ARG;
@@ -337,6 +374,8 @@ recflex_status_t recflex_plan_create(const recflex_feature_spec_t *specs, int32_
         d.col = (int32_t)col;
         d.pool = specs[f].pool;
         d.in_feature = f;
+        d.dtype = specs[f].dtype;
+        d.row_bytes = row_bytes_of(specs[f].dim, specs[f].dtype);
         d.cap = 0;
         d.slots = slots_for(max_batch, specs[f].max_len);
         d.slot_base = (int32_t)slot;
@@ -351,7 +390,12 @@ recflex_status_t recflex_plan_create(const recflex_feature_spec_t *specs, int32_
     p->task_lookups = task_lookups_target(specs, F, max_batch, p->num_sms);
     for (int f = 0; f < F; ++f) {
         recflex_schedule_t s = default_schedule(specs[f], p->task_lookups);
-        if (!schedule_valid_for(s, p->desc[f].dim, p->desc[f].col, (int)d_tot)) {
+        if (!schedule_valid_for(s, p->desc[f].dim, p->desc[f].dtype, p->desc[f].col, (int)d_tot)) {
+            if (specs[f].dtype != RECFLEX_DTYPE_F32) {
+                // reduced-precision entries need a 16-byte-aligned output column
+                delete p;
+                return RECFLEX_ERR_NOT_SUPPORTED;
+            }
             s.sched_id = find_catalog(RECFLEX_FAMILY_GROUP, std::min(32, next_pow2(specs[f].dim)), 1, 1, 4);
             s.per_block = samples_per_task_default(s.sched_id, specs[f].mean_len, specs[f].coverage, p->task_lookups);
         }
@@ -391,10 +435,10 @@ void recflex_destroy(recflex_plan_t p) {
     delete p;
 }
 
-static recflex_status_t sync_tables(recflex_plan_s *p, const float *const *tables, cudaStream_t stream) {
+static recflex_status_t sync_tables(recflex_plan_s *p, const void *const *tables, cudaStream_t stream) {
     bool changed = false;
     for (int f = 0; f < p->F; ++f) {
-        const float *t = tables[f];
+        const void *t = tables[f];
         if (!t) return RECFLEX_ERR_INVALID_ARG;
         if (t != p->tables[f]) {
             const CatalogEntry &e = kCatalog[p->desc[f].sched];
@@ -409,7 +453,7 @@ static recflex_status_t sync_tables(recflex_plan_s *p, const float *const *table
 }
 
 recflex_status_t recflex_forward(recflex_plan_t p, const int32_t *indices, const int32_t *offsets, int32_t B,
-                                 const float *const *tables, float *out, void *stream_) {
+                                 const void *const *tables, float *out, void *stream_) {
     if (!p || !tables) return RECFLEX_ERR_INVALID_ARG;
     if (B < 0 || B > p->max_batch) return RECFLEX_ERR_INVALID_ARG;
     if (B == 0) return RECFLEX_OK;
@@ -440,7 +484,7 @@ recflex_status_t recflex_forward(recflex_plan_t p, const int32_t *indices, const
 }
 
 recflex_status_t recflex_forward_routed(recflex_plan_t p, const int32_t *indices, const int32_t *offsets, int32_t B,
-                                        const float *const *tables, float *const *host_dst, int32_t num_dst,
+                                        const void *const *tables, float *const *host_dst, int32_t num_dst,
                                         int32_t rows_per_dst, int32_t dst_stride, int32_t col_base, void *stream_) {
     if (!p || !tables || !host_dst || num_dst <= 0 || num_dst > 1024 || rows_per_dst <= 0 || dst_stride <= 0 ||
         col_base < 0 || col_base + p->d_tot > dst_stride)
@@ -513,7 +557,7 @@ recflex_status_t recflex_ipc_close(void *d_ptr) {
 }
 
 recflex_status_t recflex_forward_host(recflex_plan_t p, const int32_t *h_indices, int64_t nnz, const int32_t *h_offsets,
-                                      int32_t B, const float *const *tables, float *h_out, void *stream_) {
+                                      int32_t B, const void *const *tables, float *h_out, void *stream_) {
     if (!p || !tables || B < 0 || B > p->max_batch || nnz < 0) return RECFLEX_ERR_INVALID_ARG;
     if (B == 0) return RECFLEX_OK;
     if (!h_offsets || !h_out || (nnz > 0 && !h_indices)) return RECFLEX_ERR_INVALID_ARG;
@@ -569,7 +613,8 @@ recflex_status_t recflex_get_schedule(recflex_plan_t p, int32_t f, recflex_sched
 
 recflex_status_t recflex_set_schedule(recflex_plan_t p, int32_t f, const recflex_schedule_t *s) {
     if (!p || !s || f < 0 || f >= p->F) return RECFLEX_ERR_INVALID_ARG;
-    if (!schedule_valid_for(*s, p->desc[f].dim, p->desc[f].col, (int)p->d_tot)) return RECFLEX_ERR_INVALID_ARG;
+    if (!schedule_valid_for(*s, p->desc[f].dim, p->desc[f].dtype, p->desc[f].col, (int)p->d_tot))
+        return RECFLEX_ERR_INVALID_ARG;
     p->desc[f].sched = s->sched_id;
     p->desc[f].part = s->part;
     p->desc[f].per_block = s->per_block;
@@ -591,7 +636,7 @@ recflex_status_t recflex_get_occupancy(recflex_plan_t p, int32_t *k) {
 
 recflex_status_t recflex_occupancy_check(int32_t device, int32_t k, int32_t *active, int32_t *regs, int32_t *spill) {
     if (k < 1 || k > kMaxOcc) return RECFLEX_ERR_INVALID_ARG;
-    recflex_feature_spec_t spec = {1000, 16, 0, 1.f, 1.f, 1.f};
+    recflex_feature_spec_t spec = {1000, 16, 0, 1.f, 1.f, 1.f, 0};
     recflex_plan_t p = nullptr;
     recflex_status_t st = recflex_plan_create(&spec, 1, 1, device, &p);
     if (st != RECFLEX_OK) return st;
@@ -782,7 +827,9 @@ recflex_status_t recflex_plan_import(recflex_plan_t p, const char *json) {
     long v = 0;
     if (!c) return RECFLEX_ERR_INVALID_ARG;
     c += 14;
-    if (!parse_int_after(c, &v) || v != kCatalogSize) return RECFLEX_ERR_NOT_SUPPORTED;
+    // the catalog is append-only: a plan exported with a smaller catalog names
+    // the same entries
+    if (!parse_int_after(c, &v) || v < 1 || v > kCatalogSize) return RECFLEX_ERR_NOT_SUPPORTED;
     c = std::strstr(json, "\"num_features\"");
     if (!c) return RECFLEX_ERR_INVALID_ARG;
     c += 14;
@@ -806,7 +853,8 @@ recflex_status_t recflex_plan_import(recflex_plan_t p, const char *json) {
         if (!parse_int_after(c, &a) || !parse_int_after(c, &b) || !parse_int_after(c, &d))
             return RECFLEX_ERR_INVALID_ARG;
         ss[f] = {(int32_t)a, (int32_t)b, (int32_t)d};
-        if (!schedule_valid_for(ss[f], p->desc[f].dim, p->desc[f].col, (int)p->d_tot)) return RECFLEX_ERR_INVALID_ARG;
+        if (!schedule_valid_for(ss[f], p->desc[f].dim, p->desc[f].dtype, p->desc[f].col, (int)p->d_tot))
+            return RECFLEX_ERR_INVALID_ARG;
     }
     for (int f = 0; f < p->F; ++f) recflex_set_schedule(p, f, &ss[f]);
     p->k = k;

@@ -42,7 +42,7 @@ struct recflex_plan_s {
     std::vector<recflex_feature_spec_t> specs;
     std::vector<recflex::FeatureDesc> desc;  // host mirror
     std::vector<int32_t> part1;              // features with part == 1
-    std::vector<const float *> tables;       // cached table pointers
+    std::vector<const void *> tables;        // cached table pointers
     int k = 4;
     int task_lookups = 4096;  // lookups per task targeted by the default schedules
     bool desc_dirty = true;
@@ -89,9 +89,10 @@ int min_dyn_smem(int F);
 recflex_status_t run_pipeline(recflex_plan_s *p, const Exec &ex, const int32_t *indices, const int32_t *offsets, int B,
                               float *out, int out_stride, int k, cudaStream_t stream, EventTriple *ev);
 recflex_status_t upload_desc(recflex_plan_s *p, cudaStream_t stream);
-bool schedule_valid_for(const recflex_schedule_t &s, int dim, int col, int d_tot);
+bool schedule_valid_for(const recflex_schedule_t &s, int dim, int dtype, int col, int d_tot);
+int row_bytes_of(int dim, int dtype);
 recflex_schedule_t default_schedule(const recflex_feature_spec_t &spec, int target);
-int find_catalog(int family, int G, int VEC, int C, int U);
+int find_catalog(int family, int G, int VEC, int C, int U, int ET = 0);
 int samples_per_task_default(int sched_id, float mean_len, float coverage, int target);
 int slots_for(int max_batch, float max_len);
 

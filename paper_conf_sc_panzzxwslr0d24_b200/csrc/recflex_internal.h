@@ -14,7 +14,7 @@ constexpr int kSmemBlockStartCap = 4096;   // features whose block_start fits in
 // Per-feature device descriptor: the paper's `args + arg_offsets[f]` and
 // `schedule_map[f]` (Fig. 8) folded into one record.
 struct __align__(16) FeatureDesc {
-    const float *table;   // T_f, [rows][dim]
+    const void *table;    // T_f, [rows][row_bytes] in the feature's dtype
     int64_t rows;
     int32_t dim;
     int32_t col;          // col_f
@@ -26,6 +26,8 @@ struct __align__(16) FeatureDesc {
     int32_t slots;        // reserved task-range slots (part 1), incl. sentinel
     int32_t slot_base;    // first slot of this feature in task_range scratch (part 1)
     int32_t in_feature;   // which KJT feature slot this descriptor reads (identity for plans)
+    int32_t row_bytes;    // bytes per table row (d*4, d*2, or RECFLEX_I8_ROW_BYTES(d))
+    int32_t dtype;        // recflex_dtype_t (the schedule's entry has the same ET)
 };
 static_assert(sizeof(FeatureDesc) == 64, "FeatureDesc layout");
 
@@ -73,72 +75,101 @@ struct FusedArgs {
 };
 
 // ---------------------------------------------------------------------------
-// Schedule catalog: X(family, G, VEC, C, U).  The id of an entry is its
+// Schedule catalog: X(family, ET, G, VEC, C, U), ET = recflex_dtype_t of the rows.  The id of an entry is its
 // position.  Hand-written templates ("schedule templates").
 // ---------------------------------------------------------------------------
 #define RECFLEX_CATALOG(X)                                                      \
     /* GROUP, 128-bit rows, one column chunk per lane */                        \
-    X(0, 1, 4, 1, 2) X(0, 1, 4, 1, 4) X(0, 1, 4, 1, 8)                          \
-    X(0, 2, 4, 1, 2) X(0, 2, 4, 1, 4) X(0, 2, 4, 1, 8)                          \
-    X(0, 4, 4, 1, 2) X(0, 4, 4, 1, 4) X(0, 4, 4, 1, 8)                          \
-    X(0, 8, 4, 1, 2) X(0, 8, 4, 1, 4) X(0, 8, 4, 1, 8)                          \
-    X(0, 16, 4, 1, 2) X(0, 16, 4, 1, 4) X(0, 16, 4, 1, 8)                       \
-    X(0, 32, 4, 1, 2) X(0, 32, 4, 1, 4) X(0, 32, 4, 1, 8)                       \
+    X(0, 0, 1, 4, 1, 2) X(0, 0, 1, 4, 1, 4) X(0, 0, 1, 4, 1, 8)                          \
+    X(0, 0, 2, 4, 1, 2) X(0, 0, 2, 4, 1, 4) X(0, 0, 2, 4, 1, 8)                          \
+    X(0, 0, 4, 4, 1, 2) X(0, 0, 4, 4, 1, 4) X(0, 0, 4, 4, 1, 8)                          \
+    X(0, 0, 8, 4, 1, 2) X(0, 0, 8, 4, 1, 4) X(0, 0, 8, 4, 1, 8)                          \
+    X(0, 0, 16, 4, 1, 2) X(0, 0, 16, 4, 1, 4) X(0, 0, 16, 4, 1, 8)                       \
+    X(0, 0, 32, 4, 1, 2) X(0, 0, 32, 4, 1, 4) X(0, 0, 32, 4, 1, 8)                       \
     /* GROUP, 128-bit rows, two column chunks per lane */                       \
-    X(0, 1, 4, 2, 2) X(0, 1, 4, 2, 4)                                           \
-    X(0, 2, 4, 2, 2) X(0, 2, 4, 2, 4)                                           \
-    X(0, 4, 4, 2, 2) X(0, 4, 4, 2, 4)                                           \
-    X(0, 8, 4, 2, 2) X(0, 8, 4, 2, 4)                                           \
-    X(0, 16, 4, 2, 2) X(0, 16, 4, 2, 4)                                         \
-    X(0, 32, 4, 2, 2) X(0, 32, 4, 2, 4)                                         \
+    X(0, 0, 1, 4, 2, 2) X(0, 0, 1, 4, 2, 4)                                           \
+    X(0, 0, 2, 4, 2, 2) X(0, 0, 2, 4, 2, 4)                                           \
+    X(0, 0, 4, 4, 2, 2) X(0, 0, 4, 4, 2, 4)                                           \
+    X(0, 0, 8, 4, 2, 2) X(0, 0, 8, 4, 2, 4)                                           \
+    X(0, 0, 16, 4, 2, 2) X(0, 0, 16, 4, 2, 4)                                         \
+    X(0, 0, 32, 4, 2, 2) X(0, 0, 32, 4, 2, 4)                                         \
     /* GROUP, 256-bit rows (LDG.256) */                                         \
-    X(0, 1, 8, 1, 2) X(0, 1, 8, 1, 4)                                           \
-    X(0, 2, 8, 1, 2) X(0, 2, 8, 1, 4)                                           \
-    X(0, 4, 8, 1, 2) X(0, 4, 8, 1, 4)                                           \
-    X(0, 8, 8, 1, 2) X(0, 8, 8, 1, 4)                                           \
-    X(0, 16, 8, 1, 2) X(0, 16, 8, 1, 4)                                         \
-    X(0, 32, 8, 1, 2) X(0, 32, 8, 1, 4)                                         \
+    X(0, 0, 1, 8, 1, 2) X(0, 0, 1, 8, 1, 4)                                           \
+    X(0, 0, 2, 8, 1, 2) X(0, 0, 2, 8, 1, 4)                                           \
+    X(0, 0, 4, 8, 1, 2) X(0, 0, 4, 8, 1, 4)                                           \
+    X(0, 0, 8, 8, 1, 2) X(0, 0, 8, 8, 1, 4)                                           \
+    X(0, 0, 16, 8, 1, 2) X(0, 0, 16, 8, 1, 4)                                         \
+    X(0, 0, 32, 8, 1, 2) X(0, 0, 32, 8, 1, 4)                                         \
     /* GROUP, scalar rows (any dim / alignment) */                              \
-    X(0, 1, 1, 1, 4) X(0, 2, 1, 1, 4) X(0, 4, 1, 1, 4)                          \
-    X(0, 8, 1, 1, 4) X(0, 16, 1, 1, 4) X(0, 32, 1, 1, 4)                        \
+    X(0, 0, 1, 1, 1, 4) X(0, 0, 2, 1, 1, 4) X(0, 0, 4, 1, 1, 4)                          \
+    X(0, 0, 8, 1, 1, 4) X(0, 0, 16, 1, 1, 4) X(0, 0, 32, 1, 1, 4)                        \
     /* BLOCK: whole CTA on one bag, 128-bit rows */                             \
-    X(1, 1, 4, 1, 4) X(1, 2, 4, 1, 4) X(1, 4, 4, 1, 4)                          \
-    X(1, 8, 4, 1, 4) X(1, 16, 4, 1, 4) X(1, 32, 4, 1, 2) X(1, 32, 4, 1, 4)     \
+    X(1, 0, 1, 4, 1, 4) X(1, 0, 2, 4, 1, 4) X(1, 0, 4, 4, 1, 4)                          \
+    X(1, 0, 8, 4, 1, 4) X(1, 0, 16, 4, 1, 4) X(1, 0, 32, 4, 1, 2) X(1, 0, 32, 4, 1, 4)     \
     /* BLOCK, 256-bit rows */                                                   \
-    X(1, 16, 8, 1, 2) X(1, 16, 8, 1, 4)                                         \
+    X(1, 0, 16, 8, 1, 2) X(1, 0, 16, 8, 1, 4)                                         \
     /* FLAT: runs of bags walked as one lookup range, 128-bit rows */           \
-    X(2, 1, 4, 1, 2) X(2, 1, 4, 1, 4) X(2, 2, 4, 1, 2) X(2, 2, 4, 1, 4)         \
-    X(2, 4, 4, 1, 2) X(2, 4, 4, 1, 4) X(2, 8, 4, 1, 2) X(2, 8, 4, 1, 4)         \
-    X(2, 16, 4, 1, 2) X(2, 16, 4, 1, 4) X(2, 32, 4, 1, 2) X(2, 32, 4, 1, 4)     \
+    X(2, 0, 1, 4, 1, 2) X(2, 0, 1, 4, 1, 4) X(2, 0, 2, 4, 1, 2) X(2, 0, 2, 4, 1, 4)         \
+    X(2, 0, 4, 4, 1, 2) X(2, 0, 4, 4, 1, 4) X(2, 0, 8, 4, 1, 2) X(2, 0, 8, 4, 1, 4)         \
+    X(2, 0, 16, 4, 1, 2) X(2, 0, 16, 4, 1, 4) X(2, 0, 32, 4, 1, 2) X(2, 0, 32, 4, 1, 4)     \
     /* FLAT, 256-bit rows */                                                    \
-    X(2, 1, 8, 1, 2) X(2, 1, 8, 1, 4) X(2, 2, 8, 1, 2) X(2, 2, 8, 1, 4)         \
-    X(2, 4, 8, 1, 2) X(2, 4, 8, 1, 4) X(2, 8, 8, 1, 2) X(2, 8, 8, 1, 4)         \
-    X(2, 16, 8, 1, 2) X(2, 16, 8, 1, 4) RECFLEX_CATALOG_EXPERIMENTAL(X)
+    X(2, 0, 1, 8, 1, 2) X(2, 0, 1, 8, 1, 4) X(2, 0, 2, 8, 1, 2) X(2, 0, 2, 8, 1, 4)         \
+    X(2, 0, 4, 8, 1, 2) X(2, 0, 4, 8, 1, 4) X(2, 0, 8, 8, 1, 2) X(2, 0, 8, 8, 1, 4)         \
+    X(2, 0, 16, 8, 1, 2) X(2, 0, 16, 8, 1, 4) RECFLEX_CATALOG_EXPERIMENTAL(X)        \
+    RECFLEX_CATALOG_LOWP(X)
+#define RECFLEX_CATALOG_LOWP(X) RECFLEX_CATALOG_HALF(X, 1) RECFLEX_CATALOG_HALF(X, 2) RECFLEX_CATALOG_I8(X)
+
+// Reduced-precision rows, appended so the fp32 ids above
+// stay stable.  VEC counts ELEMENTS per lane per load: for 16-bit types
+// 4 -> 64-bit, 8 -> 128-bit, 16 -> 256-bit loads; for int8 8 -> 64-bit,
+// 16 -> 128-bit.  Accumulation is fp32 as for float32 rows.
+#define RECFLEX_CATALOG_HALF(X, T)                                              \
+    X(0, T, 1, 8, 1, 2) X(0, T, 1, 8, 1, 4) X(0, T, 2, 8, 1, 2) X(0, T, 2, 8, 1, 4) \
+    X(0, T, 4, 8, 1, 2) X(0, T, 4, 8, 1, 4) X(0, T, 8, 8, 1, 2) X(0, T, 8, 8, 1, 4) \
+    X(0, T, 16, 8, 1, 2) X(0, T, 16, 8, 1, 4) X(0, T, 32, 8, 1, 2) X(0, T, 32, 8, 1, 4) \
+    X(0, T, 1, 16, 1, 2) X(0, T, 1, 16, 1, 4) X(0, T, 2, 16, 1, 2) X(0, T, 2, 16, 1, 4) \
+    X(0, T, 4, 16, 1, 2) X(0, T, 4, 16, 1, 4) X(0, T, 8, 16, 1, 2) X(0, T, 8, 16, 1, 4) \
+    X(0, T, 16, 16, 1, 2) X(0, T, 16, 16, 1, 4) X(0, T, 32, 16, 1, 2) X(0, T, 32, 16, 1, 4) \
+    X(0, T, 1, 4, 1, 4) X(0, T, 2, 4, 1, 4) X(0, T, 4, 4, 1, 4) X(0, T, 8, 4, 1, 4)  \
+    X(1, T, 16, 8, 1, 4) X(1, T, 8, 16, 1, 4)                                   \
+    X(2, T, 1, 8, 1, 4) X(2, T, 2, 8, 1, 4) X(2, T, 4, 8, 1, 4) X(2, T, 8, 8, 1, 4)
+#define RECFLEX_CATALOG_I8(X)                                                   \
+    X(0, 3, 1, 8, 1, 2) X(0, 3, 1, 8, 1, 4) X(0, 3, 2, 8, 1, 2) X(0, 3, 2, 8, 1, 4) \
+    X(0, 3, 4, 8, 1, 2) X(0, 3, 4, 8, 1, 4) X(0, 3, 8, 8, 1, 2) X(0, 3, 8, 8, 1, 4) \
+    X(0, 3, 16, 8, 1, 2) X(0, 3, 16, 8, 1, 4)                                  \
+    X(0, 3, 1, 16, 1, 2) X(0, 3, 1, 16, 1, 4) X(0, 3, 2, 16, 1, 2) X(0, 3, 2, 16, 1, 4) \
+    X(0, 3, 4, 16, 1, 2) X(0, 3, 4, 16, 1, 4) X(0, 3, 8, 16, 1, 2) X(0, 3, 8, 16, 1, 4) \
+    X(0, 3, 16, 16, 1, 2) X(0, 3, 16, 16, 1, 4) X(0, 3, 32, 16, 1, 2) X(0, 3, 32, 16, 1, 4) \
+    X(1, 3, 8, 16, 1, 4)                                                        \
+    X(2, 3, 1, 16, 1, 4) X(2, 3, 2, 16, 1, 4) X(2, 3, 4, 16, 1, 4) X(2, 3, 8, 16, 1, 4)
 
 // BULK (rows by TMA bulk copy into smem stages) is built only on request:
 // per-row cp.async.bulk of random rows from multi-GB tables measured 10-100x
 // slower than register loads on B200 (the copy engine's address translation
 // thrashes), see DESIGN.md §6.
 #ifdef RECFLEX_EXPERIMENTAL_BULK
-#define RECFLEX_CATALOG_EXPERIMENTAL(X) X(3, 32, 4, 1, 2) X(3, 32, 4, 1, 4) X(3, 32, 4, 1, 8)
+#define RECFLEX_CATALOG_EXPERIMENTAL(X) X(3, 0, 32, 4, 1, 2) X(3, 0, 32, 4, 1, 4) X(3, 0, 32, 4, 1, 8)
 #else
 #define RECFLEX_CATALOG_EXPERIMENTAL(X)
 #endif
 
 struct CatalogEntry {
-    int family, G, VEC, C, U;
+    int family, ET, G, VEC, C, U;
 };
 
-#define RECFLEX_CAT_ENTRY(fam, g, v, c, u) {fam, g, v, c, u},
+#define RECFLEX_CAT_ENTRY(fam, et, g, v, c, u) {fam, et, g, v, c, u},
 static constexpr CatalogEntry kCatalog[] = {RECFLEX_CATALOG(RECFLEX_CAT_ENTRY)};
 #undef RECFLEX_CAT_ENTRY
 constexpr int kCatalogSize = sizeof(kCatalog) / sizeof(kCatalog[0]);
 
-// Can entry e run a feature of dimension d?  (vector width divides d; at least
-// a quarter of the lanes hold real columns; wide rows take several passes)
-inline bool catalog_valid(const CatalogEntry &e, int d) {
+// Can entry e run a feature of dimension d stored as dtype?  (same element
+// type; vector width divides d; at least a quarter of the lanes hold real
+// columns; wide rows take several passes)
+inline bool catalog_valid(const CatalogEntry &e, int d, int dtype = RECFLEX_DTYPE_F32) {
     if (d <= 0) return false;
+    if (e.ET != dtype) return false;
     if (d % e.VEC != 0) return false;
+    if (dtype == RECFLEX_DTYPE_I8 && d % 8 != 0) return false;  // scale/bias 8-byte aligned
     int span = e.G * e.VEC * e.C;
     if (4 * d < span) return false;
     if (e.family == 3 && (d < 32 || d > 128)) return false;  // BULK: 128..512-byte rows, one pass

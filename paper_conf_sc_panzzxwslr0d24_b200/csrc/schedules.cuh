@@ -49,6 +49,116 @@ __device__ __forceinline__ void ld_row<8>(const float *p, float (&v)[8]) {
 
 __device__ __forceinline__ int ld_idx(const int32_t *p) { return __ldg(p); }
 
+// ---- typed row loads -------------------------------------
+// RowFrag<ET, VEC>: VEC consecutive elements of one table row starting at
+// column col, held in registers in their STORED form between the load and
+// the accumulation (so U rows in flight cost U * VEC * sizeof(elem) bytes of
+// registers, not U * VEC floats), widened to fp32 only in add_to.  `row` is
+// the row's first byte (table base + id * row_bytes).  ET = recflex_dtype_t:
+//   F32  : 4/16/32-byte loads
+//   F16  : 8/16/32-byte loads of binary16, exact widening (cvt.f32.f16)
+//   BF16 : same loads, widening = the 16 bits placed in the upper half
+//   I8   : 8/16-byte loads of int8 codes plus the row's float32 scale and bias
+//          (bytes [d, d+8) of the row); value = fma(scale, q, bias) in fp32.
+//          q -> fp32 without I2F: the code byte is placed in the mantissa of
+//          2^23 (PRMT) and 2^23 + 128 subtracted (exact).
+template <int NW>
+__device__ __forceinline__ void ld_words(const void *p, unsigned (&w)[NW]) {
+    if constexpr (NW == 1) {
+        asm("ld.global.nc.L1::no_allocate.b32 %0, [%1];" : "=r"(w[0]) : "l"(p));
+    } else if constexpr (NW == 2) {
+        asm("ld.global.nc.L1::no_allocate.v2.b32 {%0, %1}, [%2];" : "=r"(w[0]), "=r"(w[1]) : "l"(p));
+    } else if constexpr (NW == 4) {
+        asm("ld.global.nc.L1::no_allocate.v4.b32 {%0, %1, %2, %3}, [%4];"
+            : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3])
+            : "l"(p));
+    } else {
+        static_assert(NW == 8, "1, 2, 4 or 8 words");
+        asm("ld.global.nc.L1::no_allocate.v8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
+            : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]), "=r"(w[4]), "=r"(w[5]), "=r"(w[6]), "=r"(w[7])
+            : "l"(p));
+    }
+}
+
+__device__ __forceinline__ float f16_lo(unsigned w) {
+    float f;
+    asm("{\n\t.reg .b16 l, h;\n\tmov.b32 {l, h}, %1;\n\tcvt.f32.f16 %0, l;\n\t}" : "=f"(f) : "r"(w));
+    return f;
+}
+__device__ __forceinline__ float f16_hi(unsigned w) {
+    float f;
+    asm("{\n\t.reg .b16 l, h;\n\tmov.b32 {l, h}, %1;\n\tcvt.f32.f16 %0, h;\n\t}" : "=f"(f) : "r"(w));
+    return f;
+}
+// int8 code (byte k of w) -> fp32, exact: 2^23 + (q + 128) - (2^23 + 128)
+template <int K>
+__device__ __forceinline__ float i8_at(unsigned w) {
+    const unsigned biased = __byte_perm(w ^ 0x80808080u, 0x4B000000u, 0x7640 | K);  // {0x4B,0,0,byte^0x80}
+    return __uint_as_float(biased) - 8388736.0f;
+}
+
+template <int ET, int VEC>
+struct RowFrag;
+
+template <int VEC>
+struct RowFrag<RECFLEX_DTYPE_F32, VEC> {
+    float x[VEC];
+    __device__ __forceinline__ void load(const char *row, int col, int) {
+        ld_row<VEC>(reinterpret_cast<const float *>(row) + col, x);
+    }
+    __device__ __forceinline__ void add_to(float (&acc)[VEC]) const {
+#pragma unroll
+        for (int e = 0; e < VEC; ++e) acc[e] += x[e];
+    }
+};
+
+template <int VEC>
+struct RowFrag<RECFLEX_DTYPE_F16, VEC> {
+    unsigned w[VEC / 2];
+    __device__ __forceinline__ void load(const char *row, int col, int) { ld_words<VEC / 2>(row + 2 * col, w); }
+    __device__ __forceinline__ void add_to(float (&acc)[VEC]) const {
+#pragma unroll
+        for (int i = 0; i < VEC / 2; ++i) {
+            acc[2 * i] += f16_lo(w[i]);
+            acc[2 * i + 1] += f16_hi(w[i]);
+        }
+    }
+};
+
+template <int VEC>
+struct RowFrag<RECFLEX_DTYPE_BF16, VEC> {
+    unsigned w[VEC / 2];
+    __device__ __forceinline__ void load(const char *row, int col, int) { ld_words<VEC / 2>(row + 2 * col, w); }
+    __device__ __forceinline__ void add_to(float (&acc)[VEC]) const {
+#pragma unroll
+        for (int i = 0; i < VEC / 2; ++i) {
+            acc[2 * i] += __uint_as_float(w[i] << 16);
+            acc[2 * i + 1] += __uint_as_float(w[i] & 0xffff0000u);
+        }
+    }
+};
+
+template <int VEC>
+struct RowFrag<RECFLEX_DTYPE_I8, VEC> {
+    static_assert(VEC % 4 == 0, "int8 rows: 4 codes per word");
+    unsigned w[VEC / 4];
+    unsigned sb[2];  // scale, bias
+    __device__ __forceinline__ void load(const char *row, int col, int d) {
+        ld_words<VEC / 4>(row + col, w);
+        ld_words<2>(row + d, sb);  // 8-byte aligned: d % 8 == 0
+    }
+    __device__ __forceinline__ void add_to(float (&acc)[VEC]) const {
+        const float sc = __uint_as_float(sb[0]), bi = __uint_as_float(sb[1]);
+#pragma unroll
+        for (int i = 0; i < VEC / 4; ++i) {
+            acc[4 * i + 0] += fmaf(sc, i8_at<0>(w[i]), bi);
+            acc[4 * i + 1] += fmaf(sc, i8_at<1>(w[i]), bi);
+            acc[4 * i + 2] += fmaf(sc, i8_at<2>(w[i]), bi);
+            acc[4 * i + 3] += fmaf(sc, i8_at<3>(w[i]), bi);
+        }
+    }
+};
+
 template <int VEC>
 __device__ __forceinline__ void st_out(float *p, const float (&v)[VEC]) {
     if constexpr (VEC == 1) {
@@ -56,8 +166,9 @@ __device__ __forceinline__ void st_out(float *p, const float (&v)[VEC]) {
     } else if constexpr (VEC == 4) {
         *reinterpret_cast<float4 *>(p) = make_float4(v[0], v[1], v[2], v[3]);
     } else {
-        reinterpret_cast<float4 *>(p)[0] = make_float4(v[0], v[1], v[2], v[3]);
-        reinterpret_cast<float4 *>(p)[1] = make_float4(v[4], v[5], v[6], v[7]);
+#pragma unroll
+        for (int i = 0; i < VEC / 4; ++i)
+            reinterpret_cast<float4 *>(p)[i] = make_float4(v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
     }
 }
 
@@ -110,7 +221,8 @@ __device__ __forceinline__ float *out_row(float *out, int s, const OutRoute &r) 
 // Everything a schedule needs for one task, passed by value (registers): the
 // paper's `args + arg_offsets[feature_idx]` (Fig. 8 line 17) resolved.
 struct TaskCtx {
-    const float *table;     // T_f
+    const char *table;      // T_f (first byte of row 0)
+    unsigned rowb;          // bytes per row
     const int32_t *offs;    // this feature's B+1 offsets
     const int32_t *idx;     // all lookup IDs
     float *out;             // out + col_f
@@ -125,10 +237,11 @@ struct TaskCtx {
 // ---- GROUP family --------------------------------------------------------
 // One bag [lo, hi) pooled by the G lanes of a group: lane lg holds columns
 // p*SPAN + c*G*VEC + lg*VEC (+0..VEC-1); U rows in flight per lane.
-template <int G, int VEC, int C, int U>
-__device__ __forceinline__ void group_bag(const float *__restrict__ T, const int32_t *__restrict__ idx, int d,
-                                          int pool, float *__restrict__ orow, int lo, int hi, int lg) {
-    constexpr int SPAN = G * VEC * C;
+template <int ET, int GT, int VEC, int C, int U>
+__device__ __forceinline__ void group_bag(const char *__restrict__ T, unsigned rowb, const int32_t *__restrict__ idx, int d,
+                                          int pool, float *__restrict__ orow, int lo, int hi, int lg, int gr) {
+    const int G = GT ? GT : gr;  // GT == 0: lane-group size at run time (see kRuntimeG)
+    const int SPAN = G * VEC * C;
     const int passes = (d + SPAN - 1) / SPAN;
     {
         for (int p = 0; p < passes; ++p) {
@@ -146,7 +259,7 @@ __device__ __forceinline__ void group_bag(const float *__restrict__ T, const int
                 for (int e = 0; e < VEC; ++e) acc[c][e] = 0.f;
 
 #ifdef RECFLEX_FASTLOOP
-            if constexpr (U <= G && G >= 4 && C == 1) {
+            if constexpr (ET == RECFLEX_DTYPE_F32 && GT != 0 && U <= GT && GT >= 4 && C == 1) {
                 if ((p + 1) * SPAN <= d) {
                     // EXPERIMENT, off by default (measured 16% SLOWER on heavy,
                     // 7% on sharded1000): the row addresses of iteration i+1
@@ -156,8 +269,7 @@ __device__ __forceinline__ void group_bag(const float *__restrict__ T, const int
                     // them, so nothing is gained and the loop gets longer.
                     const int lane = threadIdx.x & 31;
                     const unsigned gmask = (G == 32) ? 0xffffffffu : (((1u << G) - 1u) << (lane & ~(G - 1)));
-                    const char *base = reinterpret_cast<const char *>(T + colv[0]);
-                    const unsigned rowb = (unsigned)d * 4u;
+                    const char *base = T + 4 * colv[0];
                     int cb = lo;
                     int cur = (lo + lg < hi) ? ld_idx(idx + lo + lg) : 0;
                     int nxt = (lo + G + lg < hi) ? ld_idx(idx + lo + G + lg) : 0;
@@ -216,7 +328,7 @@ __device__ __forceinline__ void group_bag(const float *__restrict__ T, const int
             }
 #endif
 #ifndef RECFLEX_NO_SHFL_IDX
-            if constexpr (U <= G && G >= 4) {
+            if (U <= G && G >= 4) {
                 // Lookup IDs through registers: lane lg holds ID cb+lg of the
                 // current chunk of G IDs (one coalesced load per chunk) and the
                 // next chunk is already in flight; each iteration broadcasts its
@@ -238,19 +350,18 @@ __device__ __forceinline__ void group_bag(const float *__restrict__ T, const int
                     unsigned id[U];
 #pragma unroll
                     for (int u = 0; u < U; ++u) id[u] = (unsigned)__shfl_sync(gmask, cur, (j - cb) + u, G);
-                    float v[U][C][VEC];
+                    RowFrag<ET, VEC> v[U][C];
 #pragma unroll
                     for (int u = 0; u < U; ++u)
 #pragma unroll
                         for (int c = 0; c < C; ++c)
-                            if (ok[c]) ld_row<VEC>(T + (size_t)id[u] * (unsigned)d + colv[c], v[u][c]);
+                            if (ok[c]) v[u][c].load(T + (size_t)id[u] * rowb, colv[c], d);
 #pragma unroll
                     for (int u = 0; u < U; ++u)
 #pragma unroll
                         for (int c = 0; c < C; ++c)
                             if (ok[c])
-#pragma unroll
-                                for (int e = 0; e < VEC; ++e) acc[c][e] += v[u][c][e];
+                                v[u][c].add_to(acc[c]);
                 }
                 if (j < hi) {
                     if (j - cb >= G) {
@@ -261,20 +372,19 @@ __device__ __forceinline__ void group_bag(const float *__restrict__ T, const int
                     unsigned id[U];
 #pragma unroll
                     for (int u = 0; u < U; ++u) id[u] = (unsigned)__shfl_sync(gmask, cur, (j - cb) + u, G);
-                    float v[U][C][VEC];
+                    RowFrag<ET, VEC> v[U][C];
 #pragma unroll
                     for (int u = 0; u < U; ++u)
 #pragma unroll
                         for (int c = 0; c < C; ++c)
-                            if (u < n && ok[c]) ld_row<VEC>(T + (size_t)id[u] * (unsigned)d + colv[c], v[u][c]);
+                            if (u < n && ok[c]) v[u][c].load(T + (size_t)id[u] * rowb, colv[c], d);
 #pragma unroll
                     for (int u = 0; u < U; ++u)
                         if (u < n)
 #pragma unroll
                             for (int c = 0; c < C; ++c)
                                 if (ok[c])
-#pragma unroll
-                                    for (int e = 0; e < VEC; ++e) acc[c][e] += v[u][c][e];
+                                    v[u][c].add_to(acc[c]);
                 }
 #pragma unroll
                 for (int c = 0; c < C; ++c) {
@@ -296,39 +406,37 @@ __device__ __forceinline__ void group_bag(const float *__restrict__ T, const int
                 int id[U];
 #pragma unroll
                 for (int u = 0; u < U; ++u) id[u] = ld_idx(idx + j + u);
-                float v[U][C][VEC];
+                RowFrag<ET, VEC> v[U][C];
 #pragma unroll
                 for (int u = 0; u < U; ++u)
 #pragma unroll
                     for (int c = 0; c < C; ++c)
-                        if (ok[c]) ld_row<VEC>(T + (size_t)id[u] * d + colv[c], v[u][c]);
+                        if (ok[c]) v[u][c].load(T + (size_t)id[u] * rowb, colv[c], d);
 #pragma unroll
                 for (int u = 0; u < U; ++u)
 #pragma unroll
                     for (int c = 0; c < C; ++c)
                         if (ok[c])
-#pragma unroll
-                            for (int e = 0; e < VEC; ++e) acc[c][e] += v[u][c][e];
+                            v[u][c].add_to(acc[c]);
             }
             if (j < hi) {  // ragged tail of the bag: n < U rows
                 const int n = hi - j;
                 int id[U];
 #pragma unroll
                 for (int u = 0; u < U; ++u) id[u] = (u < n) ? ld_idx(idx + j + u) : 0;
-                float v[U][C][VEC];
+                RowFrag<ET, VEC> v[U][C];
 #pragma unroll
                 for (int u = 0; u < U; ++u)
 #pragma unroll
                     for (int c = 0; c < C; ++c)
-                        if (u < n && ok[c]) ld_row<VEC>(T + (size_t)id[u] * d + colv[c], v[u][c]);
+                        if (u < n && ok[c]) v[u][c].load(T + (size_t)id[u] * rowb, colv[c], d);
 #pragma unroll
                 for (int u = 0; u < U; ++u)
                     if (u < n)
 #pragma unroll
                         for (int c = 0; c < C; ++c)
                             if (ok[c])
-#pragma unroll
-                                for (int e = 0; e < VEC; ++e) acc[c][e] += v[u][c][e];
+                                v[u][c].add_to(acc[c]);
             }
 #pragma unroll
             for (int c = 0; c < C; ++c) {
@@ -346,10 +454,11 @@ __device__ __forceinline__ void group_bag(const float *__restrict__ T, const int
 // its own group; the next bag's offsets are loaded while the current bag is
 // pooled.  Which group pools a bag does not change the bag's arithmetic (rows
 // in ascending lookup order) -> results are independent of the claim order.
-template <int G, int VEC, int C, int U>
-__device__ __noinline__ void sched_group(const float *__restrict__ T, const int32_t *__restrict__ offs,
+template <int ET, int GT, int VEC, int C, int U>
+__device__ __noinline__ void sched_group(const char *__restrict__ T, unsigned rowb, int gr, const int32_t *__restrict__ offs,
                                         const int32_t *__restrict__ idx, float *__restrict__ out, int d, int pool,
                                         const OutRoute ro, int s0, int s1, int *bag_ctr) {
+    const int G = GT ? GT : gr;
     const int lane = threadIdx.x & 31;
     const int lg = lane & (G - 1);
     const unsigned gmask = (G == 32) ? 0xffffffffu : (((1u << G) - 1u) << (lane & ~(G - 1)));
@@ -382,7 +491,7 @@ __device__ __noinline__ void sched_group(const float *__restrict__ T, const int3
             lon = ld_idx(offs + sn);
             hin = ld_idx(offs + sn + 1);
         }
-        group_bag<G, VEC, C, U>(T, idx, d, pool, out_row(out, s, ro), lo, hi, lg);
+        group_bag<ET, GT, VEC, C, U>(T, rowb, idx, d, pool, out_row(out, s, ro), lo, hi, lg, G);
         s = sn;
         lo = lon;
         hi = hin;
@@ -399,14 +508,15 @@ __device__ __noinline__ void sched_group(const float *__restrict__ T, const int3
 // ascending lookup order (same arithmetic as GROUP).
 constexpr int kFlatRun = 8;
 
-template <int G, int VEC, int U>
-__device__ __noinline__ void sched_flat(const float *__restrict__ T, const int32_t *__restrict__ offs,
+template <int ET, int GT, int VEC, int U>
+__device__ __noinline__ void sched_flat(const char *__restrict__ T, unsigned rowb, int gr, const int32_t *__restrict__ offs,
                                        const int32_t *__restrict__ idx, float *__restrict__ out, int d, int pool,
                                        const OutRoute ro, int s0, int s1, int *bag_ctr) {
+    const int G = GT ? GT : gr;
     const int lane = threadIdx.x & 31;
     const int lg = lane & (G - 1);
     const unsigned gmask = (G == 32) ? 0xffffffffu : (((1u << G) - 1u) << (lane & ~(G - 1)));
-    constexpr int SPAN = G * VEC;
+    const int SPAN = G * VEC;
     const int passes = (d + SPAN - 1) / SPAN;
     while (true) {
         int v = 0;
@@ -440,16 +550,15 @@ __device__ __noinline__ void sched_flat(const float *__restrict__ T, const int32
                 unsigned id[U];
 #pragma unroll
                 for (int u = 0; u < U; ++u) id[u] = (j + u < Z) ? (unsigned)ld_idx(idx + j + u) : 0u;
-                float r[U][VEC];
+                RowFrag<ET, VEC> r[U];
 #pragma unroll
                 for (int u = 0; u < U; ++u)
-                    if (j + u < Z && ok) ld_row<VEC>(T + (size_t)id[u] * (unsigned)d + col, r[u]);
+                    if (j + u < Z && ok) r[u].load(T + (size_t)id[u] * rowb, col, d);
 #pragma unroll
                 for (int u = 0; u < U; ++u) {
                     if (j + u < Z) {
                         while (j + u >= bend) finish_bag();
-#pragma unroll
-                        for (int e = 0; e < VEC; ++e) acc[e] += r[u][e];
+                        r[u].add_to(acc);
                     }
                 }
             }
@@ -518,8 +627,8 @@ __device__ __noinline__ void sched_bulk(const float *__restrict__ T, const int32
             if (s >= s1) return;
             const int se = min(s1, s + kFlatRun);
             for (int b = s; b < se; ++b)
-                group_bag<32, 4, 1, 4>(T, idx, d, pool, out_row(out, b, ro), ld_idx(offs + b),
-                                       ld_idx(offs + b + 1), lane);
+                group_bag<0, 32, 4, 1, 4>(reinterpret_cast<const char *>(T), (unsigned)d * 4u, idx, d, pool,
+                                          out_row(out, b, ro), ld_idx(offs + b), ld_idx(offs + b + 1), lane, 32);
         }
     }
     if (lane == 0) {
@@ -601,12 +710,13 @@ __device__ __noinline__ void sched_bulk(const float *__restrict__ T, const int32
 // (adjacent groups read adjacent IDs: coalesced index loads).  Partials:
 // xor-butterfly across the groups of a warp (every lane gets bit-identical
 // sums), then the 8 warp partials are summed in warp order from shared memory.
-template <int G, int VEC, int C, int U>
-__device__ __noinline__ void sched_block(const float *__restrict__ T, const int32_t *__restrict__ offs,
+template <int ET, int GT, int VEC, int C, int U>
+__device__ __noinline__ void sched_block(const char *__restrict__ T, unsigned rowb, int gr, const int32_t *__restrict__ offs,
                                         const int32_t *__restrict__ idx, float *__restrict__ out, int d, int pool,
                                         const OutRoute ro, int s0, int s1, float *red /* [8][SPAN] */) {
-    constexpr int NG = kBlockThreads / G;
-    constexpr int SPAN = G * VEC * C;
+    const int G = GT ? GT : gr;
+    const int NG = kBlockThreads / G;
+    const int SPAN = G * VEC * C;
     constexpr int NW = kBlockThreads / 32;
     const int tid = threadIdx.x;
     const int gid = tid / G;
@@ -639,38 +749,36 @@ __device__ __noinline__ void sched_block(const float *__restrict__ T, const int3
                 int id[U];
 #pragma unroll
                 for (int u = 0; u < U; ++u) id[u] = ld_idx(idx + j + u * NG);
-                float v[U][C][VEC];
+                RowFrag<ET, VEC> v[U][C];
 #pragma unroll
                 for (int u = 0; u < U; ++u)
 #pragma unroll
                     for (int c = 0; c < C; ++c)
-                        if (ok[c]) ld_row<VEC>(T + (size_t)id[u] * d + colv[c], v[u][c]);
+                        if (ok[c]) v[u][c].load(T + (size_t)id[u] * rowb, colv[c], d);
 #pragma unroll
                 for (int u = 0; u < U; ++u)
 #pragma unroll
                     for (int c = 0; c < C; ++c)
                         if (ok[c])
-#pragma unroll
-                            for (int e = 0; e < VEC; ++e) acc[c][e] += v[u][c][e];
+                            v[u][c].add_to(acc[c]);
             }
             {
                 int id[U];
 #pragma unroll
                 for (int u = 0; u < U; ++u) id[u] = (j + u * NG < hi) ? ld_idx(idx + j + u * NG) : 0;
-                float v[U][C][VEC];
+                RowFrag<ET, VEC> v[U][C];
 #pragma unroll
                 for (int u = 0; u < U; ++u)
 #pragma unroll
                     for (int c = 0; c < C; ++c)
-                        if (j + u * NG < hi && ok[c]) ld_row<VEC>(T + (size_t)id[u] * d + colv[c], v[u][c]);
+                        if (j + u * NG < hi && ok[c]) v[u][c].load(T + (size_t)id[u] * rowb, colv[c], d);
 #pragma unroll
                 for (int u = 0; u < U; ++u)
                     if (j + u * NG < hi)
 #pragma unroll
                         for (int c = 0; c < C; ++c)
                             if (ok[c])
-#pragma unroll
-                                for (int e = 0; e < VEC; ++e) acc[c][e] += v[u][c][e];
+                                v[u][c].add_to(acc[c]);
             }
             // groups of one warp -> one partial (butterfly: identical on all lanes)
 #pragma unroll

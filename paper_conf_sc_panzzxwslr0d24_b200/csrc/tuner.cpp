@@ -517,7 +517,7 @@ std::vector<recflex_schedule_t> candidates_for(const recflex_plan_s *p, int f, i
             const CatalogEntry &e = kCatalog[id];
             recflex_schedule_t s = {id, 0, 1};
             s.per_block = samples_per_task_default(id, sp.mean_len, sp.coverage, p->task_lookups);
-            if (!schedule_valid_for(s, d.dim, d.col, (int)p->d_tot)) continue;
+            if (!schedule_valid_for(s, d.dim, d.dtype, d.col, (int)p->d_tot)) continue;
             const int span = e.G * e.VEC * e.C;
             const int passes = (d.dim + span - 1) / span;
             if (relax == 0 && (passes > 1 || e.C > 1)) continue;
@@ -537,7 +537,7 @@ std::vector<recflex_schedule_t> candidates_for(const recflex_plan_s *p, int f, i
 
 extern "C" recflex_status_t recflex_tune_ex(recflex_plan_t p, int32_t N, const int32_t *const *indices,
                                             const int32_t *const *offsets, const int32_t *batch_sizes,
-                                            const float *const *tables, void *stream_,
+                                            const void *const *tables, void *stream_,
                                             const recflex_tune_options_t *opt, recflex_tune_stats_t *stats) {
     if (!p || N <= 0 || !indices || !offsets || !batch_sizes || !tables) return RECFLEX_ERR_INVALID_ARG;
     auto t_start = std::chrono::steady_clock::now();
@@ -701,6 +701,6 @@ extern "C" recflex_status_t recflex_tune_ex(recflex_plan_t p, int32_t N, const i
 
 extern "C" recflex_status_t recflex_tune(recflex_plan_t p, int32_t N, const int32_t *const *indices,
                                          const int32_t *const *offsets, const int32_t *batch_sizes,
-                                         const float *const *tables, void *stream) {
+                                         const void *const *tables, void *stream) {
     return recflex_tune_ex(p, N, indices, offsets, batch_sizes, tables, stream, nullptr, nullptr);
 }

@@ -18,6 +18,29 @@ from ._lib import check, lib
 POOL_SUM = 0
 POOL_MEAN = 1
 
+# table row storage types (recflex_dtype_t)
+DTYPES = {'f32': 0, 'f16': 1, 'bf16': 2, 'i8': 3}
+DTYPE_NAMES = {v: k for k, v in DTYPES.items()}
+
+
+def dtype_code(dt) -> int:
+    return DTYPES[dt] if isinstance(dt, str) else int(dt)
+
+
+def i8_row_bytes(dim: int) -> int:
+    """RECFLEX_I8_ROW_BYTES: d int8 codes + fp32 scale + fp32 bias, padded to 16 bytes."""
+    return (dim + 8 + 15) // 16 * 16
+
+
+def check_table(t: torch.Tensor, dim: int, dtype) -> None:
+    """The tensor layout recflex_forward expects for a table of this dim / dtype."""
+    code = dtype_code(dtype)
+    want = {0: (torch.float32, dim), 1: (torch.float16, dim), 2: (torch.bfloat16, dim),
+            3: (torch.uint8, i8_row_bytes(dim))}[code]
+    if not (t.is_cuda and t.dtype == want[0] and t.is_contiguous() and t.dim() == 2 and t.shape[1] == want[1]):
+        raise ValueError(f'table: need contiguous CUDA {want[0]} [rows, {want[1]}] for dim {dim} '
+                         f'dtype {DTYPE_NAMES[code]}, got {t.dtype} {tuple(t.shape)}')
+
 
 def catalog():
     """List of dicts describing every catalog entry (schedule templates)."""
@@ -26,7 +49,7 @@ def catalog():
         ci = _lib.CatalogInfo()
         check(lib.recflex_catalog_info(i, ctypes.byref(ci)), 'recflex_catalog_info')
         out.append(dict(id=i, family=('group', 'block', 'flat', 'bulk')[ci.family], G=ci.group, VEC=ci.vec, C=ci.cols,
-                        U=ci.unroll))
+                        U=ci.unroll, dtype=DTYPE_NAMES[ci.dtype]))
     return out
 
 
@@ -56,7 +79,8 @@ def _dptr(t: torch.Tensor, dtype, name):
 class Plan:
     """recflex_plan_create / recflex_destroy around a list of feature specs.
 
-    specs: sequence of dicts with keys rows, dim, pool, mean_len, max_len, coverage.
+    specs: sequence of dicts with keys rows, dim, pool, mean_len, max_len, coverage
+    and optionally dtype ('f32' default, 'f16', 'bf16', 'i8' -- see check_table).
     """
 
     def __init__(self, specs: Sequence[dict], max_batch: int, device: int = 0):
@@ -69,11 +93,13 @@ class Plan:
             arr[i].mean_len = float(s.get('mean_len', 1.0))
             arr[i].max_len = float(s.get('max_len', 1.0))
             arr[i].coverage = float(s.get('coverage', 1.0))
+            arr[i].dtype = dtype_code(s.get('dtype', 0))
         self._h = ctypes.c_void_p()
         check(lib.recflex_plan_create(arr, F, int(max_batch), int(device), ctypes.byref(self._h)),
               'recflex_plan_create')
         self.F = F
         self.dims = [int(s['dim']) for s in specs]
+        self.dtypes = [dtype_code(s.get('dtype', 0)) for s in specs]
         self.d_tot = sum(self.dims)
         self.max_batch = int(max_batch)
         self.device = int(device)
@@ -81,9 +107,9 @@ class Plan:
         self._tables_arr = None
 
     @classmethod
-    def from_model(cls, model, max_batch: Optional[int] = None, device: int = 0) -> 'Plan':
+    def from_model(cls, model, max_batch: Optional[int] = None, device: int = 0, dtype='f32') -> 'Plan':
         specs = [dict(rows=f.rows, dim=f.dim, pool=f.pool, mean_len=f.mean_len(), max_len=f.max_len(),
-                      coverage=f.coverage) for f in model.features]
+                      coverage=f.coverage, dtype=dtype) for f in model.features]
         return cls(specs, max_batch or model.batch, device)
 
     # -------------------------------------------------------------- lifecycle
@@ -105,9 +131,10 @@ class Plan:
         key = tuple(t.data_ptr() for t in tables)
         if key != self._tables_key:
             for f, t in enumerate(tables):
-                if not (t.is_cuda and t.dtype == torch.float32 and t.is_contiguous() and t.dim() == 2
-                        and t.shape[1] == self.dims[f]):
-                    raise ValueError(f'table {f}: need contiguous CUDA float32 [rows, {self.dims[f]}]')
+                try:
+                    check_table(t, self.dims[f], self.dtypes[f])
+                except ValueError as ex:
+                    raise ValueError(f'table {f}: {ex}') from None
             self._tables_arr = (ctypes.c_void_p * self.F)(*key)
             self._tables_key = key
         return self._tables_arr

@@ -23,9 +23,15 @@ from typing import List, Sequence
 import numpy as np
 
 
-def feature_cost(feat, B: int) -> float:
+def row_bytes(dim: int, dtype: str = 'f32') -> int:
+    """Bytes one lookup gathers: the stored row (int8: codes + scale + bias)."""
+    return {'f32': 4 * dim, 'f16': 2 * dim, 'bf16': 2 * dim, 'i8': dim + 8}[dtype]
+
+
+def feature_cost(feat, B: int, dtype: str = 'f32') -> float:
+    """Estimated bytes per batch (reading C24): lookups x (row + ID) + pooled output."""
     el = feat.mean_len() * feat.coverage
-    return el * (4 * feat.dim + 4) * B + 4.0 * feat.dim * B
+    return el * (row_bytes(feat.dim, dtype) + 4) * B + 4.0 * feat.dim * B
 
 
 def lpt_partition(costs: Sequence[float], W: int) -> List[List[int]]:
@@ -42,8 +48,8 @@ def lpt_partition(costs: Sequence[float], W: int) -> List[List[int]]:
     return [sorted(p) for p in parts]
 
 
-def partition_model(model, W: int) -> List[List[int]]:
-    return lpt_partition([feature_cost(f, model.batch) for f in model.features], W)
+def partition_model(model, W: int, dtype: str = 'f32') -> List[List[int]]:
+    return lpt_partition([feature_cost(f, model.batch, dtype) for f in model.features], W)
 
 
 def column_order(model, parts: List[List[int]]) -> np.ndarray:
@@ -105,16 +111,16 @@ def exchange(send, dims_per_rank: Sequence[int], B: int, group=None):
 class ShardedEmbedding:
     """One rank's slice of a table-wise sharded model: plan + exchange + relayout."""
 
-    def __init__(self, model, rank: int, world: int, device: int = 0, parts=None):
+    def __init__(self, model, rank: int, world: int, device: int = 0, parts=None, dtype: str = 'f32'):
         from .plan import Plan
         self.model = model
         self.rank, self.world = rank, world
-        self.parts = parts if parts is not None else partition_model(model, world)
+        self.parts = parts if parts is not None else partition_model(model, world, dtype)
         self.features = self.parts[rank]
         self.dims_per_rank = [sum(model.dims[f] for f in p) for p in self.parts]
         specs = [dict(rows=model.features[f].rows, dim=model.features[f].dim, pool=model.features[f].pool,
                       mean_len=model.features[f].mean_len(), max_len=model.features[f].max_len(),
-                      coverage=model.features[f].coverage) for f in self.features]
+                      coverage=model.features[f].coverage, dtype=dtype) for f in self.features]
         self.plan = Plan(specs, model.batch, device)
         self.d_local = self.dims_per_rank[rank]
         self.d_tot = sum(self.dims_per_rank)
@@ -143,10 +149,10 @@ class FusedShardedEmbedding(ShardedEmbedding):
     orders the destination's reads after every writer (stream-ordered
     all_reduce on NCCL; host barrier on gloo)."""
 
-    def __init__(self, model, rank: int, world: int, device: int = 0, parts=None, group=None):
+    def __init__(self, model, rank: int, world: int, device: int = 0, parts=None, group=None, dtype: str = 'f32'):
         import torch.distributed as dist
         from .plan import DeviceBuffer, ipc_handle, ipc_open
-        super().__init__(model, rank, world, device, parts)
+        super().__init__(model, rank, world, device, parts, dtype)
         if model.batch % world:
             raise ValueError('fused exchange needs B % W == 0 (reading C23)')
         self.group = group

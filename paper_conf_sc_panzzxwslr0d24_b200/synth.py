@@ -328,6 +328,83 @@ def make_table(table_id: int, rows: int, dim: int, mode: str = 'float', device='
     return out
 
 
+# ---------------------------------------------------------------------------
+# Reduced-precision storage: the same seeded tables, stored
+# as float16 / bfloat16 (round-to-nearest casts of the fp32 values) or as
+# rowwise int8 (codes + per-row fp32 scale and bias, include/recflex.h).
+# Encoding inputs only: the value of a stored element is defined (and
+# computed for checking) by oracle_decode, not here.
+# ---------------------------------------------------------------------------
+STORAGE_DTYPES = ('f32', 'f16', 'bf16', 'i8')
+
+
+def i8_row_bytes(dim: int) -> int:
+    return (dim + 8 + 15) // 16 * 16
+
+
+def table_rows_stored(table_id: int, row_ids, dim: int, dtype: str = 'f32', mode: str = 'float', device='cpu',
+                      seed: int = MODEL_SEED):
+    """Stored rows of a physical table: float32 / float16 / bfloat16 [n, dim],
+    or uint8 [n, i8_row_bytes(dim)] for 'i8'.  'int' mode keeps every element
+    an exact small integer in all storage types (i8: scale 1, integer bias)."""
+    import torch
+    if dtype == 'f32':
+        return table_rows_at(table_id, row_ids, dim, mode, device, seed)
+    if dtype in ('f16', 'bf16'):
+        v = table_rows_at(table_id, row_ids, dim, mode, device, seed)
+        return v.to(torch.float16 if dtype == 'f16' else torch.bfloat16)
+    if dtype != 'i8':
+        raise ValueError(dtype)
+    r = torch.as_tensor(row_ids, dtype=torch.int64, device=device).reshape(-1)
+    n = r.numel()
+    h0 = _mix32(torch.tensor(((table_id * 0x2545F491) + (seed * 0x9E3779B9) + 0x51ED27) & M32, dtype=torch.int64,
+                             device=device))
+    h1 = _mix32((h0 ^ (r & M32)) & M32)
+    c = torch.arange(dim, dtype=torch.int64, device=device)
+    h2 = _mix32((h1[:, None] + ((c * 0x61C88647) & M32)[None, :]) & M32)
+    hs = _mix32((h1 + 0x3C6EF372) & M32)
+    hb = _mix32((h1 + 0x7F4A7C15) & M32)
+    if mode == 'float':
+        q = (h2 >> 24) - 128                                             # [-128, 127]
+        scale = ((hs >> 8).to(torch.float64) * 2.0 ** -24 + 1.0) * 2.0 ** -7  # [2^-7, 2^-6)
+        bias = (hb >> 8).to(torch.float64) * 2.0 ** -23 - 1.0               # [-1, 1)
+    elif mode == 'int':
+        q = (h2 >> 28) - 8                                               # [-8, 7]
+        scale = torch.ones(n, dtype=torch.float64, device=device)
+        bias = ((hb >> 29) - 4).to(torch.float64)                         # [-4, 3]
+    else:
+        raise ValueError(mode)
+    out = torch.zeros((n, i8_row_bytes(dim)), dtype=torch.uint8, device=device)
+    out[:, :dim] = (q & 0xFF).to(torch.uint8)
+    sb = torch.stack([scale.to(torch.float32), bias.to(torch.float32)], dim=1).contiguous()
+    out[:, dim:dim + 8] = sb.view(torch.uint8).reshape(n, 8)
+    return out
+
+
+def make_table_stored(table_id: int, rows: int, dim: int, dtype: str = 'f32', mode: str = 'float', device='cpu',
+                      seed: int = MODEL_SEED, chunk_rows: Optional[int] = None):
+    """A whole physical table in storage type `dtype` (see table_rows_stored)."""
+    import torch
+    if dtype == 'f32':
+        return make_table(table_id, rows, dim, mode, device, seed, chunk_rows)
+    width = i8_row_bytes(dim) if dtype == 'i8' else dim
+    tdt = {'f16': torch.float16, 'bf16': torch.bfloat16, 'i8': torch.uint8}[dtype]
+    out = torch.empty((rows, width), dtype=tdt, device=device)
+    if chunk_rows is None:
+        chunk_rows = max(1, (1 << 24) // max(1, dim))
+    for a in range(0, rows, chunk_rows):
+        b = min(rows, a + chunk_rows)
+        out[a:b] = table_rows_stored(table_id, torch.arange(a, b, dtype=torch.int64, device=device), dim, dtype,
+                                     mode, device, seed)
+    return out
+
+
+def row_bytes(dim: int, dtype: str = 'f32') -> int:
+    """Algorithmic bytes of one stored row (C26 generalised): the element bytes,
+    plus scale and bias for int8 (padding excluded)."""
+    return {'f32': 4 * dim, 'f16': 2 * dim, 'bf16': 2 * dim, 'i8': dim + 8}[dtype]
+
+
 def make_tables(model: Model, mode: str = 'float', device='cpu'):
     """Physical tables of a model (list indexed by table id)."""
     return [make_table(t, rows, dim, mode, device, model.seed) for t, (rows, dim) in enumerate(model.tables)]
@@ -337,14 +414,16 @@ def make_tables(model: Model, mode: str = 'float', device='cpu'):
 # Byte accounting (C26): what the method must move per batch
 # ---------------------------------------------------------------------------
 
-def algorithmic_bytes(model: Model, batch: Batch) -> dict:
-    """indices + gathered rows + outputs (reading C26); offsets reported apart."""
+def algorithmic_bytes(model: Model, batch: Batch, dtype: str = 'f32') -> dict:
+    """indices + gathered rows + outputs (reading C26); offsets reported apart.
+    Rows count their stored bytes (row_bytes: int8 = codes + scale + bias)."""
     F, B = batch.F, batch.B
     offs = batch.offsets.astype(np.int64)
     nnz_f = offs[np.arange(1, F + 1) * B] - offs[np.arange(0, F) * B]
     dims = np.asarray(model.dims, np.int64)
+    rowb = np.asarray([row_bytes(int(d), dtype) for d in dims], np.int64)
     idx_b = 4 * int(nnz_f.sum())
-    row_b = 4 * int((dims * nnz_f).sum())
+    row_b = int((rowb * nnz_f).sum())
     out_b = 4 * B * int(dims.sum())
     off_b = 4 * (F * B + 1)
     return {'index': idx_b, 'rows': row_b, 'out': out_b, 'offsets': off_b,

@@ -300,3 +300,127 @@ def test_nnz_task_ranges_partition():
         for s in range(B):
             q = (int(off[s]) - int(off[0])) // npb
             assert s0[q] <= s < s1[q]
+
+
+# ---------------------------------------------------------------- reduced-precision storage (NEXT #3)
+
+LOWP = os.path.join(os.path.dirname(__file__), 'golden', 'lowp_rows.json')
+
+
+def _lowp():
+    with open(LOWP) as fh:
+        return json.load(fh)
+
+
+def _i8_row(codes, scale, bias):
+    d = len(codes)
+    row = np.zeros(oracle.row_bytes('i8', d), np.uint8)
+    row[:d] = np.asarray(codes, np.int8).view(np.uint8)
+    row[d:d + 8] = np.asarray([scale, bias], np.float32).view(np.uint8)
+    return row
+
+
+def test_decode_f16_worked_values():
+    g = _lowp()['f16']
+    v = oracle.decode_rows(np.asarray(g['bits'], np.uint16).reshape(-1, 1), 1, 'f16')
+    assert v[:, 0].tolist() == g['values']
+
+
+def test_decode_bf16_worked_values():
+    g = _lowp()['bf16']
+    v = oracle.decode_rows(np.asarray(g['bits'], np.uint16).reshape(-1, 1), 1, 'bf16')
+    assert v[:, 0].tolist() == g['values']
+
+
+def test_decode_f16_exhaustive_vs_numpy():
+    """All 2^16 binary16 patterns against numpy's float16 -> float64 (library routine)."""
+    bits = np.arange(1 << 16, dtype=np.uint32).astype(np.uint16)
+    v = oracle.decode_rows(bits.reshape(-1, 4), 4, 'f16').reshape(-1)
+    ref = bits.view(np.float16).astype(np.float64)
+    assert np.array_equal(np.isnan(v), np.isnan(ref))
+    ok = ~np.isnan(ref)
+    assert np.array_equal(v[ok], ref[ok])
+    assert np.array_equal(np.signbit(v[ok]), np.signbit(ref[ok]))  # -0.0 stays -0.0
+
+
+def test_decode_bf16_exhaustive_vs_torch():
+    """All 2^16 bfloat16 patterns against torch's bfloat16 -> float64 (library routine)."""
+    bits = torch.arange(1 << 16, dtype=torch.int32).to(torch.int16)
+    v = oracle.decode_rows(bits.numpy().view(np.uint16).reshape(-1, 4), 4, 'bf16').reshape(-1)
+    ref = bits.view(torch.bfloat16).double().numpy()
+    assert np.array_equal(np.isnan(v), np.isnan(ref))
+    ok = ~np.isnan(ref)
+    assert np.array_equal(v[ok], ref[ok])
+
+
+def test_decode_i8_worked_row():
+    g = _lowp()['i8']
+    row = _i8_row(g['codes'], g['scale'], g['bias'])
+    v = oracle.decode_rows(row.reshape(1, -1), g['dim'], 'i8')
+    assert v[0].tolist() == g['values']
+
+
+@pytest.mark.parametrize('pool', [0, 1])
+def test_i8_bag_worked_example(pool):
+    g = _lowp()
+    r0 = _i8_row(g['i8']['codes'], g['i8']['scale'], g['i8']['bias'])
+    r1 = _i8_row(g['i8_bag']['codes_r1'], g['i8_bag']['scale_r1'], g['i8_bag']['bias_r1'])
+    T = np.stack([r0, r1])
+    out = oracle.embedding_bag([T], [8], [pool], g['i8_bag']['indices'], g['i8_bag']['offsets'], 2, dtypes=['i8'])
+    exp0 = np.asarray(g['i8_bag']['sum_s0'], np.float64)
+    if pool == 1:
+        exp0 = exp0 / 3.0
+    assert np.array_equal(out[0], exp0)
+    assert np.array_equal(out[1], np.zeros(8))  # empty bag -> 0 (reading C1)
+
+
+@pytest.mark.parametrize('dtype', ['f16', 'bf16'])
+def test_half_tables_equal_upcast_f32_tables(dtype):
+    """A 16-bit stored table pools exactly like its library up-cast to float32
+    (every 16-bit value is exactly representable in float32)."""
+    m = synth.make_model('tiny')
+    b = synth.make_batch(m, 7)
+    st = [synth.table_rows_stored(f.table, np.arange(m.tables[f.table][0]), f.dim, dtype, 'float', seed=m.seed)
+          for f in m.features]
+    up = [t.float().numpy() for t in st]
+    pools = [1, 0, 1, 0]
+    a = oracle.embedding_bag(st, m.dims, pools, b.indices, b.offsets, b.B, dtypes=[dtype] * m.F)
+    r = oracle.embedding_bag(up, m.dims, pools, b.indices, b.offsets, b.B)
+    assert np.array_equal(a, r)
+
+
+def test_i8_tables_vs_torch_weighted_embedding_bag():
+    """Rowwise int8 pooling = torch embedding_bag of the codes with per-lookup
+    weights scale[id], plus embedding_bag of the bias column (library routine,
+    fp64), since sum_j (s_j q_j + b_j) = sum_j s_j q_j + sum_j b_j."""
+    m = synth.make_model('tiny')
+    b = synth.make_batch(m, 8)
+    F, B = m.F, b.B
+    st = [synth.table_rows_stored(f.table, np.arange(m.tables[f.table][0]), f.dim, 'i8', 'float', seed=m.seed)
+          for f in m.features]
+    out = oracle.embedding_bag(st, m.dims, [0] * F, b.indices, b.offsets, B, dtypes=['i8'] * F)
+    col = 0
+    for f in range(F):
+        d = m.dims[f]
+        raw = st[f].numpy()
+        q = torch.from_numpy(raw[:, :d].view(np.int8).astype(np.float64))
+        sb = raw[:, d:d + 8].copy().view(np.float32).astype(np.float64)
+        lo, hi = b.offsets[f * B], b.offsets[(f + 1) * B]
+        ids = torch.from_numpy(b.indices[lo:hi].astype(np.int64))
+        offs = torch.from_numpy((b.offsets[f * B:(f + 1) * B + 1] - lo).astype(np.int64))
+        w = torch.from_numpy(sb[:, 0])[ids]
+        ref = torch.nn.functional.embedding_bag(ids, q, offs, mode='sum', per_sample_weights=w,
+                                                include_last_offset=True)
+        ref += torch.nn.functional.embedding_bag(ids, torch.from_numpy(sb[:, 1:2]), offs, mode='sum',
+                                                 include_last_offset=True)
+        assert np.allclose(out[:, col:col + d], ref.numpy(), rtol=1e-13, atol=1e-12)
+        col += d
+
+
+def test_i8_int_mode_exact_integers():
+    m = synth.make_model('tiny')
+    b = synth.make_batch(m, 7)
+    st = [synth.table_rows_stored(f.table, np.arange(m.tables[f.table][0]), f.dim, 'i8', 'int', seed=m.seed)
+          for f in m.features]
+    out = oracle.embedding_bag(st, m.dims, [0] * m.F, b.indices, b.offsets, b.B, dtypes=['i8'] * m.F)
+    assert np.array_equal(out, np.rint(out))

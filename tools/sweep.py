@@ -22,22 +22,23 @@ def main():
     ap.add_argument('--parts', default='0')
     ap.add_argument('--per-block', default='', help='override per_block values (comma list)')
     ap.add_argument('--reps', type=int, default=6)
+    ap.add_argument('--dtype', default='f32', choices=['f32', 'f16', 'bf16', 'i8'])
     a = ap.parse_args()
     import torch
     from paper_conf_sc_panzzxwslr0d24_b200 import synth
     from paper_conf_sc_panzzxwslr0d24_b200.plan import Plan, catalog, l2_flush
     dev = torch.device('cuda', 0)
     m = synth.make_model(a.config)
-    phys = [synth.make_table(t, r, d, 'float', device=dev) for t, (r, d) in enumerate(m.tables)]
+    phys = [synth.make_table_stored(t, r, d, a.dtype, 'float', device=dev) for t, (r, d) in enumerate(m.tables)]
     tables = [phys[f.table] for f in m.features]
     bts = [synth.make_batch(m, 7 + i) for i in range(2)]
-    alg = np.mean([synth.algorithmic_bytes(m, b)['total'] for b in bts])
+    alg = np.mean([synth.algorithmic_bytes(m, b, a.dtype)['total'] for b in bts])
     dev_b = [(torch.from_numpy(b.indices).to(dev), torch.from_numpy(b.offsets).to(dev)) for b in bts]
-    plan = Plan.from_model(m)
+    plan = Plan.from_model(m, dtype=a.dtype)
     out = torch.empty((m.batch, m.d_tot), device=dev)
     flush = torch.empty(64 << 20, device=dev)
     cat = catalog()
-    ids = [int(x) for x in a.ids.split(',')] if a.ids else [e['id'] for e in cat]
+    ids = [int(x) for x in a.ids.split(',')] if a.ids else [e['id'] for e in cat if e['dtype'] == a.dtype]
     dims = sorted(set(m.dims))
     default = [plan.get_schedule(f) for f in range(m.F)]
     print(f'# {a.config}: {alg / 1e9:.2f} GB algorithmic per batch')

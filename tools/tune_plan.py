@@ -3,7 +3,7 @@ schedules are reused for a long period, re-tuned periodically).
 
     python tools/tune_plan.py sharded1000 [--world W --rank R] [--ks 2,4,6,8] [--out DIR]
 
-Writes DIR/<config>_w<W>_r<R>.json (default DIR = gpurun_out/tuned) plus a
+Writes DIR/<config>[_<dtype>]_w<W>_r<R>.json (default DIR = gpurun_out/tuned) plus a
 .log with the tuner statistics.  bench.py loads configs/tuned/ automatically.
 """
 import argparse
@@ -25,6 +25,7 @@ def main():
     ap.add_argument('--batches', type=int, default=2)
     ap.add_argument('--reps', type=int, default=5)
     ap.add_argument('--max-candidates', type=int, default=0)
+    ap.add_argument('--dtype', default='f32', choices=['f32', 'f16', 'bf16', 'i8'])
     ap.add_argument('--out', default=os.path.join(ROOT, 'gpurun_out', 'tuned'))
     a = ap.parse_args()
     import torch
@@ -34,19 +35,19 @@ def main():
     os.makedirs(a.out, exist_ok=True)
     dev = torch.device('cuda', 0)
     model = synth.make_model(a.config)
-    parts = partition_model(model, a.world)
+    parts = partition_model(model, a.world, a.dtype)
     ranks = range(a.world) if a.rank < 0 else [a.rank]
     ks = [int(x) for x in a.ks.split(',')] if a.ks else None
     fulls = [synth.make_batch(model, 7 + i) for i in range(a.batches)]
     for r in ranks:
-        sh = ShardedEmbedding(model, r, a.world, device=0, parts=parts)
+        sh = ShardedEmbedding(model, r, a.world, device=0, parts=parts, dtype=a.dtype)
         feats = sh.features
         phys = {}
         for f in feats:
             t = model.features[f].table
             if t not in phys:
                 rows, dim = model.tables[t]
-                phys[t] = synth.make_table(t, rows, dim, 'float', device=dev, seed=model.seed)
+                phys[t] = synth.make_table_stored(t, rows, dim, a.dtype, 'float', device=dev, seed=model.seed)
         tables = [phys[model.features[f].table] for f in feats]
         hist = []
         for full in fulls:
@@ -56,7 +57,7 @@ def main():
         st = sh.plan.tune(hist, tables, occupancies=ks, reps=a.reps, max_candidates=a.max_candidates, verbose=True)
         st['wall_s'] = time.time() - t0
         state = sh.plan.export()
-        name = f'{a.config}_w{a.world}_r{r}'
+        name = f'{a.config}_w{a.world}_r{r}' if a.dtype == 'f32' else f'{a.config}_{a.dtype}_w{a.world}_r{r}'
         with open(os.path.join(a.out, name + '.json'), 'w') as fh:
             json.dump(state, fh)
         with open(os.path.join(a.out, name + '.log'), 'w') as fh:
