@@ -205,6 +205,7 @@ __global__ void __launch_bounds__(kBlockThreads, KOCC) recflex_fused_kernel(Fuse
     for (int n = 0;; ++n) {
         TaskSlot &S = ring[n % kRing];
         if (lane == 0) {
+            long long spin0 = 0;
             while (true) {
                 const int st = ld_acquire(&S.state);
                 if (st == 2) {
@@ -214,6 +215,12 @@ __global__ void __launch_bounds__(kBlockThreads, KOCC) recflex_fused_kernel(Fuse
                     break;
                 }
                 __nanosleep(32);
+                // watchdog: a slot that never becomes ready is a protocol bug;
+                // fail the launch (cudaErrorIllegalInstruction) instead of
+                // hanging the device (~10 s at 2 GHz)
+                const long long now = clock64();
+                if (spin0 == 0) spin0 = now;
+                else if (now - spin0 > 20000000000LL) asm volatile("trap;");
             }
 #ifdef RECFLEX_FILL_AHEAD
             // EXPERIMENT, off by default (heavy unchanged, sharded1000 9% slower):
