@@ -16,6 +16,8 @@ Functions and the passages they follow (PAPER.md "P:n"):
   decode_rows    -- the value of a stored row element per storage type (SURVEY
                     NEXT #3: f16 / bf16 / rowwise int8); embedding_bag takes
                     stored tables and decodes every element with it.
+  embedding_bag_backward -- the adjoint (training):
+                    dense gradient / SGD update of every table row.
   task_map       -- Fig. 8: d_blocks_map and d_task_map, reading C12.
   nnz_task_ranges-- reading C12 for nnz-partitioned schedules.
 """
@@ -70,6 +72,11 @@ def lib():
                                              P(ctypes.c_double)]
             L.oracle_row_bytes.restype = ctypes.c_int64
             L.oracle_row_bytes.argtypes = [ctypes.c_int, ctypes.c_int]
+            L.oracle_embedding_bag_backward.restype = ctypes.c_int
+            L.oracle_embedding_bag_backward.argtypes = [
+                ctypes.c_int, ctypes.c_int, P(ctypes.c_int), P(ctypes.c_int), P(ctypes.c_int64),
+                P(ctypes.c_int32), P(ctypes.c_int32), P(ctypes.c_double), ctypes.c_double,
+                P(ctypes.c_void_p), P(ctypes.c_void_p), P(ctypes.c_void_p)]
             L.oracle_task_map.restype = ctypes.c_int
             L.oracle_task_map.argtypes = [
                 ctypes.c_int, ctypes.c_int, P(ctypes.c_int), P(ctypes.c_int), P(ctypes.c_int),
@@ -161,6 +168,42 @@ def embedding_bag(tables, dims, pools, indices, offsets, B, nthreads: int = 0, d
     if rc != 0:
         raise OracleError({-1: 'index out of range', -2: 'bad offsets', -3: 'bad argument'}.get(rc, rc))
     return out
+
+
+def embedding_bag_backward(rows, dims, pools, indices, offsets, B, grad, scale=1.0, targets=None):
+    """Adjoint of embedding_bag: fp64 per-feature updates.
+
+    rows: per-feature row counts; grad: [B][sum(dims)] (cast to fp64);
+    targets: optional list of F initial arrays [rows_f][d_f] (copied to fp64;
+    default zeros).  Returns (targets, counts, abssum): the updated targets,
+    the number of terms per row and the per-element sum of |term|.
+    """
+    F = len(dims)
+    dims_a = np.asarray(dims, np.intc)
+    pools_a = np.asarray(pools, np.intc)
+    rows_a = np.asarray(rows, np.int64)
+    g = np.ascontiguousarray(grad, np.float64)
+    if g.shape != (B, int(dims_a.sum())):
+        raise ValueError(f'grad shape {g.shape}')
+    tg = [np.array(targets[f], np.float64, copy=True).reshape(int(rows_a[f]), dims[f]) if targets is not None
+          else np.zeros((int(rows_a[f]), dims[f]), np.float64) for f in range(F)]
+    cn = [np.zeros(int(rows_a[f]), np.int64) for f in range(F)]
+    ab = [np.zeros((int(rows_a[f]), dims[f]), np.float64) for f in range(F)]
+    idx = np.ascontiguousarray(indices, np.int32)
+    off = np.ascontiguousarray(offsets, np.int32)
+    if off.shape[0] != F * B + 1:
+        raise ValueError('offsets must have F*B+1 entries')
+    if idx.size == 0:
+        idx = np.zeros(1, np.int32)
+    P = ctypes.c_void_p
+    rc = lib().oracle_embedding_bag_backward(
+        F, B, _ptr(dims_a, ctypes.c_int), _ptr(pools_a, ctypes.c_int), _ptr(rows_a, ctypes.c_int64),
+        _ptr(idx, ctypes.c_int32), _ptr(off, ctypes.c_int32), _ptr(g, ctypes.c_double), float(scale),
+        (P * F)(*[t.ctypes.data for t in tg]), (P * F)(*[c.ctypes.data for c in cn]),
+        (P * F)(*[a.ctypes.data for a in ab]))
+    if rc != 0:
+        raise OracleError({-1: 'index out of range', -2: 'bad offsets', -3: 'bad argument'}.get(rc, rc))
+    return tg, cn, ab
 
 
 def task_map(B, mode, per_block, offsets, cap=None):

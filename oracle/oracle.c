@@ -35,6 +35,21 @@
  *       Pinned by tests/test_oracle.py: exhaustive over all 2^16 patterns
  *       against numpy float16 and torch bfloat16, hand-decoded I8 rows.
  *
+ *   oracle_embedding_bag_backward -- the adjoint of oracle_embedding_bag
+ *       (training; "there is no fundamental reason
+ *       limiting RecFlex from optimizing the training process"): with the
+ *       upstream gradient G = dLoss/d out [B][D_tot], row r of table f
+ *       receives  sum over bags (f,s) and positions j with indices[j] == r of
+ *       w_{f,s} * G[s][col_f + c],  w = 1 (SUM) or 1/L_{f,s} (MEAN), i.e.
+ *       the derivative of the definition above.  Written as the update
+ *       target_f[r][c] += scale * w * G[s][col_f + c] (scale = 1 into zeroed
+ *       buffers: the dense gradient; scale = -lr into the table: one SGD
+ *       step).  fp64, in ascending (f, s, j) order; also returns per element
+ *       the number of terms and the sum of their magnitudes (for the
+ *       floating-point error bound of a GPU result accumulated in any order).
+ *       Pinned by tests/test_oracle.py: hand-worked example, torch autograd
+ *       of embedding_bag in fp64, the adjoint identity <G, A T> = <A^T G, T>.
+ *
  *   oracle_task_map       -- the runtime thread map of Fig. 8:
  *       d_blocks_map[f] = feature_blocks, and d_task_map[b] = (feature_idx,
  *       rel_bidx) enumerating, feature by feature, rel = 0..feature_blocks-1.
@@ -199,6 +214,46 @@ int oracle_embedding_bag(int F, int B, const int *dims, const int *pools,
                          double *out, int nthreads) {
     return oracle_embedding_bag_typed(F, B, dims, pools, NULL, (const void *const *)tables, rows, indices, offsets,
                                       out, nthreads);
+}
+
+/*
+ * Backward of the embedding bag (the adjoint), fp64.
+ * targets[f] -> double [rows[f]][dims[f]] (accumulated into, caller-initialised);
+ * grad -> double [B][sum(dims)]; counts[f] (nullable) -> int64 [rows[f]] terms per
+ * row; abssum[f] (nullable) -> double [rows[f]][dims[f]] sum of |term| (accumulated).
+ */
+int oracle_embedding_bag_backward(int F, int B, const int *dims, const int *pools, const int64_t *rows,
+                                  const int32_t *indices, const int32_t *offsets, const double *grad, double scale,
+                                  double *const *targets, int64_t *const *counts, double *const *abssum) {
+    if (F <= 0 || B < 0) return ORACLE_ERR_ARG;
+    int64_t d_tot = 0;
+    for (int f = 0; f < F; ++f) d_tot += dims[f];
+    if (offsets[0] != 0) return ORACLE_ERR_OFFSETS;
+    for (int64_t k = 0; k < (int64_t)F * B; ++k)
+        if (offsets[k + 1] < offsets[k]) return ORACLE_ERR_OFFSETS;
+    int64_t col = 0;
+    for (int f = 0; f < F; ++f) {
+        const int d = dims[f];
+        for (int s = 0; s < B; ++s) {
+            const int64_t lo = offsets[(int64_t)f * B + s];
+            const int64_t hi = offsets[(int64_t)f * B + s + 1];
+            const int64_t L = hi - lo;
+            const double w = (pools[f] == POOL_MEAN && L > 0) ? 1.0 / (double)L : 1.0;
+            const double *g = grad + (int64_t)s * d_tot + col;
+            for (int64_t j = lo; j < hi; ++j) {
+                const int64_t r = indices[j];
+                if (r < 0 || r >= rows[f]) return ORACLE_ERR_INDEX;
+                for (int c = 0; c < d; ++c) {
+                    const double term = scale * w * g[c];
+                    targets[f][r * d + c] += term;
+                    if (abssum) abssum[f][r * d + c] += term < 0 ? -term : term;
+                }
+                if (counts) counts[f][r] += 1;
+            }
+        }
+        col += d;
+    }
+    return ORACLE_OK;
 }
 
 /*

@@ -424,3 +424,75 @@ def test_i8_int_mode_exact_integers():
           for f in m.features]
     out = oracle.embedding_bag(st, m.dims, [0] * m.F, b.indices, b.offsets, b.B, dtypes=['i8'] * m.F)
     assert np.array_equal(out, np.rint(out))
+
+
+# ---------------------------------------------------------------- backward / adjoint (NEXT #4)
+
+@pytest.mark.parametrize('pool', [0, 1])
+def test_backward_worked_example(pool):
+    g = _gold()['backward']
+    tg, cn, _ = oracle.embedding_bag_backward([g['rows']], [g['dim']], [pool], g['indices'], g['offsets'], g['B'],
+                                              np.asarray(g['grad'], np.float64))
+    if pool == 0:
+        exp = np.asarray(g['sum'], np.float64)
+    else:
+        exp = np.asarray(g['mean_num'], np.float64) / g['mean_den']
+    assert np.allclose(tg[0], exp, rtol=0, atol=1e-15)
+    assert cn[0].tolist() == g['counts']
+
+
+@pytest.mark.parametrize('name', ['tiny', 'fig3'])
+def test_backward_vs_torch_autograd(name):
+    """Library routine: torch autograd of embedding_bag (fp64) gives the same table gradients."""
+    m = synth.make_model(name)
+    b = synth.make_batch(m, 7)
+    F, B = m.F, b.B
+    pools = [f % 2 for f in range(F)]
+    rng = np.random.default_rng(3)
+    G = rng.standard_normal((B, m.d_tot))
+    tg, _, _ = oracle.embedding_bag_backward([f.rows for f in m.features], m.dims, pools, b.indices, b.offsets, B, G)
+    col = 0
+    for f in range(F):
+        d = m.dims[f]
+        W = torch.zeros((m.features[f].rows, d), dtype=torch.float64, requires_grad=True)
+        lo, hi = b.offsets[f * B], b.offsets[(f + 1) * B]
+        ids = torch.from_numpy(b.indices[lo:hi].astype(np.int64))
+        offs = torch.from_numpy((b.offsets[f * B:(f + 1) * B + 1] - lo).astype(np.int64))
+        out = torch.nn.functional.embedding_bag(ids, W, offs, mode=('sum', 'mean')[pools[f]],
+                                                include_last_offset=True)
+        out.backward(torch.from_numpy(G[:, col:col + d]))
+        assert np.allclose(tg[f], W.grad.numpy(), rtol=1e-12, atol=1e-12)
+        col += d
+
+
+def test_backward_adjoint_identity():
+    """<G, A(T)> == <A^T(G), T> for the linear map A = embedding bag (fixed indices)."""
+    m = synth.make_model('tiny')
+    b = synth.make_batch(m, 9)
+    pools = [0, 1, 1, 0]
+    rng = np.random.default_rng(5)
+    T = [rng.standard_normal((f.rows, f.dim)).astype(np.float32) for f in m.features]
+    G = rng.standard_normal((b.B, m.d_tot))
+    fwd = oracle.embedding_bag(T, m.dims, pools, b.indices, b.offsets, b.B)
+    tg, _, _ = oracle.embedding_bag_backward([f.rows for f in m.features], m.dims, pools, b.indices, b.offsets, b.B, G)
+    lhs = float(np.sum(G * fwd))
+    rhs = float(sum(np.sum(tg[f] * T[f].astype(np.float64)) for f in range(m.F)))
+    assert abs(lhs - rhs) <= 1e-10 * max(1.0, abs(lhs))
+
+
+def test_backward_scale_and_initial_targets():
+    """SGD form: targets start at T0 and receive scale * gradient (exact for scale = -0.5)."""
+    m = synth.make_model('tiny')
+    b = synth.make_batch(m, 7)
+    rows = [f.rows for f in m.features]
+    rng = np.random.default_rng(1)
+    G = rng.integers(-8, 8, (b.B, m.d_tot)).astype(np.float64)
+    T0 = [rng.integers(-8, 8, (f.rows, f.dim)).astype(np.float64) for f in m.features]
+    g1, cn, ab = oracle.embedding_bag_backward(rows, m.dims, [0] * m.F, b.indices, b.offsets, b.B, G)
+    g2, _, _ = oracle.embedding_bag_backward(rows, m.dims, [0] * m.F, b.indices, b.offsets, b.B, G, scale=-0.5,
+                                             targets=T0)
+    for f in range(m.F):
+        assert np.array_equal(g2[f], T0[f] - 0.5 * g1[f])
+        assert np.all(ab[f] >= np.abs(g1[f]))
+        nnz = b.offsets[(f + 1) * b.B] - b.offsets[f * b.B]
+        assert cn[f].sum() == nnz
