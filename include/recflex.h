@@ -295,6 +295,29 @@ recflex_status_t recflex_forward_routed(recflex_plan_t plan, const int32_t *indi
                                         int32_t num_dst, int32_t rows_per_dst, int32_t dst_stride,
                                         int32_t col_base, void *stream);
 
+/* ---- backward (training) --------------------------------- */
+
+/* The adjoint of recflex_forward (training is "not fundamentally
+ * excluded"): for every bag (f, s) of the batch and every lookup j in it,
+ *     targets[f][indices[j]][c] += scale * w * grad[s][col_f + c],   c < d_f,
+ * w = 1 (SUM) or 1/L (MEAN, L the bag length; empty bags contribute nothing).
+ * scale = 1 into zeroed buffers gives the dense table gradients; targets =
+ * the (float32) tables and scale = -lr is one fused SGD step.
+ *   grad    : DEVICE float32 [B][D_tot], 16-byte aligned (the gradient of out)
+ *   targets : HOST array of F DEVICE float32 [rows_f][d_f] buffers, 16-byte
+ *             aligned, updated in place (independent of the tables' storage
+ *             dtype: fp32 master weights / gradient buffers)
+ * Runs the plan's map kernel and a persistent scatter kernel over the same
+ * task map as the forward (one CTA-task = the forward task's samples); each
+ * bag's gradient row is loaded once and added to its rows with vector
+ * reductions in L2 (red.global.add.v4.f32).  Contributions to one row from
+ * different bags are added in no fixed order: results are exact when every
+ * partial sum is representable (integer data), else within the fp32
+ * summation bound.  Async on `stream`, no allocation after the first call. */
+recflex_status_t recflex_backward(recflex_plan_t plan, const int32_t *indices, const int32_t *offsets,
+                                  int32_t batch_size, const float *grad, float *const *targets, float scale,
+                                  void *stream);
+
 /* CUDA IPC helpers for the routed forward across processes: 64-byte handle of
  * a device allocation, map a peer process's handle, unmap. */
 recflex_status_t recflex_ipc_get_handle(const void *d_ptr, void *handle64);

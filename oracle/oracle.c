@@ -238,13 +238,15 @@ int oracle_embedding_bag_backward(int F, int B, const int *dims, const int *pool
             const int64_t lo = offsets[(int64_t)f * B + s];
             const int64_t hi = offsets[(int64_t)f * B + s + 1];
             const int64_t L = hi - lo;
-            const double w = (pools[f] == POOL_MEAN && L > 0) ? 1.0 / (double)L : 1.0;
+            /* MEAN: the term is G / L (a division, as the forward divides the sum
+             * by L): exact whenever G is a multiple of L, unlike G * fl(1/L) */
+            const int mean = pools[f] == POOL_MEAN && L > 0;
             const double *g = grad + (int64_t)s * d_tot + col;
             for (int64_t j = lo; j < hi; ++j) {
                 const int64_t r = indices[j];
                 if (r < 0 || r >= rows[f]) return ORACLE_ERR_INDEX;
                 for (int c = 0; c < d; ++c) {
-                    const double term = scale * w * g[c];
+                    const double term = scale * (mean ? g[c] / (double)L : g[c]);
                     targets[f][r * d + c] += term;
                     if (abssum) abssum[f][r * d + c] += term < 0 ? -term : term;
                 }

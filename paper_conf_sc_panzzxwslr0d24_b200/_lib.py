@@ -89,6 +89,8 @@ SIGNATURES = {
     'recflex_l2_flush': (c_int32, [c_void_p, ctypes.c_size_t, c_void_p]),
     'recflex_forward_routed': (c_int32, [c_void_p, c_void_p, c_void_p, c_int32, P(c_void_p), P(c_void_p), c_int32,
                                          c_int32, c_int32, c_int32, c_void_p]),
+    'recflex_backward': (c_int32, [c_void_p, c_void_p, c_void_p, c_int32, c_void_p, P(c_void_p), ctypes.c_float,
+                                   c_void_p]),
     'recflex_ipc_get_handle': (c_int32, [c_void_p, c_void_p]),
     'recflex_ipc_open_handle': (c_int32, [c_void_p, P(c_void_p)]),
     'recflex_ipc_close': (c_int32, [c_void_p]),

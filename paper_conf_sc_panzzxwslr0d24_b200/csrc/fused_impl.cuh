@@ -168,8 +168,10 @@ __device__ __forceinline__ void fill_slot(TaskSlot &S, int n, const FusedArgs &a
     st_release(&S.state, 2);
 }
 
-template <int KOCC>
-__global__ void __launch_bounds__(kBlockThreads, KOCC) recflex_fused_kernel(FusedArgs a) {
+// BWD = false: the forward (gather + pool, catalog dispatch).  BWD = true: the
+// backward scatter (sched_backward) over the SAME task map and task ring.
+template <int KOCC, bool BWD>
+__device__ __forceinline__ void fused_body(const FusedArgs &a) {
     extern __shared__ __align__(16) unsigned char dyn_smem[];
     __shared__ TaskSlot ring[kRing];
     float *red = reinterpret_cast<float *>(dyn_smem);                            // union member 1
@@ -242,15 +244,21 @@ __global__ void __launch_bounds__(kBlockThreads, KOCC) recflex_fused_kernel(Fuse
         const long long w0 = a.timers ? clock64() : 0;
         const int f = vld(&S.f);
         const FeatureDesc fd = a.desc[f];
-        const bool cta_wide = kFamilyDev[fd.sched] == RECFLEX_FAMILY_BLOCK;
+        const bool cta_wide = !BWD && kFamilyDev[fd.sched] == RECFLEX_FAMILY_BLOCK;
         if (cta_wide) __syncthreads();  // every warp reaches task n (they walk the same sequence)
         OutRoute ro;
         ro.ptrs = a.out_ptrs;
         ro.rows = a.route_rows;
         ro.colofs = a.col_base + fd.col;
         ro.stride = a.out_stride;
-        dispatch_task(fd.sched, static_cast<const char *>(fd.table), (unsigned)fd.row_bytes, a.offsets + (size_t)fd.in_feature * a.B, a.indices, a.out + fd.col, fd.dim,
-                      fd.pool, ro, vld(&S.s0), vld(&S.s1), red, &S.bag, wsmem, wbytes);
+        if constexpr (BWD) {
+            sched_backward(a.grad + fd.col, a.out_stride, a.targets[f], a.offsets + (size_t)fd.in_feature * a.B,
+                           a.indices, fd.dim, fd.pool, a.bscale, vld(&S.s0), vld(&S.s1), &S.bag, a.bvec != 0);
+        } else {
+            dispatch_task(fd.sched, static_cast<const char *>(fd.table), (unsigned)fd.row_bytes,
+                          a.offsets + (size_t)fd.in_feature * a.B, a.indices, a.out + fd.col, fd.dim, fd.pool, ro,
+                          vld(&S.s0), vld(&S.s1), red, &S.bag, wsmem, wbytes);
+        }
         if (cta_wide) __syncthreads();
         __syncwarp();
         if (lane == 0) {
@@ -266,6 +274,16 @@ __global__ void __launch_bounds__(kBlockThreads, KOCC) recflex_fused_kernel(Fuse
 }
 
 template <int KOCC>
+__global__ void __launch_bounds__(kBlockThreads, KOCC) recflex_fused_kernel(FusedArgs a) {
+    fused_body<KOCC, false>(a);
+}
+
+template <int KOCC>
+__global__ void __launch_bounds__(kBlockThreads, KOCC) recflex_backward_kernel(FusedArgs a) {
+    fused_body<KOCC, true>(a);
+}
+
+template <int KOCC, bool BWD>
 int fused_launch_impl(const FusedArgs &a, const LaunchCfg &cfg, void *stream) {
     cudaLaunchConfig_t lc = {};
     lc.gridDim = dim3(cfg.grid);
@@ -277,7 +295,8 @@ int fused_launch_impl(const FusedArgs &a, const LaunchCfg &cfg, void *stream) {
     attr[0].val.programmaticStreamSerializationAllowed = cfg.pdl ? 1 : 0;
     lc.attrs = attr;
     lc.numAttrs = 1;
-    return (int)cudaLaunchKernelEx(&lc, recflex_fused_kernel<KOCC>, a);
+    if constexpr (BWD) return (int)cudaLaunchKernelEx(&lc, recflex_backward_kernel<KOCC>, a);
+    else return (int)cudaLaunchKernelEx(&lc, recflex_fused_kernel<KOCC>, a);
 }
 
 template <int KOCC>
@@ -285,6 +304,11 @@ int fused_prepare_impl(int smem) {
     cudaError_t e = cudaFuncSetAttribute(recflex_fused_kernel<KOCC>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return (int)e;
     e = cudaFuncSetAttribute(recflex_fused_kernel<KOCC>, cudaFuncAttributePreferredSharedMemoryCarveout,
+                             cudaSharedmemCarveoutMaxShared);
+    if (e != cudaSuccess) return (int)e;
+    e = cudaFuncSetAttribute(recflex_backward_kernel<KOCC>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return (int)e;
+    e = cudaFuncSetAttribute(recflex_backward_kernel<KOCC>, cudaFuncAttributePreferredSharedMemoryCarveout,
                              cudaSharedmemCarveoutMaxShared);
     return (int)e;
 }
@@ -305,7 +329,10 @@ int fused_occupancy_impl(int smem, int *blocks, int *regs, int *spill) {
 #define RECFLEX_INSTANTIATE_FUSED(K)                                                                          \
     namespace recflex {                                                                                       \
     int fused_launch_k##K(const FusedArgs &a, const LaunchCfg &cfg, void *stream) {                           \
-        return fused_launch_impl<K>(a, cfg, stream);                                                          \
+        return fused_launch_impl<K, false>(a, cfg, stream);                                                   \
+    }                                                                                                         \
+    int backward_launch_k##K(const FusedArgs &a, const LaunchCfg &cfg, void *stream) {                        \
+        return fused_launch_impl<K, true>(a, cfg, stream);                                                    \
     }                                                                                                         \
     int fused_prepare_k##K(int smem) { return fused_prepare_impl<K>(smem); }                                  \
     int fused_occupancy_k##K(int smem, int *b, int *r, int *s) { return fused_occupancy_impl<K>(smem, b, r, s); } \

@@ -23,6 +23,14 @@ int fused_launch_k5(const FusedArgs &, const LaunchCfg &, void *);
 int fused_launch_k6(const FusedArgs &, const LaunchCfg &, void *);
 int fused_launch_k7(const FusedArgs &, const LaunchCfg &, void *);
 int fused_launch_k8(const FusedArgs &, const LaunchCfg &, void *);
+int backward_launch_k1(const FusedArgs &, const LaunchCfg &, void *);
+int backward_launch_k2(const FusedArgs &, const LaunchCfg &, void *);
+int backward_launch_k3(const FusedArgs &, const LaunchCfg &, void *);
+int backward_launch_k4(const FusedArgs &, const LaunchCfg &, void *);
+int backward_launch_k5(const FusedArgs &, const LaunchCfg &, void *);
+int backward_launch_k6(const FusedArgs &, const LaunchCfg &, void *);
+int backward_launch_k7(const FusedArgs &, const LaunchCfg &, void *);
+int backward_launch_k8(const FusedArgs &, const LaunchCfg &, void *);
 int fused_prepare_k1(int);
 int fused_prepare_k2(int);
 int fused_prepare_k3(int);
@@ -50,6 +58,20 @@ int fused_launch(int k, const FusedArgs &a, const LaunchCfg &cfg, void *stream) 
         case 6: return fused_launch_k6(a, cfg, stream);
         case 7: return fused_launch_k7(a, cfg, stream);
         case 8: return fused_launch_k8(a, cfg, stream);
+        default: return (int)cudaErrorInvalidValue;
+    }
+}
+
+int backward_launch(int k, const FusedArgs &a, const LaunchCfg &cfg, void *stream) {
+    switch (k) {
+        case 1: return backward_launch_k1(a, cfg, stream);
+        case 2: return backward_launch_k2(a, cfg, stream);
+        case 3: return backward_launch_k3(a, cfg, stream);
+        case 4: return backward_launch_k4(a, cfg, stream);
+        case 5: return backward_launch_k5(a, cfg, stream);
+        case 6: return backward_launch_k6(a, cfg, stream);
+        case 7: return backward_launch_k7(a, cfg, stream);
+        case 8: return backward_launch_k8(a, cfg, stream);
         default: return (int)cudaErrorInvalidValue;
     }
 }

@@ -253,14 +253,18 @@ recflex_status_t run_pipeline(recflex_plan_s *p, const Exec &ex, const int32_t *
     a.out_ptrs = ex.out_ptrs;
     a.route_rows = ex.route_rows;
     a.col_base = ex.col_base;
+    a.grad = ex.grad;
+    a.targets = ex.d_targets;
+    a.bscale = ex.bscale;
+    a.bvec = ex.bvec;
     LaunchCfg cfg;
     cfg.grid = p->num_sms * p->occ[k];
     cfg.smem = p->smem[k];
     // With events between the kernels, PDL overlap is disabled (the event is a
     // stream dependency point anyway).
     cfg.pdl = p->pdl && ev == nullptr;
-    rc = fused_launch(k, a, cfg, stream);
-    if (rc) return cuda_status_at((cudaError_t)rc, "fused kernel launch");
+    rc = ex.backward ? backward_launch(k, a, cfg, stream) : fused_launch(k, a, cfg, stream);
+    if (rc) return cuda_status_at((cudaError_t)rc, ex.backward ? "backward kernel launch" : "fused kernel launch");
     if (ev) cudaEventRecord(ev->e2, stream);
     return RECFLEX_OK;
 }
@@ -312,6 +316,7 @@ int32_t recflex_catalog_valid_dtype(int32_t id, int32_t dim, int32_t dtype) {
 
 static void plan_free_device(recflex_plan_s *p) {
     cudaFree(p->d_route);
+    cudaFree(p->d_targets);
     cudaFree(p->ex.d_desc);
     cudaFree(p->ex.d_block_start);
     cudaFree(p->ex.d_npb_eff);
@@ -519,6 +524,44 @@ recflex_status_t recflex_forward_routed(recflex_plan_t p, const int32_t *indices
     ex.route_rows = rows_per_dst;
     ex.col_base = col_base;
     return run_pipeline(p, ex, indices, offsets, B, host_dst[0], dst_stride, p->k, stream, nullptr);
+}
+
+recflex_status_t recflex_backward(recflex_plan_t p, const int32_t *indices, const int32_t *offsets, int32_t B,
+                                  const float *grad, float *const *targets, float scale, void *stream_) {
+    if (!p || !targets || B < 0 || B > p->max_batch) return RECFLEX_ERR_INVALID_ARG;
+    if (B == 0) return RECFLEX_OK;
+    if (!indices || !offsets || !grad || ((uintptr_t)grad) % 16) return RECFLEX_ERR_INVALID_ARG;
+    for (int f = 0; f < p->F; ++f)
+        if (!targets[f] || ((uintptr_t)targets[f]) % 16) return RECFLEX_ERR_INVALID_ARG;
+    cudaStream_t stream = (cudaStream_t)stream_;
+    cudaSetDevice(p->device);
+    // the task map reads the descriptors (schedules, part); tables are not read
+    if (p->desc_dirty) {
+        recflex_status_t st = upload_desc(p, stream);
+        if (st != RECFLEX_OK) return st;
+    }
+    bool same = (int)p->targets_cache.size() == p->F;
+    for (int f = 0; same && f < p->F; ++f) same = p->targets_cache[f] == targets[f];
+    if (!same) {
+        if (!p->d_targets) {
+            cudaError_t e = cudaMalloc(&p->d_targets, sizeof(float *) * p->F);
+            if (e != cudaSuccess) return cuda_status(e);
+        }
+        p->targets_cache.assign(targets, targets + p->F);
+        cudaError_t e = cudaMemcpyAsync(p->d_targets, p->targets_cache.data(), sizeof(float *) * p->F,
+                                        cudaMemcpyHostToDevice, stream);
+        if (e != cudaSuccess) return cuda_status(e);
+    }
+    Exec ex = p->ex;
+    ex.backward = true;
+    ex.grad = grad;
+    ex.d_targets = p->d_targets;
+    ex.bscale = scale;
+    int vec_ok = (p->d_tot % 4) == 0;
+    for (int f = 0; f < p->F && vec_ok; ++f)
+        if (p->desc[f].dim % 4 == 0 && p->desc[f].col % 4 != 0) vec_ok = 0;
+    ex.bvec = vec_ok;
+    return run_pipeline(p, ex, indices, offsets, B, nullptr, (int)p->d_tot, p->k, stream, nullptr);
 }
 
 recflex_status_t recflex_ipc_get_handle(const void *d_ptr, void *handle64) {

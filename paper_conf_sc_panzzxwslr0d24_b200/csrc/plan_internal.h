@@ -25,6 +25,12 @@ struct Exec {
     float *const *out_ptrs = nullptr;  // routed mode: device array of destination buffers
     int route_rows = 0;                // 0 = local output
     int col_base = 0;
+    // backward (NEXT #4)
+    bool backward = false;
+    const float *grad = nullptr;
+    float *const *d_targets = nullptr;
+    float bscale = 1.f;
+    int bvec = 0;
 };
 
 struct EventTriple {
@@ -68,6 +74,9 @@ struct recflex_plan_s {
     // routed forward: destination pointer table (device) and its host copy
     float **d_route = nullptr;
     std::vector<float *> route_cache;
+    // backward: target pointer table (device) and its host copy
+    float **d_targets = nullptr;
+    std::vector<float *> targets_cache;
     int32_t *d_stage_idx = nullptr;
     int64_t stage_idx_cap = 0;
     int32_t *d_stage_off = nullptr;

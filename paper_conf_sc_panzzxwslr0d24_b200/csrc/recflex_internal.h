@@ -72,6 +72,11 @@ struct FusedArgs {
     float *const *out_ptrs;       // device array of destination pointers (peer / IPC-mapped)
     int32_t route_rows;           // 0 = local mode (out + s * out_stride + col_f)
     int32_t col_base;
+    // backward (NEXT #4): grad [B][out_stride], targets[f] fp32 [rows_f][d_f]
+    const float *grad;
+    float *const *targets;        // device array of F target pointers
+    float bscale;
+    int32_t bvec;                 // 1: 16-byte aligned grad columns (D_tot, col_f multiples of 4)
 };
 
 // ---------------------------------------------------------------------------
@@ -184,6 +189,7 @@ struct LaunchCfg {
 };
 
 int fused_launch(int k, const FusedArgs &a, const LaunchCfg &cfg, void *stream);  // returns cudaError_t
+int backward_launch(int k, const FusedArgs &a, const LaunchCfg &cfg, void *stream);
 int fused_prepare(int k, int device, int smem_bytes);                              // cudaFuncSetAttribute
 int fused_occupancy(int k, int smem_bytes, int *blocks, int *regs, int *spill);
 int map_launch(const MapArgs &a, void *stream);

@@ -705,6 +705,71 @@ __device__ __noinline__ void sched_bulk(const float *__restrict__ T, const int32
     }
 }
 
+// ---- backward (training) --------------------------------------
+// The adjoint of the pooled gather: for every bag (f, s) of the task and every
+// lookup j of it, target[idx[j]][c] += scale * w * grad[s][col_f + c] with
+// w = 1 (SUM) or 1/L (MEAN, the correctly rounded fp32 quotient).  A group of
+// G lanes holds the bag's gradient row in registers (loaded once, 16-byte
+// loads) and scatters it to the bag's rows with vector reductions at L2
+// (red.global.add.v4.f32, sm_90+): no read-modify-write round trip through the
+// SM.  Bags are claimed dynamically as in GROUP; the reduction order across
+// bags is not fixed (fp32 adds in L2 commute only up to rounding) -> results
+// are exact when every partial sum is exactly representable (integer data)
+// and within the summation bound otherwise.
+__device__ __forceinline__ void red_add_v4(float *p, float a, float b, float c, float d) {
+    asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(p), "f"(a), "f"(b), "f"(c), "f"(d)
+                 : "memory");
+}
+
+static __device__ __noinline__ void sched_backward(const float *__restrict__ grad, int gstride, float *__restrict__ target,
+                                            const int32_t *__restrict__ offs, const int32_t *__restrict__ idx, int d,
+                                            int pool, float scale, int s0, int s1, int *bag_ctr, bool vec_ok) {
+    const bool vec = vec_ok && (d % 4) == 0;  // 16-byte aligned grad columns and target rows
+    const int per_lane = vec ? 4 : 1;
+    int G = 1;
+    while (G < 32 && G * per_lane < d) G <<= 1;
+    const int lane = threadIdx.x & 31;
+    const int lg = lane & (G - 1);
+    const unsigned gmask = (G == 32) ? 0xffffffffu : (((1u << G) - 1u) << (lane & ~(G - 1)));
+    const int span = G * per_lane;
+    while (true) {
+        int v = 0;
+        if (lg == 0) v = atomicAdd(bag_ctr, 1);
+        const int s = s0 + __shfl_sync(gmask, v, 0, G);
+        if (s >= s1) break;
+        const int lo = ld_idx(offs + s), hi = ld_idx(offs + s + 1);
+        const int L = hi - lo;
+        if (L == 0) continue;
+        const float *gr = grad + (size_t)s * gstride;
+        for (int col = lg * per_lane; col < d; col += span) {
+            if (vec) {
+                const float4 g4 = *reinterpret_cast<const float4 *>(gr + col);
+                float g[4] = {g4.x, g4.y, g4.z, g4.w};
+#pragma unroll
+                for (int e = 0; e < 4; ++e) {
+                    if (pool == RECFLEX_POOL_MEAN) g[e] = div_by_len(g[e], L);
+                    g[e] *= scale;
+                }
+                int j = lo;
+                for (; j + 4 <= hi; j += 4) {  // 4 lookup IDs in flight, then 4 reductions
+                    unsigned id[4];
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) id[u] = (unsigned)ld_idx(idx + j + u);
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) red_add_v4(target + (size_t)id[u] * (unsigned)d + col, g[0], g[1], g[2], g[3]);
+                }
+                for (; j < hi; ++j)
+                    red_add_v4(target + (size_t)(unsigned)ld_idx(idx + j) * (unsigned)d + col, g[0], g[1], g[2], g[3]);
+            } else {
+                float g = gr[col];
+                if (pool == RECFLEX_POOL_MEAN) g = div_by_len(g, L);
+                g *= scale;
+                for (int j = lo; j < hi; ++j) atomicAdd(target + (size_t)(unsigned)ld_idx(idx + j) * (unsigned)d + col, g);
+            }
+        }
+    }
+}
+
 // ---- BLOCK family ----------------------------------------------------------
 // One bag at a time for the whole CTA.  Group g takes lookups lo+g, lo+g+NG, ...
 // (adjacent groups read adjacent IDs: coalesced index loads).  Partials:

@@ -183,6 +183,31 @@ class Plan:
               'recflex_forward_host')
         return out
 
+    # -------------------------------------------------------------- backward (NEXT #4)
+    def backward(self, indices: torch.Tensor, offsets: torch.Tensor, B: int, grad: torch.Tensor,
+                 targets: Sequence[torch.Tensor], scale: float = 1.0, stream=None):
+        """recflex_backward: targets[f][id] += scale * w * grad[s][col_f:] for every lookup
+        (dense table gradients with zeroed targets and scale 1; SGD with targets = tables,
+        scale = -lr).  targets: F contiguous CUDA float32 [rows_f, d_f]."""
+        if offsets.numel() != self.F * B + 1:
+            raise ValueError('offsets must have F*B+1 entries')
+        if grad.shape != (B, self.d_tot):
+            raise ValueError(f'grad must be [B, D_tot] = [{B}, {self.d_tot}]')
+        if len(targets) != self.F:
+            raise ValueError(f'expected {self.F} targets')
+        for f, t in enumerate(targets):
+            check_table(t, self.dims[f], 0)
+        tarr = (ctypes.c_void_p * self.F)(*[t.data_ptr() for t in targets])
+        idx_ptr = _dptr(indices, torch.int32, 'indices') if indices.numel() else ctypes.c_void_p(offsets.data_ptr())
+        check(lib.recflex_backward(self._h, idx_ptr, _dptr(offsets, torch.int32, 'offsets'), int(B),
+                                   _dptr(grad, torch.float32, 'grad'), tarr, float(scale), _stream_ptr(stream)),
+              'recflex_backward')
+
+    def sgd_step(self, indices: torch.Tensor, offsets: torch.Tensor, B: int, grad: torch.Tensor,
+                 tables: Sequence[torch.Tensor], lr: float, stream=None):
+        """One fused SGD update of float32 tables: T -= lr * dLoss/dT (recflex_backward, scale = -lr)."""
+        self.backward(indices, offsets, B, grad, tables, scale=-float(lr), stream=stream)
+
     # -------------------------------------------------------------- tuner
     def tune(self, batches: Sequence[tuple], tables: Sequence[torch.Tensor], occupancies: Optional[List[int]] = None,
              reps: int = 7, pad_waves: int = 4, max_candidates: int = 0, verbose: bool = False, guard: bool = True,
