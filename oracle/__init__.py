@@ -20,6 +20,11 @@ Functions and the passages they follow (PAPER.md "P:n"):
                     dense gradient / SGD update of every table row.
   task_map       -- Fig. 8: d_blocks_map and d_task_map, reading C12.
   nnz_task_ranges-- reading C12 for nnz-partitioned schedules.
+  kjt_input_dist -- table-wise input distribution (P:350
+                    "place different embedding tables on multiple GPUs"):
+                    the data-parallel KJTs of W ranks regrouped so that every
+                    rank holds all B samples of the features it owns.  Pure
+                    integer data movement, written in numpy (no C needed).
 """
 from __future__ import annotations
 
@@ -253,6 +258,37 @@ def nnz_task_ranges(B, npb, feature_offsets, blocks):
     if rc != 0:
         raise OracleError(rc)
     return s0[:blocks].copy(), s1[:blocks].copy()
+
+
+def kjt_input_dist(local_kjts, parts, local_batch):
+    """Table-wise input distribution, the plain definition.
+
+    local_kjts[j] = (indices, offsets) of rank j: a feature-major KJT over ALL F
+    features and rank j's Bl = local_batch samples (global samples
+    j*Bl .. (j+1)*Bl-1), offsets[F*Bl+1].  parts[r] = the features rank r owns.
+    Returns, for every rank r, (indices, offsets) of the KJT over r's features
+    (in the order given by parts[r]) and all B = W*Bl global samples in global
+    order: bag (k, s) of the result = bag (parts[r][k], s mod Bl) of rank
+    s // Bl.  Bags keep their IDs in order.
+    """
+    W, Bl = len(local_kjts), int(local_batch)
+    out = []
+    for r in range(len(parts)):
+        ids, lens = [], []
+        for f in parts[r]:
+            for j in range(W):                       # global sample order = (source rank, local sample)
+                idx_j = np.asarray(local_kjts[j][0])
+                off_j = np.asarray(local_kjts[j][1], np.int64)
+                for s in range(Bl):
+                    a, b = off_j[f * Bl + s], off_j[f * Bl + s + 1]
+                    if b < a:
+                        raise OracleError('bad offsets')
+                    ids.append(idx_j[a:b])
+                    lens.append(b - a)
+        off = np.zeros(len(lens) + 1, np.int64)
+        np.cumsum(np.asarray(lens, np.int64), out=off[1:])
+        out.append((np.concatenate(ids).astype(np.int32) if ids else np.zeros(0, np.int32), off.astype(np.int32)))
+    return out
 
 
 # ---------------------------------------------------------------------------

@@ -496,3 +496,61 @@ def test_backward_scale_and_initial_targets():
         assert np.all(ab[f] >= np.abs(g1[f]))
         nnz = b.offsets[(f + 1) * b.B] - b.offsets[f * b.B]
         assert cn[f].sum() == nnz
+
+
+# ---- table-wise input distribution -------------------
+
+KJTD = os.path.join(os.path.dirname(__file__), 'golden', 'kjt_input_dist.json')
+
+
+def test_kjt_input_dist_golden():
+    """Hand-worked 2-rank example (tests/golden/kjt_input_dist.json)."""
+    g = json.load(open(KJTD))
+    locs = [(np.asarray(k['indices'], np.int32), np.asarray(k['offsets'], np.int32)) for k in g['local_kjts']]
+    # the golden local KJTs are the hand-written bags, laid out feature-major
+    for j, kjt in enumerate(locs):
+        bags = g['local_bags'][f'rank{j}']
+        flat = [bag for f in range(3) for bag in bags[f'f{f}']]
+        assert kjt[0].tolist() == [i for bag in flat for i in bag]
+        assert np.diff(kjt[1]).tolist() == [len(bag) for bag in flat]
+    got = oracle.kjt_input_dist(locs, g['parts'], g['local_batch'])
+    for r, exp in enumerate(g['expected']):
+        assert got[r][0].tolist() == exp['indices']
+        assert got[r][1].tolist() == exp['offsets']
+
+
+def _sample_split(idx, off, F, B, W):
+    """Global KJT -> W data-parallel local KJTs (rank j: samples [j*B/W, (j+1)*B/W))."""
+    Bl = B // W
+    out = []
+    for j in range(W):
+        lens = np.diff(off.astype(np.int64)).reshape(F, B)[:, j * Bl:(j + 1) * Bl]
+        ids = np.concatenate([idx[off[f * B + j * Bl]:off[f * B + (j + 1) * Bl]] for f in range(F)])
+        o = np.concatenate([[0], np.cumsum(lens.reshape(-1))]).astype(np.int32)
+        out.append((ids.astype(np.int32), o))
+    return out
+
+
+@pytest.mark.parametrize('W', [1, 2, 4])
+def test_kjt_input_dist_equals_feature_restriction(W):
+    """Splitting a global KJT by samples and redistributing it by features gives
+    exactly the global KJT restricted to each rank's features (the operation's
+    defining property; both sides written here with plain slicing)."""
+    m = synth.make_model('tiny')
+    b = synth.make_batch(m, 11)
+    F, B = m.F, b.B
+    rng = np.random.default_rng(W)
+    owner = rng.integers(0, W, F)
+    parts = [[f for f in range(F) if owner[f] == r] for r in range(W)]
+    got = oracle.kjt_input_dist(_sample_split(b.indices, b.offsets, F, B, W), parts, B // W)
+    for r in range(W):
+        ids = [b.indices[b.offsets[f * B]:b.offsets[(f + 1) * B]] for f in parts[r]]
+        lens = [np.diff(b.offsets[f * B:(f + 1) * B + 1]) for f in parts[r]]
+        exp_idx = np.concatenate(ids) if ids else np.zeros(0, np.int32)
+        exp_off = np.concatenate([[0], np.cumsum(np.concatenate(lens))]) if lens else np.zeros(1)
+        assert np.array_equal(got[r][0], exp_idx)
+        assert np.array_equal(got[r][1], exp_off)
+    # invariants: every ID arrives exactly once, W = 1 with all features is the identity
+    assert sum(g[0].size for g in got) == b.indices.size
+    if W == 1:
+        assert np.array_equal(got[0][0], b.indices) and np.array_equal(got[0][1], b.offsets)
