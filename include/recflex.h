@@ -336,6 +336,48 @@ recflex_status_t recflex_device_free(void *d_ptr);
 recflex_status_t recflex_shard_concat(const float *recv, int32_t num_ranks, int32_t rows,
                                       const int32_t *host_dims, float *out, void *stream);
 
+/* ---- table-wise input distribution ----------------- */
+
+/* The KJT all-to-all in front of a table-wise sharded forward (TorchRec's
+ * "input dist"; PAPER.md P:350 places whole tables on GPUs).  W ranks; rank j
+ * holds a data-parallel KJT over ALL F features and its Bl local samples
+ * (global samples j*Bl .. j*Bl+Bl-1): indices int32[nnz_j], offsets
+ * int32[F*Bl+1], feature-major as in recflex_forward.  After pack ->
+ * alltoallv (caller's, e.g. NCCL) -> unpack, rank r holds the KJT of the
+ * features it owns (ascending feature id) over all B = W*Bl samples in global
+ * order -- exactly the input recflex_forward of its plan takes.
+ *
+ * create: feature_owner[F] (host) = owning rank of every feature; the handle
+ *   owns small device scratch (O(F + W*F_r)); device = CUDA ordinal.
+ *   F*Bl and W*Bl must be < 2^31.  Errors: INVALID_ARG, CUDA/OOM. */
+typedef struct recflex_kjt_dist_s *recflex_kjt_dist_t;
+recflex_status_t recflex_kjt_dist_create(int32_t num_features, const int32_t *feature_owner, int32_t num_ranks,
+                                         int32_t rank, int32_t local_batch, int32_t device,
+                                         recflex_kjt_dist_t *out);
+void recflex_kjt_dist_destroy(recflex_kjt_dist_t dist);
+/* Host-known alltoallv sizes of the LENGTHS exchange (in int32 elements, per
+ * peer, arrays of num_ranks) and the number of owned features F_r. */
+recflex_status_t recflex_kjt_dist_sizes(recflex_kjt_dist_t dist, int32_t *send_length_counts,
+                                        int32_t *recv_length_counts, int32_t *num_owned);
+/* Sender side (all DEVICE pointers, async on stream, no allocation):
+ *   send_lengths int32[F*Bl]: for every destination r in rank order, for every
+ *     feature r owns (ascending id), the Bl bag lengths of this rank's samples;
+ *   send_indices int32[nnz_local]: the same (destination, feature) order, each
+ *     feature's IDs as one contiguous run (sample order kept);
+ *   dest_counts int32[W]: IDs sent to each rank (the IDs alltoallv splits).
+ * Offsets must be monotone (undefined otherwise, as in recflex_forward). */
+recflex_status_t recflex_kjt_pack(recflex_kjt_dist_t dist, const int32_t *indices, const int32_t *offsets,
+                                  int32_t *send_lengths, int32_t *send_indices, int32_t *dest_counts,
+                                  void *stream);
+/* Receiver side (DEVICE pointers, async on stream, no allocation):
+ *   recv_lengths int32[W*F_r*Bl]: what pack sent here, concatenated in source
+ *     rank order ([j][k][s]); recv_indices: the received IDs, same order;
+ *   indices_out int32[sum of recv IDs], offsets_out int32[F_r*W*Bl+1]: the
+ *     owned features' KJT, feature-major, samples in global order. */
+recflex_status_t recflex_kjt_unpack(recflex_kjt_dist_t dist, const int32_t *recv_lengths,
+                                    const int32_t *recv_indices, int32_t *indices_out, int32_t *offsets_out,
+                                    void *stream);
+
 /* Writes `bytes` of a device scratch buffer to evict L2 (timing hygiene). */
 recflex_status_t recflex_l2_flush(void *d_scratch, size_t bytes, void *stream);
 

@@ -348,3 +348,71 @@ def ipc_close(ptr: int):
 def l2_flush(buf: torch.Tensor, stream=None):
     check(lib.recflex_l2_flush(ctypes.c_void_p(buf.data_ptr()), buf.numel() * buf.element_size(),
                                _stream_ptr(stream)), 'recflex_l2_flush')
+
+
+class KJTDist:
+    """recflex_kjt_dist_* : the table-wise input distribution's two device
+    passes around the caller's alltoallv (include/recflex.h).
+
+    owner[f] = rank owning feature f; this object is rank `rank`'s view with
+    `local_batch` samples per rank.  pack/unpack take and fill caller-owned
+    int32 CUDA tensors (no allocation inside the library)."""
+
+    def __init__(self, owner: Sequence[int], world: int, rank: int, local_batch: int, device: int = 0):
+        F = len(owner)
+        arr = (ctypes.c_int32 * F)(*[int(o) for o in owner])
+        self._h = ctypes.c_void_p()
+        check(lib.recflex_kjt_dist_create(F, arr, int(world), int(rank), int(local_batch), int(device),
+                                          ctypes.byref(self._h)), 'recflex_kjt_dist_create')
+        self.F, self.world, self.rank, self.local_batch = F, int(world), int(rank), int(local_batch)
+        sl = (ctypes.c_int32 * world)()
+        rl = (ctypes.c_int32 * world)()
+        fr = ctypes.c_int32()
+        check(lib.recflex_kjt_dist_sizes(self._h, sl, rl, ctypes.byref(fr)), 'recflex_kjt_dist_sizes')
+        self.send_length_counts = list(sl)
+        self.recv_length_counts = list(rl)
+        self.num_owned = fr.value
+
+    def close(self):
+        if getattr(self, '_h', None) and self._h.value:
+            lib.recflex_kjt_dist_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def pack(self, indices: torch.Tensor, offsets: torch.Tensor, send_lengths: torch.Tensor,
+             send_indices: torch.Tensor, dest_counts: torch.Tensor, stream=None):
+        """recflex_kjt_pack: local KJT -> destination-major lengths / IDs + per-destination ID counts."""
+        if offsets.numel() != self.F * self.local_batch + 1:
+            raise ValueError('offsets must have F*Bl+1 entries')
+        if send_lengths.numel() != self.F * self.local_batch or dest_counts.numel() != self.world:
+            raise ValueError('send_lengths must hold F*Bl, dest_counts W entries')
+        if send_indices.numel() < indices.numel():
+            raise ValueError('send_indices smaller than the local IDs')
+        nul = ctypes.c_void_p(offsets.data_ptr())
+        check(lib.recflex_kjt_pack(self._h, _dptr(indices, torch.int32, 'indices') if indices.numel() else nul,
+                                   _dptr(offsets, torch.int32, 'offsets'),
+                                   _dptr(send_lengths, torch.int32, 'send_lengths') if send_lengths.numel() else nul,
+                                   _dptr(send_indices, torch.int32, 'send_indices') if send_indices.numel() else nul,
+                                   _dptr(dest_counts, torch.int32, 'dest_counts'), _stream_ptr(stream)),
+              'recflex_kjt_pack')
+
+    def unpack(self, recv_lengths: torch.Tensor, recv_indices: torch.Tensor, indices_out: torch.Tensor,
+               offsets_out: torch.Tensor, stream=None):
+        """recflex_kjt_unpack: source-major received buffers -> owned features' KJT (global sample order)."""
+        B = self.world * self.local_batch
+        if recv_lengths.numel() != self.world * self.num_owned * self.local_batch:
+            raise ValueError('recv_lengths must hold W*F_r*Bl entries')
+        if offsets_out.numel() != self.num_owned * B + 1 or indices_out.numel() < recv_indices.numel():
+            raise ValueError('offsets_out must hold F_r*B+1 entries, indices_out the received IDs')
+        nul = ctypes.c_void_p(offsets_out.data_ptr())
+        check(lib.recflex_kjt_unpack(self._h,
+                                     _dptr(recv_lengths, torch.int32, 'recv_lengths') if recv_lengths.numel() else nul,
+                                     _dptr(recv_indices, torch.int32, 'recv_indices') if recv_indices.numel() else nul,
+                                     _dptr(indices_out, torch.int32, 'indices_out') if indices_out.numel() else nul,
+                                     _dptr(offsets_out, torch.int32, 'offsets_out'), _stream_ptr(stream)),
+              'recflex_kjt_unpack')

@@ -88,13 +88,11 @@ def split_sizes(B: int, W: int, dims_per_rank: Sequence[int], rank: int):
     return inp, out
 
 
-def exchange(send, dims_per_rank: Sequence[int], B: int, group=None):
-    """Pooled-output alltoallv: send [B][D_r] -> recv [sum_i B/W*D_i] (chunks in rank order)."""
+def alltoallv(send, input_splits: Sequence[int], output_splits: Sequence[int], group=None):
+    """all_to_all_single with element split sizes; returns the received flat tensor."""
     import torch
     import torch.distributed as dist
-    W = dist.get_world_size(group)
-    rank = dist.get_rank(group)
-    inp, out = split_sizes(B, W, dims_per_rank, rank)
+    inp, out = [int(x) for x in input_splits], [int(x) for x in output_splits]
     recv = torch.empty(sum(out), dtype=send.dtype, device=send.device)
     if send.is_cuda and dist.get_backend(group) == 'gloo':
         # test plumbing only (several ranks sharing one GPU, where NCCL refuses):
@@ -106,6 +104,83 @@ def exchange(send, dims_per_rank: Sequence[int], B: int, group=None):
         return recv
     dist.all_to_all_single(recv, send.reshape(-1), output_split_sizes=out, input_split_sizes=inp, group=group)
     return recv
+
+
+def exchange(send, dims_per_rank: Sequence[int], B: int, group=None):
+    """Pooled-output alltoallv: send [B][D_r] -> recv [sum_i B/W*D_i] (chunks in rank order)."""
+    import torch.distributed as dist
+    W = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    inp, out = split_sizes(B, W, dims_per_rank, rank)
+    return alltoallv(send, inp, out, group)
+
+
+def feature_owner(parts: List[List[int]], F: int) -> List[int]:
+    """owner[f] = the rank whose part holds f (parts must cover 0..F-1 once, each sorted)."""
+    owner = [-1] * F
+    for r, p in enumerate(parts):
+        if list(p) != sorted(p):
+            raise ValueError('each part must list its features in ascending order')
+        for f in p:
+            if not 0 <= f < F or owner[f] != -1:
+                raise ValueError(f'feature {f} out of range or owned twice')
+            owner[f] = r
+    if -1 in owner:
+        raise ValueError('every feature needs an owner')
+    return owner
+
+
+def exchange_kjt(send_lengths, send_indices, dest_counts, send_length_counts: Sequence[int],
+                 recv_length_counts: Sequence[int], group=None):
+    """The collective half of the input distribution (layouts: include/recflex.h
+    recflex_kjt_pack / recflex_kjt_unpack): the per-destination ID counts first
+    (W ints), one host read of them (the alltoallv split sizes NCCL takes from
+    the host), then the lengths (host-known sizes) and the IDs.
+    Returns (recv_lengths, recv_indices, recv_counts list)."""
+    import torch
+    import torch.distributed as dist
+    W = dist.get_world_size(group)
+    recv_counts = alltoallv(dest_counts, [1] * W, [1] * W, group)
+    both = torch.cat([dest_counts.reshape(-1), recv_counts]).cpu().tolist()  # the one host sync
+    send_counts, rc = both[:W], both[W:]
+    recv_lengths = alltoallv(send_lengths, send_length_counts, recv_length_counts, group)
+    recv_indices = alltoallv(send_indices[:sum(send_counts)], send_counts, rc, group)
+    return recv_lengths, recv_indices, rc
+
+
+class KJTInputDist:
+    """Table-wise input distribution: data-parallel local
+    KJTs (all features, Bl samples per rank) -> each rank's owned features over
+    all B = W*Bl samples, ready for its plan's forward.  Device passes in the
+    library (recflex_kjt_pack / recflex_kjt_unpack), collective over
+    torch.distributed (NCCL on GPUs)."""
+
+    def __init__(self, parts: List[List[int]], F: int, rank: int, world: int, local_batch: int, device: int = 0):
+        import torch
+        from .plan import KJTDist
+        self.parts, self.rank, self.world, self.local_batch = parts, rank, world, local_batch
+        self.kd = KJTDist(feature_owner(parts, F), world, rank, local_batch, device)
+        dev = torch.device('cuda', device)
+        self.dev = dev
+        self.send_lengths = torch.empty(F * local_batch, dtype=torch.int32, device=dev)
+        self.dest_counts = torch.empty(world, dtype=torch.int32, device=dev)
+        self.offsets_out = torch.empty(self.kd.num_owned * world * local_batch + 1, dtype=torch.int32, device=dev)
+        self._send_idx = torch.empty(0, dtype=torch.int32, device=dev)
+
+    def forward(self, indices, offsets, group=None, stream=None):
+        """Returns (indices, offsets) of the owned features' global-batch KJT."""
+        import torch
+        if self._send_idx.numel() < indices.numel():
+            self._send_idx = torch.empty(indices.numel(), dtype=torch.int32, device=self.dev)
+        self.kd.pack(indices, offsets, self.send_lengths, self._send_idx, self.dest_counts, stream=stream)
+        rl, ri, rc = exchange_kjt(self.send_lengths, self._send_idx, self.dest_counts, self.kd.send_length_counts,
+                                  self.kd.recv_length_counts, group)
+        idx_out = torch.empty(sum(rc), dtype=torch.int32, device=self.dev)
+        self.kd.unpack(rl, ri, idx_out, self.offsets_out, stream=stream)
+        return idx_out, self.offsets_out
+
+    def close(self):
+        self.kd.close()
 
 
 class ShardedEmbedding:

@@ -126,3 +126,91 @@ def test_gloo_world2_exchange_matches_oracle_slices():
         order = column_order(m, parts)
         exp = full[rank * rows:(rank + 1) * rows][:, order]
         assert np.array_equal(got, exp)
+
+
+# ---- input distribution (KJT all-to-all) ------------
+
+def test_feature_owner():
+    from paper_conf_sc_panzzxwslr0d24_b200.shard import feature_owner
+    assert feature_owner([[0, 2], [1], []], 3) == [0, 1, 0]
+    with pytest.raises(ValueError):
+        feature_owner([[2, 0], [1]], 3)   # unsorted part
+    with pytest.raises(ValueError):
+        feature_owner([[0, 1], [1, 2]], 3)  # owned twice
+    with pytest.raises(ValueError):
+        feature_owner([[0], [2]], 3)  # feature 1 unowned
+
+
+def _np_pack(idx, off, parts, Bl):
+    """The send layout recflex_kjt_pack documents (include/recflex.h), written
+    with plain slicing: destination-major, each owned feature's lengths / IDs."""
+    lens, ids, counts = [], [], []
+    for p in parts:
+        c = 0
+        for f in p:
+            lens.append(np.diff(off[f * Bl:(f + 1) * Bl + 1]))
+            seg = idx[off[f * Bl]:off[(f + 1) * Bl]]
+            ids.append(seg)
+            c += seg.size
+        counts.append(c)
+    cat = lambda xs: np.concatenate(xs).astype(np.int32) if xs else np.zeros(0, np.int32)  # noqa: E731
+    return cat(lens), cat(ids), np.asarray(counts, np.int32)
+
+
+def _np_unpack(recv_lengths, recv_ids, W, Fr, Bl):
+    """The receive layout recflex_kjt_unpack documents: [j][k][s] -> feature-major global order."""
+    L = recv_lengths.reshape(W, Fr, Bl)
+    seg_len = L.sum(axis=2)
+    src = np.concatenate([[0], np.cumsum(seg_len.reshape(-1))])
+    ids, lens = [], []
+    for k in range(Fr):
+        for j in range(W):
+            a = src[j * Fr + k]
+            ids.append(recv_ids[a:a + seg_len[j, k]])
+            lens.append(L[j, k])
+    off = np.concatenate([[0], np.cumsum(np.concatenate(lens))]) if lens else np.zeros(1)
+    return (np.concatenate(ids) if ids else np.zeros(0, np.int32)).astype(np.int32), off.astype(np.int32)
+
+
+def _kjt_worker(rank, world, port, result_q):
+    os.environ['MASTER_ADDR'] = '127.0.0.1'
+    os.environ['MASTER_PORT'] = str(port)
+    dist.init_process_group('gloo', rank=rank, world_size=world)
+    try:
+        from paper_conf_sc_panzzxwslr0d24_b200.shard import exchange_kjt
+        m = synth.make_model('tiny')
+        Bl = m.batch // world
+        loc = synth.make_batch(m, 100 + rank, B=Bl)   # this rank's data-parallel slice
+        parts = partition_model(m, world)
+        sl, si, sc = _np_pack(loc.indices, loc.offsets, parts, Bl)
+        Fr = len(parts[rank])
+        rl, ri, rc = exchange_kjt(torch.from_numpy(sl), torch.from_numpy(si), torch.from_numpy(sc),
+                                  [len(p) * Bl for p in parts], [Fr * Bl] * world)
+        got = _np_unpack(rl.numpy(), ri.numpy(), world, Fr, Bl)
+        result_q.put((rank, got[0], got[1], rc, parts))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_gloo_world2_kjt_input_dist_matches_oracle():
+    """exchange_kjt (the collective half) between the documented pack / unpack
+    layouts reproduces oracle.kjt_input_dist on every rank."""
+    world = 2
+    ctx = mp.get_context('spawn')
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_kjt_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=120) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    m = synth.make_model('tiny')
+    Bl = m.batch // world
+    locs = [synth.make_batch(m, 100 + j, B=Bl) for j in range(world)]
+    parts = res[0][4]
+    exp = oracle.kjt_input_dist([(b.indices, b.offsets) for b in locs], parts, Bl)
+    for rank, idx, off, rc, _ in res:
+        assert np.array_equal(idx, exp[rank][0]) and np.array_equal(off, exp[rank][1])
+        assert sum(rc) == exp[rank][0].size
