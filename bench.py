@@ -211,6 +211,9 @@ def main():
     ap.add_argument('--profile-only', action='store_true', help='short run for ncu (no e2e / cpu / clocks)')
     ap.add_argument('--exchange', default='nccl', choices=['nccl', 'fused'],
                     help='N>1: NCCL alltoallv + relayout kernel, or peer stores fused into the kernel epilogue')
+    ap.add_argument('--input-dist', action='store_true',
+                    help='start each step from data-parallel local batches (B/W samples, all features) and run '
+                         'the KJT input distribution (pack -> alltoallv -> unpack) inside the timed step')
     args = ap.parse_args()
 
     world = int(os.environ.get('WORLD_SIZE', '1'))
@@ -223,7 +226,8 @@ def main():
     import torch
     import torch.distributed as dist
     from paper_conf_sc_panzzxwslr0d24_b200 import synth
-    from paper_conf_sc_panzzxwslr0d24_b200.shard import ShardedEmbedding, partition_model, shard_batch
+    from paper_conf_sc_panzzxwslr0d24_b200.shard import (KJTInputDist, ShardedEmbedding, partition_model,
+                                                          sample_slice, shard_batch)
 
     torch.cuda.set_device(local_rank)
     dev = torch.device('cuda', local_rank)
@@ -251,7 +255,7 @@ def main():
     tables = [phys[model.features[f].table] for f in feats]
 
     # batches: the global batch for my features, resident in HBM
-    batches, host_batches, alg_bytes = [], [], []
+    batches, host_batches, alg_bytes, local_batches = [], [], [], []
     dims_local = np.asarray([model.dims[f] for f in feats], np.int64)
     rowb_local = np.asarray([synth.row_bytes(model.dims[f], args.dtype) for f in feats], np.int64)
     for i in range(args.batches):
@@ -259,6 +263,9 @@ def main():
         idx, off = shard_batch(full, feats)
         host_batches.append((idx, off))
         batches.append((torch.from_numpy(idx).to(dev), torch.from_numpy(off).to(dev)))
+        if args.input_dist:
+            li, lo = sample_slice(full, rank, world)
+            local_batches.append((torch.from_numpy(li).to(dev), torch.from_numpy(lo).to(dev)))
         o = off.astype(np.int64)
         nnz_f = o[np.arange(1, len(feats) + 1) * B] - o[np.arange(0, len(feats)) * B]
         # C26: IDs + gathered rows (stored bytes) + pooled fp32 output
@@ -291,8 +298,13 @@ def main():
     flush_buf = torch.empty(2 * L2_BYTES // 4, dtype=torch.float32, device=dev) if flush_between else None
     stream = torch.cuda.current_stream()
 
+    ind = KJTInputDist(parts, model.F, rank, world, B // world, device=local_rank) if args.input_dist else None
+
     def step(i):
-        bi, bo = batches[i % len(batches)]
+        if ind is not None:
+            bi, bo = ind.forward(*local_batches[i % len(local_batches)])
+        else:
+            bi, bo = batches[i % len(batches)]
         return sh.forward(bi, bo, B, tables, out_local=out_local, out=out_x)
 
     def barrier():
@@ -420,6 +432,7 @@ def main():
 
     launches_per_step = 2 + (1 if plan.export() and any(s[1] == 1 for s in plan.export()['schedules']) else 0)
     launches_per_step += 1 if (world > 1 and args.exchange == 'nccl') else 0   # relayout kernel
+    launches_per_step += 5 if args.input_dist else 0  # pack scan + copy, unpack reduce + scan + main
     if rank == 0:
         line = {
             'metric': _baseline_metric(),
@@ -437,6 +450,8 @@ def main():
             'config': {'workload': args.config, 'global_batch': B, 'fields': model.F, 'table_dtype': args.dtype,
                        'parallelism': f'tablewise{world}', 'plan': plan_src, 'occupancy': plan.occupancy,
                        'exchange': (args.exchange if world > 1 else 'none'),
+                       'input': ('data-parallel local batches + KJT input dist in the timed step'
+                                 if args.input_dist else 'table-wise KJT resident per rank'),
                        'l2': 'flushed between steps' if flush_between else
                              f'inputs > L2 ({alg_local / 1e9:.2f} GB algorithmic per step per rank, '
                              f'{args.batches} rotating batches)'},

@@ -78,6 +78,19 @@ def shard_batch(batch, features: Sequence[int]):
     return idx.astype(np.int32), np.concatenate(off_parts).astype(np.int32)
 
 
+def sample_slice(batch, j: int, W: int):
+    """Data-parallel slice of a global KJT: all features, samples [j*B/W, (j+1)*B/W) (rebased)."""
+    B, F = batch.B, batch.F
+    if B % W:
+        raise ValueError('B % W != 0')
+    Bl = B // W
+    offs = batch.offsets.astype(np.int64)
+    lens = np.diff(offs).reshape(F, B)[:, j * Bl:(j + 1) * Bl]
+    idx = np.concatenate([batch.indices[offs[f * B + j * Bl]:offs[f * B + (j + 1) * Bl]] for f in range(F)])
+    off = np.concatenate([[0], np.cumsum(lens.reshape(-1))])
+    return idx.astype(np.int32), off.astype(np.int32)
+
+
 def split_sizes(B: int, W: int, dims_per_rank: Sequence[int], rank: int):
     """alltoallv element counts for rank `rank`: (input_splits, output_splits)."""
     if B % W:
@@ -139,6 +152,9 @@ def exchange_kjt(send_lengths, send_indices, dest_counts, send_length_counts: Se
     Returns (recv_lengths, recv_indices, recv_counts list)."""
     import torch
     import torch.distributed as dist
+    if len(send_length_counts) == 1:  # one rank: the send buffers are the receive buffers
+        n = int(dest_counts.reshape(-1)[0].item())
+        return send_lengths, send_indices[:n], [n]
     W = dist.get_world_size(group)
     recv_counts = alltoallv(dest_counts, [1] * W, [1] * W, group)
     both = torch.cat([dest_counts.reshape(-1), recv_counts]).cpu().tolist()  # the one host sync

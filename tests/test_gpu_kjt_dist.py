@@ -197,3 +197,14 @@ def test_input_dist_then_sharded_forward(world):
         b = locs[rank]
         exp = oracle.embedding_bag(tabs, m.dims, [f.pool for f in m.features], b.indices, b.offsets, Bl)
         assert np.array_equal(got, exp[:, column_order(m, parts)].astype(np.float32))
+
+
+def test_input_dist_single_rank_is_identity():
+    """W = 1 (no process group): pack + unpack reproduce the input KJT."""
+    from paper_conf_sc_panzzxwslr0d24_b200.shard import KJTInputDist
+    m = synth.make_model('industrial')
+    b = synth.make_batch(m, 7, B=512)
+    ind = KJTInputDist([list(range(m.F))], m.F, 0, 1, 512)
+    idx, off = ind.forward(torch.from_numpy(b.indices).to(_dev()), torch.from_numpy(b.offsets).to(_dev()))
+    assert np.array_equal(idx.cpu().numpy(), b.indices) and np.array_equal(off.cpu().numpy(), b.offsets)
+    ind.close()
