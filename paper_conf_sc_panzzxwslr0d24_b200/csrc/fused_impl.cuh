@@ -300,16 +300,16 @@ int fused_launch_impl(const FusedArgs &a, const LaunchCfg &cfg, void *stream) {
 }
 
 template <int KOCC>
-int fused_prepare_impl(int smem) {
+int fused_prepare_impl(int smem, int carveout) {
     cudaError_t e = cudaFuncSetAttribute(recflex_fused_kernel<KOCC>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return (int)e;
     e = cudaFuncSetAttribute(recflex_fused_kernel<KOCC>, cudaFuncAttributePreferredSharedMemoryCarveout,
-                             cudaSharedmemCarveoutMaxShared);
+                             carveout);
     if (e != cudaSuccess) return (int)e;
     e = cudaFuncSetAttribute(recflex_backward_kernel<KOCC>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return (int)e;
     e = cudaFuncSetAttribute(recflex_backward_kernel<KOCC>, cudaFuncAttributePreferredSharedMemoryCarveout,
-                             cudaSharedmemCarveoutMaxShared);
+                             carveout);
     return (int)e;
 }
 
@@ -334,6 +334,6 @@ int fused_occupancy_impl(int smem, int *blocks, int *regs, int *spill) {
     int backward_launch_k##K(const FusedArgs &a, const LaunchCfg &cfg, void *stream) {                        \
         return fused_launch_impl<K, true>(a, cfg, stream);                                                    \
     }                                                                                                         \
-    int fused_prepare_k##K(int smem) { return fused_prepare_impl<K>(smem); }                                  \
+    int fused_prepare_k##K(int smem, int cv) { return fused_prepare_impl<K>(smem, cv); }                      \
     int fused_occupancy_k##K(int smem, int *b, int *r, int *s) { return fused_occupancy_impl<K>(smem, b, r, s); } \
     }

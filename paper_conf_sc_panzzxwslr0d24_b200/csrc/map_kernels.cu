@@ -31,14 +31,14 @@ int backward_launch_k5(const FusedArgs &, const LaunchCfg &, void *);
 int backward_launch_k6(const FusedArgs &, const LaunchCfg &, void *);
 int backward_launch_k7(const FusedArgs &, const LaunchCfg &, void *);
 int backward_launch_k8(const FusedArgs &, const LaunchCfg &, void *);
-int fused_prepare_k1(int);
-int fused_prepare_k2(int);
-int fused_prepare_k3(int);
-int fused_prepare_k4(int);
-int fused_prepare_k5(int);
-int fused_prepare_k6(int);
-int fused_prepare_k7(int);
-int fused_prepare_k8(int);
+int fused_prepare_k1(int, int);
+int fused_prepare_k2(int, int);
+int fused_prepare_k3(int, int);
+int fused_prepare_k4(int, int);
+int fused_prepare_k5(int, int);
+int fused_prepare_k6(int, int);
+int fused_prepare_k7(int, int);
+int fused_prepare_k8(int, int);
 int fused_occupancy_k1(int, int *, int *, int *);
 int fused_occupancy_k2(int, int *, int *, int *);
 int fused_occupancy_k3(int, int *, int *, int *);
@@ -76,18 +76,18 @@ int backward_launch(int k, const FusedArgs &a, const LaunchCfg &cfg, void *strea
     }
 }
 
-int fused_prepare(int k, int device, int smem) {
+int fused_prepare(int k, int device, int smem, int carveout) {
     cudaError_t e = cudaSetDevice(device);
     if (e != cudaSuccess) return (int)e;
     switch (k) {
-        case 1: return fused_prepare_k1(smem);
-        case 2: return fused_prepare_k2(smem);
-        case 3: return fused_prepare_k3(smem);
-        case 4: return fused_prepare_k4(smem);
-        case 5: return fused_prepare_k5(smem);
-        case 6: return fused_prepare_k6(smem);
-        case 7: return fused_prepare_k7(smem);
-        case 8: return fused_prepare_k8(smem);
+        case 1: return fused_prepare_k1(smem, carveout);
+        case 2: return fused_prepare_k2(smem, carveout);
+        case 3: return fused_prepare_k3(smem, carveout);
+        case 4: return fused_prepare_k4(smem, carveout);
+        case 5: return fused_prepare_k5(smem, carveout);
+        case 6: return fused_prepare_k6(smem, carveout);
+        case 7: return fused_prepare_k7(smem, carveout);
+        case 8: return fused_prepare_k8(smem, carveout);
         default: return (int)cudaErrorInvalidValue;
     }
 }

@@ -150,35 +150,56 @@ int min_dyn_smem(int F) {
     return (m + 127) / 128 * 128;
 }
 
-// Shared-memory padding so that exactly k CTAs fit per SM (C15).
+// Occupancy control (C15): exactly k CTAs per SM.  The register cap of
+// __launch_bounds__(256, k) alone enforces k whenever the kernel uses its full
+// cap (the fused kernel does at every k); then the CTA keeps only the dynamic
+// shared memory it needs and the carveout leaves the rest of the SM's 256 KB
+// to L1 -- padding shared memory as well (the paper's second knob) shrank L1
+// to ~30 KB at k = 4, so the per-bag register spills of the schedule
+// functions went to L2 (1.2 GB of local-memory traffic per heavy batch).
+// Shared-memory padding is used only when registers do not already limit the
+// kernel to k (or when RECFLEX_SMEM_PAD=1 forces the old behaviour).
 recflex_status_t prepare_occupancy(recflex_plan_s *p, int k) {
     if (k < 1 || k > kMaxOcc) return RECFLEX_ERR_INVALID_ARG;
     if (p->prepared[k]) return RECFLEX_OK;
     cudaError_t e = cudaSetDevice(p->device);
     if (e != cudaSuccess) return cuda_status(e);
     const int sm_total = 233472;  // 228 KB per SM
-    int dyn = ((sm_total / k - 1152) / 128) * 128;
-    if (p->no_smem_pad) dyn = min_dyn_smem(p->F);  // experiment: leave L1 its capacity
-    dyn = std::max(dyn, min_dyn_smem(p->F));
-    dyn = std::min(dyn, 232448 - 1024);  // 227 KB opt-in max minus static smem (<= 1 KB)
-    int rc = fused_prepare(k, p->device, 232448 - 1024);
+    const int mind = min_dyn_smem(p->F);
+    int rc = fused_prepare(k, p->device, 232448 - 1024, (int)cudaSharedmemCarveoutMaxShared);
     if (rc) return cuda_status((cudaError_t)rc);
     int blocks = 0, regs = 0, spill = 0;
-    // walk the padding until the occupancy API reports exactly k (or as close as possible)
-    for (int it = 0; it < 64; ++it) {
-        rc = fused_occupancy(k, dyn, &blocks, &regs, &spill);
-        if (rc) return cuda_status((cudaError_t)rc);
-        if (blocks > k) {
-            dyn += 128;
-        } else if (blocks < k && dyn - 128 >= min_dyn_smem(p->F)) {
-            int b2 = 0;
-            fused_occupancy(k, dyn - 128, &b2, &regs, &spill);
-            if (b2 <= k) dyn -= 128;
-            else break;
-            if (b2 == k) break;
-        } else {
-            break;
+    rc = fused_occupancy(k, mind, &blocks, &regs, &spill);
+    if (rc) return cuda_status((cudaError_t)rc);
+    int dyn = mind;
+    if (p->force_smem_pad || blocks > k) {
+        dyn = ((sm_total / k - 1152) / 128) * 128;
+        dyn = std::max(dyn, mind);
+        dyn = std::min(dyn, 232448 - 1024);  // 227 KB opt-in max minus static smem (<= 1 KB)
+        // walk the padding until the occupancy API reports exactly k (or as close as possible)
+        for (int it = 0; it < 64; ++it) {
+            rc = fused_occupancy(k, dyn, &blocks, &regs, &spill);
+            if (rc) return cuda_status((cudaError_t)rc);
+            if (blocks > k) {
+                dyn += 128;
+            } else if (blocks < k && dyn - 128 >= mind) {
+                int b2 = 0;
+                fused_occupancy(k, dyn - 128, &b2, &regs, &spill);
+                if (b2 <= k) dyn -= 128;
+                else break;
+                if (b2 == k) break;
+            } else {
+                break;
+            }
         }
+        p->carveout[k] = 100;
+    } else {
+        // smallest carveout (percent of 228 KB) that holds k CTAs' shared memory
+        // (dynamic + <= 1 KB static + 1 KB per-CTA reservation)
+        const int need = k * (dyn + 2048);
+        p->carveout[k] = std::min(100, (need * 100 + sm_total - 1) / sm_total);
+        rc = fused_prepare(k, p->device, 232448 - 1024, p->carveout[k]);
+        if (rc) return cuda_status((cudaError_t)rc);
     }
     rc = fused_occupancy(k, dyn, &blocks, &regs, &spill);
     if (rc) return cuda_status((cudaError_t)rc);
@@ -428,7 +449,7 @@ recflex_status_t recflex_plan_create(const recflex_feature_spec_t *specs, int32_
         if (k >= 1 && k <= kMaxOcc) p->k = k;
     }
     if (const char *env = std::getenv("RECFLEX_NO_PDL")) p->pdl = !(env[0] == '1');
-    if (const char *env = std::getenv("RECFLEX_NO_SMEM_PAD")) p->no_smem_pad = (env[0] == '1');
+    if (const char *env = std::getenv("RECFLEX_SMEM_PAD")) p->force_smem_pad = (env[0] == '1');
     *out = p;
     return RECFLEX_OK;
 }

@@ -53,7 +53,7 @@ struct recflex_plan_s {
     int task_lookups = 4096;  // lookups per task targeted by the default schedules
     bool desc_dirty = true;
     bool pdl = true;
-    bool no_smem_pad = false;  // RECFLEX_NO_SMEM_PAD=1: occupancy by grid size + registers only
+    bool force_smem_pad = false;  // RECFLEX_SMEM_PAD=1: always pad shared memory to k CTAs/SM (A/B)
     int64_t slots_total = 0;
 
     recflex::Exec ex;  // plan-owned device scratch
@@ -62,6 +62,7 @@ struct recflex_plan_s {
     int smem[recflex::kMaxOcc + 1] = {0};
     int occ[recflex::kMaxOcc + 1] = {0};
     bool prepared[recflex::kMaxOcc + 1] = {false};
+    int carveout[recflex::kMaxOcc + 1] = {0};  // shared-memory carveout (percent) chosen for k
 
     // profiling
     bool profiling = false;

@@ -190,7 +190,7 @@ struct LaunchCfg {
 
 int fused_launch(int k, const FusedArgs &a, const LaunchCfg &cfg, void *stream);  // returns cudaError_t
 int backward_launch(int k, const FusedArgs &a, const LaunchCfg &cfg, void *stream);
-int fused_prepare(int k, int device, int smem_bytes);                              // cudaFuncSetAttribute
+int fused_prepare(int k, int device, int smem_bytes, int carveout);                              // cudaFuncSetAttribute
 int fused_occupancy(int k, int smem_bytes, int *blocks, int *regs, int *spill);
 int map_launch(const MapArgs &a, void *stream);
 int fill_launch(const FillArgs &a, int grid_x, bool pdl, void *stream);

@@ -46,8 +46,21 @@ def run(model, label, ids=(15, 16), ks=(4, 6), reps=5):
     torch.cuda.empty_cache()
 
 
+def base_heavy():
+    from paper_conf_sc_panzzxwslr0d24_b200 import synth
+    return synth.make_model('heavy')
+
+
 def main():
     from paper_conf_sc_panzzxwslr0d24_b200 import synth
+    if len(sys.argv) > 2 and sys.argv[1] == 'heavy':  # one short run of heavy on one schedule (for ncu)
+        run(base_heavy(), 'heavy', ids=(int(sys.argv[2]),), ks=(int(sys.argv[3]) if len(sys.argv) > 3 else 4,), reps=1)
+        return
+    if len(sys.argv) > 1 and sys.argv[1] == 'fixedL100':  # one short run (for ncu)
+        feats = [synth.Feature(rows=10_000_000, dim=128, pool=0, kind='fixed', mu=100, lmax=100, table=f % 16)
+                 for f in range(100)]
+        run(synth.custom_model('fixedL100', feats, 8192), 'fixed L=100, 100 fields', ids=(15,), ks=(4,), reps=1)
+        return
     base = synth.make_model('heavy')
     run(base, 'heavy (lognormal L, 100 fields)')
     feats = [synth.Feature(rows=10_000_000, dim=128, pool=0, kind='fixed', mu=100, lmax=100, table=f % 16)
@@ -59,6 +72,11 @@ def main():
     feats = [synth.Feature(rows=10_000_000, dim=128, pool=0, kind='lognormal', mu=100, sigma=0.9, lmax=1000,
                            table=0)]
     run(synth.custom_model('onefield', feats, 819200), 'lognormal, 1 field x 819200 samples')
+    # table footprint (TLB reach / DRAM page spread): heavy's lengths, 1 and 4 physical tables
+    for nt in (1, 4):
+        feats = [synth.Feature(rows=10_000_000, dim=128, pool=0, kind='lognormal', mu=100, sigma=0.9, lmax=1000,
+                               table=f % nt) for f in range(100)]
+        run(synth.custom_model(f'heavy_t{nt}', feats, 8192), f'heavy lengths, {nt} physical table(s)')
 
 
 if __name__ == '__main__':
