@@ -179,7 +179,9 @@ __device__ __forceinline__ void fused_body(const FusedArgs &a) {
     const int tid = threadIdx.x;
     const int lane = tid & 31;
     const int F = a.F;
-    const bool bs_in_smem = (F + 1) <= kSmemBlockStartCap;
+    // block_start cached in shared memory when it fits in the launch's dynamic
+    // smem (tuning launches run more -- virtual -- features than the plan sized for)
+    const bool bs_in_smem = (F + 1) <= kSmemBlockStartCap && kRedFloats * 4 + 4 * (F + 1) <= a.smem_bytes;
     // BULK-family stage slices: whatever dynamic smem the occupancy padding
     // leaves after the reduction scratch and the block_start cache, split 8 ways
     const int bulk_off = (kRedFloats * 4 + (bs_in_smem ? 4 * (F + 1) : 0) + 127) & ~127;
