@@ -103,6 +103,10 @@ struct RowFrag;
 template <int VEC>
 struct RowFrag<RECFLEX_DTYPE_F32, VEC> {
     float x[VEC];
+    __device__ __forceinline__ void zero() {
+#pragma unroll
+        for (int e = 0; e < VEC; ++e) x[e] = 0.f;
+    }
     __device__ __forceinline__ void load(const char *row, int col, int) {
         ld_row<VEC>(reinterpret_cast<const float *>(row) + col, x);
     }
@@ -115,6 +119,10 @@ struct RowFrag<RECFLEX_DTYPE_F32, VEC> {
 template <int VEC>
 struct RowFrag<RECFLEX_DTYPE_F16, VEC> {
     unsigned w[VEC / 2];
+    __device__ __forceinline__ void zero() {
+#pragma unroll
+        for (int e = 0; e < VEC / 2; ++e) w[e] = 0u;
+    }
     __device__ __forceinline__ void load(const char *row, int col, int) { ld_words<VEC / 2>(row + 2 * col, w); }
     __device__ __forceinline__ void add_to(float (&acc)[VEC]) const {
 #pragma unroll
@@ -128,6 +136,10 @@ struct RowFrag<RECFLEX_DTYPE_F16, VEC> {
 template <int VEC>
 struct RowFrag<RECFLEX_DTYPE_BF16, VEC> {
     unsigned w[VEC / 2];
+    __device__ __forceinline__ void zero() {
+#pragma unroll
+        for (int e = 0; e < VEC / 2; ++e) w[e] = 0u;
+    }
     __device__ __forceinline__ void load(const char *row, int col, int) { ld_words<VEC / 2>(row + 2 * col, w); }
     __device__ __forceinline__ void add_to(float (&acc)[VEC]) const {
 #pragma unroll
@@ -143,6 +155,11 @@ struct RowFrag<RECFLEX_DTYPE_I8, VEC> {
     static_assert(VEC % 4 == 0, "int8 rows: 4 codes per word");
     unsigned w[VEC / 4];
     unsigned sb[2];  // scale, bias
+    __device__ __forceinline__ void zero() {
+#pragma unroll
+        for (int e = 0; e < VEC / 4; ++e) w[e] = 0u;
+        sb[0] = sb[1] = 0u;
+    }
     __device__ __forceinline__ void load(const char *row, int col, int d) {
         ld_words<VEC / 4>(row + col, w);
         ld_words<2>(row + d, sb);  // 8-byte aligned: d % 8 == 0
@@ -158,6 +175,18 @@ struct RowFrag<RECFLEX_DTYPE_I8, VEC> {
         }
     }
 };
+
+// Registers of a U x C row-fragment set start at zero: a fragment that a
+// predicated-off load leaves unwritten must not make the compiler keep the
+// array in local memory to preserve "old" contents (measured: every ragged
+// bag tail stored its just-loaded rows to the stack).
+template <int ET, int VEC, int U, int C>
+__device__ __forceinline__ void rf_zero(RowFrag<ET, VEC> (&v)[U][C]) {
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+#pragma unroll
+        for (int c = 0; c < C; ++c) v[u][c].zero();
+}
 
 template <int VEC>
 __device__ __forceinline__ void st_out(float *p, const float (&v)[VEC]) {
@@ -360,6 +389,7 @@ __device__ __forceinline__ void group_bag(const char *__restrict__ T, unsigned r
 #pragma unroll
                     for (int u = 0; u < U; ++u) id[u] = (unsigned)__shfl_sync(gmask, cur, (j - cb) + u, G);
                     RowFrag<ET, VEC> v[U][C];
+                    rf_zero<ET, VEC, U, C>(v);
 #ifdef RECFLEX_MERGED_TAIL
                     const int n = hi - j;
 #pragma unroll
@@ -398,6 +428,7 @@ __device__ __forceinline__ void group_bag(const char *__restrict__ T, unsigned r
 #pragma unroll
                     for (int u = 0; u < U; ++u) id[u] = (unsigned)__shfl_sync(gmask, cur, (j - cb) + u, G);
                     RowFrag<ET, VEC> v[U][C];
+                    rf_zero<ET, VEC, U, C>(v);
 #pragma unroll
                     for (int u = 0; u < U; ++u)
 #pragma unroll
@@ -433,6 +464,7 @@ __device__ __forceinline__ void group_bag(const char *__restrict__ T, unsigned r
 #pragma unroll
                 for (int u = 0; u < U; ++u) id[u] = ld_idx(idx + j + u);
                 RowFrag<ET, VEC> v[U][C];
+                rf_zero<ET, VEC, U, C>(v);
 #pragma unroll
                 for (int u = 0; u < U; ++u)
 #pragma unroll
@@ -451,6 +483,7 @@ __device__ __forceinline__ void group_bag(const char *__restrict__ T, unsigned r
 #pragma unroll
                 for (int u = 0; u < U; ++u) id[u] = (u < n) ? ld_idx(idx + j + u) : 0;
                 RowFrag<ET, VEC> v[U][C];
+                rf_zero<ET, VEC, U, C>(v);
 #pragma unroll
                 for (int u = 0; u < U; ++u)
 #pragma unroll
@@ -577,6 +610,8 @@ __device__ __noinline__ void sched_flat(const char *__restrict__ T, unsigned row
 #pragma unroll
                 for (int u = 0; u < U; ++u) id[u] = (j + u < Z) ? (unsigned)ld_idx(idx + j + u) : 0u;
                 RowFrag<ET, VEC> r[U];
+                #pragma unroll
+                for (int u = 0; u < U; ++u) r[u].zero();
 #pragma unroll
                 for (int u = 0; u < U; ++u)
                     if (j + u < Z && ok) r[u].load(T + (size_t)id[u] * rowb, col, d);
@@ -841,6 +876,7 @@ __device__ __noinline__ void sched_block(const char *__restrict__ T, unsigned ro
 #pragma unroll
                 for (int u = 0; u < U; ++u) id[u] = ld_idx(idx + j + u * NG);
                 RowFrag<ET, VEC> v[U][C];
+                rf_zero<ET, VEC, U, C>(v);
 #pragma unroll
                 for (int u = 0; u < U; ++u)
 #pragma unroll
@@ -858,6 +894,7 @@ __device__ __noinline__ void sched_block(const char *__restrict__ T, unsigned ro
 #pragma unroll
                 for (int u = 0; u < U; ++u) id[u] = (j + u * NG < hi) ? ld_idx(idx + j + u * NG) : 0;
                 RowFrag<ET, VEC> v[U][C];
+                rf_zero<ET, VEC, U, C>(v);
 #pragma unroll
                 for (int u = 0; u < U; ++u)
 #pragma unroll

@@ -33,6 +33,10 @@ KEYS = [
     ('l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum', 'global load sectors'),
     ('l1tex__t_requests_pipe_lsu_mem_global_op_ld.sum', 'global load requests'),
     ('smsp__issue_active.avg.pct_of_peak_sustained_active', 'issue active %'),
+    ('l1tex__t_sectors_pipe_lsu_mem_local_op_ld.sum', 'local-memory (spill) load sectors'),
+    ('l1tex__t_sectors_pipe_lsu_mem_local_op_st.sum', 'local-memory (spill) store sectors'),
+    ('l1tex__m_l1tex2xbar_write_bytes.sum', 'L1 -> L2 write bytes (stores + local evictions)'),
+    ('launch__shared_mem_config_size', 'shared memory config per SM'),
 ]
 
 
