@@ -165,6 +165,21 @@ recflex_status_t recflex_forward_host(recflex_plan_t plan, const int32_t *h_indi
                                       const int32_t *h_offsets, int32_t batch_size,
                                       const void *const *tables, float *h_out, void *stream);
 
+/* The serving loop over host-resident batches (end-to-end path): batch i's
+ * KJT (h_indices[i][nnz[i]], h_offsets[i][F*B_i+1], pinned host memory for
+ * full copy bandwidth) is copied in, pooled, and its output copied to
+ * h_out[i] [B_i][D_tot], exactly as recflex_forward_host does per batch, but
+ * pipelined over two plan-owned device staging slots and two copy streams:
+ * the H2D of batch i+1 and the D2H of batch i-1 overlap the forward of batch
+ * i.  Blocks until every h_out[i] is written.  Host arrays of num_batches
+ * entries; staging grows on demand (may allocate); results identical to
+ * recflex_forward per batch.  Errors: INVALID_ARG (null/negative/too-large
+ * arguments, checked before any copy), CUDA/OOM. */
+recflex_status_t recflex_forward_host_batches(recflex_plan_t plan, int32_t num_batches,
+                                              const int32_t *const *h_indices, const int64_t *nnz,
+                                              const int32_t *const *h_offsets, const int32_t *batch_sizes,
+                                              const void *const *tables, float *const *h_out, void *stream);
+
 /* ---- tuner (§IV-A) ------------------------------------------------------ */
 
 typedef struct {

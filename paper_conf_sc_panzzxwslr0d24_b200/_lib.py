@@ -96,6 +96,8 @@ SIGNATURES = {
     'recflex_ipc_close': (c_int32, [c_void_p]),
     'recflex_device_alloc': (c_int32, [ctypes.c_size_t, c_int32, P(c_void_p)]),
     'recflex_device_free': (c_int32, [c_void_p]),
+    'recflex_forward_host_batches': (c_int32, [c_void_p, c_int32, P(c_void_p), P(c_int64), P(c_void_p), P(c_int32),
+                                               P(c_void_p), P(c_void_p), c_void_p]),
     'recflex_kjt_dist_create': (c_int32, [c_int32, P(c_int32), c_int32, c_int32, c_int32, c_int32, P(c_void_p)]),
     'recflex_kjt_dist_destroy': (None, [c_void_p]),
     'recflex_kjt_dist_sizes': (c_int32, [c_void_p, P(c_int32), P(c_int32), P(c_int32)]),

@@ -347,6 +347,7 @@ static void plan_free_device(recflex_plan_s *p) {
     cudaFree(p->d_stage_idx);
     cudaFree(p->d_stage_off);
     cudaFree(p->d_stage_out);
+    host_pipe_free(p);
     for (auto &t : p->ev_pending) {
         cudaEventDestroy(t.e0);
         cudaEventDestroy(t.e1);

@@ -84,6 +84,8 @@ struct recflex_plan_s {
     int64_t stage_off_cap = 0;
     float *d_stage_out = nullptr;
     int64_t stage_out_cap = 0;
+    // recflex_forward_host_batches: double-buffered staging + copy streams
+    struct HostPipe *pipe = nullptr;
 
     recflex_tune_stats_t last_stats = {};
 };
@@ -94,6 +96,7 @@ recflex_status_t cuda_status(cudaError_t e);
 recflex_status_t cuda_status_at(cudaError_t e, const char *where);
 void set_last_error(const char *msg);
 recflex_status_t prepare_occupancy(recflex_plan_s *p, int k);
+void host_pipe_free(recflex_plan_s *p);
 int min_dyn_smem(int F);
 // Launch map (+fill) + fused for an Exec.  Events (optional) bracket map and fused.
 recflex_status_t run_pipeline(recflex_plan_s *p, const Exec &ex, const int32_t *indices, const int32_t *offsets, int B,

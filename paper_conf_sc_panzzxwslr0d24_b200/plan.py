@@ -183,6 +183,29 @@ class Plan:
               'recflex_forward_host')
         return out
 
+    def forward_host_batches(self, batches: Sequence[tuple], tables: Sequence[torch.Tensor],
+                             outs: Sequence[torch.Tensor], stream=None):
+        """recflex_forward_host_batches: [(indices, offsets, B)] host (pinned) int32 -> host float32
+        outs[i] [B_i, D_tot]; H2D / forward / D2H of consecutive batches overlapped; blocking."""
+        n = len(batches)
+        if len(outs) != n:
+            raise ValueError('one output per batch')
+        for i, ((ind, off, B), out) in enumerate(zip(batches, outs)):
+            for name, t, dt in (('indices', ind, torch.int32), ('offsets', off, torch.int32),
+                                ('out', out, torch.float32)):
+                if t.is_cuda or t.dtype != dt or not t.is_contiguous():
+                    raise ValueError(f'batch {i}: {name} must be a contiguous host {dt} tensor')
+            if off.numel() != self.F * B + 1 or out.shape != (B, self.d_tot):
+                raise ValueError(f'batch {i}: offsets must hold F*B+1 entries, out [B, D_tot]')
+        tarr = self._tables(tables)
+        P = ctypes.c_void_p
+        check(lib.recflex_forward_host_batches(
+            self._h, n, (P * n)(*[b[0].data_ptr() for b in batches]),
+            (ctypes.c_int64 * n)(*[b[0].numel() for b in batches]), (P * n)(*[b[1].data_ptr() for b in batches]),
+            (ctypes.c_int32 * n)(*[int(b[2]) for b in batches]), tarr, (P * n)(*[o.data_ptr() for o in outs]),
+            _stream_ptr(stream)), 'recflex_forward_host_batches')
+        return outs
+
     # -------------------------------------------------------------- backward (NEXT #4)
     def backward(self, indices: torch.Tensor, offsets: torch.Tensor, B: int, grad: torch.Tensor,
                  targets: Sequence[torch.Tensor], scale: float = 1.0, stream=None):
