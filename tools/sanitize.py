@@ -23,8 +23,46 @@ phys = [synth.make_table(t, r, d, 'int', device=dev) for t, (r, d) in enumerate(
 tables = [phys[f.table] for f in m.features]
 bi, bo = torch.from_numpy(b.indices).to(dev), torch.from_numpy(b.offsets).to(dev)
 cat = catalog()
-fams = sys.argv[1:] or ['group', 'flat', 'block']
+fams = sys.argv[1:] or ['group', 'flat', 'block', 'bwd', 'kjt', 'host']
 for fam in fams:
+    if fam == 'bwd':
+        plan = Plan.from_model(m)
+        grad = torch.randn((b.B, m.d_tot), device=dev)
+        tg = [torch.zeros((f.rows, f.dim), device=dev) for f in m.features]
+        plan.backward(bi, bo, b.B, grad, tg)
+        torch.cuda.synchronize()
+        print('bwd ok')
+        continue
+    if fam == 'kjt':
+        from paper_conf_sc_panzzxwslr0d24_b200.plan import KJTDist
+        W, Bl = 3, 32
+        owner = [f % W for f in range(m.F)]
+        locs = [synth.make_batch(m, 50 + j, B=Bl) for j in range(W)]
+        kds = [KJTDist(owner, W, j, Bl) for j in range(W)]
+        sends = []
+        for j, lb in enumerate(locs):
+            i_d, o_d = torch.from_numpy(lb.indices).to(dev), torch.from_numpy(lb.offsets).to(dev)
+            sl = torch.empty(m.F * Bl, dtype=torch.int32, device=dev)
+            si = torch.empty(max(1, lb.indices.size), dtype=torch.int32, device=dev)
+            dc = torch.empty(W, dtype=torch.int32, device=dev)
+            kds[j].pack(i_d, o_d, sl, si, dc)
+            sends.append((sl, si, dc.cpu().tolist(), kds[j].send_length_counts))
+        for r in range(W):
+            rl = torch.cat([sl[sum(lc[:r]):sum(lc[:r]) + lc[r]] for sl, _, _, lc in sends])
+            ri = torch.cat([si[sum(dc[:r]):sum(dc[:r]) + dc[r]] for _, si, dc, _ in sends])
+            io = torch.empty(max(1, ri.numel()), dtype=torch.int32, device=dev)
+            oo = torch.empty(kds[r].num_owned * W * Bl + 1, dtype=torch.int32, device=dev)
+            kds[r].unpack(rl, ri, io, oo)
+        torch.cuda.synchronize()
+        print('kjt ok')
+        continue
+    if fam == 'host':
+        plan = Plan.from_model(m)
+        hb = [(torch.from_numpy(b.indices).pin_memory(), torch.from_numpy(b.offsets).pin_memory(), b.B)] * 3
+        outs = [torch.empty((b.B, m.d_tot)).pin_memory() for _ in range(3)]
+        plan.forward_host_batches(hb, tables, outs)
+        print('host ok')
+        continue
     ids = [e['id'] for e in cat if e['family'] == fam]
     plan = Plan.from_model(m)
     plan.occupancy = 8 if fam != 'block' else 4
