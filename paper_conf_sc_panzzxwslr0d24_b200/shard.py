@@ -3,9 +3,11 @@ embedding tables on multiple GPUs through heuristics ... and then use RecFlex to
 optimize the embedding operations on each GPU") with the pooled-output
 exchange TorchRec-style table-wise sharding needs.
 
-  * partition: greedy LPT over features by estimated bytes per batch
-    (reading C24): E[L]*cov*(4d+4)*B + 4*d*B, largest first, to the least
-    loaded rank (ties: lower feature id first, lower rank).
+  * partition: greedy LPT over features, largest first, to the least loaded
+    rank (ties: lower feature id first, lower rank), by estimated device time
+    (`feature_time`: distinct-row DRAM fetches at the random-access rate + L2
+    re-hits + bytes at HBM rate; reading C24') or by bytes per batch
+    (`feature_cost`, reading C24: E[L]*cov*(4d+4)*B + 4*d*B).
   * each rank runs its own fused RecFlex plan over ALL B samples of its
     features -> out_r [B][D_r] (row-major, so rank j's B/W-sample block is
     contiguous: no pre-permutation before the all-to-all);
@@ -34,6 +36,32 @@ def feature_cost(feat, B: int, dtype: str = 'f32') -> float:
     return el * (row_bytes(feat.dim, dtype) + 4) * B + 4.0 * feat.dim * B
 
 
+# Device-time model for the partitioner (reading C24'): random row
+# fetches are limited by the access rate (~40 G random accesses/s on B200 for
+# rows <= 128 B, tools/gather_probe.cu), a repeated row of the batch hits L2 at
+# a fraction of that cost, bytes move at HBM bandwidth, and every bag (feature,
+# sample) has a fixed cost (offsets, output row, claim).  Coefficients: least
+# squares over 28 measured per-rank times of sharded1000 at W = 1, 2, 4, 8
+# (tools/rank_sim.py, profiles/r01_rank_sim_sharded1000_*.jsonl; rms error 4 %).
+ACCESS_RATE = 44e9
+HBM_BPS = 8.4e12
+L2_HIT_COST = 0.33
+BAG_SECONDS = 4.4e-11
+
+
+def feature_time(feat, B: int, dtype: str = 'f32') -> float:
+    """Estimated seconds per batch: DRAM row fetches (distinct rows of the batch,
+    uniform IDs) + L2 re-hits at the access rate, plus DRAM bytes at HBM rate."""
+    import math
+    nnz = feat.mean_len() * feat.coverage * B
+    R = float(feat.rows)
+    distinct = R * (1.0 - math.exp(-nnz / R)) if R > 0 else 0.0
+    rb = row_bytes(feat.dim, dtype)
+    gran = max(32, (rb + 31) // 32 * 32)  # 32-byte sectors
+    return ((distinct + (nnz - distinct) * L2_HIT_COST) / ACCESS_RATE
+            + (distinct * gran + 4.0 * nnz + 4.0 * feat.dim * B) / HBM_BPS + BAG_SECONDS * B)
+
+
 def lpt_partition(costs: Sequence[float], W: int) -> List[List[int]]:
     """Greedy longest-processing-time partition; each part sorted by feature id."""
     if W <= 0:
@@ -48,8 +76,10 @@ def lpt_partition(costs: Sequence[float], W: int) -> List[List[int]]:
     return [sorted(p) for p in parts]
 
 
-def partition_model(model, W: int, dtype: str = 'f32') -> List[List[int]]:
-    return lpt_partition([feature_cost(f, model.batch, dtype) for f in model.features], W)
+def partition_model(model, W: int, dtype: str = 'f32', cost: str = 'time') -> List[List[int]]:
+    """LPT over features by estimated device time ('time', default) or bytes ('bytes', reading C24)."""
+    fn = feature_time if cost == 'time' else feature_cost
+    return lpt_partition([fn(f, model.batch, dtype) for f in model.features], W)
 
 
 def column_order(model, parts: List[List[int]]) -> np.ndarray:

@@ -39,12 +39,28 @@ def test_lpt_small_exact():
 
 
 def test_sharded1000_balance():
+    """LPT balances the cost it partitions by: estimated device time (default) and bytes."""
+    from paper_conf_sc_panzzxwslr0d24_b200.shard import feature_cost, feature_time
     m = synth.make_model('sharded1000')
-    for W in (2, 4, 8):
-        parts = partition_model(m, W)
-        from paper_conf_sc_panzzxwslr0d24_b200.shard import feature_cost
-        loads = [sum(feature_cost(m.features[f], m.batch) for f in p) for p in parts]
-        assert max(loads) / (sum(loads) / W) < 1.01
+    for cost, fn in (('time', feature_time), ('bytes', feature_cost)):
+        for W in (2, 4, 8):
+            parts = partition_model(m, W, cost=cost)
+            loads = [sum(fn(m.features[f], m.batch) for f in p) for p in parts]
+            assert max(loads) / (sum(loads) / W) < 1.01, (cost, W)
+
+
+def test_feature_time_model():
+    """The time model's limits: rows <= 32 B cost one access each; a table far
+    smaller than the batch's lookups is fetched once per row (the rest hit L2)."""
+    from paper_conf_sc_panzzxwslr0d24_b200.shard import ACCESS_RATE, BAG_SECONDS, HBM_BPS, L2_HIT_COST, feature_time
+    big = synth.Feature(rows=10 ** 9, dim=4, pool=0, kind='fixed', mu=10, lmax=10, coverage=1.0)
+    t = feature_time(big, 1000)
+    nnz = 10 * 1000   # all distinct: one access + one 32-byte sector + one ID per lookup, 16 B out per sample
+    exp = nnz / ACCESS_RATE + (nnz * 32 + 4 * nnz + 16 * 1000) / HBM_BPS + BAG_SECONDS * 1000
+    assert abs(t / exp - 1.0) < 1e-3
+    small = synth.Feature(rows=10, dim=4, pool=0, kind='fixed', mu=10, lmax=10, coverage=1.0)
+    ts = feature_time(small, 1000)
+    assert ts < t * (L2_HIT_COST + 0.1)
 
 
 def test_shard_batch_slices_features():
