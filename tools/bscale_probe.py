@@ -7,14 +7,14 @@ m = synth.make_model('heavy')
 phys = [torch.empty((r, d), device=dev) for r, d in m.tables]
 tables = [phys[f.table] for f in m.features]
 flush = torch.empty(64 << 20, device=dev)
-for B in (2048, 8192, 24576):
+for B in (8192, 16384, 24576):
     b = synth.make_batch(m, 7, B=B)
     alg = synth.algorithmic_bytes(m, b)['total']
     bi, bo = torch.from_numpy(b.indices).to(dev), torch.from_numpy(b.offsets).to(dev)
     out = torch.empty((B, m.d_tot), device=dev)
     plan = Plan.from_model(m, max_batch=B)
-    for sid in (15, 16):
-        for k in (4, 5):
+    for sid in (16,):
+        for k in (4,):
             for f in range(m.F):
                 plan.set_schedule(f, sid, 0, 40)
             plan.occupancy = k
