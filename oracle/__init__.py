@@ -107,7 +107,7 @@ def max_threads() -> int:
     return int(lib().oracle_max_threads())
 
 
-DTYPES = {'f32': 0, 'f16': 1, 'bf16': 2, 'i8': 3}
+DTYPES = {'f32': 0, 'f16': 1, 'bf16': 2, 'i8': 3, 'fp8': 4}
 
 
 def row_bytes(dtype, dim: int) -> int:

@@ -31,9 +31,12 @@
  *       binary32; I8 = scale * q + bias with q the signed code and scale, bias
  *       the row's two float32 after its d codes (rowwise-quantised row: d
  *       codes, scale, bias, zero padding to a multiple of 16 bytes),
- *       evaluated in fp64.
+ *       evaluated in fp64; FP8 = OCP E4M3 ("e4m3fn": 4-bit exponent with
+ *       bias 7, 3-bit fraction, subnormals, S.1111.111 = NaN, no infinities)
+ *       written out from its fields, one byte per element.
  *       Pinned by tests/test_oracle.py: exhaustive over all 2^16 patterns
- *       against numpy float16 and torch bfloat16, hand-decoded I8 rows.
+ *       against numpy float16 and torch bfloat16, all 256 FP8 codes against
+ *       torch float8_e4m3fn, hand-decoded I8 and FP8 rows.
  *
  *   oracle_embedding_bag_backward -- the adjoint of oracle_embedding_bag
  *       (training; "there is no fundamental reason
@@ -83,6 +86,7 @@
 #define DT_F16 1
 #define DT_BF16 2
 #define DT_I8 3
+#define DT_FP8 4
 
 /* bytes per stored row of dimension d */
 int64_t oracle_row_bytes(int dtype, int d) {
@@ -90,6 +94,7 @@ int64_t oracle_row_bytes(int dtype, int d) {
         case DT_F16:
         case DT_BF16: return 2 * (int64_t)d;
         case DT_I8: return ((int64_t)d + 8 + 15) / 16 * 16;
+        case DT_FP8: return (int64_t)d;
         default: return 4 * (int64_t)d;
     }
 }
@@ -110,6 +115,17 @@ double oracle_decode(int dtype, const unsigned char *row, int c, int d) {
         float f;
         memcpy(&f, &u, 4);
         return (double)f;
+    }
+    if (dtype == DT_FP8) {
+        /* OCP FP8 E4M3 ("fn"): sign, 4-bit exponent with bias 7, 3-bit
+         * fraction; exponent 0 = subnormal m * 2^-9; S.1111.111 = NaN; no inf */
+        unsigned b = row[c];
+        int sign = (b >> 7) & 1, e = (b >> 3) & 15, m = b & 7;
+        double v;
+        if (e == 0) v = ldexp((double)m, -9);
+        else if (e == 15 && m == 7) v = NAN;
+        else v = ldexp((double)(8 + m), e - 10);               /* (1 + m/8) * 2^(e-7) */
+        return sign ? -v : v;
     }
     if (dtype == DT_I8) {
         int q = (int)(signed char)row[c];

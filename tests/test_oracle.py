@@ -353,6 +353,40 @@ def test_decode_bf16_exhaustive_vs_torch():
     assert np.array_equal(v[ok], ref[ok])
 
 
+def test_decode_fp8_worked_values():
+    g = _lowp()['fp8']
+    v = oracle.decode_rows(np.asarray(g['bits'], np.uint8).reshape(-1, 1), 1, 'fp8')[:, 0]
+    assert v.tolist() == g['values']
+    assert np.signbit(v[-1])  # 0x80 = -0.0
+    nan = oracle.decode_rows(np.asarray(g['nan_bits'], np.uint8).reshape(-1, 1), 1, 'fp8')[:, 0]
+    assert np.all(np.isnan(nan))
+
+
+def test_decode_fp8_exhaustive_vs_torch():
+    """All 256 FP8 E4M3 codes against torch's float8_e4m3fn -> float64 (library routine)."""
+    bits = torch.arange(256, dtype=torch.int32).to(torch.uint8)
+    v = oracle.decode_rows(bits.numpy().reshape(-1, 8), 8, 'fp8').reshape(-1)
+    ref = bits.view(torch.float8_e4m3fn).double().numpy()
+    assert np.array_equal(np.isnan(v), np.isnan(ref))
+    ok = ~np.isnan(ref)
+    assert np.array_equal(v[ok], ref[ok])
+    assert np.array_equal(np.signbit(v[ok]), np.signbit(ref[ok]))
+
+
+def test_fp8_tables_equal_upcast_f32_tables():
+    """An FP8 stored table pools exactly like its library up-cast to float32."""
+    m = synth.make_model('tiny')
+    b = synth.make_batch(m, 7)
+    rng = np.random.default_rng(2)
+    codes = [rng.integers(0, 256, (f.rows, f.dim)).astype(np.uint8) for f in m.features]
+    codes = [np.where((c & 0x7F) == 0x7F, 0x38, c).astype(np.uint8) for c in codes]   # no NaN codes
+    up = [torch.from_numpy(c).view(torch.float8_e4m3fn).float().numpy() for c in codes]
+    pools = [0, 1, 0, 1]
+    got = oracle.embedding_bag(codes, m.dims, pools, b.indices, b.offsets, b.B, dtypes=['fp8'] * m.F)
+    exp = oracle.embedding_bag(up, m.dims, pools, b.indices, b.offsets, b.B)
+    assert np.array_equal(got, exp)
+
+
 def test_decode_i8_worked_row():
     g = _lowp()['i8']
     row = _i8_row(g['codes'], g['scale'], g['bias'])
