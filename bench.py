@@ -197,7 +197,7 @@ def main():
     ap.add_argument('--impl', default='ours', choices=['ours', 'reference'])
     ap.add_argument('--config', default='sharded1000')
     ap.add_argument('--mode', default='float', choices=['float', 'int'])
-    ap.add_argument('--dtype', default='f32', choices=['f32', 'f16', 'bf16', 'i8'],
+    ap.add_argument('--dtype', default='f32', choices=['f32', 'f16', 'bf16', 'i8', 'fp8'],
                     help='table row storage (SURVEY NEXT #3); accumulation and output stay fp32')
     ap.add_argument('--batches', type=int, default=3)
     ap.add_argument('--plan', default='auto', help="tuned plan JSON, 'auto' (configs/tuned/) or 'none'")

@@ -36,6 +36,7 @@
  *               F32  float32  [rows_f][d_f]                      (default)
  *               F16  binary16 [rows_f][d_f]
  *               BF16 bfloat16 [rows_f][d_f]
+ *               FP8  OCP E4M3 codes [rows_f][d_f] (1 byte each)
  *               I8   rowwise-quantised: row r is RECFLEX_I8_ROW_BYTES(d_f)
  *                    bytes = d_f int8 codes q, then float32 scale, float32
  *                    bias, zero padding to a multiple of 16 bytes; the row's
@@ -67,7 +68,10 @@ typedef enum {
     RECFLEX_DTYPE_F32 = 0,  /* float32                                                   */
     RECFLEX_DTYPE_F16 = 1,  /* IEEE binary16; needs d_f % 4 == 0                         */
     RECFLEX_DTYPE_BF16 = 2, /* bfloat16 (upper half of a float32); needs d_f % 4 == 0    */
-    RECFLEX_DTYPE_I8 = 3    /* int8 codes + per-row float32 scale and bias; d_f % 8 == 0 */
+    RECFLEX_DTYPE_I8 = 3,   /* int8 codes + per-row float32 scale and bias; d_f % 8 == 0 */
+    RECFLEX_DTYPE_FP8 = 4   /* OCP FP8 E4M3 ("e4m3fn") codes, d_f bytes per row, no
+                               scale (a per-table scale is linear in the pooled output
+                               and folds into its consumer); d_f % 8 == 0             */
 } recflex_dtype_t;
 
 /* Bytes per row of an I8 table: d codes + 8 bytes scale/bias, padded to 16. */

@@ -21,9 +21,9 @@
 
 namespace recflex {
 
-template <int I>
-__device__ __forceinline__ void dispatch_schedule(int id, const TaskCtx &x, float *red, int *bag_ctr) {
-    if constexpr (I < kCatalogSize) {
+template <int I, int END>
+__device__ __forceinline__ void dispatch_chain(int id, const TaskCtx &x, float *red, int *bag_ctr) {
+    if constexpr (I < END && I < kCatalogSize) {
         if (id == I) {
             constexpr CatalogEntry e = kCatalog[I];
             // fp32 entries: G compiled in (the tuned path); reduced-precision
@@ -44,9 +44,20 @@ __device__ __forceinline__ void dispatch_schedule(int id, const TaskCtx &x, floa
                 sched_block<e.ET, GT, e.VEC, e.C, e.U>(x.table, x.rowb, e.G, x.offs, x.idx, x.out, x.dim, x.pool, x.ro,
                                                         x.s0, x.s1, red);
         } else {
-            dispatch_schedule<I + 1>(id, x, red, bag_ctr);
+            dispatch_chain<I + 1, END>(id, x, red, bag_ctr);
         }
     }
+}
+
+// The if-else chain over the catalog, cut into runs of 64 entries so
+// the template recursion stays shallow (fp32 entries keep their place in the
+// first run).
+__device__ __forceinline__ void dispatch_schedule(int id, const TaskCtx &x, float *red, int *bag_ctr) {
+    static_assert(kCatalogSize <= 256, "extend dispatch_schedule");
+    if (id < 64) dispatch_chain<0, 64>(id, x, red, bag_ctr);
+    else if (id < 128) dispatch_chain<64, 128>(id, x, red, bag_ctr);
+    else if (id < 192) dispatch_chain<128, 192>(id, x, red, bag_ctr);
+    else dispatch_chain<192, 256>(id, x, red, bag_ctr);
 }
 
 // Single call site for the whole catalog: the kernel calls this once per task
@@ -68,7 +79,7 @@ static __device__ __noinline__ void dispatch_task(int id, const char *T, unsigne
     x.ro = ro;
     x.s0 = s0;
     x.s1 = s1;
-    dispatch_schedule<0>(id, x, red, bag);
+    dispatch_schedule(id, x, red, bag);
 }
 
 constexpr int kRedFloats = 8 * 256;  // BLOCK family: [8 warps][SPAN <= 256]

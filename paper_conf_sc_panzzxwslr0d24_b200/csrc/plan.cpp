@@ -51,6 +51,7 @@ int row_bytes_of(int dim, int dtype) {
         case RECFLEX_DTYPE_F16:
         case RECFLEX_DTYPE_BF16: return 2 * dim;
         case RECFLEX_DTYPE_I8: return (int)RECFLEX_I8_ROW_BYTES(dim);
+        case RECFLEX_DTYPE_FP8: return dim;
         default: return 4 * dim;
     }
 }
@@ -92,7 +93,11 @@ recflex_schedule_t default_schedule(const recflex_feature_spec_t &spec, int targ
         // (int8), one lane group per row, U = 2 for one-hot bags.
         const int et = spec.dtype;
         const int U = spec.mean_len >= 2.5f ? 4 : 2;
-        if (et == RECFLEX_DTYPE_I8) {
+        if (et == RECFLEX_DTYPE_FP8) {
+            // 16-byte lanes (16 codes), one lane group per row
+            if (d % 16 == 0) id = find_catalog(RECFLEX_FAMILY_GROUP, std::min(32, next_pow2(d / 16)), 16, 1, U, et);
+            if (id < 0) id = find_catalog(RECFLEX_FAMILY_GROUP, std::min(16, next_pow2(d / 8)), 8, 1, U, et);
+        } else if (et == RECFLEX_DTYPE_I8) {
             if (d % 16 == 0) id = find_catalog(RECFLEX_FAMILY_GROUP, std::min(32, next_pow2(d / 16)), 16, 1, U, et);
             if (id < 0) id = find_catalog(RECFLEX_FAMILY_GROUP, std::min(16, next_pow2(d / 8)), 8, 1, U, et);
         } else {
@@ -372,10 +377,11 @@ recflex_status_t recflex_plan_create(const recflex_feature_spec_t *specs, int32_
         if (s.pool != RECFLEX_POOL_SUM && s.pool != RECFLEX_POOL_MEAN) return RECFLEX_ERR_INVALID_ARG;
         if (!(s.mean_len >= 0.f) || !(s.max_len >= 0.f) || !(s.coverage >= 0.f) || s.coverage > 1.f)
             return RECFLEX_ERR_INVALID_ARG;
-        if (s.dtype < RECFLEX_DTYPE_F32 || s.dtype > RECFLEX_DTYPE_I8) return RECFLEX_ERR_INVALID_ARG;
+        if (s.dtype < RECFLEX_DTYPE_F32 || s.dtype > RECFLEX_DTYPE_FP8) return RECFLEX_ERR_INVALID_ARG;
         if ((s.dtype == RECFLEX_DTYPE_F16 || s.dtype == RECFLEX_DTYPE_BF16) && s.dim % 4 != 0)
             return RECFLEX_ERR_INVALID_ARG;
-        if (s.dtype == RECFLEX_DTYPE_I8 && s.dim % 8 != 0) return RECFLEX_ERR_INVALID_ARG;
+        if ((s.dtype == RECFLEX_DTYPE_I8 || s.dtype == RECFLEX_DTYPE_FP8) && s.dim % 8 != 0)
+            return RECFLEX_ERR_INVALID_ARG;
         d_tot += s.dim;
     }
     if (d_tot >= (int64_t(1) << 31) || (int64_t)max_batch * d_tot >= (int64_t(1) << 40)) return RECFLEX_ERR_INVALID_ARG;

@@ -122,7 +122,8 @@ struct FusedArgs {
     X(2, 0, 4, 8, 1, 2) X(2, 0, 4, 8, 1, 4) X(2, 0, 8, 8, 1, 2) X(2, 0, 8, 8, 1, 4)         \
     X(2, 0, 16, 8, 1, 2) X(2, 0, 16, 8, 1, 4) RECFLEX_CATALOG_EXPERIMENTAL(X)        \
     RECFLEX_CATALOG_LOWP(X)
-#define RECFLEX_CATALOG_LOWP(X) RECFLEX_CATALOG_HALF(X, 1) RECFLEX_CATALOG_HALF(X, 2) RECFLEX_CATALOG_I8(X)
+#define RECFLEX_CATALOG_LOWP(X) RECFLEX_CATALOG_HALF(X, 1) RECFLEX_CATALOG_HALF(X, 2) RECFLEX_CATALOG_I8(X) \
+    RECFLEX_CATALOG_FP8(X)
 
 // Reduced-precision rows, appended so the fp32 ids above
 // stay stable.  VEC counts ELEMENTS per lane per load: for 16-bit types
@@ -147,6 +148,19 @@ struct FusedArgs {
     X(0, 3, 16, 16, 1, 2) X(0, 3, 16, 16, 1, 4) X(0, 3, 32, 16, 1, 2) X(0, 3, 32, 16, 1, 4) \
     X(1, 3, 8, 16, 1, 4)                                                        \
     X(2, 3, 1, 16, 1, 4) X(2, 3, 2, 16, 1, 4) X(2, 3, 4, 16, 1, 4) X(2, 3, 8, 16, 1, 4)
+
+// FP8 E4M3 rows (1 byte per element, no scale): VEC 8 -> 64-bit, 16 -> 128-bit,
+// 32 -> 256-bit loads; widened exactly with cvt.rn.f16x2.e4m3x2.
+#define RECFLEX_CATALOG_FP8(X)                                                  \
+    X(0, 4, 1, 8, 1, 2) X(0, 4, 1, 8, 1, 4) X(0, 4, 2, 8, 1, 2) X(0, 4, 2, 8, 1, 4) \
+    X(0, 4, 4, 8, 1, 2) X(0, 4, 4, 8, 1, 4) X(0, 4, 8, 8, 1, 2) X(0, 4, 8, 8, 1, 4) \
+    X(0, 4, 16, 8, 1, 2) X(0, 4, 16, 8, 1, 4)                                  \
+    X(0, 4, 1, 16, 1, 2) X(0, 4, 1, 16, 1, 4) X(0, 4, 2, 16, 1, 2) X(0, 4, 2, 16, 1, 4) \
+    X(0, 4, 4, 16, 1, 2) X(0, 4, 4, 16, 1, 4) X(0, 4, 8, 16, 1, 2) X(0, 4, 8, 16, 1, 4) \
+    X(0, 4, 16, 16, 1, 2) X(0, 4, 16, 16, 1, 4) X(0, 4, 32, 16, 1, 2) X(0, 4, 32, 16, 1, 4) \
+    X(0, 4, 1, 32, 1, 2) X(0, 4, 2, 32, 1, 2) X(0, 4, 4, 32, 1, 2) X(0, 4, 4, 32, 1, 4) \
+    X(1, 4, 8, 16, 1, 4)                                                        \
+    X(2, 4, 1, 16, 1, 4) X(2, 4, 2, 16, 1, 4) X(2, 4, 4, 16, 1, 4) X(2, 4, 8, 16, 1, 4)
 
 // BULK (rows by TMA bulk copy into smem stages) is built only on request:
 // per-row cp.async.bulk of random rows from multi-GB tables measured 10-100x
@@ -175,6 +189,7 @@ inline bool catalog_valid(const CatalogEntry &e, int d, int dtype = RECFLEX_DTYP
     if (e.ET != dtype) return false;
     if (d % e.VEC != 0) return false;
     if (dtype == RECFLEX_DTYPE_I8 && d % 8 != 0) return false;  // scale/bias 8-byte aligned
+    if (dtype == RECFLEX_DTYPE_FP8 && d % 8 != 0) return false;  // rows 8-byte aligned
     int span = e.G * e.VEC * e.C;
     if (4 * d < span) return false;
     if (e.family == 3 && (d < 32 || d > 128)) return false;  // BULK: 128..512-byte rows, one pass

@@ -150,6 +150,40 @@ struct RowFrag<RECFLEX_DTYPE_BF16, VEC> {
     }
 };
 
+// FP8 E4M3: two codes -> f16x2 (exact: E4M3 is a subset of binary16) -> two fp32.
+__device__ __forceinline__ void e4m3x4_to_f32(unsigned w, float &a, float &b, float &c, float &d) {
+    unsigned lo, hi;
+    asm("{\n\t.reg .b16 l, h;\n\tmov.b32 {l, h}, %2;\n\tcvt.rn.f16x2.e4m3x2 %0, l;\n\tcvt.rn.f16x2.e4m3x2 %1, h;\n\t}"
+        : "=r"(lo), "=r"(hi)
+        : "r"(w));
+    a = f16_lo(lo);
+    b = f16_hi(lo);
+    c = f16_lo(hi);
+    d = f16_hi(hi);
+}
+
+template <int VEC>
+struct RowFrag<RECFLEX_DTYPE_FP8, VEC> {
+    static_assert(VEC % 4 == 0, "fp8 rows: 4 codes per word");
+    unsigned w[VEC / 4];
+    __device__ __forceinline__ void zero() {
+#pragma unroll
+        for (int e = 0; e < VEC / 4; ++e) w[e] = 0u;
+    }
+    __device__ __forceinline__ void load(const char *row, int col, int) { ld_words<VEC / 4>(row + col, w); }
+    __device__ __forceinline__ void add_to(float (&acc)[VEC]) const {
+#pragma unroll
+        for (int i = 0; i < VEC / 4; ++i) {
+            float a, b, c, d;
+            e4m3x4_to_f32(w[i], a, b, c, d);
+            acc[4 * i + 0] += a;
+            acc[4 * i + 1] += b;
+            acc[4 * i + 2] += c;
+            acc[4 * i + 3] += d;
+        }
+    }
+};
+
 template <int VEC>
 struct RowFrag<RECFLEX_DTYPE_I8, VEC> {
     static_assert(VEC % 4 == 0, "int8 rows: 4 codes per word");

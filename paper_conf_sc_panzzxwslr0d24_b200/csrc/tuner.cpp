@@ -642,7 +642,7 @@ extern "C" recflex_status_t recflex_tune_ex(recflex_plan_t p, int32_t N, const i
             const recflex_feature_spec_t &sp = p->specs[f];
             const float el = sp.mean_len;
             const int lb = sp.max_len <= 1.f ? 0 : (el < 4.f ? 1 : (el < 32.f ? 2 : 3));
-            const long key = ((long)sp.dim * 16 + lb * 4 + (int)T.cands[f].size() % 4) * 4 + sp.dtype;
+            const long key = ((long)sp.dim * 16 + lb * 4 + (int)T.cands[f].size() % 4) * 8 + sp.dtype;
             size_t c = 0;
             while (c < keys.size() && keys[c] != key) ++c;
             if (c == keys.size()) {

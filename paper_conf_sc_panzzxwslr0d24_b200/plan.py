@@ -19,7 +19,7 @@ POOL_SUM = 0
 POOL_MEAN = 1
 
 # table row storage types (recflex_dtype_t)
-DTYPES = {'f32': 0, 'f16': 1, 'bf16': 2, 'i8': 3}
+DTYPES = {'f32': 0, 'f16': 1, 'bf16': 2, 'i8': 3, 'fp8': 4}
 DTYPE_NAMES = {v: k for k, v in DTYPES.items()}
 
 
@@ -36,8 +36,9 @@ def check_table(t: torch.Tensor, dim: int, dtype) -> None:
     """The tensor layout recflex_forward expects for a table of this dim / dtype."""
     code = dtype_code(dtype)
     want = {0: (torch.float32, dim), 1: (torch.float16, dim), 2: (torch.bfloat16, dim),
-            3: (torch.uint8, i8_row_bytes(dim))}[code]
-    if not (t.is_cuda and t.dtype == want[0] and t.is_contiguous() and t.dim() == 2 and t.shape[1] == want[1]):
+            3: (torch.uint8, i8_row_bytes(dim)), 4: (torch.uint8, dim)}[code]
+    tdt = torch.uint8 if (code == 4 and t.dtype == torch.float8_e4m3fn) else t.dtype  # fp8: codes as uint8 or e4m3fn
+    if not (t.is_cuda and tdt == want[0] and t.is_contiguous() and t.dim() == 2 and t.shape[1] == want[1]):
         raise ValueError(f'table: need contiguous CUDA {want[0]} [rows, {want[1]}] for dim {dim} '
                          f'dtype {DTYPE_NAMES[code]}, got {t.dtype} {tuple(t.shape)}')
 

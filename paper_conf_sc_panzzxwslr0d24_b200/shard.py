@@ -27,7 +27,7 @@ import numpy as np
 
 def row_bytes(dim: int, dtype: str = 'f32') -> int:
     """Bytes one lookup gathers: the stored row (int8: codes + scale + bias)."""
-    return {'f32': 4 * dim, 'f16': 2 * dim, 'bf16': 2 * dim, 'i8': dim + 8}[dtype]
+    return {'f32': 4 * dim, 'f16': 2 * dim, 'bf16': 2 * dim, 'i8': dim + 8, 'fp8': dim}[dtype]
 
 
 def feature_cost(feat, B: int, dtype: str = 'f32') -> float:

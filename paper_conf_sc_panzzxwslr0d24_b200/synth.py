@@ -335,7 +335,7 @@ def make_table(table_id: int, rows: int, dim: int, mode: str = 'float', device='
 # Encoding inputs only: the value of a stored element is defined (and
 # computed for checking) by oracle_decode, not here.
 # ---------------------------------------------------------------------------
-STORAGE_DTYPES = ('f32', 'f16', 'bf16', 'i8')
+STORAGE_DTYPES = ('f32', 'f16', 'bf16', 'i8', 'fp8')
 
 
 def i8_row_bytes(dim: int) -> int:
@@ -353,6 +353,11 @@ def table_rows_stored(table_id: int, row_ids, dim: int, dtype: str = 'f32', mode
     if dtype in ('f16', 'bf16'):
         v = table_rows_at(table_id, row_ids, dim, mode, device, seed)
         return v.to(torch.float16 if dtype == 'f16' else torch.bfloat16)
+    if dtype == 'fp8':
+        # E4M3 codes (uint8) of the same values, rounded to nearest by the library
+        # conversion; 'int' mode values (integers in [-8, 7]) are exact in E4M3
+        v = table_rows_at(table_id, row_ids, dim, mode, device, seed)
+        return v.to(torch.float8_e4m3fn).view(torch.uint8)
     if dtype != 'i8':
         raise ValueError(dtype)
     r = torch.as_tensor(row_ids, dtype=torch.int64, device=device).reshape(-1)
@@ -388,7 +393,7 @@ def make_table_stored(table_id: int, rows: int, dim: int, dtype: str = 'f32', mo
     if dtype == 'f32':
         return make_table(table_id, rows, dim, mode, device, seed, chunk_rows)
     width = i8_row_bytes(dim) if dtype == 'i8' else dim
-    tdt = {'f16': torch.float16, 'bf16': torch.bfloat16, 'i8': torch.uint8}[dtype]
+    tdt = {'f16': torch.float16, 'bf16': torch.bfloat16, 'i8': torch.uint8, 'fp8': torch.uint8}[dtype]
     out = torch.empty((rows, width), dtype=tdt, device=device)
     if chunk_rows is None:
         chunk_rows = max(1, (1 << 24) // max(1, dim))
@@ -402,7 +407,7 @@ def make_table_stored(table_id: int, rows: int, dim: int, dtype: str = 'f32', mo
 def row_bytes(dim: int, dtype: str = 'f32') -> int:
     """Algorithmic bytes of one stored row (C26 generalised): the element bytes,
     plus scale and bias for int8 (padding excluded)."""
-    return {'f32': 4 * dim, 'f16': 2 * dim, 'bf16': 2 * dim, 'i8': dim + 8}[dtype]
+    return {'f32': 4 * dim, 'f16': 2 * dim, 'bf16': 2 * dim, 'i8': dim + 8, 'fp8': dim}[dtype]
 
 
 def make_tables(model: Model, mode: str = 'float', device='cpu'):

@@ -1,5 +1,5 @@
 """GPU parity for reduced-precision table rows: float16,
-bfloat16 and rowwise int8 storage, fp32 accumulation, fp32 output.
+bfloat16, rowwise int8 and FP8 E4M3 storage, fp32 accumulation, fp32 output.
 
 The oracle decodes every stored element in fp64 (oracle_decode: IEEE binary16
 from its fields, bfloat16 as the upper half of a binary32, int8 as scale*q+bias)
@@ -20,7 +20,7 @@ from test_gpu_parity import bitexact, check_tol
 
 pytestmark = pytest.mark.gpu
 
-LOWP = ('f16', 'bf16', 'i8')
+LOWP = ('f16', 'bf16', 'i8', 'fp8')
 
 
 def _P():
@@ -121,7 +121,8 @@ def test_industrial_sampled(dtype):
     _check(case, out, np.unique(np.concatenate([[0, b.B - 1], rng.integers(0, b.B, 150)])))
 
 
-@pytest.mark.parametrize('name,dtype', [('heavy', 'bf16'), ('heavy', 'i8'), ('sharded1000', 'f16')])
+@pytest.mark.parametrize('name,dtype', [('heavy', 'bf16'), ('heavy', 'i8'), ('heavy', 'fp8'), ('sharded1000', 'f16'),
+                                        ('sharded1000', 'fp8')])
 def test_full_size_sampled(name, dtype):
     """BASELINE.json full sizes in the default launch configuration; sampled rows, int bit-exact."""
     m = synth.make_model(name)
@@ -137,7 +138,7 @@ def test_full_size_sampled(name, dtype):
 # ---------------------------------------------------------------------------- every entry
 
 def _lowp_model(dtype):
-    dims = ([8, 16, 24, 32, 48, 64, 96, 128, 256, 8, 16, 40] if dtype == 'i8'
+    dims = ([8, 16, 24, 32, 48, 64, 96, 128, 256, 8, 16, 40] if dtype in ('i8', 'fp8')
             else [4, 8, 12, 16, 24, 32, 64, 96, 128, 256, 40, 20])
     feats = []
     for i, d in enumerate(dims):
@@ -194,6 +195,8 @@ def test_fp32_entries_rejected_for_lowp_features_and_vice_versa():
         P.Plan([dict(rows=10, dim=6, dtype='f16')], 8)   # 16-bit rows need dim % 4 == 0
     with pytest.raises(Exception):
         P.Plan([dict(rows=10, dim=12, dtype='i8')], 8)   # int8 rows need dim % 8 == 0
+    with pytest.raises(Exception):
+        P.Plan([dict(rows=10, dim=12, dtype='fp8')], 8)  # fp8 rows need dim % 8 == 0
     with pytest.raises(ValueError):
         plan.forward(case.idx, case.off, case.B, [t.float() if t.dtype == torch.bfloat16 else t
                                                    for t in case.tables])
@@ -202,8 +205,9 @@ def test_fp32_entries_rejected_for_lowp_features_and_vice_versa():
 # ---------------------------------------------------------------------------- mixed storage in one kernel
 
 def _mixed_dtypes(m):
-    cyc = ['f32', 'f16', 'bf16', 'i8']
-    return [cyc[i % 4] if (cyc[i % 4] != 'i8' or f.dim % 8 == 0) else 'bf16' for i, f in enumerate(m.features)]
+    cyc = ['f32', 'f16', 'bf16', 'i8', 'fp8']
+    return [cyc[i % 5] if (cyc[i % 5] not in ('i8', 'fp8') or f.dim % 8 == 0) else 'bf16'
+            for i, f in enumerate(m.features)]
 
 
 @pytest.mark.parametrize('mode', ['int', 'float'])

@@ -22,7 +22,7 @@ def main():
     ap.add_argument('--parts', default='0')
     ap.add_argument('--per-block', default='', help='override per_block values (comma list)')
     ap.add_argument('--reps', type=int, default=6)
-    ap.add_argument('--dtype', default='f32', choices=['f32', 'f16', 'bf16', 'i8'])
+    ap.add_argument('--dtype', default='f32', choices=['f32', 'f16', 'bf16', 'i8', 'fp8'])
     a = ap.parse_args()
     import torch
     from paper_conf_sc_panzzxwslr0d24_b200 import synth

@@ -25,7 +25,7 @@ def main():
     ap.add_argument('--batches', type=int, default=2)
     ap.add_argument('--reps', type=int, default=5)
     ap.add_argument('--max-candidates', type=int, default=0)
-    ap.add_argument('--dtype', default='f32', choices=['f32', 'f16', 'bf16', 'i8'])
+    ap.add_argument('--dtype', default='f32', choices=['f32', 'f16', 'bf16', 'i8', 'fp8'])
     ap.add_argument('--out', default=os.path.join(ROOT, 'gpurun_out', 'tuned'))
     a = ap.parse_args()
     import torch
