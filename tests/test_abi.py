@@ -52,21 +52,21 @@ def test_catalog_consistency():
         seen.add(key)
         fams.add(ci.family)
         assert ci.group in (1, 2, 4, 8, 16, 32)
-        # vec counts elements: fp32 4/16/32-byte loads, 16-bit 8/16/32-byte, int8 8/16-byte
-        assert ci.vec in {0: (1, 4, 8), 1: (4, 8, 16), 2: (4, 8, 16), 3: (8, 16)}[ci.dtype]
+        # vec counts elements: fp32 4/16/32-byte loads, 16-bit 8/16/32-byte, int8 8/16-byte, fp8 8/16/32-byte
+        assert ci.vec in {0: (1, 4, 8), 1: (4, 8, 16), 2: (4, 8, 16), 3: (8, 16), 4: (8, 16, 32)}[ci.dtype]
         # append-only catalog: every fp32 entry precedes every reduced-precision one
         if ci.dtype == 0:
             assert all(k[1] == 0 for k in seen)
         # an entry is valid only for its own storage type
         assert L.lib.recflex_catalog_valid_dtype(i, 128, ci.dtype) == 1
-        assert all(L.lib.recflex_catalog_valid_dtype(i, 128, o) == 0 for o in range(4) if o != ci.dtype)
+        assert all(L.lib.recflex_catalog_valid_dtype(i, 128, o) == 0 for o in range(5) if o != ci.dtype)
     assert fams == {0, 1, 2}  # BULK (3) only in RECFLEX_EXPERIMENTAL_BULK builds
     assert L.lib.recflex_catalog_info(n, ctypes.byref(L.CatalogInfo())) != 0
     # every dim 1..256 has at least one valid fp32 entry; every dim % 4 == 0 a
     # 16-bit one, every dim % 8 == 0 an int8 one
     for d in range(1, 257):
         assert any(L.lib.recflex_catalog_valid(i, d) for i in range(n)), d
-        for dt, mult in ((1, 4), (2, 4), (3, 8)):
+        for dt, mult in ((1, 4), (2, 4), (3, 8), (4, 8)):
             if d % mult == 0:
                 assert any(L.lib.recflex_catalog_valid_dtype(i, d, dt) for i in range(n)), (d, dt)
 
