@@ -149,8 +149,10 @@ struct FusedArgs {
     X(1, 3, 8, 16, 1, 4)                                                        \
     X(2, 3, 1, 16, 1, 4) X(2, 3, 2, 16, 1, 4) X(2, 3, 4, 16, 1, 4) X(2, 3, 8, 16, 1, 4)
 
-// FP8 E4M3 rows (1 byte per element, no scale): VEC 8 -> 64-bit, 16 -> 128-bit,
-// 32 -> 256-bit loads; widened exactly with cvt.rn.f16x2.e4m3x2.
+// FP8 E4M3 rows (1 byte per element, no scale): VEC 4 -> 32-bit, 8 -> 64-bit,
+// 16 -> 128-bit, 32 -> 256-bit loads; widened exactly with cvt.rn.f16x2.e4m3x2.
+// (A 128-byte row is one cache line: 32 lanes x 4 codes keeps only 4
+// accumulators per lane, so U = 8 rows fit in flight under the k = 6..8 caps.)
 #define RECFLEX_CATALOG_FP8(X)                                                  \
     X(0, 4, 1, 8, 1, 2) X(0, 4, 1, 8, 1, 4) X(0, 4, 2, 8, 1, 2) X(0, 4, 2, 8, 1, 4) \
     X(0, 4, 4, 8, 1, 2) X(0, 4, 4, 8, 1, 4) X(0, 4, 8, 8, 1, 2) X(0, 4, 8, 8, 1, 4) \
@@ -159,6 +161,7 @@ struct FusedArgs {
     X(0, 4, 4, 16, 1, 2) X(0, 4, 4, 16, 1, 4) X(0, 4, 8, 16, 1, 2) X(0, 4, 8, 16, 1, 4) \
     X(0, 4, 16, 16, 1, 2) X(0, 4, 16, 16, 1, 4) X(0, 4, 32, 16, 1, 2) X(0, 4, 32, 16, 1, 4) \
     X(0, 4, 1, 32, 1, 2) X(0, 4, 2, 32, 1, 2) X(0, 4, 4, 32, 1, 2) X(0, 4, 4, 32, 1, 4) \
+    X(0, 4, 32, 4, 1, 4) X(0, 4, 32, 4, 1, 8) X(0, 4, 16, 4, 1, 8) X(0, 4, 16, 8, 1, 8) \
     X(1, 4, 8, 16, 1, 4)                                                        \
     X(2, 4, 1, 16, 1, 4) X(2, 4, 2, 16, 1, 4) X(2, 4, 4, 16, 1, 4) X(2, 4, 8, 16, 1, 4)
 
