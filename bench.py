@@ -287,9 +287,12 @@ def main():
         if args.dtype != 'f32' and args.plan == 'auto':
             path = os.path.join(ROOT, 'configs', 'tuned', f'{args.config}_{args.dtype}_w{world}_r{rank}.json')
         if os.path.exists(path):
-            with open(path) as fh:
-                plan.import_(json.load(fh))
-            plan_src = os.path.relpath(path, ROOT)
+            try:
+                with open(path) as fh:
+                    plan.import_(json.load(fh))
+                plan_src = os.path.relpath(path, ROOT)
+            except Exception as ex:  # stale plan (e.g. a different partition): keep the heuristic defaults
+                plan_src = f'default (untuned heuristic; {os.path.relpath(path, ROOT)} rejected: {ex})
     if args.occupancy:
         plan.occupancy = args.occupancy
 
