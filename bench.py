@@ -292,7 +292,7 @@ def main():
                     plan.import_(json.load(fh))
                 plan_src = os.path.relpath(path, ROOT)
             except Exception as ex:  # stale plan (e.g. a different partition): keep the heuristic defaults
-                plan_src = f'default (untuned heuristic; {os.path.relpath(path, ROOT)} rejected: {ex})
+                plan_src = f'default (untuned heuristic; {os.path.relpath(path, ROOT)} rejected: {ex})'
     if args.occupancy:
         plan.occupancy = args.occupancy
 
