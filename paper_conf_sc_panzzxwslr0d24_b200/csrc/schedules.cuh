@@ -404,16 +404,7 @@ __device__ __forceinline__ void group_bag(const char *__restrict__ T, unsigned r
                 int cur = (lo + lg < hi) ? ld_idx(idx + lo + lg) : 0;
                 int nxt = (lo + G + lg < hi) ? ld_idx(idx + lo + G + lg) : 0;
                 int j = lo;
-#ifdef RECFLEX_MERGED_TAIL
-                // One loop for the full iterations and the ragged tail (loads
-                // and adds predicated on u < hi - j): a separate tail block
-                // needs its own U-row register set on top of the loop's live
-                // state and spilled under the occupancy register caps (local
-                // memory traffic through L2 on every bag).
-                for (; j < hi; j += U) {
-#else
                 for (; j + U <= hi; j += U) {
-#endif
                     if (j - cb >= G) {
                         cb += G;
                         cur = nxt;
@@ -424,20 +415,6 @@ __device__ __forceinline__ void group_bag(const char *__restrict__ T, unsigned r
                     for (int u = 0; u < U; ++u) id[u] = (unsigned)__shfl_sync(gmask, cur, (j - cb) + u, G);
                     RowFrag<ET, VEC> v[U][C];
                     rf_zero<ET, VEC, U, C>(v);
-#ifdef RECFLEX_MERGED_TAIL
-                    const int n = hi - j;
-#pragma unroll
-                    for (int u = 0; u < U; ++u)
-#pragma unroll
-                        for (int c = 0; c < C; ++c)
-                            if ((U == 1 || u < n) && ok[c]) v[u][c].load(T + (size_t)id[u] * rowb, colv[c], d);
-#pragma unroll
-                    for (int u = 0; u < U; ++u)
-                        if (U == 1 || u < n)
-#pragma unroll
-                            for (int c = 0; c < C; ++c)
-                                if (ok[c]) v[u][c].add_to(acc[c]);
-#else
 #pragma unroll
                     for (int u = 0; u < U; ++u)
 #pragma unroll
@@ -449,9 +426,7 @@ __device__ __forceinline__ void group_bag(const char *__restrict__ T, unsigned r
                         for (int c = 0; c < C; ++c)
                             if (ok[c])
                                 v[u][c].add_to(acc[c]);
-#endif
                 }
-#ifndef RECFLEX_MERGED_TAIL
                 if (j < hi) {
                     if (j - cb >= G) {
                         cb += G;
@@ -476,7 +451,6 @@ __device__ __forceinline__ void group_bag(const char *__restrict__ T, unsigned r
                                 if (ok[c])
                                     v[u][c].add_to(acc[c]);
                 }
-#endif
 #pragma unroll
                 for (int c = 0; c < C; ++c) {
                     if (ok[c]) {
