@@ -123,11 +123,20 @@ def test_industrial_sampled(dtype):
 
 @pytest.mark.parametrize('name,dtype', [('heavy', 'bf16'), ('heavy', 'i8'), ('heavy', 'fp8'), ('sharded1000', 'f16')])
 def test_full_size_sampled(name, dtype):
-    """BASELINE.json full sizes in the default launch configuration; sampled rows, int bit-exact."""
+    """BASELINE.json full sizes in bench.py's launch configuration (tuned plan if present); sampled rows,
+    int bit-exact."""
+    import json
+    import os
     m = synth.make_model(name)
     b = synth.make_batch(m, 7)
     case = TypedCase(m, b, dtype, 'int')
-    out = case.run(case.plan())
+    plan = case.plan()
+    # the tuned plan bench.py --dtype loads, when there is one (its launch configuration)
+    path = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), 'configs', 'tuned',
+                        f'{name}_{dtype}_w1_r0.json')
+    if os.path.exists(path):
+        plan.import_(json.load(open(path)))
+    out = case.run(plan)
     rng = np.random.default_rng(2)
     _check(case, out, np.unique(np.concatenate([[0, b.B - 1], rng.integers(0, b.B, 40)])))
     del case
