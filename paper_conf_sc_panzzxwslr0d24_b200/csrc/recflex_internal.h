@@ -123,7 +123,7 @@ struct FusedArgs {
     X(2, 0, 16, 8, 1, 2) X(2, 0, 16, 8, 1, 4) RECFLEX_CATALOG_EXPERIMENTAL(X)        \
     RECFLEX_CATALOG_LOWP(X)
 #define RECFLEX_CATALOG_LOWP(X) RECFLEX_CATALOG_HALF(X, 1) RECFLEX_CATALOG_HALF(X, 2) RECFLEX_CATALOG_I8(X) \
-    RECFLEX_CATALOG_FP8(X)
+    RECFLEX_CATALOG_FP8(X) RECFLEX_CATALOG_HALF_U8(X, 1) RECFLEX_CATALOG_HALF_U8(X, 2)
 
 // Reduced-precision rows, appended so the fp32 ids above
 // stay stable.  VEC counts ELEMENTS per lane per load: for 16-bit types
@@ -164,6 +164,10 @@ struct FusedArgs {
     X(0, 4, 32, 4, 1, 4) X(0, 4, 32, 4, 1, 8) X(0, 4, 16, 4, 1, 8) X(0, 4, 16, 8, 1, 8) \
     X(1, 4, 8, 16, 1, 4)                                                        \
     X(2, 4, 1, 16, 1, 4) X(2, 4, 2, 16, 1, 4) X(2, 4, 4, 16, 1, 4) X(2, 4, 8, 16, 1, 4)
+
+// 16-bit rows, 8 rows in flight per lane group (appended: ids above stay stable);
+// 32 lanes x 4 elements keep 4 accumulators per lane (cf. the FP8 entries).
+#define RECFLEX_CATALOG_HALF_U8(X, T) X(0, T, 16, 8, 1, 8) X(0, T, 32, 4, 1, 8) X(0, T, 8, 8, 1, 8)
 
 // BULK (rows by TMA bulk copy into smem stages) is built only on request:
 // per-row cp.async.bulk of random rows from multi-GB tables measured 10-100x
