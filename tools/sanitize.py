@@ -56,6 +56,29 @@ for fam in fams:
         torch.cuda.synchronize()
         print('kjt ok')
         continue
+    if fam == 'lowp':
+        lfeats = [synth.Feature(rows=300 + i, dim=d, pool=i % 2, kind='uniform', coverage=1.0, lo=0, hi=30, lmax=30,
+                                table=i) for i, d in enumerate([8, 16, 32, 64, 128, 24])]
+        lm = synth.custom_model('san_lowp', lfeats, 64)
+        lb = synth.make_batch(lm, 3)
+        li, lo = torch.from_numpy(lb.indices).to(dev), torch.from_numpy(lb.offsets).to(dev)
+        n = 0
+        for dt in ('f16', 'bf16', 'i8', 'fp8'):
+            tabs = [synth.make_table_stored(f.table, f.rows, f.dim, dt, 'int', device=dev) for f in lm.features]
+            specs = [dict(rows=f.rows, dim=f.dim, pool=f.pool, mean_len=15, max_len=30, coverage=1.0, dtype=dt)
+                     for f in lm.features]
+            plan = Plan(specs, lb.B)
+            for e in [e for e in cat if e['dtype'] == dt][::2]:
+                for f in range(lm.F):
+                    try:
+                        plan.set_schedule(f, e['id'], 0, 8)
+                    except Exception:
+                        pass
+                plan.forward(li, lo, lb.B, tabs)
+                n += 1
+        torch.cuda.synchronize()
+        print('lowp forwards', n)
+        continue
     if fam == 'host':
         plan = Plan.from_model(m)
         hb = [(torch.from_numpy(b.indices).pin_memory(), torch.from_numpy(b.offsets).pin_memory(), b.B)] * 3
