@@ -219,6 +219,11 @@ def main():
     world = int(os.environ.get('WORLD_SIZE', '1'))
     rank = int(os.environ.get('RANK', '0'))
     local_rank = int(os.environ.get('LOCAL_RANK', '0'))
+    # test plumbing only: run the N > 1 path with several ranks on ONE GPU (gloo,
+    # exchange staged through host memory) -- RECFLEX_DIST_BACKEND=gloo RECFLEX_BENCH_DEVICE=0
+    backend = os.environ.get('RECFLEX_DIST_BACKEND', 'nccl')
+    if os.environ.get('RECFLEX_BENCH_DEVICE') is not None:
+        local_rank = int(os.environ['RECFLEX_BENCH_DEVICE'])
 
     if args.impl == 'reference':
         return run_reference(args, rank, world)
@@ -232,7 +237,10 @@ def main():
     torch.cuda.set_device(local_rank)
     dev = torch.device('cuda', local_rank)
     if world > 1:
-        dist.init_process_group('nccl', device_id=dev)
+        if backend == 'nccl':
+            dist.init_process_group('nccl', device_id=dev)
+        else:
+            dist.init_process_group(backend)
 
     model = synth.make_model(args.config)
     B = model.batch
@@ -347,7 +355,7 @@ def main():
     clk = clocks.stop() if clocks else None
 
     if world > 1:
-        t = torch.tensor([elapsed_ms], dtype=torch.float64, device=dev)
+        t = torch.tensor([elapsed_ms], dtype=torch.float64, device=dev if backend == 'nccl' else 'cpu')
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         elapsed_ms = float(t.item())
     ms_per_step = elapsed_ms / args.steps
@@ -412,7 +420,7 @@ def main():
                 hout.copy_(o, non_blocking=True)
                 torch.cuda.current_stream().synchronize()
             dt = time.perf_counter() - t0
-            t = torch.tensor([dt], dtype=torch.float64, device=dev)
+            t = torch.tensor([dt], dtype=torch.float64, device=dev if backend == 'nccl' else 'cpu')
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             dt = float(t.item())
             h2d = float(np.mean([hi.numel() * 4 + ho.numel() * 4 for hi, ho in hb]))
@@ -457,6 +465,7 @@ def main():
             'data': 'synthetic (seeded generator, SURVEY §8d recipe; tables: counter-based hash U[-1,1))',
             'config': {'workload': args.config, 'global_batch': B, 'fields': model.F, 'table_dtype': args.dtype,
                        'parallelism': f'tablewise{world}', 'plan': plan_src, 'occupancy': plan.occupancy,
+                       **({'dist_backend': backend} if world > 1 else {}),
                        'exchange': (args.exchange if world > 1 else 'none'),
                        'input': ('data-parallel local batches + KJT input dist in the timed step'
                                  if args.input_dist else 'table-wise KJT resident per rank'),
