@@ -211,6 +211,8 @@ def main():
     ap.add_argument('--profile-only', action='store_true', help='short run for ncu (no e2e / cpu / clocks)')
     ap.add_argument('--exchange', default='nccl', choices=['nccl', 'fused'],
                     help='N>1: NCCL alltoallv + relayout kernel, or peer stores fused into the kernel epilogue')
+    ap.add_argument('--no-graph', action='store_true',
+                    help='N=1: launch each step eagerly instead of replaying its captured CUDA graph')
     ap.add_argument('--input-dist', action='store_true',
                     help='start each step from data-parallel local batches (B/W samples, all features) and run '
                          'the KJT input distribution (pack -> alltoallv -> unpack) inside the timed step')
@@ -327,6 +329,33 @@ def main():
     for i in range(args.warmup):
         step(i)
     torch.cuda.synchronize()
+
+    # N = 1: each rotating batch's forward (map + fused kernel, PDL-chained) captured
+    # once as a CUDA graph and replayed per step -- no host launch work in the loop
+    graphs = None
+    eager_step = step
+    if world == 1 and ind is None and not args.no_graph and not args.profile_only:
+        try:
+            graphs = []
+            cap = torch.cuda.Stream()
+            cap.wait_stream(torch.cuda.current_stream())
+            for j in range(len(batches)):
+                g = torch.cuda.CUDAGraph()
+                with torch.cuda.graph(g, stream=cap):
+                    step(j)
+                graphs.append(g)
+            torch.cuda.current_stream().wait_stream(cap)
+            torch.cuda.synchronize()
+
+            def step(i):  # noqa: F811
+                graphs[i % len(graphs)].replay()
+            for i in range(args.warmup):
+                step(i)
+            torch.cuda.synchronize()
+        except Exception as ex:  # capture unsupported here: stay eager
+            print(f'[bench] CUDA graph capture failed ({ex}); timing eager launches', file=sys.stderr)
+            graphs = None
+            step = eager_step
 
     clocks = ClockSampler(local_rank) if not args.profile_only else None
     if clocks:
@@ -467,6 +496,7 @@ def main():
                        'parallelism': f'tablewise{world}', 'plan': plan_src, 'occupancy': plan.occupancy,
                        **({'dist_backend': backend} if world > 1 else {}),
                        'exchange': (args.exchange if world > 1 else 'none'),
+                       'launch': 'CUDA graph replay per step' if graphs else 'eager',
                        'input': ('data-parallel local batches + KJT input dist in the timed step'
                                  if args.input_dist else 'table-wise KJT resident per rank'),
                        'l2': 'flushed between steps' if flush_between else
