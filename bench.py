@@ -233,7 +233,7 @@ def main():
     import torch
     import torch.distributed as dist
     from paper_conf_sc_panzzxwslr0d24_b200 import synth
-    from paper_conf_sc_panzzxwslr0d24_b200.shard import (KJTInputDist, ShardedEmbedding, partition_model,
+    from paper_conf_sc_panzzxwslr0d24_b200.shard import (KJTInputDist, ShardedEmbedding, model_parts,
                                                           sample_slice, shard_batch)
 
     torch.cuda.set_device(local_rank)
@@ -246,7 +246,7 @@ def main():
 
     model = synth.make_model(args.config)
     B = model.batch
-    parts = partition_model(model, world, args.dtype)
+    parts = model_parts(model, world, args.dtype, args.config, os.path.join(ROOT, 'configs', 'tuned'))
     if world > 1 and args.exchange == 'fused':
         from paper_conf_sc_panzzxwslr0d24_b200.shard import FusedShardedEmbedding
         sh = FusedShardedEmbedding(model, rank, world, device=local_rank, parts=parts, dtype=args.dtype)

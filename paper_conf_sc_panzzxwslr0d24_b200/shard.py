@@ -82,6 +82,31 @@ def partition_model(model, W: int, dtype: str = 'f32', cost: str = 'time') -> Li
     return lpt_partition([fn(f, model.batch, dtype) for f in model.features], W)
 
 
+def check_parts(parts: List[List[int]], F: int, W: int) -> List[List[int]]:
+    """A table-wise partition must cover every feature exactly once, W non-empty parts."""
+    if len(parts) != W or any(len(p) == 0 for p in parts):
+        raise ValueError(f'partition needs {W} non-empty parts')
+    flat = sorted(f for p in parts for f in p)
+    if flat != list(range(F)):
+        raise ValueError('partition does not cover every feature exactly once')
+    return [sorted(int(f) for f in p) for p in parts]
+
+
+def model_parts(model, W: int, dtype: str = 'f32', config: str = '', tuned_dir: str = '') -> List[List[int]]:
+    """The partition a run uses: the measured refinement `<tuned_dir>/<config>[_<dtype>]_w<W>_parts.json`
+    (written by tools/rebalance.py together with the per-rank plans it retuned) if present,
+    else the model LPT (`partition_model`)."""
+    import json
+    import os
+    if config and tuned_dir and W > 1:
+        name = f'{config}_w{W}_parts.json' if dtype == 'f32' else f'{config}_{dtype}_w{W}_parts.json'
+        path = os.path.join(tuned_dir, name)
+        if os.path.exists(path):
+            with open(path) as fh:
+                return check_parts(json.load(fh)['parts'], len(model.features), W)
+    return partition_model(model, W, dtype)
+
+
 def column_order(model, parts: List[List[int]]) -> np.ndarray:
     """Global column index of every column of the exchanged [B/W][D_tot'] output."""
     col = np.cumsum([0] + model.dims)

@@ -230,3 +230,27 @@ def test_gloo_world2_kjt_input_dist_matches_oracle():
     for rank, idx, off, rc, _ in res:
         assert np.array_equal(idx, exp[rank][0]) and np.array_equal(off, exp[rank][1])
         assert sum(rc) == exp[rank][0].size
+
+
+def test_model_parts_override(tmp_path):
+    """model_parts: the LPT partition unless a measured refinement file exists; the
+    file must be a partition (every feature once, W non-empty parts) or it is rejected."""
+    import json
+    from paper_conf_sc_panzzxwslr0d24_b200.shard import check_parts, model_parts
+    m = synth.make_model('medium')
+    F = len(m.features)
+    assert model_parts(m, 2, 'f32', 'medium', str(tmp_path)) == partition_model(m, 2)
+    lpt = partition_model(m, 2)
+    moved = [list(p) for p in lpt]
+    f = moved[0].pop()
+    moved[1].append(f)
+    (tmp_path / 'medium_w2_parts.json').write_text(json.dumps({'parts': moved}))
+    got = model_parts(m, 2, 'f32', 'medium', str(tmp_path))
+    assert got == [sorted(p) for p in moved] and got != lpt
+    assert model_parts(m, 4, 'f32', 'medium', str(tmp_path)) == partition_model(m, 4)  # other W: no file
+    with pytest.raises(ValueError):
+        check_parts([moved[0], moved[1] + [0]], F, 2)  # feature twice
+    with pytest.raises(ValueError):
+        check_parts([moved[0][1:], moved[1]], F, 2)  # feature missing
+    with pytest.raises(ValueError):
+        check_parts([list(range(F)), []], F, 2)  # empty rank

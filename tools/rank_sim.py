@@ -31,7 +31,7 @@ def main():
     import torch
     from paper_conf_sc_panzzxwslr0d24_b200 import synth
     from paper_conf_sc_panzzxwslr0d24_b200.plan import l2_flush
-    from paper_conf_sc_panzzxwslr0d24_b200.shard import ShardedEmbedding, partition_model, shard_batch
+    from paper_conf_sc_panzzxwslr0d24_b200.shard import ShardedEmbedding, model_parts, shard_batch
     dev = torch.device('cuda', 0)
     model = synth.make_model(a.config)
     B = model.batch
@@ -41,7 +41,7 @@ def main():
         phys[t] = synth.make_table_stored(t, rows, dim, 'f32', 'float', device=dev, seed=model.seed)
     flush = torch.empty(64 << 20, device=dev)
     for W in [int(x) for x in a.worlds.split(',')]:
-        parts = partition_model(model, W)
+        parts = model_parts(model, W, 'f32', a.config, os.path.join(ROOT, 'configs', 'tuned'))
         per_rank = []
         for r in range(W):
             sh = ShardedEmbedding(model, r, W, device=0, parts=parts)

@@ -30,12 +30,12 @@ def main():
     a = ap.parse_args()
     import torch
     from paper_conf_sc_panzzxwslr0d24_b200 import synth
-    from paper_conf_sc_panzzxwslr0d24_b200.shard import ShardedEmbedding, partition_model, shard_batch
+    from paper_conf_sc_panzzxwslr0d24_b200.shard import ShardedEmbedding, model_parts, shard_batch
 
     os.makedirs(a.out, exist_ok=True)
     dev = torch.device('cuda', 0)
     model = synth.make_model(a.config)
-    parts = partition_model(model, a.world, a.dtype)
+    parts = model_parts(model, a.world, a.dtype, a.config, os.path.join(ROOT, 'configs', 'tuned'))
     ranks = range(a.world) if a.rank < 0 else [a.rank]
     ks = [int(x) for x in a.ks.split(',')] if a.ks else None
     fulls = [synth.make_batch(model, 7 + i) for i in range(a.batches)]
