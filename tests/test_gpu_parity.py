@@ -410,3 +410,35 @@ def test_tuner_runs_counts_and_keeps_parity():
     _, out = run_plan(case, plan)
     ref, _ = case.oracle()
     assert bitexact(out, ref)
+
+
+def test_sharded1000_rank_plans_sampled():
+    """Every rank plan bench.py loads at W = 2/4/8 (the measured partition refinement
+    configs/tuned/sharded1000_w{W}_parts.json + its per-rank tuned plans): each rank's
+    fused forward over all B samples of its features, integer tables, sampled rows
+    bit-exact against the oracle's columns of those features."""
+    import json
+    import os
+    from paper_conf_sc_panzzxwslr0d24_b200.shard import ShardedEmbedding, model_parts, shard_batch
+    tuned = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), 'configs', 'tuned')
+    m = synth.make_model('sharded1000')
+    b = synth.make_batch(m, 7)
+    case = Case(m, b, 'int')
+    rng = np.random.default_rng(2)
+    samples = np.unique(np.concatenate([[0, b.B - 1], rng.integers(0, b.B, 24)]))
+    ref, _ = case.oracle(samples)
+    col = np.cumsum([0] + m.dims)
+    dev = torch.device('cuda', 0)
+    for W in (2, 4, 8):
+        parts = model_parts(m, W, 'f32', 'sharded1000', tuned)
+        for r in range(W):
+            sh = ShardedEmbedding(m, r, W, device=0, parts=parts)
+            sh.plan.import_(json.load(open(os.path.join(tuned, f'sharded1000_w{W}_r{r}.json'))))
+            idx, off = shard_batch(b, sh.features)
+            out = sh.plan.forward(torch.from_numpy(idx).to(dev), torch.from_numpy(off).to(dev), b.B,
+                                  [case.tables[f] for f in sh.features]).cpu().numpy()
+            cols = np.concatenate([np.arange(col[f], col[f + 1]) for f in sh.features])
+            assert bitexact(out[samples], ref[:, cols]), (W, r)
+            del sh, out
+    del case
+    torch.cuda.empty_cache()
