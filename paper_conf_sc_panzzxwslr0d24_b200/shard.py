@@ -92,6 +92,51 @@ def check_parts(parts: List[List[int]], F: int, W: int) -> List[List[int]]:
     return [sorted(int(f) for f in p) for p in parts]
 
 
+def refine_partition(parts: List[List[int]], measure, est: Sequence[float], moves: int = 8, tries: int = 6):
+    """Measured refinement of a partition (tools/rebalance.py).
+
+    `measure(parts, r)` returns rank r's measured time under `parts`; `est[f]` is the
+    modelled cost of feature f.  Repeatedly: a = slowest rank, b = fastest; try moving
+    one feature of a to b (candidates ordered by |est[f] * t_a / est(a) - gap/2|); accept
+    the first whose two new rank times are both below t_a.  Stops after `moves`
+    accepted moves or when no candidate helps.  Returns (parts, times, log); a candidate
+    whose measurement raises (e.g. a schedule invalid at the new column) is skipped."""
+    F = sum(len(p) for p in parts)
+    W = len(parts)
+    parts = check_parts(parts, F, W)
+    t = [float(measure(parts, r)) for r in range(W)]
+    log = [dict(step='start', ms=list(t), max=max(t), max_over_mean=max(t) * W / sum(t))]
+    for _ in range(moves):
+        ra = max(range(W), key=lambda r: (t[r], -r))
+        rb = min(range(W), key=lambda r: (t[r], r))
+        if ra == rb or len(parts[ra]) < 2:
+            break
+        gap = 0.5 * (t[ra] - t[rb])
+        scale = t[ra] / max(sum(est[f] for f in parts[ra]), 1e-30)
+        cands = sorted(parts[ra], key=lambda f: (abs(est[f] * scale - gap), f))[:tries]
+        accepted = None
+        for f in cands:
+            trial = [list(p) for p in parts]
+            trial[ra].remove(f)
+            trial[rb].append(f)
+            trial = check_parts(trial, F, W)
+            try:
+                ta, tb = float(measure(trial, ra)), float(measure(trial, rb))
+            except Exception as ex:  # noqa: BLE001 -- reported in the log, candidate skipped
+                log.append(dict(step='skip', feature=f, why=str(ex)[:120]))
+                continue
+            log.append(dict(step='try', feature=f, src=ra, dst=rb, ta=ta, tb=tb, old_max=t[ra]))
+            if max(ta, tb) < t[ra]:
+                accepted = (f, trial, ta, tb)
+                break
+        if accepted is None:
+            break
+        f, parts, t[ra], t[rb] = accepted
+        log.append(dict(step='move', feature=f, src=ra, dst=rb, ms=list(t), max=max(t),
+                        max_over_mean=max(t) * W / sum(t)))
+    return parts, t, log
+
+
 def model_parts(model, W: int, dtype: str = 'f32', config: str = '', tuned_dir: str = '') -> List[List[int]]:
     """The partition a run uses: the measured refinement `<tuned_dir>/<config>[_<dtype>]_w<W>_parts.json`
     (written by tools/rebalance.py together with the per-rank plans it retuned) if present,

@@ -41,8 +41,8 @@ def main():
     import torch
     from paper_conf_sc_panzzxwslr0d24_b200 import synth
     from paper_conf_sc_panzzxwslr0d24_b200.plan import l2_flush
-    from paper_conf_sc_panzzxwslr0d24_b200.shard import (ShardedEmbedding, check_parts, feature_time, model_parts,
-                                                          shard_batch)
+    from paper_conf_sc_panzzxwslr0d24_b200.shard import (ShardedEmbedding, feature_time, model_parts,
+                                                          refine_partition, shard_batch)
     os.makedirs(a.out, exist_ok=True)
     dev = torch.device('cuda', 0)
     model = synth.make_model(a.config)
@@ -87,38 +87,12 @@ def main():
         del sh, bi, bo, out
         return float(np.median(ts))
 
-    t = [measure(parts, r, occ[r]) for r in range(W)]
-    log = [dict(step='start', ms=t, max=max(t), max_over_mean=max(t) / np.mean(t))]
-    print(json.dumps(log[-1]), flush=True)
-    est = {f: feature_time(model.features[f], B) for f in range(F)}
-    changed = set()
-    for _ in range(a.moves):
-        ra, rb = int(np.argmax(t)), int(np.argmin(t))
-        gap = 0.5 * (t[ra] - t[rb])
-        scale = t[ra] / (1e3 * sum(est[f] for f in parts[ra]))  # measured ms per modelled s on rank a
-        cands = sorted(parts[ra], key=lambda f: abs(1e3 * est[f] * scale - gap))[:a.tries]
-        accepted = None
-        for f in cands:
-            trial = [list(p) for p in parts]
-            trial[ra].remove(f)
-            trial[rb] = sorted(trial[rb] + [f])
-            trial = check_parts(trial, F, W)
-            try:
-                ta, tb = measure(trial, ra, occ[ra]), measure(trial, rb, occ[rb])
-            except Exception as ex:  # schedule not valid at the new column offset
-                print(json.dumps(dict(skip=f, why=str(ex)[:120])), flush=True)
-                continue
-            print(json.dumps(dict(try_feature=f, src=ra, dst=rb, ta=ta, tb=tb, old_max=t[ra])), flush=True)
-            if max(ta, tb) < t[ra]:
-                accepted = (f, trial, ta, tb)
-                break
-        if accepted is None:
-            break
-        f, parts, t[ra], t[rb] = accepted
-        changed.update((ra, rb))
-        log.append(dict(step='move', feature=f, src=ra, dst=rb, ms=list(t), max=max(t),
-                        max_over_mean=max(t) / np.mean(t)))
-        print(json.dumps(log[-1]), flush=True)
+    est = [feature_time(model.features[f], B) for f in range(F)]
+    parts0 = parts
+    parts, t, log = refine_partition(parts, lambda p, r: measure(p, r, occ[r]), est, a.moves, a.tries)
+    for entry in log:
+        print(json.dumps(entry), flush=True)
+    changed = {r for r in range(W) if parts[r] != parts0[r]}
 
     with open(os.path.join(a.out, f'{a.config}_w{W}_parts.json'), 'w') as fh:
         json.dump(dict(config=a.config, world=W, parts=parts, log=log,
@@ -126,8 +100,7 @@ def main():
     for r in range(W):  # every rank's plan follows the (possibly new) partition
         with open(os.path.join(a.out, f'{a.config}_w{W}_r{r}.json'), 'w') as fh:
             json.dump(state(parts[r], occ[r]), fh)
-    print(json.dumps(dict(done=True, changed=sorted(changed), max=max(t), max_over_mean=max(t) / np.mean(t))),
-          flush=True)
+    print(json.dumps(dict(done=True, changed=sorted(changed), max=max(t), max_over_mean=max(t) * W / sum(t))), flush=True)
 
 
 if __name__ == '__main__':
