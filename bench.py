@@ -105,6 +105,26 @@ class ClockSampler:
                 'reasons': sorted(seen), 'samples': len(rows)}
 
 
+def _cpu_model():
+    try:
+        with open('/proc/cpuinfo') as fh:
+            for line in fh:
+                if line.startswith('model name'):
+                    return line.split(':', 1)[1].strip()
+    except Exception:
+        pass
+    import platform
+    return platform.processor() or 'unknown'
+
+
+def _workload_config(args, model, world):
+    """The `config` dict both arms print (identical keys and values for the same run):
+    the workload only -- implementation details go to `impl_config`."""
+    return {'workload': args.config, 'global_batch': model.batch, 'fields': model.F, 'table_dtype': args.dtype,
+            'parallelism': f'tablewise{world}',
+            'l2': f'inputs > L2 ({args.batches} rotating batches, each larger than L2) or flushed between steps'}
+
+
 # ------------------------------------------------------------------------- CPU oracle arm
 def oracle_sample_rate(model, batch, n_samples: int, seed: int = 0, nthreads: int = 0, min_seconds: float = 0.0,
                        max_reps: int = 1000, dtype: str = 'f32'):
@@ -175,12 +195,12 @@ def run_reference(args, rank, world):
     line = {
         'impl': 'reference', 'metric': _baseline_metric(), 'value': value, 'unit': 'samples/s',
         'n_gpus': world, 'steps': args.steps, 'warmup': args.warmup, 'ms_per_step': 1e3 * tot_t / args.steps,
-        'higher_is_better': True, 'scaling': 'strong' if world > 1 else 'weak', 'vs_baseline': None,
+        'higher_is_better': True, 'scaling': 'strong', 'vs_baseline': None,
         'dtype': 'f64', 'data': 'synthetic',
-        'config': {'workload': args.config, 'global_batch': model.batch, 'fields': model.F,
-                   'parallelism': f'tablewise{world}'},
+        'config': _workload_config(args, model, world),
         'effective_gbs': tot_b / tot_t / 1e9,
         'cpu_baseline': {'value': value, 'unit': 'samples/s', 'cores': cores, 'kind': 'oracle',
+                         'cpu_model': _cpu_model(),
                          'sample': f'{args.steps} steps x {n} random samples (all {model.F} fields) of batch seed 7'},
         'e2e': {'value': value, 'unit': 'samples/s', 'h2d_bytes_per_step': 0, 'd2h_bytes_per_step': 0},
     }
@@ -211,6 +231,10 @@ def main():
     ap.add_argument('--profile-only', action='store_true', help='short run for ncu (no e2e / cpu / clocks)')
     ap.add_argument('--exchange', default='nccl', choices=['nccl', 'fused'],
                     help='N>1: NCCL alltoallv + relayout kernel, or peer stores fused into the kernel epilogue')
+    ap.add_argument('--no-heavy', action='store_true',
+                    help='N=1: skip timing the heavy (north-star >= 70 %% HBM) workload in the same run')
+    ap.add_argument('--no-jit', action='store_true',
+                    help='time the precompiled catalog kernel instead of the plan-specialised (NVRTC) one')
     ap.add_argument('--no-graph', action='store_true',
                     help='N=1: launch each step eagerly instead of replaying its captured CUDA graph')
     ap.add_argument('--input-dist', action='store_true',
@@ -233,7 +257,8 @@ def main():
     import torch
     import torch.distributed as dist
     from paper_conf_sc_panzzxwslr0d24_b200 import synth
-    from paper_conf_sc_panzzxwslr0d24_b200.shard import (KJTInputDist, ShardedEmbedding, model_parts,
+    from paper_conf_sc_panzzxwslr0d24_b200.plan import shard_concat
+    from paper_conf_sc_panzzxwslr0d24_b200.shard import (KJTInputDist, ShardedEmbedding, exchange, model_parts,
                                                           sample_slice, shard_batch)
 
     torch.cuda.set_device(local_rank)
@@ -305,6 +330,10 @@ def main():
                 plan_src = f'default (untuned heuristic; {os.path.relpath(path, ROOT)} rejected: {ex})'
     if args.occupancy:
         plan.occupancy = args.occupancy
+    # the paper's fusion compiler: the plan's schedules inlined into one kernel (NVRTC)
+    jit = None
+    if not args.no_jit:
+        jit = plan.compile()
 
     out_local = torch.empty((B, sh.d_local), dtype=torch.float32, device=dev)
     out_x = torch.empty((B // world, sh.d_tot), dtype=torch.float32, device=dev) if world > 1 else None
@@ -363,32 +392,40 @@ def main():
         time.sleep(0.3)
     barrier()
     torch.cuda.synchronize()
-    if flush_between:
-        evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-        for i in range(args.steps):
+    # every step bracketed by events on the launching stream: the headline is the
+    # first-to-last span (or, with L2 flushes between steps, the sum of the steps)
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    for i in range(args.steps):
+        if flush_between:
             l2_flush(flush_buf)
-            evs[i][0].record(stream)
-            step(i)
-            evs[i][1].record(stream)
-        torch.cuda.synchronize()
-        elapsed_ms = sum(a.elapsed_time(b) for a, b in evs)
-    else:
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
-        for i in range(args.steps):
-            step(i)
-        e1.record(stream)
-        torch.cuda.synchronize()
-        elapsed_ms = e0.elapsed_time(e1)
+        evs[i][0].record(stream)
+        step(i)
+        evs[i][1].record(stream)
+    torch.cuda.synchronize()
+    per_step = [a_.elapsed_time(b_) for a_, b_ in evs]
+    elapsed_ms = sum(per_step) if flush_between else evs[0][0].elapsed_time(evs[-1][1])
     barrier()
     clk = clocks.stop() if clocks else None
 
-    if world > 1:
-        t = torch.tensor([elapsed_ms], dtype=torch.float64, device=dev if backend == 'nccl' else 'cpu')
+    def max_over_ranks(x):
+        if world == 1:
+            return float(x)
+        t = torch.tensor([float(x)], dtype=torch.float64, device=dev if backend == 'nccl' else 'cpu')
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        elapsed_ms = float(t.item())
+        return float(t.item())
+
+    def sum_over_ranks(x):
+        if world == 1:
+            return float(x)
+        t = torch.tensor([float(x)], dtype=torch.float64, device=dev if backend == 'nccl' else 'cpu')
+        dist.all_reduce(t, op=dist.ReduceOp.SUM)
+        return float(t.item())
+
+    elapsed_ms = max_over_ranks(elapsed_ms)
+    median_ms = max_over_ranks(float(np.median(per_step)))
     ms_per_step = elapsed_ms / args.steps
     value = B * args.steps / (elapsed_ms / 1e3)
+    alg_all = sum_over_ranks(alg_local)  # every rank's algorithmic bytes of one step
 
     # per-kernel device time (events on the launch stream; PDL off in this pass)
     plan.set_profiling(True)
@@ -404,11 +441,63 @@ def main():
     map_ms = kt['map_ms'] / max(1, kt['forwards'])
     peak, peak_src = _peaks()
     achieved = alg_local / (fused_ms / 1e3) / 1e9
-    eff_gbs_step = alg_local / (ms_per_step / 1e3) / 1e9
+    eff_gbs_step = alg_all / (ms_per_step / 1e3) / 1e9
 
+    # N > 1: the step split into this rank's compute (map + fused) and the exchange,
+    # per-rank medians, max over ranks; bounds from the NVLink all-to-all
+    multi = None
+    if world > 1 and ind is None:
+        comp, tot = [], []
+        for i in range(max(3, min(args.steps, 10))):
+            bi, bo = batches[i % len(batches)]
+            barrier()
+            e = [torch.cuda.Event(enable_timing=True) for _ in range(3)]
+            e[0].record(stream)
+            plan.forward(bi, bo, B, tables, out=out_local)
+            e[1].record(stream)
+            if args.exchange == 'nccl':
+                # the exchange alone: alltoallv of this rank's pooled rows + relayout kernel
+                recv = exchange(out_local, sh.dims_per_rank, B)
+                shard_concat(recv, sh.dims_per_rank, B // world, out_x)
+            else:
+                step(i)  # fused: compute + peer stores + completion wait, as timed
+            e[2].record(stream)
+            torch.cuda.synchronize()
+            comp.append(e[0].elapsed_time(e[1]))
+            tot.append(e[1].elapsed_time(e[2]))
+        comp_ms = float(np.median(comp))
+        # nccl: step = compute + exchange; fused: the fused step itself
+        step_ms = comp_ms + float(np.median(tot)) if args.exchange == 'nccl' else float(np.median(tot))
+        rows = B // world
+        send = rows * sh.d_local * 4 * (world - 1)
+        recv = rows * (sh.d_tot - sh.d_local) * 4
+        a2a_bytes = max(send, recv)
+        nvlink = 900e9
+        a2a_ms = a2a_bytes / nvlink * 1e3
+        relayout_ms = (2.0 * rows * sh.d_tot * 4) / (peak * 1e9) * 1e3 if args.exchange == 'nccl' else 0.0
+        comp_max = max_over_ranks(comp_ms)
+        a2a_max = max_over_ranks(a2a_ms)
+        multi = {
+            'compute_ms_max_rank': comp_max,
+            'compute_ms_this_rank': comp_ms,
+            'step_ms_max_rank': max_over_ranks(step_ms),
+            'exchange_ms_max_rank': max_over_ranks(step_ms - comp_ms),
+            'exchange': ('NCCL alltoallv + relayout kernel' if args.exchange == 'nccl' else
+                         'peer stores in the fused kernel epilogue + device-side flags (recflex_forward_exchange)'),
+            'nvlink': {'a2a_bytes_max_rank': max_over_ranks(a2a_bytes), 'gbs_per_direction': nvlink / 1e9,
+                       'a2a_ms_at_peak': a2a_max, 'relayout_ms_at_hbm_peak': max_over_ranks(relayout_ms),
+                       'serial_bound_ms': comp_max + a2a_max + max_over_ranks(relayout_ms),
+                       'overlapped_bound_ms': max(comp_max, a2a_max),
+                       'samples_per_s_serial_bound': B / ((comp_max + a2a_max + max_over_ranks(relayout_ms)) / 1e3),
+                       'samples_per_s_overlapped_bound': B / (max(comp_max, a2a_max) / 1e3)},
+            'note': 'compute = this plan\'s map + fused kernels alone; step = the timed step (compute + exchange)',
+        }
+
+    # DRAM traffic of the fused kernel from a committed ncu capture of THIS workload and rank plan
     traffic = None
-    tp = os.path.join(ROOT, 'profiles', f'ncu_traffic_{args.config}' + ('' if args.dtype == 'f32' else f'_{args.dtype}')
-                      + '.json')
+    tname = f'ncu_traffic_{args.config}' + ('' if args.dtype == 'f32' else f'_{args.dtype}') + \
+        ('' if world == 1 else f'_w{world}_r{rank}') + '.json'
+    tp = os.path.join(ROOT, 'profiles', tname)
     if os.path.exists(tp):
         try:
             with open(tp) as fh:
@@ -449,9 +538,7 @@ def main():
                 hout.copy_(o, non_blocking=True)
                 torch.cuda.current_stream().synchronize()
             dt = time.perf_counter() - t0
-            t = torch.tensor([dt], dtype=torch.float64, device=dev if backend == 'nccl' else 'cpu')
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            dt = float(t.item())
+            dt = max_over_ranks(dt)
             h2d = float(np.mean([hi.numel() * 4 + ho.numel() * 4 for hi, ho in hb]))
             d2h = hout.numel() * 4
         e2e = {'value': B * ke / dt, 'unit': 'samples/s', 'h2d_bytes_per_step': int(h2d),
@@ -468,7 +555,7 @@ def main():
             cores = len(os.sched_getaffinity(0))
             S, dt, alg = oracle_sample_rate(model, full, args.cpu_samples, seed=0, nthreads=cores,
                                             min_seconds=args.cpu_seconds, dtype=args.dtype)
-            cpu = {'value': S / dt, 'unit': 'samples/s', 'cores': cores, 'kind': 'oracle',
+            cpu = {'value': S / dt, 'unit': 'samples/s', 'cores': cores, 'kind': 'oracle', 'cpu_model': _cpu_model(),
                    'sample': f'{args.cpu_samples} random samples x all {model.F} fields of batch seed 7, '
                              f'oracle repeated to {dt:.1f} s ({S} samples total; fp64 C oracle, OpenMP)',
                    'effective_gbs': alg / dt / 1e9, 'seconds': dt}
@@ -477,7 +564,20 @@ def main():
 
     launches_per_step = 2 + (1 if plan.export() and any(s[1] == 1 for s in plan.export()['schedules']) else 0)
     launches_per_step += 1 if (world > 1 and args.exchange == 'nccl') else 0   # relayout kernel
+    launches_per_step += 1 if (world > 1 and args.exchange == 'fused') else 0  # exchange wait kernel
     launches_per_step += 5 if args.input_dist else 0  # pack scan + copy, unpack reduce + scan + main
+
+    # the north-star target configuration (>= 70 % of HBM on the large multi-hot
+    # model), timed in the same run at N = 1 (the headline stays the config above)
+    heavy = None
+    if world == 1 and args.config != 'heavy' and not args.no_heavy and not args.profile_only:
+        del tables, phys, batches, graphs
+        torch.cuda.empty_cache()
+        try:
+            heavy = time_config('heavy', args, dev, peak)
+        except Exception as ex:  # never fail the bench line on the extra leg
+            heavy = {'failed': str(ex)[:300]}
+
     if rank == 0:
         line = {
             'metric': _baseline_metric(),
@@ -487,27 +587,36 @@ def main():
             'steps': args.steps,
             'warmup': args.warmup,
             'ms_per_step': ms_per_step,
+            'ms_per_step_median': median_ms,
             'higher_is_better': True,
-            'scaling': 'strong' if world > 1 else 'weak',
+            'scaling': 'strong',
             'vs_baseline': None,
             'dtype': 'f32' if args.dtype == 'f32' else f'{args.dtype} rows, f32 accumulate/output',
             'data': 'synthetic (seeded generator, SURVEY §8d recipe; tables: counter-based hash U[-1,1))',
-            'config': {'workload': args.config, 'global_batch': B, 'fields': model.F, 'table_dtype': args.dtype,
-                       'parallelism': f'tablewise{world}', 'plan': plan_src, 'occupancy': plan.occupancy,
-                       **({'dist_backend': backend} if world > 1 else {}),
-                       'exchange': (args.exchange if world > 1 else 'none'),
-                       'launch': 'CUDA graph replay per step' if graphs else 'eager',
-                       'input': ('data-parallel local batches + KJT input dist in the timed step'
-                                 if args.input_dist else 'table-wise KJT resident per rank'),
-                       'l2': 'flushed between steps' if flush_between else
-                             f'inputs > L2 ({alg_local / 1e9:.2f} GB algorithmic per step per rank, '
-                             f'{args.batches} rotating batches)'},
-            'effective_hbm_gbs': eff_gbs_step * (world if world > 1 else 1),
-            'pct_of_8tbs': 100.0 * eff_gbs_step / 8000.0,
+            'config': _workload_config(args, model, world),
+            'impl_config': {'plan': plan_src, 'occupancy': plan.occupancy,
+                            **({'dist_backend': backend} if world > 1 else {}),
+                            'exchange': (args.exchange if world > 1 else 'none'),
+                            'launch': 'CUDA graph replay per step' if graphs else 'eager',
+                            'kernel': (f"plan-specialised (NVRTC, {jit['variants']} variants, {jit['registers']} "
+                                       f"regs, {jit['local_bytes']} B local)" if jit and jit['active'] else 'catalog'),
+                            'input': ('data-parallel local batches + KJT input dist in the timed step'
+                                      if args.input_dist else 'table-wise KJT resident per rank'),
+                            'l2': 'flushed between steps' if flush_between else
+                                  f'inputs > L2 ({alg_local / 1e9:.2f} GB algorithmic per step per rank, '
+                                  f'{args.batches} rotating batches)'},
+            'effective_hbm_gbs': eff_gbs_step,
+            'pct_of_8tbs': 100.0 * eff_gbs_step / (8000.0 * world),
             'roofline': {'bound': 'hbm', 'achieved': achieved, 'peak': peak, 'unit': 'GB/s',
-                         'frac': achieved / peak, 'traffic': traffic, 'kernel': 'recflex_fused_kernel',
+                         'frac': achieved / peak, 'traffic': traffic,
+                         'kernel': (f'recflex_fused_jit_k{plan.occupancy}' if jit and jit['active']
+                                    else 'recflex_fused_kernel'),
                          'peak_source': peak_src, 'fused_ms': fused_ms, 'map_ms': map_ms,
-                         'algorithmic_bytes_per_launch': alg_local},
+                         'algorithmic_bytes_per_launch': alg_local,
+                         'traffic_source': (os.path.relpath(tp, ROOT) if traffic is not None else
+                                            'no ncu capture of this workload / rank plan committed')},
+            'multi_gpu': multi,
+            'heavy': heavy,
             'e2e': e2e,
             'gpu_launches': launches_per_step * args.steps,
             'clocks': clk,
@@ -518,6 +627,81 @@ def main():
         dist.barrier()
         dist.destroy_process_group()
     return 0
+
+
+def time_config(config, args, dev, peak, steps=20, warmup=5, nbatches=3):
+    """One extra workload at N = 1 in the same run: tuned plan, plan-specialised
+    kernel, CUDA-graph replay per rotating batch, event-timed K steps (inputs >
+    L2), clocks sampled during the timed region, fused-kernel roofline."""
+    import torch
+    from paper_conf_sc_panzzxwslr0d24_b200 import synth
+    from paper_conf_sc_panzzxwslr0d24_b200.plan import Plan
+    m = synth.make_model(config)
+    phys = {}
+    for f in m.features:
+        if f.table not in phys:
+            rows, dim = m.tables[f.table]
+            phys[f.table] = synth.make_table_stored(f.table, rows, dim, 'f32', 'float', device=dev, seed=m.seed)
+    tables = [phys[f.table] for f in m.features]
+    plan = Plan.from_model(m)
+    path = os.path.join(ROOT, 'configs', 'tuned', f'{config}_w1_r0.json')
+    if os.path.exists(path):
+        with open(path) as fh:
+            plan.import_(json.load(fh))
+    info = plan.compile()
+    bts, alg = [], []
+    for i in range(nbatches):
+        b = synth.make_batch(m, 7 + i)
+        bts.append((torch.from_numpy(b.indices).to(dev), torch.from_numpy(b.offsets).to(dev)))
+        alg.append(synth.algorithmic_bytes(m, b, 'f32')['total'])
+    alg_b = float(np.mean(alg))
+    out = torch.empty((m.batch, m.d_tot), dtype=torch.float32, device=dev)
+    for i in range(warmup):
+        plan.forward(*bts[i % nbatches], m.batch, tables, out=out)
+    cap = torch.cuda.Stream()
+    cap.wait_stream(torch.cuda.current_stream())
+    graphs = []
+    for j in range(nbatches):
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=cap):
+            plan.forward(*bts[j], m.batch, tables, out=out, stream=cap)
+        graphs.append(g)
+    torch.cuda.current_stream().wait_stream(cap)
+    for i in range(warmup):
+        graphs[i % nbatches].replay()
+    torch.cuda.synchronize()
+    clocks = ClockSampler(dev.index)
+    clocks.start()
+    time.sleep(0.3)
+    stream = torch.cuda.current_stream()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for i in range(steps):
+        graphs[i % nbatches].replay()
+    e1.record(stream)
+    torch.cuda.synchronize()
+    clk = clocks.stop()
+    ms = e0.elapsed_time(e1) / steps
+    plan.set_profiling(True)
+    plan.kernel_times(reset=True)
+    for i in range(steps):
+        plan.forward(*bts[i % nbatches], m.batch, tables, out=out)
+    kt = plan.kernel_times(reset=True)
+    plan.set_profiling(False)
+    fused_ms = kt['fused_ms'] / max(1, kt['forwards'])
+    res = {'workload': config, 'global_batch': m.batch, 'fields': m.F, 'steps': steps, 'warmup': warmup,
+           'ms_per_step': ms, 'samples_per_s': m.batch / (ms / 1e3),
+           'effective_hbm_gbs': alg_b / (ms / 1e3) / 1e9, 'pct_of_8tbs': 100.0 * alg_b / (ms / 1e3) / 8e12,
+           'roofline': {'bound': 'hbm', 'achieved': alg_b / (fused_ms / 1e3) / 1e9, 'peak': peak, 'unit': 'GB/s',
+                        'frac': alg_b / (fused_ms / 1e3) / 1e9 / peak, 'fused_ms': fused_ms,
+                        'kernel': f'recflex_fused_jit_k{plan.occupancy}' if info['active'] else 'recflex_fused_kernel',
+                        'algorithmic_bytes_per_launch': alg_b},
+           'plan': os.path.relpath(path, ROOT), 'occupancy': plan.occupancy,
+           'l2': f'inputs > L2 ({alg_b / 1e9:.1f} GB algorithmic per step, {nbatches} rotating batches)',
+           'launch': 'CUDA graph replay per step', 'clocks': clk}
+    del graphs, tables, phys, bts
+    torch.cuda.empty_cache()
+    return res
 
 
 if __name__ == '__main__':

@@ -49,14 +49,24 @@
 #ifndef RECFLEX_H_
 #define RECFLEX_H_
 
+#ifdef __CUDACC_RTC__
+/* device-side compilation of the plan-specialised fused kernel (NVRTC, no libc headers) */
+typedef signed char int8_t;
+typedef int int32_t;
+typedef unsigned int uint32_t;
+typedef long long int64_t;
+typedef unsigned long long uint64_t;
+typedef unsigned long long uintptr_t;
+#else
 #include <stddef.h>
 #include <stdint.h>
+#endif
 
 #ifdef __cplusplus
 extern "C" {
 #endif
 
-#define RECFLEX_ABI_VERSION 2
+#define RECFLEX_ABI_VERSION 3
 #define RECFLEX_MAX_OCCUPANCY 8          /* CTAs of 256 threads per SM: K = 8 (reading C14) */
 
 typedef struct recflex_plan_s *recflex_plan_t; /* opaque, library-owned */
@@ -101,23 +111,30 @@ typedef struct {
 /* A feature's schedule: catalog entry + its runtime thread-mapping parameters
  * ("tunable parameters").  part 0: a task (CTA work unit) covers
  * per_block consecutive samples; part 1: a task covers the bags whose first
- * lookup falls in a window of per_block lookups (adaptive to the batch);
- * part 2: STATIC mapping -- exactly per_block tasks whatever the batch, each
- * covering ceil(B/per_block) samples (the paper's ablation straw man, P:81,
- * P:328-338; for experiments, never chosen by the tuner). */
+ * lookup falls in a window of per_block lookups (adaptive to the batch).
+ * Either way the batch NEEDS blocks_f = ceil(B/per_block) (part 0) or
+ * floor(nnz_f/npb)+1 (part 1) tasks, computed on the device per batch: the
+ * runtime thread mapping of §IV-B.
+ * static_blocks > 0 replaces it by the paper's STATIC thread mapping (the
+ * ablation straw man): exactly static_blocks tasks are allocated
+ * whatever the batch, and allocated task a performs the needed tasks
+ * a, a + static_blocks, a + 2*static_blocks, ... one after another ("if we
+ * allocate two blocks ... while the input workload requires three blocks at
+ * runtime, the first block will perform the computation of two blocks
+ * sequentially"; reading C31); allocated tasks with nothing to do idle.
+ * Never chosen by the tuner; for experiments. */
 typedef struct {
-    int32_t sched_id;  /* index into the catalog (recflex_catalog_info)         */
-    int32_t part;      /* 0 sample-, 1 lookup(nnz)-partitioned, 2 static         */
-    int32_t per_block; /* samples per task (0), lookups per task (1), tasks (2)  */
+    int32_t sched_id;      /* index into the catalog (recflex_catalog_info)         */
+    int32_t part;          /* 0 sample-, 1 lookup(nnz)-partitioned                   */
+    int32_t per_block;     /* samples per task (part 0), lookups per task (part 1)   */
+    int32_t static_blocks; /* 0: runtime thread mapping; > 0: static, that many tasks */
 } recflex_schedule_t;
 
 /* Catalog entry description (hand-written sm_100a schedule templates). */
 typedef enum {
     RECFLEX_FAMILY_GROUP = 0, /* G lanes per bag; 256/G bags in flight per CTA (G=32: warp per sample) */
     RECFLEX_FAMILY_BLOCK = 1, /* all 256 threads on one bag; smem partials + fixed-order reduction    */
-    RECFLEX_FAMILY_FLAT = 2,  /* G lanes walk a run of 8 consecutive bags as one lookup range       */
-    RECFLEX_FAMILY_BULK = 3   /* warp per run of bags; rows by TMA bulk copies into smem stages
-                                 (only in experimental builds; not in the default catalog)         */
+    RECFLEX_FAMILY_FLAT = 2   /* G lanes walk a run of 8 consecutive bags as one lookup range       */
 } recflex_family_t;
 
 typedef struct {
@@ -267,6 +284,60 @@ int32_t recflex_catalog_valid_dtype(int32_t sched_id, int32_t dim, int32_t dtype
 recflex_status_t recflex_occupancy_check(int32_t device, int32_t k, int32_t *active_blocks_per_sm,
                                          int32_t *registers_per_thread, int32_t *spill_bytes);
 
+/* ---- plan-specialised fused kernel (the paper's fusion compiler) --------- */
+
+/* The paper compiles one fused kernel per model with every feature's tuned
+ * schedule inlined into the if-else dispatch (§IV-B, Fig. 8; P:178
+ * "make all functions inline within the branches").  recflex_plan_compile
+ * generates that kernel for the plan's CURRENT schedules -- one branch per
+ * distinct (catalog entry, d_f, pool, row pitch), the entry's template called
+ * with those values as compile-time literals -- and compiles it for sm_100a
+ * with NVRTC (libnvrtc.so.12, loaded at run time), once per occupancy listed
+ * (occupancies = NULL / num = 0: the plan's current k).  Blocking; compiles
+ * concurrently; cubins are cached on disk (recflex_set_jit_cache_dir, else
+ * env RECFLEX_JIT_CACHE, else no cache).  From then on recflex_forward and
+ * recflex_forward_routed at occupancy k launch the compiled kernel as long as
+ * no feature's sched_id has changed since (recflex_set_schedule, import and
+ * tuning invalidate it; forwards then use the precompiled catalog kernel
+ * until the next compile -- same results, bit for bit, by construction: the
+ * same schedule templates in the same order).  RECFLEX_ERR_NOT_SUPPORTED if
+ * NVRTC or the driver entry points are unavailable (recflex_last_error says
+ * which). */
+recflex_status_t recflex_plan_compile(recflex_plan_t plan, const int32_t *occupancies, int32_t num_occupancies);
+
+typedef struct {
+    int32_t compiled;      /* a kernel exists for this k                          */
+    int32_t active;        /* it matches the current schedules and is used        */
+    int32_t variants;      /* distinct (entry, d, pool, pitch) branches           */
+    int32_t registers;     /* per thread (cuFuncGetAttribute)                     */
+    int32_t local_bytes;   /* local memory per thread (spills / stack)            */
+    int32_t blocks_per_sm; /* occupancy after smem / carveout setup (== k)        */
+    int32_t smem_bytes;    /* dynamic shared memory per CTA                       */
+    int32_t cache_hit;     /* cubin came from the disk cache                      */
+    float compile_ms;      /* NVRTC (or cache read) wall time                      */
+} recflex_jit_info_t;
+/* k = 0: the plan's current occupancy. */
+recflex_status_t recflex_jit_info(recflex_plan_t plan, int32_t k, recflex_jit_info_t *info);
+/* enable = 0: forwards ignore compiled kernels (A/B against the catalog kernel). */
+recflex_status_t recflex_set_jit(recflex_plan_t plan, int32_t enable);
+/* Directory for cached cubins (created on first write); NULL or "" = none. */
+recflex_status_t recflex_set_jit_cache_dir(const char *dir);
+/* The generator alone (no GPU needed): CUDA source of the specialised kernel
+ * for num_features features (catalog ids, dims, pools, dtypes -- dtypes NULL =
+ * all F32) at occupancy k; buf (nullable) receives up to cap-1 bytes + NUL,
+ * *len the full length; variant_of_feature[F] (nullable) the branch each
+ * feature takes; *num_variants the branch count.  INVALID_ARG if an entry is
+ * not valid for its feature. */
+recflex_status_t recflex_jit_generate(const int32_t *sched_ids, const int32_t *dims, const int32_t *pools,
+                                      const int32_t *dtypes, int32_t num_features, int32_t k, char *buf,
+                                      size_t cap, size_t *len, int32_t *variant_of_feature,
+                                      int32_t *num_variants);
+/* NVRTC-compile generated source to an sm_100a cubin (no GPU needed).
+ * cubin_buf (nullable, cap bytes) receives the cubin if it fits, *cubin_len
+ * its size; log_buf (nullable) the NVRTC log (ptxas -v lines included). */
+recflex_status_t recflex_jit_compile_source(const char *source, void *cubin_buf, size_t cap, size_t *cubin_len,
+                                            char *log_buf, size_t log_cap, int32_t *cache_hit);
+
 /* ---- introspection / validation / persistence ---------------------------- */
 
 /* Runs the map (+ fill) kernels for offsets (device) and copies the task map
@@ -277,6 +348,18 @@ recflex_status_t recflex_occupancy_check(int32_t device, int32_t k, int32_t *act
 recflex_status_t recflex_debug_task_map(recflex_plan_t plan, const int32_t *offsets, int32_t batch_size,
                                         int32_t *host_block_start, int32_t *host_task_range,
                                         int64_t task_range_capacity, void *stream);
+
+/* Task-range slots the plan reserved for feature f (lookup-partitioned
+ * schedules): max(64, max_batch * max_len / 128 + 3).  A batch whose
+ * floor(nnz_f/npb)+1 tasks would not fit in slots - 1 runs with npb raised to
+ * ceil(nnz_f / (slots - 2)) (reading C12). */
+recflex_status_t recflex_get_task_slots(recflex_plan_t plan, int32_t f, int32_t *slots);
+
+/* Tasks every feature NEEDED in the plan's last map (forward or
+ * recflex_debug_task_map): ceil(B/per_block) or floor(nnz_f/npb)+1 -- equal to
+ * the feature's task count unless a static mapping (static_blocks > 0) folds
+ * them onto fewer.  host_need[F].  Blocking. */
+recflex_status_t recflex_debug_task_need(recflex_plan_t plan, int32_t *host_need);
 
 /* Checks offsets (offsets[0]==0, monotone, F*B+1 entries) and that every ID of
  * feature f is in [0, rows_f).  Blocking.  RECFLEX_ERR_INDEX_OOB / INVALID_ARG. */
@@ -313,6 +396,49 @@ recflex_status_t recflex_forward_routed(recflex_plan_t plan, const int32_t *indi
                                         int32_t batch_size, const void *const *tables, float *const *host_dst,
                                         int32_t num_dst, int32_t rows_per_dst, int32_t dst_stride,
                                         int32_t col_base, void *stream);
+
+/* The safe form of the fused exchange for a step loop (P:350 table-wise
+ * placement): double-buffered destinations and a
+ * device-side completion signal, no host or collective barrier per step.
+ *   world, rank   : W ranks, this rank's index
+ *   rows_per_dst  : B / W (samples each rank receives)
+ *   dst_stride    : columns of the exchanged [rows][stride] float32 layout
+ *   col_base      : first column of this rank's features in it
+ *   dst[b][j]     : host arrays of W DEVICE pointers -- buffer b (0, 1) of rank
+ *                   j (local, NVLink peer-enabled or CUDA-IPC mapped), 16-byte
+ *                   aligned
+ *   flags[j]      : host array of W DEVICE pointers -- rank j's flag array of W
+ *                   uint32 (zero-initialised before the first step, owned by
+ *                   rank j, mapped here like the buffers)
+ *   local_flags   : this rank's own flag array (flags[rank] as seen locally)
+ * Step n of this plan (n = 0, 1, ... counted per plan) writes buffer n & 1 of
+ * every destination; *buffer_index receives n & 1 for the caller's own
+ * buffer.  The fused kernel's last CTA publishes n + 1 into every
+ * destination's flags[rank] with a system-scope release after all of the
+ * step's pooled rows are stored; a one-warp wait kernel, enqueued after it on
+ * `stream`, acquires flags[j] >= n + 1 for every writer j.  So work enqueued
+ * on `stream` after this call sees the complete exchanged rows of step n.
+ * Write-after-read safety: step n + 2 reuses buffer n & 1; a writer starts
+ * step n + 2 only after its own wait of step n + 1, i.e. after every rank's
+ * kernel of step n + 1 ran -- and each rank launches step n + 1 after the
+ * work it enqueued on `stream` before that call.  Hence the returned buffer
+ * is valid for work enqueued on `stream` before this plan's next-but-one
+ * exchange call (consume it on the same stream, or copy it).  Every rank must
+ * call this the same number of times; a writer that never arrives makes the
+ * wait kernel trap after ~60 s.  Async; B == world * rows_per_dst. */
+typedef struct {
+    int32_t world;
+    int32_t rank;
+    int32_t rows_per_dst;
+    int32_t dst_stride;
+    int32_t col_base;
+    float *const *dst[2];
+    uint32_t *const *flags;
+    uint32_t *local_flags;
+} recflex_exchange_t;
+recflex_status_t recflex_forward_exchange(recflex_plan_t plan, const int32_t *indices, const int32_t *offsets,
+                                          int32_t batch_size, const void *const *tables,
+                                          const recflex_exchange_t *exchange, int32_t *buffer_index, void *stream);
 
 /* ---- backward (training) --------------------------------- */
 

@@ -18,7 +18,10 @@ Functions and the passages they follow (PAPER.md "P:n"):
                     stored tables and decodes every element with it.
   embedding_bag_backward -- the adjoint (training):
                     dense gradient / SGD update of every table row.
-  task_map       -- Fig. 8: d_blocks_map and d_task_map, reading C12.
+  task_map       -- Fig. 8: d_blocks_map and d_task_map, reading C12
+                    (incl. the npb raise for reserved task slots).
+  static_assignment -- P:338 static thread mapping: which allocated block runs
+                    which needed block, in which order (reading C31).
   nnz_task_ranges-- reading C12 for nnz-partitioned schedules.
   kjt_input_dist -- table-wise input distribution (P:350
                     "place different embedding tables on multiple GPUs"):
@@ -84,9 +87,11 @@ def lib():
                 P(ctypes.c_void_p), P(ctypes.c_void_p), P(ctypes.c_void_p)]
             L.oracle_task_map.restype = ctypes.c_int
             L.oracle_task_map.argtypes = [
-                ctypes.c_int, ctypes.c_int, P(ctypes.c_int), P(ctypes.c_int), P(ctypes.c_int),
-                P(ctypes.c_int32), P(ctypes.c_int), P(ctypes.c_int), P(ctypes.c_int),
-                ctypes.c_int64, P(ctypes.c_int64)]
+                ctypes.c_int, ctypes.c_int, P(ctypes.c_int), P(ctypes.c_int), P(ctypes.c_int), P(ctypes.c_int),
+                P(ctypes.c_int), P(ctypes.c_int32), P(ctypes.c_int), P(ctypes.c_int), P(ctypes.c_int),
+                P(ctypes.c_int), P(ctypes.c_int), ctypes.c_int64, P(ctypes.c_int64)]
+            L.oracle_static_assignment.restype = ctypes.c_int
+            L.oracle_static_assignment.argtypes = [ctypes.c_int, ctypes.c_int, P(ctypes.c_int), P(ctypes.c_int)]
             L.oracle_nnz_task_ranges.restype = ctypes.c_int
             L.oracle_nnz_task_ranges.argtypes = [
                 ctypes.c_int, ctypes.c_int, P(ctypes.c_int32), ctypes.c_int, P(ctypes.c_int), P(ctypes.c_int)]
@@ -211,34 +216,55 @@ def embedding_bag_backward(rows, dims, pools, indices, offsets, B, grad, scale=1
     return tg, cn, ab
 
 
-def task_map(B, mode, per_block, offsets, cap=None):
-    """Fig. 8 arrays: (blocks_map[F], task_feature[T], task_rel[T])."""
+def task_map(B, mode, per_block, offsets, cap=None, slots=None, static_blocks=None, full=False):
+    """Fig. 8 arrays: (blocks_map[F], task_feature[T], task_rel[T]); with full=True also
+    need_map[F] (blocks the batch needs) and npb_map[F] (effective lookups per block)."""
     F = len(mode)
     mode_a = np.asarray(mode, np.intc)
     pb = np.asarray(per_block, np.intc)
-    cap_a = np.asarray(cap if cap is not None else [0] * F, np.intc)
+    z = [0] * F
+    cap_a = np.asarray(cap if cap is not None else z, np.intc)
+    slots_a = np.asarray(slots if slots is not None else z, np.intc)
+    st_a = np.asarray(static_blocks if static_blocks is not None else z, np.intc)
     off = np.ascontiguousarray(offsets, np.int32)
     # upper bound on tasks for the output buffers
     ub = 0
     for f in range(F):
-        if mode[f] == 0:
+        if st_a[f] > 0:
+            ub += int(st_a[f])
+        elif mode[f] == 0:
             ub += (B + pb[f] - 1) // pb[f]
-        elif mode[f] == 2:
-            ub += int(pb[f])
         else:
-            ub += (int(off[(f + 1) * B]) - int(off[f * B])) // pb[f] + 1
+            ub += (int(off[(f + 1) * B]) - int(off[f * B])) // max(1, int(pb[f])) + 1
     ub = max(ub, 1)
     blocks = np.zeros(F, np.intc)
+    need = np.zeros(F, np.intc)
+    npb = np.zeros(F, np.intc)
     tf = np.zeros(ub, np.intc)
     tr = np.zeros(ub, np.intc)
     n = ctypes.c_int64(0)
     rc = lib().oracle_task_map(F, B, _ptr(mode_a, ctypes.c_int), _ptr(pb, ctypes.c_int),
+                               _ptr(slots_a, ctypes.c_int), _ptr(st_a, ctypes.c_int),
                                _ptr(cap_a, ctypes.c_int), _ptr(off, ctypes.c_int32),
+                               _ptr(need, ctypes.c_int), _ptr(npb, ctypes.c_int),
                                _ptr(blocks, ctypes.c_int), _ptr(tf, ctypes.c_int), _ptr(tr, ctypes.c_int),
                                ub, ctypes.byref(n))
     if rc != 0:
         raise OracleError(rc)
+    if full:
+        return blocks, tf[:n.value].copy(), tr[:n.value].copy(), need, npb
     return blocks, tf[:n.value].copy(), tr[:n.value].copy()
+
+
+def static_assignment(need: int, nalloc: int):
+    """P:338 static mapping: (alloc_of[need], seq_of[need]) -- the allocated block that
+    performs needed block q, and at which sequential step."""
+    a = np.zeros(max(1, need), np.intc)
+    q = np.zeros(max(1, need), np.intc)
+    rc = lib().oracle_static_assignment(int(need), int(nalloc), _ptr(a, ctypes.c_int), _ptr(q, ctypes.c_int))
+    if rc != 0:
+        raise OracleError(rc)
+    return a[:need].copy(), q[:need].copy()
 
 
 def block_start_from_task_map(F, task_feature):

@@ -56,11 +56,24 @@
  *   oracle_task_map       -- the runtime thread map of Fig. 8:
  *       d_blocks_map[f] = feature_blocks, and d_task_map[b] = (feature_idx,
  *       rel_bidx) enumerating, feature by feature, rel = 0..feature_blocks-1.
- *       feature_blocks follows reading C12 (blocks "adaptive" to the batch's
- *       workload): sample-partitioned schedules take ceil(B/spb),
- *       nnz-partitioned schedules take floor(nnz_f/npb) + 1; an optional cap
- *       (tuning padding) limits it.  Pinned by brute-force enumeration
- *       and invariants in tests/test_oracle.py.
+ *       The blocks a batch NEEDS follow reading C12 (blocks "adaptive" to the
+ *       batch's workload): sample-partitioned schedules take
+ *       ceil(B/spb); nnz-partitioned schedules take floor(nnz_f/npb) + 1, where
+ *       npb is raised to ceil(nnz_f/(slots_f - 2)) when the feature's reserved
+ *       task slots would not hold the batch (reading C12).
+ *       Under a static thread mapping the feature instead gets a
+ *       fixed number of allocated blocks whatever the batch.  An optional cap
+ *       (tuning padding) limits the count.  Pinned by hand-worked
+ *       goldens (tests/golden/worked_example.json) and brute-force
+ *       enumeration in tests/test_oracle.py.
+ *
+ *   oracle_static_assignment -- the static thread mapping of P:338: "if we
+ *       allocate two blocks to a specific feature at compile time while the
+ *       input workload requires three blocks at runtime, the first block will
+ *       perform the computation of two blocks sequentially".  Needed block q
+ *       (0 <= q < need) is performed by allocated block q mod nalloc as its
+ *       (q div nalloc)-th step (reading C31: round robin).  Pinned by the
+ *       P:338 golden.
  *
  *   oracle_nnz_task_ranges -- for an nnz-partitioned feature, the samples a
  *       task owns: {s : floor((off[s]-off[0]) / npb) == rel}, written out by
@@ -276,31 +289,46 @@ int oracle_embedding_bag_backward(int F, int B, const int *dims, const int *pool
 
 /*
  * Task map of Fig. 8.
- *   mode[f]: 0 = sample-partitioned (per_block[f] = samples per block)
- *            1 = nnz-partitioned    (per_block[f] = lookups per block)
- *            2 = static             (per_block[f] = fixed block count)
- *   cap[f]:  0 = none, else feature_blocks = min(feature_blocks, cap[f])
- * Outputs blocks_map[F] (d_blocks_map), task_feature/task_rel[max_tasks]
- * (d_task_map .x/.y), *num_tasks.  Returns ORACLE_ERR_ARG if max_tasks is short.
+ *   mode[f]:  0 = sample-partitioned (per_block[f] = samples per block)
+ *             1 = nnz-partitioned    (per_block[f] = lookups per block)
+ *   slots[f]: nnz-partitioned only: task slots reserved for the feature (0 =
+ *             unlimited); npb_eff = max(per_block, ceil(nnz_f / (slots - 2)))
+ *   static_blocks[f]: 0 = runtime mapping, > 0 = static mapping with that
+ *             many allocated blocks
+ *   cap[f]:   0 = none, else feature_blocks = min(feature_blocks, cap[f])
+ * Any of slots / static_blocks / cap may be NULL (all zero).
+ * Outputs need_map[F] (blocks the batch needs), npb_map[F] (effective lookups
+ * per block; per_block for mode 0), blocks_map[F] (d_blocks_map),
+ * task_feature/task_rel[max_tasks] (d_task_map .x/.y), *num_tasks.
+ * Returns ORACLE_ERR_ARG if max_tasks is short or a parameter is invalid.
  */
-int oracle_task_map(int F, int B, const int *mode, const int *per_block, const int *cap,
-                    const int32_t *offsets, int *blocks_map, int *task_feature, int *task_rel,
-                    int64_t max_tasks, int64_t *num_tasks) {
+int oracle_task_map(int F, int B, const int *mode, const int *per_block, const int *slots, const int *static_blocks,
+                    const int *cap, const int32_t *offsets, int *need_map, int *npb_map, int *blocks_map,
+                    int *task_feature, int *task_rel, int64_t max_tasks, int64_t *num_tasks) {
     int64_t n = 0;
     for (int f = 0; f < F; ++f) {
-        int64_t blocks;
+        int64_t need, npb = per_block[f];
+        if (per_block[f] < 1) return ORACLE_ERR_ARG;
         if (mode[f] == 0) {
-            blocks = ((int64_t)B + per_block[f] - 1) / per_block[f];
-        } else if (mode[f] == 2) {
-            /* static thread mapping (P:328-338 ablation): a fixed block count */
-            blocks = per_block[f];
-            if (B == 0) blocks = 0;
-        } else {
+            need = ((int64_t)B + per_block[f] - 1) / per_block[f];
+        } else if (mode[f] == 1) {
             int64_t nnz_f = (int64_t)offsets[(int64_t)(f + 1) * B] - offsets[(int64_t)f * B];
-            blocks = nnz_f / per_block[f] + 1;
-            if (B == 0) blocks = 0;
+            if (slots && slots[f] > 0) {
+                int64_t room = slots[f] - 2;
+                if (room < 1) return ORACLE_ERR_ARG;
+                int64_t lo = (nnz_f + room - 1) / room;
+                if (lo > npb) npb = lo;
+            }
+            need = nnz_f / npb + 1;
+        } else {
+            return ORACLE_ERR_ARG;
         }
+        if (B == 0) need = 0;
+        int64_t blocks = need;
+        if (static_blocks && static_blocks[f] > 0 && B > 0) blocks = static_blocks[f];
         if (cap && cap[f] > 0 && blocks > cap[f]) blocks = cap[f];
+        if (need_map) need_map[f] = (int)need;
+        if (npb_map) npb_map[f] = (int)npb;
         blocks_map[f] = (int)blocks;
         for (int64_t rel = 0; rel < blocks; ++rel) {
             if (n >= max_tasks) return ORACLE_ERR_ARG;
@@ -310,6 +338,20 @@ int oracle_task_map(int F, int B, const int *mode, const int *per_block, const i
         }
     }
     *num_tasks = n;
+    return ORACLE_OK;
+}
+
+/*
+ * Static thread mapping: needed block q runs on allocated block
+ * alloc_of[q] = q mod nalloc as its seq_of[q] = q div nalloc -th sequential
+ * step (reading C31).  Allocated blocks a >= need run nothing.
+ */
+int oracle_static_assignment(int need, int nalloc, int *alloc_of, int *seq_of) {
+    if (need < 0 || nalloc < 1) return ORACLE_ERR_ARG;
+    for (int q = 0; q < need; ++q) {
+        alloc_of[q] = q % nalloc;
+        seq_of[q] = q / nalloc;
+    }
     return ORACLE_OK;
 }
 

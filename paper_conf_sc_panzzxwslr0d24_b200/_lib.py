@@ -26,7 +26,8 @@ class FeatureSpec(ctypes.Structure):
 
 
 class Schedule(ctypes.Structure):
-    _fields_ = [('sched_id', ctypes.c_int32), ('part', ctypes.c_int32), ('per_block', ctypes.c_int32)]
+    _fields_ = [('sched_id', ctypes.c_int32), ('part', ctypes.c_int32), ('per_block', ctypes.c_int32),
+                ('static_blocks', ctypes.c_int32)]
 
 
 class CatalogInfo(ctypes.Structure):
@@ -47,6 +48,18 @@ class TuneStats(ctypes.Structure):
                 ('guard_evals', ctypes.c_int64), ('guard_won', ctypes.c_int32),
                 ('best_occupancy', ctypes.c_int32), ('best_ms', ctypes.c_double), ('tune_seconds', ctypes.c_double),
                 ('refine_evals', ctypes.c_int64), ('refine_gain', ctypes.c_double)]
+
+
+class JitInfo(ctypes.Structure):
+    _fields_ = [('compiled', ctypes.c_int32), ('active', ctypes.c_int32), ('variants', ctypes.c_int32),
+                ('registers', ctypes.c_int32), ('local_bytes', ctypes.c_int32), ('blocks_per_sm', ctypes.c_int32),
+                ('smem_bytes', ctypes.c_int32), ('cache_hit', ctypes.c_int32), ('compile_ms', ctypes.c_float)]
+
+
+class Exchange(ctypes.Structure):
+    _fields_ = [('world', ctypes.c_int32), ('rank', ctypes.c_int32), ('rows_per_dst', ctypes.c_int32),
+                ('dst_stride', ctypes.c_int32), ('col_base', ctypes.c_int32), ('dst', ctypes.c_void_p * 2),
+                ('flags', ctypes.c_void_p), ('local_flags', ctypes.c_void_p)]
 
 
 LOCAL_COST_FN = ctypes.CFUNCTYPE(None, c_void_p, c_int32, c_int32, P(ctypes.c_double))
@@ -103,6 +116,18 @@ SIGNATURES = {
     'recflex_kjt_dist_sizes': (c_int32, [c_void_p, P(c_int32), P(c_int32), P(c_int32)]),
     'recflex_kjt_pack': (c_int32, [c_void_p, c_void_p, c_void_p, c_void_p, c_void_p, c_void_p, c_void_p]),
     'recflex_kjt_unpack': (c_int32, [c_void_p, c_void_p, c_void_p, c_void_p, c_void_p, c_void_p]),
+    'recflex_plan_compile': (c_int32, [c_void_p, P(c_int32), c_int32]),
+    'recflex_forward_exchange': (c_int32, [c_void_p, c_void_p, c_void_p, c_int32, P(c_void_p), P(Exchange),
+                                           P(c_int32), c_void_p]),
+    'recflex_debug_task_need': (c_int32, [c_void_p, P(c_int32)]),
+    'recflex_get_task_slots': (c_int32, [c_void_p, c_int32, P(c_int32)]),
+    'recflex_jit_info': (c_int32, [c_void_p, c_int32, P(JitInfo)]),
+    'recflex_set_jit': (c_int32, [c_void_p, c_int32]),
+    'recflex_set_jit_cache_dir': (c_int32, [ctypes.c_char_p]),
+    'recflex_jit_generate': (c_int32, [P(c_int32), P(c_int32), P(c_int32), P(c_int32), c_int32, c_int32,
+                                       ctypes.c_char_p, ctypes.c_size_t, P(ctypes.c_size_t), P(c_int32), P(c_int32)]),
+    'recflex_jit_compile_source': (c_int32, [ctypes.c_char_p, c_void_p, ctypes.c_size_t, P(ctypes.c_size_t),
+                                             ctypes.c_char_p, ctypes.c_size_t, P(c_int32)]),
 }
 
 
@@ -130,6 +155,11 @@ def _load():
 
 
 lib = _load()
+
+# Compiled plan-specialised kernels (recflex_plan_compile) are cached in-tree
+# next to the library unless RECFLEX_JIT_CACHE names another directory.
+JIT_CACHE = os.environ.get('RECFLEX_JIT_CACHE') or os.path.join(HERE, 'jit_cache')
+lib.recflex_set_jit_cache_dir(JIT_CACHE.encode())
 
 
 def check(code, where=''):

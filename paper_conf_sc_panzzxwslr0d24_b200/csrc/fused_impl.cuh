@@ -21,6 +21,7 @@
 
 namespace recflex {
 
+#ifndef RECFLEX_JIT
 template <int I, int END>
 __device__ __forceinline__ void dispatch_chain(int id, const TaskCtx &x, float *red, int *bag_ctr) {
     if constexpr (I < END && I < kCatalogSize) {
@@ -37,9 +38,6 @@ __device__ __forceinline__ void dispatch_chain(int id, const TaskCtx &x, float *
             else if constexpr (e.family == RECFLEX_FAMILY_FLAT)
                 sched_flat<e.ET, GT, e.VEC, e.U>(x.table, x.rowb, e.G, x.offs, x.idx, x.out, x.dim, x.pool, x.ro, x.s0,
                                                   x.s1, bag_ctr);
-            else if constexpr (e.family == RECFLEX_FAMILY_BULK)
-                sched_bulk<e.U>(reinterpret_cast<const float *>(x.table), x.offs, x.idx, x.out, x.dim, x.pool, x.ro,
-                                x.s0, x.s1, bag_ctr, x.wsmem, x.wbytes);
             else
                 sched_block<e.ET, GT, e.VEC, e.C, e.U>(x.table, x.rowb, e.G, x.offs, x.idx, x.out, x.dim, x.pool, x.ro,
                                                         x.s0, x.s1, red);
@@ -63,12 +61,9 @@ __device__ __forceinline__ void dispatch_schedule(int id, const TaskCtx &x, floa
 // Single call site for the whole catalog: the kernel calls this once per task
 // (few live values cross the call), and it branches to the schedule.
 static __device__ __noinline__ void dispatch_task(int id, const char *T, unsigned rowb, const int32_t *offs,
-                                                  const int32_t *idx, float *out,
-                                           int d, int pool, const OutRoute ro, int s0, int s1, float *red, int *bag,
-                                           unsigned char *wsmem, int wbytes) {
+                                                  const int32_t *idx, float *out, int d, int pool, const OutRoute ro,
+                                                  int s0, int s1, float *red, int *bag) {
     TaskCtx x;
-    x.wsmem = wsmem;
-    x.wbytes = wbytes;
     x.table = T;
     x.rowb = rowb;
     x.offs = offs;
@@ -81,6 +76,8 @@ static __device__ __noinline__ void dispatch_task(int id, const char *T, unsigne
     x.s1 = s1;
     dispatch_schedule(id, x, red, bag);
 }
+
+#endif  // !RECFLEX_JIT
 
 constexpr int kRedFloats = 8 * 256;  // BLOCK family: [8 warps][SPAN <= 256]
 constexpr int kWarps = kBlockThreads / 32;
@@ -133,6 +130,20 @@ __device__ __forceinline__ int find_feature(const int *bs, int F, int t) {
     return lo;
 }
 
+// Samples [s0, s1) of needed task q of feature f (the runtime thread map's
+// task, Fig. 8): sample-partitioned -> per_block consecutive samples;
+// lookup-partitioned -> the range the fill kernel wrote.
+__device__ __forceinline__ void task_range(const FeatureDesc &fd, int q, const FusedArgs &a, int &s0, int &s1) {
+    if (fd.part == 0) {
+        s0 = min(a.B, q * fd.per_block);
+        s1 = min(a.B, s0 + fd.per_block);
+    } else {
+        const int32_t *ts = a.task_start + fd.slot_base;
+        s0 = ts[q];
+        s1 = ts[q + 1];
+    }
+}
+
 // Claim the next task from the device counter and decode it into slot S
 // (called by one lane that won the slot's 0 -> 1 CAS); publishes with a
 // release store of state = 2.
@@ -147,19 +158,8 @@ __device__ __forceinline__ void fill_slot(TaskSlot &S, int n, const FusedArgs &a
         const int f = find_feature(bs, F, t);
         const int rel = t - bs[f];
         const FeatureDesc &fd = a.desc[f];
-        int s0, s1;
-        if (fd.part == 0) {
-            s0 = rel * fd.per_block;
-            s1 = min(a.B, s0 + fd.per_block);
-        } else if (fd.part == 2) {
-            const int per = (a.B + fd.per_block - 1) / fd.per_block;
-            s0 = min(a.B, rel * per);
-            s1 = min(a.B, s0 + per);
-        } else {
-            const int32_t *ts = a.task_start + fd.slot_base;
-            s0 = ts[rel];
-            s1 = ts[rel + 1];
-        }
+        int s0 = 0, s1 = 0;
+        if (fd.nalloc == 0) task_range(fd, rel, a, s0, s1);  // static tasks resolve their ranges in the loop
         S.f = f;
         S.s0 = s0;
         S.s1 = s1;
@@ -193,16 +193,14 @@ __device__ __forceinline__ void fused_body(const FusedArgs &a) {
     // block_start cached in shared memory when it fits in the launch's dynamic
     // smem (tuning launches run more -- virtual -- features than the plan sized for)
     const bool bs_in_smem = (F + 1) <= kSmemBlockStartCap && kRedFloats * 4 + 4 * (F + 1) <= a.smem_bytes;
-    // BULK-family stage slices: whatever dynamic smem the occupancy padding
-    // leaves after the reduction scratch and the block_start cache, split 8 ways
-    const int bulk_off = (kRedFloats * 4 + (bs_in_smem ? 4 * (F + 1) : 0) + 127) & ~127;
-    const int wbytes = ((a.smem_bytes - bulk_off) / kWarps) & ~127;
-    unsigned char *wsmem = dyn_smem + bulk_off + (tid >> 5) * (wbytes > 0 ? wbytes : 0);
 
     // PDL: everything above overlapped the map kernel; wait for its results.
     asm volatile("griddepcontrol.wait;" ::: "memory");
 
     const int total = a.block_start[F];
+    // exchange mode: this step's destination buffers (double-buffered by epoch parity)
+    float *const *optrs = a.out_ptrs;
+    if (!BWD && a.route_epoch) optrs += (size_t)(vld(a.route_epoch) & 1) * a.route_world;
     if (bs_in_smem)
         for (int i = tid; i <= F; i += kBlockThreads) bs_s[i] = a.block_start[i];
     const int *bs = bs_in_smem ? bs_s : a.block_start;
@@ -237,13 +235,6 @@ __device__ __forceinline__ void fused_body(const FusedArgs &a) {
                 if (spin0 == 0) spin0 = now;
                 else if (now - spin0 > 20000000000LL) asm volatile("trap;");
             }
-#ifdef RECFLEX_FILL_AHEAD
-            // EXPERIMENT, off by default (heavy unchanged, sharded1000 9% slower):
-            // claim and decode task n+1 now, so the warps that reach it later
-            // find it ready instead of waiting on its fill
-            TaskSlot &N = ring[(n + 1) % kRing];
-            if (ld_acquire(&N.state) == 0 && atomicCAS(&N.state, 0, 1) == 0) fill_slot(N, n + 1, a, bs, F, total);
-#endif
         }
         __syncwarp();
         __threadfence_block();
@@ -257,20 +248,67 @@ __device__ __forceinline__ void fused_body(const FusedArgs &a) {
         const long long w0 = a.timers ? clock64() : 0;
         const int f = vld(&S.f);
         const FeatureDesc fd = a.desc[f];
-        const bool cta_wide = !BWD && kFamilyDev[fd.sched] == RECFLEX_FAMILY_BLOCK;
+#ifdef RECFLEX_JIT
+        const int jv = a.jit_var[f];
+        const bool block_family = jit_is_block(jv);
+#else
+        const bool block_family = kFamilyDev[fd.sched] == RECFLEX_FAMILY_BLOCK;
+#endif
+        // static thread mapping runs its needed tasks CTA-synchronously;
+        // compiled only into plan-specialised kernels of plans that use it
+        // (its loop state would cost registers in every other kernel)
+#if defined(RECFLEX_JIT) && RECFLEX_JIT_STATIC
+        const bool stat = !BWD && fd.nalloc > 0;
+#else
+        constexpr bool stat = false;
+#endif
+        const bool cta_wide = !BWD && (block_family || stat);
         if (cta_wide) __syncthreads();  // every warp reaches task n (they walk the same sequence)
         OutRoute ro;
-        ro.ptrs = a.out_ptrs;
+        ro.ptrs = optrs;
         ro.rows = a.route_rows;
         ro.colofs = a.col_base + fd.col;
         ro.stride = a.out_stride;
-        if constexpr (BWD) {
-            sched_backward(a.grad + fd.col, a.out_stride, a.targets[f], a.offsets + (size_t)fd.in_feature * a.B,
-                           a.indices, fd.dim, fd.pool, a.bscale, vld(&S.s0), vld(&S.s1), &S.bag, a.bvec != 0);
-        } else {
-            dispatch_task(fd.sched, static_cast<const char *>(fd.table), (unsigned)fd.row_bytes,
-                          a.offsets + (size_t)fd.in_feature * a.B, a.indices, a.out + fd.col, fd.dim, fd.pool, ro,
-                          vld(&S.s0), vld(&S.s1), red, &S.bag, wsmem, wbytes);
+        // Static thread mapping (the paper's ablation straw man):
+        // allocated task rel performs the needed tasks rel, rel + nalloc,
+        // rel + 2*nalloc, ... one after another (reading C31); an allocated
+        // task beyond the batch's need idles.  Runtime mapping: one pass.
+        // (One call site for the dispatch: the schedules are inlined once.)
+        int q = stat ? t - bs[f] : 0;
+        const int need = stat ? a.need[f] : 1;
+        while (q < need) {
+            int s0, s1;
+            if (stat) {
+                task_range(fd, q, a, s0, s1);
+            } else {
+                s0 = vld(&S.s0);
+                s1 = vld(&S.s1);
+            }
+            if constexpr (BWD) {
+                sched_backward(a.grad + fd.col, a.out_stride, a.targets[f], a.offsets + (size_t)fd.in_feature * a.B,
+                               a.indices, fd.dim, fd.pool, a.bscale, s0, s1, &S.bag, a.bvec != 0);
+            } else {
+#ifdef RECFLEX_JIT
+                TaskCtx x;
+                x.table = static_cast<const char *>(fd.table);
+                x.offs = a.offsets + (size_t)fd.in_feature * a.B;
+                x.idx = a.indices;
+                x.out = a.out + fd.col;
+                x.ro = ro;
+                x.s0 = s0;
+                x.s1 = s1;
+                jit_dispatch(jv, x, red, &S.bag);
+#else
+                dispatch_task(fd.sched, static_cast<const char *>(fd.table), (unsigned)fd.row_bytes,
+                              a.offsets + (size_t)fd.in_feature * a.B, a.indices, a.out + fd.col, fd.dim, fd.pool, ro,
+                              s0, s1, red, &S.bag);
+#endif
+            }
+            if (!stat) break;
+            __syncthreads();           // every warp is done with needed task q
+            if (tid == 0) S.bag = 0;   // fresh bag counter for the next one
+            __syncthreads();
+            q += fd.nalloc;
         }
         if (cta_wide) __syncthreads();
         __syncwarp();
@@ -281,6 +319,31 @@ __device__ __forceinline__ void fused_body(const FusedArgs &a) {
                 if (a.timers && t < a.timers_cap) a.timers[t] = (long long)(vld64(&S.wtime) / kWarps);
                 S.seq = -1;
                 st_release(&S.state, 0);
+            }
+        }
+    }
+    if constexpr (!BWD) {
+        if (a.route_flags) {
+            // Exchange completion (recflex_forward_exchange): every CTA makes its
+            // peer stores visible system-wide, then counts itself done; the last
+            // one bumps the epoch and publishes it into each destination's flag
+            // array with a system-scope release (the destination's wait kernel
+            // acquires it).  The fence -> atomic -> fence chain orders all CTAs'
+            // stores before the flag.
+            __syncthreads();
+            if (tid == 0) {
+                __threadfence_system();
+                if (atomicAdd(a.route_done, 1) == (int)gridDim.x - 1) {
+                    __threadfence_system();
+                    const int e = vld(a.route_epoch) + 1;
+                    vst(a.route_epoch, e);
+                    vst(a.route_done, 0);
+                    __threadfence_system();
+                    for (int j = 0; j < a.route_world; ++j)
+                        asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(a.route_flags[j] + a.route_rank),
+                                     "r"((unsigned)e)
+                                     : "memory");
+                }
             }
         }
     }
@@ -296,6 +359,7 @@ __global__ void __launch_bounds__(kBlockThreads, KOCC) recflex_backward_kernel(F
     fused_body<KOCC, true>(a);
 }
 
+#ifndef __CUDACC_RTC__
 template <int KOCC, bool BWD>
 int fused_launch_impl(const FusedArgs &a, const LaunchCfg &cfg, void *stream) {
     cudaLaunchConfig_t lc = {};
@@ -336,6 +400,8 @@ int fused_occupancy_impl(int smem, int *blocks, int *regs, int *spill) {
     e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks, recflex_fused_kernel<KOCC>, kBlockThreads, smem);
     return (int)e;
 }
+
+#endif  // !__CUDACC_RTC__
 
 }  // namespace recflex
 

@@ -4,9 +4,10 @@
 // The paper computes the map on the host ("host-side workload analysis",
 // P:170); here one CTA reads the batch's offsets and scans, so the forward has
 // no host round trip (reading C13).  Same integers as the oracle's formula:
-//   part 0 (sample-partitioned): feature_blocks = ceil(B / per_block)
+//   part 0 (sample-partitioned): need_f = ceil(B / per_block)
 //   part 1 (lookup-partitioned): npb = max(per_block, ceil(nnz_f/(slots-2)))
-//                                feature_blocks = floor(nnz_f / npb) + 1
+//                                need_f = floor(nnz_f / npb) + 1
+//   feature_blocks = need_f, or nalloc_f under a static mapping
 //   cap > 0: feature_blocks = min(feature_blocks, cap)
 //   block_start = exclusive scan of feature_blocks in feature order.
 #include <cuda_runtime.h>
@@ -127,10 +128,6 @@ __global__ void __launch_bounds__(kMapThreads) recflex_map_kernel(MapArgs a) {
             const FeatureDesc &fd = a.desc[f];
             if (fd.part == 0) {
                 blocks = (a.B + fd.per_block - 1) / fd.per_block;
-            } else if (fd.part == 2) {
-                // static mapping (paper's ablation straw man): a fixed
-                // number of blocks whatever the batch; each takes ceil(B/blocks)
-                blocks = fd.per_block;
             } else {
                 const int64_t fi = fd.in_feature;
                 const int nnz = a.offsets[(fi + 1) * a.B] - a.offsets[fi * a.B];
@@ -141,6 +138,10 @@ __global__ void __launch_bounds__(kMapThreads) recflex_map_kernel(MapArgs a) {
                 a.npb_eff[f] = npb;
                 blocks = nnz / npb + 1;
             }
+            a.need[f] = blocks;
+            // static thread mapping: a fixed number of allocated
+            // tasks whatever the batch; they fold the needed ones (fused kernel)
+            if (fd.nalloc > 0) blocks = fd.nalloc;
             if (fd.cap > 0 && blocks > fd.cap) blocks = fd.cap;
         }
         // block-wide exclusive scan
@@ -193,7 +194,7 @@ __global__ void __launch_bounds__(256) recflex_fill_kernel(FillArgs a) {
         const int32_t *offs = a.offsets + (size_t)fd.in_feature * a.B;
         const int base = offs[0];
         const int npb = a.npb_eff[f];
-        const int blocks = a.block_start[f + 1] - a.block_start[f];
+        const int blocks = a.need[f];  // needed tasks (a static feature allocates a different count)
         int32_t *ts = a.task_start + fd.slot_base;
         const int q_hi = (offs[s] - base) / npb;
         const int q_lo = (s == 0) ? -1 : (offs[s - 1] - base) / npb;
@@ -283,6 +284,31 @@ int concat_launch(const float *recv, int W, int rows, const int32_t *d_dims, con
     int grid = (int)((n + 255) / 256);
     if (grid > 148 * 16) grid = 148 * 16;
     recflex_concat_kernel<<<grid, 256, 0, (cudaStream_t)stream>>>(recv, W, rows, d_dims, d_cols, d_tot, out);
+    return (int)cudaGetLastError();
+}
+
+// Exchange wait (recflex_forward_exchange): lane j spins until writer j has
+// published this rank's current epoch (acquire at system scope), so work
+// ordered after this kernel on the stream sees every peer's pooled rows.  A
+// writer that never arrives (a dead peer) traps after ~60 s instead of hanging.
+__global__ void recflex_route_wait_kernel(const uint32_t *flags, const int32_t *epoch, int world) {
+    const int j = threadIdx.x;
+    if (j >= world) return;
+    const unsigned target = (unsigned)*reinterpret_cast<const volatile int32_t *>(epoch);
+    unsigned long long t0 = 0, now;
+    while (true) {
+        unsigned v;
+        asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(flags + j) : "memory");
+        if ((int)(v - target) >= 0) break;
+        __nanosleep(200);
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(now));
+        if (t0 == 0) t0 = now;
+        else if (now - t0 > 60ull * 1000000000ull) asm volatile("trap;");
+    }
+}
+
+int route_wait_launch(const uint32_t *local_flags, const int32_t *epoch, int world, void *stream) {
+    recflex_route_wait_kernel<<<1, 32 * ((world + 31) / 32), 0, (cudaStream_t)stream>>>(local_flags, epoch, world);
     return (int)cudaGetLastError();
 }
 

@@ -62,7 +62,7 @@ int row_bytes_of(int dim, int dtype) {
 int samples_per_task_default(int sched_id, float mean_len, float coverage, int target) {
     const CatalogEntry &e = kCatalog[sched_id];
     const int slots = (e.family == RECFLEX_FAMILY_GROUP) ? kBlockThreads / e.G
-                      : (e.family == RECFLEX_FAMILY_FLAT || e.family == RECFLEX_FAMILY_BULK)
+                      : (e.family == RECFLEX_FAMILY_FLAT)
                           ? (kBlockThreads / e.G) * 8
                           : 1;
     double el = std::max(0.25, (double)mean_len * std::max(0.05, (double)coverage));
@@ -84,7 +84,7 @@ int task_lookups_target(const recflex_feature_spec_t *specs, int F, int max_batc
 }
 
 recflex_schedule_t default_schedule(const recflex_feature_spec_t &spec, int target) {
-    recflex_schedule_t s = {0, 0, 1};
+    recflex_schedule_t s = {0, 0, 1, 0};
     const int d = spec.dim;
     int id = -1;
     if (spec.dtype != RECFLEX_DTYPE_F32) {
@@ -140,8 +140,8 @@ int slots_for(int max_batch, float max_len) {
 
 bool schedule_valid_for(const recflex_schedule_t &s, int dim, int dtype, int col, int d_tot) {
     if (s.sched_id < 0 || s.sched_id >= kCatalogSize) return false;
-    if (s.part < 0 || s.part > 2) return false;
-    if (s.per_block < 1) return false;
+    if (s.part < 0 || s.part > 1) return false;
+    if (s.per_block < 1 || s.static_blocks < 0) return false;
     const CatalogEntry &e = kCatalog[s.sched_id];
     if (!catalog_valid(e, dim, dtype)) return false;
     // vector stores need 16-byte aligned output columns
@@ -214,18 +214,56 @@ recflex_status_t prepare_occupancy(recflex_plan_s *p, int k) {
     return RECFLEX_OK;
 }
 
+// Async host -> device copy of a small plan array through pinned staging (so
+// it is truly asynchronous and never reads pageable memory).  Refuses to run
+// inside a stream capture: the captured copy would read the staging slot at
+// every replay, after later uploads reused it (run one forward before capturing).
+recflex_status_t staged_copy(recflex_plan_s *p, void *d_dst, const void *src, size_t bytes, cudaStream_t stream) {
+    if (bytes == 0) return RECFLEX_OK;
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    cudaStreamIsCapturing(stream, &cs);
+    if (cs != cudaStreamCaptureStatusNone) {
+        set_last_error("plan descriptors / pointer tables changed inside a CUDA graph capture: run one forward "
+                       "with these tables and destinations before capturing");
+        return RECFLEX_ERR_INVALID_ARG;
+    }
+    StageSlot &sl = p->stage[p->stage_next];
+    p->stage_next = (p->stage_next + 1) % kStageSlots;
+    cudaError_t e = cudaSuccess;
+    if (!sl.ev) e = cudaEventCreateWithFlags(&sl.ev, cudaEventDisableTiming);
+    if (e != cudaSuccess) return cuda_status(e);
+    if (sl.pending) {
+        e = cudaEventSynchronize(sl.ev);  // the copy that last used this slot has run (normally long ago)
+        if (e != cudaSuccess) return cuda_status(e);
+        sl.pending = false;
+    }
+    if (sl.cap < bytes) {
+        cudaFreeHost(sl.h);
+        sl.h = nullptr;
+        sl.cap = 0;
+        e = cudaMallocHost(&sl.h, bytes);
+        if (e != cudaSuccess) return cuda_status(e);
+        sl.cap = bytes;
+    }
+    std::memcpy(sl.h, src, bytes);
+    e = cudaMemcpyAsync(d_dst, sl.h, bytes, cudaMemcpyHostToDevice, stream);
+    if (e != cudaSuccess) return cuda_status(e);
+    e = cudaEventRecord(sl.ev, stream);
+    if (e != cudaSuccess) return cuda_status(e);
+    sl.pending = true;
+    return RECFLEX_OK;
+}
+
 recflex_status_t upload_desc(recflex_plan_s *p, cudaStream_t stream) {
     for (int f = 0; f < p->F; ++f) p->desc[f].table = p->tables[f];
     p->part1.clear();
     for (int f = 0; f < p->F; ++f)
         if (p->desc[f].part == 1) p->part1.push_back(f);
-    cudaError_t e = cudaMemcpyAsync(p->ex.d_desc, p->desc.data(), sizeof(FeatureDesc) * p->F,
-                                    cudaMemcpyHostToDevice, stream);
-    if (e != cudaSuccess) return cuda_status(e);
+    recflex_status_t st = staged_copy(p, p->ex.d_desc, p->desc.data(), sizeof(FeatureDesc) * p->F, stream);
+    if (st != RECFLEX_OK) return st;
     if (!p->part1.empty()) {
-        e = cudaMemcpyAsync(p->ex.d_part1, p->part1.data(), sizeof(int32_t) * p->part1.size(), cudaMemcpyHostToDevice,
-                            stream);
-        if (e != cudaSuccess) return cuda_status(e);
+        st = staged_copy(p, p->ex.d_part1, p->part1.data(), sizeof(int32_t) * p->part1.size(), stream);
+        if (st != RECFLEX_OK) return st;
     }
     p->ex.num_part1 = (int)p->part1.size();
     p->desc_dirty = false;
@@ -245,6 +283,7 @@ recflex_status_t run_pipeline(recflex_plan_s *p, const Exec &ex, const int32_t *
     ma.in_F = ex.in_F;
     ma.block_start = ex.d_block_start;
     ma.npb_eff = ex.d_npb_eff;
+    ma.need = ex.d_need;
     ma.counter = ex.d_counter;
     int rc = map_launch(ma, stream);
     if (rc) return cuda_status_at((cudaError_t)rc, "map kernel launch");
@@ -254,6 +293,7 @@ recflex_status_t run_pipeline(recflex_plan_s *p, const Exec &ex, const int32_t *
         fa.offsets = offsets;
         fa.block_start = ex.d_block_start;
         fa.npb_eff = ex.d_npb_eff;
+        fa.need = ex.d_need;
         fa.part1_features = ex.d_part1;
         fa.num_part1 = ex.num_part1;
         fa.B = B;
@@ -266,6 +306,7 @@ recflex_status_t run_pipeline(recflex_plan_s *p, const Exec &ex, const int32_t *
     a.desc = ex.d_desc;
     a.block_start = ex.d_block_start;
     a.task_start = ex.d_task_start;
+    a.need = ex.d_need;
     a.indices = indices;
     a.offsets = offsets;
     a.out = out;
@@ -279,6 +320,11 @@ recflex_status_t run_pipeline(recflex_plan_s *p, const Exec &ex, const int32_t *
     a.out_ptrs = ex.out_ptrs;
     a.route_rows = ex.route_rows;
     a.col_base = ex.col_base;
+    a.route_epoch = ex.route_epoch;
+    a.route_done = ex.route_done;
+    a.route_flags = ex.route_flags;
+    a.route_rank = ex.route_rank;
+    a.route_world = ex.route_world;
     a.grad = ex.grad;
     a.targets = ex.d_targets;
     a.bscale = ex.bscale;
@@ -289,7 +335,16 @@ recflex_status_t run_pipeline(recflex_plan_s *p, const Exec &ex, const int32_t *
     // With events between the kernels, PDL overlap is disabled (the event is a
     // stream dependency point anyway).
     cfg.pdl = p->pdl && ev == nullptr;
-    rc = ex.backward ? backward_launch(k, a, cfg, stream) : fused_launch(k, a, cfg, stream);
+    a.jit_var = nullptr;
+    if (ex.d_desc == p->ex.d_desc && p->num_static > 0 && (ex.backward || !jit_ready(p, k))) {
+        set_last_error("a static thread mapping (static_blocks > 0) runs only in the plan-specialised kernel: "
+                       "call recflex_plan_compile (forward only)");
+        return RECFLEX_ERR_NOT_SUPPORTED;
+    }
+    if (!ex.backward && ex.d_desc == p->ex.d_desc && jit_ready(p, k))
+        rc = jit_launch(p, k, a, cfg.pdl, stream);  // the plan-specialised kernel (jit.cpp)
+    else
+        rc = ex.backward ? backward_launch(k, a, cfg, stream) : fused_launch(k, a, cfg, stream);
     if (rc) return cuda_status_at((cudaError_t)rc, ex.backward ? "backward kernel launch" : "fused kernel launch");
     if (ev) cudaEventRecord(ev->e2, stream);
     return RECFLEX_OK;
@@ -341,11 +396,22 @@ int32_t recflex_catalog_valid_dtype(int32_t id, int32_t dim, int32_t dtype) {
 }
 
 static void plan_free_device(recflex_plan_s *p) {
+    jit_release(p);
+    for (auto &sl : p->stage) {
+        if (sl.pending) cudaEventSynchronize(sl.ev);
+        if (sl.ev) cudaEventDestroy(sl.ev);
+        cudaFreeHost(sl.h);
+        sl = StageSlot();
+    }
+    cudaFree(p->d_xroute);
+    cudaFree(p->d_xflags);
+    cudaFree(p->d_xcount);
     cudaFree(p->d_route);
     cudaFree(p->d_targets);
     cudaFree(p->ex.d_desc);
     cudaFree(p->ex.d_block_start);
     cudaFree(p->ex.d_npb_eff);
+    cudaFree(p->ex.d_need);
     cudaFree(p->ex.d_counter);
     cudaFree(p->ex.d_task_start);
     cudaFree(p->ex.d_part1);
@@ -402,7 +468,7 @@ recflex_status_t recflex_plan_create(const recflex_feature_spec_t *specs, int32_
     for (int f = 0; f < F; ++f) {
         FeatureDesc &d = p->desc[f];
         std::memset(&d, 0, sizeof(d));
-        d.rows = specs[f].num_rows;
+        d.rows = (int32_t)specs[f].num_rows;
         d.dim = specs[f].dim;
         d.col = (int32_t)col;
         d.pool = specs[f].pool;
@@ -442,6 +508,7 @@ recflex_status_t recflex_plan_create(const recflex_feature_spec_t *specs, int32_
     if (e == cudaSuccess) e = cudaMalloc(&p->ex.d_desc, sizeof(FeatureDesc) * F);
     if (e == cudaSuccess) e = cudaMalloc(&p->ex.d_block_start, sizeof(int32_t) * (F + 1));
     if (e == cudaSuccess) e = cudaMalloc(&p->ex.d_npb_eff, sizeof(int32_t) * F);
+    if (e == cudaSuccess) e = cudaMalloc(&p->ex.d_need, sizeof(int32_t) * F);
     if (e == cudaSuccess) e = cudaMalloc(&p->ex.d_counter, sizeof(int32_t) * 4);
     if (e == cudaSuccess) e = cudaMalloc(&p->ex.d_task_start, sizeof(int32_t) * std::max<int64_t>(1, slot));
     if (e == cudaSuccess) e = cudaMalloc(&p->ex.d_part1, sizeof(int32_t) * F);
@@ -485,6 +552,21 @@ static recflex_status_t sync_tables(recflex_plan_s *p, const void *const *tables
     return RECFLEX_OK;
 }
 
+namespace {
+// Makes the plan's device current for the call and restores the caller's.
+struct DeviceGuard {
+    int prev = -1;
+    explicit DeviceGuard(int dev) {
+        if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+        if (prev != dev) cudaSetDevice(dev);
+    }
+    ~DeviceGuard() {
+        int cur = -1;
+        if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+    }
+};
+}  // namespace
+
 recflex_status_t recflex_forward(recflex_plan_t p, const int32_t *indices, const int32_t *offsets, int32_t B,
                                  const void *const *tables, float *out, void *stream_) {
     if (!p || !tables) return RECFLEX_ERR_INVALID_ARG;
@@ -493,9 +575,7 @@ recflex_status_t recflex_forward(recflex_plan_t p, const int32_t *indices, const
     if (!indices || !offsets || !out) return RECFLEX_ERR_INVALID_ARG;
     if (((uintptr_t)out) % 16 != 0) return RECFLEX_ERR_INVALID_ARG;
     cudaStream_t stream = (cudaStream_t)stream_;
-    int cur = -1;
-    cudaGetDevice(&cur);
-    if (cur != p->device) cudaSetDevice(p->device);
+    DeviceGuard guard(p->device);
     recflex_status_t st = sync_tables(p, tables, stream);
     if (st != RECFLEX_OK) return st;
     EventTriple *ev = nullptr;
@@ -530,7 +610,7 @@ recflex_status_t recflex_forward_routed(recflex_plan_t p, const int32_t *indices
     for (int j = 0; j < num_dst; ++j)
         if (!host_dst[j] || ((uintptr_t)host_dst[j]) % 16) return RECFLEX_ERR_INVALID_ARG;
     cudaStream_t stream = (cudaStream_t)stream_;
-    cudaSetDevice(p->device);
+    DeviceGuard guard(p->device);
     recflex_status_t st = sync_tables(p, tables, stream);
     if (st != RECFLEX_OK) return st;
     bool same = (int)p->route_cache.size() == num_dst;
@@ -543,15 +623,79 @@ recflex_status_t recflex_forward_routed(recflex_plan_t p, const int32_t *indices
             if (e != cudaSuccess) return cuda_status(e);
         }
         p->route_cache.assign(host_dst, host_dst + num_dst);
-        cudaError_t e = cudaMemcpyAsync(p->d_route, p->route_cache.data(), sizeof(float *) * num_dst,
-                                        cudaMemcpyHostToDevice, stream);
-        if (e != cudaSuccess) return cuda_status(e);
+        st = staged_copy(p, p->d_route, p->route_cache.data(), sizeof(float *) * num_dst, stream);
+        if (st != RECFLEX_OK) return st;
     }
     Exec ex = p->ex;
     ex.out_ptrs = p->d_route;
     ex.route_rows = rows_per_dst;
     ex.col_base = col_base;
     return run_pipeline(p, ex, indices, offsets, B, host_dst[0], dst_stride, p->k, stream, nullptr);
+}
+
+recflex_status_t recflex_forward_exchange(recflex_plan_t p, const int32_t *indices, const int32_t *offsets, int32_t B,
+                                          const void *const *tables, const recflex_exchange_t *x,
+                                          int32_t *buffer_index, void *stream_) {
+    if (!p || !tables || !x) return RECFLEX_ERR_INVALID_ARG;
+    const int W = x->world;
+    if (W <= 0 || W > 1024 || x->rank < 0 || x->rank >= W || x->rows_per_dst <= 0 || x->dst_stride <= 0 ||
+        x->col_base < 0 || x->col_base + p->d_tot > x->dst_stride || !x->dst[0] || !x->dst[1] || !x->flags ||
+        !x->local_flags)
+        return RECFLEX_ERR_INVALID_ARG;
+    if (B != (int64_t)W * x->rows_per_dst || B > p->max_batch || B <= 0) return RECFLEX_ERR_INVALID_ARG;
+    if (!indices || !offsets) return RECFLEX_ERR_INVALID_ARG;
+    if ((x->dst_stride % 4) || (x->col_base % 4)) return RECFLEX_ERR_INVALID_ARG;
+    for (int b = 0; b < 2; ++b)
+        for (int j = 0; j < W; ++j)
+            if (!x->dst[b][j] || ((uintptr_t)x->dst[b][j]) % 16) return RECFLEX_ERR_INVALID_ARG;
+    for (int j = 0; j < W; ++j)
+        if (!x->flags[j]) return RECFLEX_ERR_INVALID_ARG;
+    cudaStream_t stream = (cudaStream_t)stream_;
+    DeviceGuard guard(p->device);
+    recflex_status_t st = sync_tables(p, tables, stream);
+    if (st != RECFLEX_OK) return st;
+    // pointer tables: [2W] destinations then [W] flag arrays, cached
+    std::vector<void *> want;
+    for (int b = 0; b < 2; ++b)
+        for (int j = 0; j < W; ++j) want.push_back(x->dst[b][j]);
+    for (int j = 0; j < W; ++j) want.push_back(x->flags[j]);
+    if (want != p->xroute_cache) {
+        if (p->xroute_cache.size() != want.size()) {
+            cudaFree(p->d_xroute);
+            cudaFree(p->d_xflags);
+            p->d_xroute = nullptr;
+            p->d_xflags = nullptr;
+            cudaError_t e = cudaMalloc(&p->d_xroute, sizeof(float *) * 2 * W);
+            if (e == cudaSuccess) e = cudaMalloc(&p->d_xflags, sizeof(uint32_t *) * W);
+            if (e != cudaSuccess) return cuda_status(e);
+        }
+        if (!p->d_xcount) {
+            cudaError_t e = cudaMalloc(&p->d_xcount, sizeof(int32_t) * 4);
+            if (e == cudaSuccess) e = cudaMemsetAsync(p->d_xcount, 0, sizeof(int32_t) * 4, stream);
+            if (e != cudaSuccess) return cuda_status(e);
+            p->x_steps = 0;
+        }
+        st = staged_copy(p, p->d_xroute, want.data(), sizeof(void *) * 2 * W, stream);
+        if (st == RECFLEX_OK) st = staged_copy(p, p->d_xflags, want.data() + 2 * W, sizeof(void *) * W, stream);
+        if (st != RECFLEX_OK) return st;
+        p->xroute_cache = want;
+    }
+    Exec ex = p->ex;
+    ex.out_ptrs = p->d_xroute;
+    ex.route_rows = x->rows_per_dst;
+    ex.col_base = x->col_base;
+    ex.route_epoch = p->d_xcount;
+    ex.route_done = p->d_xcount + 1;
+    ex.route_flags = p->d_xflags;
+    ex.route_rank = x->rank;
+    ex.route_world = W;
+    st = run_pipeline(p, ex, indices, offsets, B, x->dst[0][0], x->dst_stride, p->k, stream, nullptr);
+    if (st != RECFLEX_OK) return st;
+    int rc = route_wait_launch(x->local_flags, p->d_xcount, W, stream);
+    if (rc) return cuda_status_at((cudaError_t)rc, "exchange wait kernel launch");
+    if (buffer_index) *buffer_index = (int32_t)(p->x_steps & 1);
+    ++p->x_steps;
+    return RECFLEX_OK;
 }
 
 recflex_status_t recflex_backward(recflex_plan_t p, const int32_t *indices, const int32_t *offsets, int32_t B,
@@ -677,6 +821,7 @@ recflex_status_t recflex_get_schedule(recflex_plan_t p, int32_t f, recflex_sched
         s->sched_id = p->desc[f].sched;
         s->part = p->desc[f].part;
         s->per_block = p->desc[f].per_block;
+        s->static_blocks = p->desc[f].nalloc;
     }
     if (blocks_per_sm) *blocks_per_sm = p->k;
     return RECFLEX_OK;
@@ -686,9 +831,14 @@ recflex_status_t recflex_set_schedule(recflex_plan_t p, int32_t f, const recflex
     if (!p || !s || f < 0 || f >= p->F) return RECFLEX_ERR_INVALID_ARG;
     if (!schedule_valid_for(*s, p->desc[f].dim, p->desc[f].dtype, p->desc[f].col, (int)p->d_tot))
         return RECFLEX_ERR_INVALID_ARG;
+    // a compiled JIT kernel no longer matches if the entry or the presence of a
+    // static mapping (compiled in only when used) changes
+    if (p->desc[f].sched != s->sched_id || (p->desc[f].nalloc > 0) != (s->static_blocks > 0)) ++p->sched_version;
+    p->num_static += (s->static_blocks > 0 ? 1 : 0) - (p->desc[f].nalloc > 0 ? 1 : 0);
     p->desc[f].sched = s->sched_id;
     p->desc[f].part = s->part;
     p->desc[f].per_block = s->per_block;
+    p->desc[f].nalloc = s->static_blocks;
     p->desc_dirty = true;
     return RECFLEX_OK;
 }
@@ -743,6 +893,7 @@ recflex_status_t recflex_debug_task_map(recflex_plan_t p, const int32_t *offsets
     ma.in_F = p->F;
     ma.block_start = p->ex.d_block_start;
     ma.npb_eff = p->ex.d_npb_eff;
+    ma.need = p->ex.d_need;
     ma.counter = p->ex.d_counter;
     int rc = map_launch(ma, stream);
     if (rc) return cuda_status((cudaError_t)rc);
@@ -752,6 +903,7 @@ recflex_status_t recflex_debug_task_map(recflex_plan_t p, const int32_t *offsets
         fa.offsets = offsets;
         fa.block_start = p->ex.d_block_start;
         fa.npb_eff = p->ex.d_npb_eff;
+        fa.need = p->ex.d_need;
         fa.part1_features = p->ex.d_part1;
         fa.num_part1 = p->ex.num_part1;
         fa.B = B;
@@ -775,7 +927,7 @@ recflex_status_t recflex_debug_task_map(recflex_plan_t p, const int32_t *offsets
         for (int f = 0; f < p->F; ++f) {
             for (int64_t t = h_bs[f]; t < h_bs[f + 1]; ++t) {
                 const int rel = (int)(t - h_bs[f]);
-                if (p->desc[f].part == 1) {
+                if (p->desc[f].part == 1 && p->desc[f].nalloc == 0) {
                     h_ranges[2 * t] = ts[p->desc[f].slot_base + rel];
                     h_ranges[2 * t + 1] = ts[p->desc[f].slot_base + rel + 1];
                 } else {
@@ -786,6 +938,19 @@ recflex_status_t recflex_debug_task_map(recflex_plan_t p, const int32_t *offsets
         }
     }
     return RECFLEX_OK;
+}
+
+recflex_status_t recflex_get_task_slots(recflex_plan_t p, int32_t f, int32_t *slots) {
+    if (!p || !slots || f < 0 || f >= p->F) return RECFLEX_ERR_INVALID_ARG;
+    *slots = p->desc[f].slots;
+    return RECFLEX_OK;
+}
+
+recflex_status_t recflex_debug_task_need(recflex_plan_t p, int32_t *host_need) {
+    if (!p || !host_need) return RECFLEX_ERR_INVALID_ARG;
+    cudaSetDevice(p->device);
+    cudaError_t e = cudaMemcpy(host_need, p->ex.d_need, sizeof(int32_t) * p->F, cudaMemcpyDeviceToHost);
+    return e == cudaSuccess ? RECFLEX_OK : cuda_status(e);
 }
 
 recflex_status_t recflex_validate(recflex_plan_t p, const int32_t *indices, const int32_t *offsets, int32_t B,
@@ -859,15 +1024,33 @@ recflex_status_t recflex_get_kernel_times(recflex_plan_t p, double *map_ms, doub
     return RECFLEX_OK;
 }
 
+// Fingerprint of the first n catalog entries (family, ET, G, VEC, C, U): a plan
+// names schedules by catalog id, so an import must see the same entries.
+static uint64_t catalog_fingerprint(int n) {
+    uint64_t h = 1469598103934665603ull;
+    for (int i = 0; i < n && i < kCatalogSize; ++i) {
+        const CatalogEntry &e = kCatalog[i];
+        const int v[6] = {e.family, e.ET, e.G, e.VEC, e.C, e.U};
+        for (int x : v) {
+            h ^= (uint64_t)(uint32_t)x;
+            h *= 1099511628211ull;
+        }
+    }
+    return h & 0xffffffffffffull;  // 48 bits: exact in a JSON number
+}
+
 recflex_status_t recflex_plan_export(recflex_plan_t p, char *buf, size_t cap, size_t *len) {
     if (!p) return RECFLEX_ERR_INVALID_ARG;
     std::string s = "{\"abi\": " + std::to_string(RECFLEX_ABI_VERSION) + ", \"catalog_size\": " +
-                    std::to_string(kCatalogSize) + ", \"num_features\": " + std::to_string(p->F) +
-                    ", \"occupancy\": " + std::to_string(p->k) + ", \"schedules\": [";
+                    std::to_string(kCatalogSize) + ", \"catalog_fingerprint\": " +
+                    std::to_string(catalog_fingerprint(kCatalogSize)) + ", \"num_features\": " +
+                    std::to_string(p->F) + ", \"occupancy\": " + std::to_string(p->k) + ", \"schedules\": [";
     for (int f = 0; f < p->F; ++f) {
         if (f) s += ", ";
         s += "[" + std::to_string(p->desc[f].sched) + ", " + std::to_string(p->desc[f].part) + ", " +
-             std::to_string(p->desc[f].per_block) + "]";
+             std::to_string(p->desc[f].per_block);
+        if (p->desc[f].nalloc > 0) s += ", " + std::to_string(p->desc[f].nalloc);
+        s += "]";
     }
     s += "]}";
     if (len) *len = s.size() + 1;
@@ -901,6 +1084,16 @@ recflex_status_t recflex_plan_import(recflex_plan_t p, const char *json) {
     // the catalog is append-only: a plan exported with a smaller catalog names
     // the same entries
     if (!parse_int_after(c, &v) || v < 1 || v > kCatalogSize) return RECFLEX_ERR_NOT_SUPPORTED;
+    const int exported_catalog = (int)v;
+    if (const char *fp = std::strstr(json, "\"catalog_fingerprint\"")) {
+        fp += 21;
+        while (*fp && (*fp < '0' || *fp > '9')) ++fp;
+        const unsigned long long got = std::strtoull(fp, nullptr, 10);
+        if (got != catalog_fingerprint(exported_catalog)) {
+            set_last_error("plan import: catalog fingerprint mismatch (the plan names other schedules)");
+            return RECFLEX_ERR_NOT_SUPPORTED;
+        }
+    }
     c = std::strstr(json, "\"num_features\"");
     if (!c) return RECFLEX_ERR_INVALID_ARG;
     c += 14;
@@ -920,10 +1113,15 @@ recflex_status_t recflex_plan_import(recflex_plan_t p, const char *json) {
         c = std::strchr(c, '[');
         if (!c) return RECFLEX_ERR_INVALID_ARG;
         ++c;
-        long a = 0, b = 0, d = 0;
+        long a = 0, b = 0, d = 0, st = 0;
         if (!parse_int_after(c, &a) || !parse_int_after(c, &b) || !parse_int_after(c, &d))
             return RECFLEX_ERR_INVALID_ARG;
-        ss[f] = {(int32_t)a, (int32_t)b, (int32_t)d};
+        const char *save = c;
+        if (!parse_int_after(c, &st)) {  // optional 4th entry: static_blocks
+            st = 0;
+            c = save;
+        }
+        ss[f] = {(int32_t)a, (int32_t)b, (int32_t)d, (int32_t)st};
         if (!schedule_valid_for(ss[f], p->desc[f].dim, p->desc[f].dtype, p->desc[f].col, (int)p->d_tot))
             return RECFLEX_ERR_INVALID_ARG;
     }

@@ -16,6 +16,7 @@ struct Exec {
     FeatureDesc *d_desc = nullptr;
     int32_t *d_block_start = nullptr;
     int32_t *d_npb_eff = nullptr;
+    int32_t *d_need = nullptr;      // [F] needed tasks per feature (map kernel)
     int32_t *d_counter = nullptr;
     int32_t *d_task_start = nullptr;
     int32_t *d_part1 = nullptr;
@@ -25,6 +26,11 @@ struct Exec {
     float *const *out_ptrs = nullptr;  // routed mode: device array of destination buffers
     int route_rows = 0;                // 0 = local output
     int col_base = 0;
+    // exchange mode (recflex_forward_exchange): double buffers + completion flags
+    int32_t *route_epoch = nullptr;
+    int32_t *route_done = nullptr;
+    uint32_t *const *route_flags = nullptr;
+    int route_rank = 0, route_world = 0;
     // backward (NEXT #4)
     bool backward = false;
     const float *grad = nullptr;
@@ -35,6 +41,29 @@ struct Exec {
 
 struct EventTriple {
     cudaEvent_t e0, e1, e2;
+};
+
+// Pinned host staging for the plan's small async uploads (descriptors, pointer
+// tables): a pageable source would make cudaMemcpyAsync synchronous and is not
+// graph-capturable.  Slots rotate; a slot is reused only after its copy ran.
+struct StageSlot {
+    void *h = nullptr;
+    size_t cap = 0;
+    cudaEvent_t ev = nullptr;
+    bool pending = false;
+};
+constexpr int kStageSlots = 4;
+
+// A plan-specialised fused kernel (jit.cpp) compiled for one occupancy k.
+struct JitKernel {
+    void *module = nullptr;    // CUmodule
+    void *function = nullptr;  // CUfunction
+    int64_t version = -1;      // plan->sched_version it was generated from
+    int variants = 0;
+    int smem = 0, occ = 0, carveout = 0;
+    int regs = 0, local_bytes = 0;
+    bool cache_hit = false;
+    double compile_ms = 0;
 };
 
 }  // namespace recflex
@@ -88,6 +117,24 @@ struct recflex_plan_s {
     struct HostPipe *pipe = nullptr;
 
     recflex_tune_stats_t last_stats = {};
+
+    recflex::StageSlot stage[recflex::kStageSlots];
+    int stage_next = 0;
+
+    // recflex_forward_exchange state (device scratch + host caches)
+    float **d_xroute = nullptr;       // 2 x W destination pointers
+    uint32_t **d_xflags = nullptr;    // W flag-array pointers
+    int32_t *d_xcount = nullptr;      // [0] epoch (completed steps), [1] CTAs done in the launch
+    std::vector<void *> xroute_cache;
+    int64_t x_steps = 0;              // host mirror of the epoch (eager calls)
+
+    // plan-specialised fused kernels (jit.cpp): used by forwards at occupancy k
+    // while jit[k].version == sched_version (any schedule change bumps it)
+    recflex::JitKernel jit[recflex::kMaxOcc + 1];
+    int32_t *jit_var = nullptr;  // device: variant id of every feature
+    int64_t sched_version = 0;
+    int num_static = 0;          // features with a static thread mapping (P:338 ablation)
+    bool use_jit = true;
 };
 
 namespace recflex {
@@ -102,11 +149,17 @@ int min_dyn_smem(int F);
 recflex_status_t run_pipeline(recflex_plan_s *p, const Exec &ex, const int32_t *indices, const int32_t *offsets, int B,
                               float *out, int out_stride, int k, cudaStream_t stream, EventTriple *ev);
 recflex_status_t upload_desc(recflex_plan_s *p, cudaStream_t stream);
+recflex_status_t staged_copy(recflex_plan_s *p, void *d_dst, const void *src, size_t bytes, cudaStream_t stream);
 bool schedule_valid_for(const recflex_schedule_t &s, int dim, int dtype, int col, int d_tot);
 int row_bytes_of(int dim, int dtype);
 recflex_schedule_t default_schedule(const recflex_feature_spec_t &spec, int target);
 int find_catalog(int family, int G, int VEC, int C, int U, int ET = 0);
 int samples_per_task_default(int sched_id, float mean_len, float coverage, int target);
 int slots_for(int max_batch, float max_len);
+// plan-specialised fused kernel (jit.cpp)
+bool jit_ready(const recflex_plan_s *p, int k);
+int jit_launch(const recflex_plan_s *p, int k, const FusedArgs &a, bool pdl, cudaStream_t stream);
+recflex_status_t jit_compile_plan(recflex_plan_s *p, const int *ks, int nk);
+void jit_release(recflex_plan_s *p);
 
 }  // namespace recflex

@@ -1,7 +1,9 @@
 // recflex_internal.h -- shared between host plan code and device kernels of
 // librecflex.so (NOT shared with oracle/).
 #pragma once
+#ifndef __CUDACC_RTC__
 #include <stdint.h>
+#endif
 
 #include "../../include/recflex.h"
 
@@ -15,7 +17,8 @@ constexpr int kSmemBlockStartCap = 4096;   // features whose block_start fits in
 // `schedule_map[f]` (Fig. 8) folded into one record.
 struct __align__(16) FeatureDesc {
     const void *table;    // T_f, [rows][row_bytes] in the feature's dtype
-    int64_t rows;
+    int32_t rows;         // < 2^31 (recflex_plan_create)
+    int32_t nalloc;       // static thread mapping: allocated tasks, 0 = runtime mapping
     int32_t dim;
     int32_t col;          // col_f
     int32_t pool;         // 0 sum, 1 mean
@@ -39,6 +42,7 @@ struct MapArgs {
     int32_t in_F;          // number of KJT features in offsets (F_in), offsets has in_F*B+1 entries
     int32_t *block_start;  // [F+1]
     int32_t *npb_eff;      // [F] effective lookups per task (part 1)
+    int32_t *need;         // [F] tasks the batch needs (runtime mapping); = block count unless static
     int32_t *counter;      // task counter for the persistent fused kernel
 };
 
@@ -47,6 +51,7 @@ struct FillArgs {
     const int32_t *offsets;
     const int32_t *block_start;
     const int32_t *npb_eff;
+    const int32_t *need;            // [F] needed tasks (static features allocate fewer)
     const int32_t *part1_features;  // list of part-1 feature ids
     int32_t num_part1;
     int32_t B;
@@ -57,6 +62,7 @@ struct FusedArgs {
     const FeatureDesc *desc;
     const int32_t *block_start;   // [F+1]
     const int32_t *task_start;    // part-1 slots
+    const int32_t *need;          // [F] needed tasks (static thread mapping folds them onto nalloc)
     const int32_t *indices;
     const int32_t *offsets;
     float *out;
@@ -66,7 +72,7 @@ struct FusedArgs {
     int32_t B;
     int32_t out_stride;           // D_tot
     int32_t timers_cap;
-    int32_t smem_bytes;           // dynamic shared memory of the launch (BULK stages live in it)
+    int32_t smem_bytes;           // dynamic shared memory of the launch
     // fused pooled-output exchange (routed mode): sample s is stored into
     // out_ptrs[s / route_rows] at row s % route_rows, column col_base + col_f
     float *const *out_ptrs;       // device array of destination pointers (peer / IPC-mapped)
@@ -77,6 +83,17 @@ struct FusedArgs {
     float *const *targets;        // device array of F target pointers
     float bscale;
     int32_t bvec;                 // 1: 16-byte aligned grad columns (D_tot, col_f multiples of 4)
+    // plan-specialised (JIT-compiled) fused kernel: variant id of every feature
+    const int32_t *jit_var;
+    // exchange mode (recflex_forward_exchange): out_ptrs holds 2 x route_world
+    // destination pointers, buffer = *route_epoch & 1; the last CTA to finish
+    // bumps *route_epoch and publishes it into every destination's flag array
+    // (slot route_rank) with a system-scope release.  nullptr: plain routed mode.
+    int32_t *route_epoch;
+    int32_t *route_done;
+    uint32_t *const *route_flags;
+    int32_t route_rank;
+    int32_t route_world;
 };
 
 // ---------------------------------------------------------------------------
@@ -120,7 +137,7 @@ struct FusedArgs {
     /* FLAT, 256-bit rows */                                                    \
     X(2, 0, 1, 8, 1, 2) X(2, 0, 1, 8, 1, 4) X(2, 0, 2, 8, 1, 2) X(2, 0, 2, 8, 1, 4)         \
     X(2, 0, 4, 8, 1, 2) X(2, 0, 4, 8, 1, 4) X(2, 0, 8, 8, 1, 2) X(2, 0, 8, 8, 1, 4)         \
-    X(2, 0, 16, 8, 1, 2) X(2, 0, 16, 8, 1, 4) RECFLEX_CATALOG_EXPERIMENTAL(X)        \
+    X(2, 0, 16, 8, 1, 2) X(2, 0, 16, 8, 1, 4)                                  \
     RECFLEX_CATALOG_LOWP(X)
 #define RECFLEX_CATALOG_LOWP(X) RECFLEX_CATALOG_HALF(X, 1) RECFLEX_CATALOG_HALF(X, 2) RECFLEX_CATALOG_I8(X) \
     RECFLEX_CATALOG_FP8(X) RECFLEX_CATALOG_HALF_U8(X, 1) RECFLEX_CATALOG_HALF_U8(X, 2)
@@ -169,16 +186,6 @@ struct FusedArgs {
 // 32 lanes x 4 elements keep 4 accumulators per lane (cf. the FP8 entries).
 #define RECFLEX_CATALOG_HALF_U8(X, T) X(0, T, 16, 8, 1, 8) X(0, T, 32, 4, 1, 8) X(0, T, 8, 8, 1, 8)
 
-// BULK (rows by TMA bulk copy into smem stages) is built only on request:
-// per-row cp.async.bulk of random rows from multi-GB tables measured 10-100x
-// slower than register loads on B200 (the copy engine's address translation
-// thrashes), see DESIGN.md §6.
-#ifdef RECFLEX_EXPERIMENTAL_BULK
-#define RECFLEX_CATALOG_EXPERIMENTAL(X) X(3, 0, 32, 4, 1, 2) X(3, 0, 32, 4, 1, 4) X(3, 0, 32, 4, 1, 8)
-#else
-#define RECFLEX_CATALOG_EXPERIMENTAL(X)
-#endif
-
 struct CatalogEntry {
     int family, ET, G, VEC, C, U;
 };
@@ -199,7 +206,6 @@ inline bool catalog_valid(const CatalogEntry &e, int d, int dtype = RECFLEX_DTYP
     if (dtype == RECFLEX_DTYPE_FP8 && d % 8 != 0) return false;  // rows 8-byte aligned
     int span = e.G * e.VEC * e.C;
     if (4 * d < span) return false;
-    if (e.family == 3 && (d < 32 || d > 128)) return false;  // BULK: 128..512-byte rows, one pass
     return true;
 }
 
@@ -222,5 +228,6 @@ int remap_launch(const int32_t *src, int32_t *dst, int64_t n, int64_t shift, int
 int concat_launch(const float *recv, int W, int rows, const int32_t *d_dims, const int32_t *d_cols, int d_tot,
                   float *out, void *stream);
 int flush_launch(void *buf, size_t bytes, void *stream);
+int route_wait_launch(const uint32_t *local_flags, const int32_t *epoch, int world, void *stream);
 
 }  // namespace recflex

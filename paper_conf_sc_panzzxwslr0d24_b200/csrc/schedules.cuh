@@ -15,14 +15,23 @@
 //
 // Accumulation is fp32 in registers in a fixed order per (plan, batch):
 // GROUP adds a bag's rows strictly in ascending lookup order, so its result is
-// the sequential fp32 sum; BLOCK uses a fixed strided split + fixed tree.  No
-// floating-point atomics anywhere -> bitwise run-to-run determinism (C22).
+// the sequential fp32 sum; BLOCK uses a fixed strided split + fixed tree.  The
+// forward uses no floating-point atomics -> bitwise run-to-run determinism
+// (C22).  The backward (sched_backward) does: its scatter reduces with
+// red.global.add in L2, in an order that is not fixed (exact on integer data,
+// within the fp32 summation bound otherwise).
 #pragma once
+#ifndef __CUDACC_RTC__
 #include <cuda_runtime.h>
+#endif
 
 #include "recflex_internal.h"
 
 namespace recflex {
+
+#ifndef RECFLEX_SCHED_FN
+#define RECFLEX_SCHED_FN __device__ __noinline__
+#endif
 
 // ---- loads ---------------------------------------------------------------
 // Rows are gathered once and never reused by the CTA: bypass L1 allocation so
@@ -293,8 +302,6 @@ struct TaskCtx {
     int pool;
     OutRoute ro;            // output placement (local or routed to peers)
     int s0, s1;             // samples of this task
-    unsigned char *wsmem;   // this warp's private shared-memory slice (BULK stages)
-    int wbytes;             // its size
 };
 
 // ---- GROUP family --------------------------------------------------------
@@ -321,75 +328,6 @@ __device__ __forceinline__ void group_bag(const char *__restrict__ T, unsigned r
 #pragma unroll
                 for (int e = 0; e < VEC; ++e) acc[c][e] = 0.f;
 
-#ifdef RECFLEX_FASTLOOP
-            if constexpr (ET == RECFLEX_DTYPE_F32 && GT != 0 && U <= GT && GT >= 4 && C == 1) {
-                if ((p + 1) * SPAN <= d) {
-                    // EXPERIMENT, off by default (measured 16% SLOWER on heavy,
-                    // 7% on sharded1000): the row addresses of iteration i+1
-                    // (shuffle + one IMAD.WIDE each) are formed while the rows of
-                    // iteration i are in flight.  The shuffles issued behind the
-                    // outstanding row loads appear to complete in order behind
-                    // them, so nothing is gained and the loop gets longer.
-                    const int lane = threadIdx.x & 31;
-                    const unsigned gmask = (G == 32) ? 0xffffffffu : (((1u << G) - 1u) << (lane & ~(G - 1)));
-                    const char *base = T + 4 * colv[0];
-                    int cb = lo;
-                    int cur = (lo + lg < hi) ? ld_idx(idx + lo + lg) : 0;
-                    int nxt = (lo + G + lg < hi) ? ld_idx(idx + lo + G + lg) : 0;
-                    int j = lo;
-                    const float *pa[U];
-                    if (j + U <= hi) {
-#pragma unroll
-                        for (int u = 0; u < U; ++u)
-                            pa[u] = reinterpret_cast<const float *>(
-                                base + (size_t)(unsigned)__shfl_sync(gmask, cur, u, G) * rowb);
-                    }
-                    while (j + U <= hi) {
-                        float v[U][VEC];
-#pragma unroll
-                        for (int u = 0; u < U; ++u) ld_row<VEC>(pa[u], v[u]);
-                        const int jn = j + U;
-                        if (jn + U <= hi) {
-                            if (jn - cb >= G) {
-                                cb += G;
-                                cur = nxt;
-                                nxt = (cb + G + lg < hi) ? ld_idx(idx + cb + G + lg) : 0;
-                            }
-#pragma unroll
-                            for (int u = 0; u < U; ++u)
-                                pa[u] = reinterpret_cast<const float *>(
-                                    base + (size_t)(unsigned)__shfl_sync(gmask, cur, (jn - cb) + u, G) * rowb);
-                        }
-#pragma unroll
-                        for (int u = 0; u < U; ++u)
-#pragma unroll
-                            for (int e = 0; e < VEC; ++e) acc[0][e] += v[u][e];
-                        j = jn;
-                    }
-                    if (j < hi) {  // ragged tail: n < U rows
-                        if (j - cb >= G) {
-                            cb += G;
-                            cur = nxt;
-                        }
-                        const int n = hi - j;
-                        float v[U][VEC];
-#pragma unroll
-                        for (int u = 0; u < U; ++u) {
-                            const unsigned id = (unsigned)__shfl_sync(gmask, cur, (j - cb) + u, G);
-                            if (u < n) ld_row<VEC>(reinterpret_cast<const float *>(base + (size_t)id * rowb), v[u]);
-                        }
-#pragma unroll
-                        for (int u = 0; u < U; ++u)
-                            if (u < n)
-#pragma unroll
-                                for (int e = 0; e < VEC; ++e) acc[0][e] += v[u][e];
-                    }
-                    pool_finish<VEC>(acc[0], pool, hi - lo);
-                    st_out<VEC>(orow + colv[0], acc[0]);
-                    continue;
-                }
-            }
-#endif
 #ifndef RECFLEX_NO_SHFL_IDX
             if (U <= G && G >= 4) {
                 // Lookup IDs through registers: lane lg holds ID cb+lg of the
@@ -522,29 +460,18 @@ __device__ __forceinline__ void group_bag(const char *__restrict__ T, unsigned r
 // pooled.  Which group pools a bag does not change the bag's arithmetic (rows
 // in ascending lookup order) -> results are independent of the claim order.
 template <int ET, int GT, int VEC, int C, int U>
-__device__ __noinline__ void sched_group(const char *__restrict__ T, unsigned rowb, int gr, const int32_t *__restrict__ offs,
+RECFLEX_SCHED_FN void sched_group(const char *__restrict__ T, unsigned rowb, int gr, const int32_t *__restrict__ offs,
                                         const int32_t *__restrict__ idx, float *__restrict__ out, int d, int pool,
                                         const OutRoute ro, int s0, int s1, int *bag_ctr) {
     const int G = GT ? GT : gr;
     const int lane = threadIdx.x & 31;
     const int lg = lane & (G - 1);
     const unsigned gmask = (G == 32) ? 0xffffffffu : (((1u << G) - 1u) << (lane & ~(G - 1)));
-#ifdef RECFLEX_STATIC_CLAIM
-    int next_static = threadIdx.x / G;
-    auto claim = [&]() -> int {
-        const int v = next_static;
-        next_static += kBlockThreads / G;
-        (void)gmask;
-        (void)bag_ctr;
-        return s0 + v;
-    };
-#else
     auto claim = [&]() -> int {
         int v = 0;
         if (lg == 0) v = atomicAdd(bag_ctr, 1);
         return s0 + __shfl_sync(gmask, v, 0, G);
     };
-#endif
     int s = claim();
     int lo = 0, hi = 0;
     if (s < s1) {
@@ -576,7 +503,7 @@ __device__ __noinline__ void sched_group(const char *__restrict__ T, unsigned ro
 constexpr int kFlatRun = 8;
 
 template <int ET, int GT, int VEC, int U>
-__device__ __noinline__ void sched_flat(const char *__restrict__ T, unsigned rowb, int gr, const int32_t *__restrict__ offs,
+RECFLEX_SCHED_FN void sched_flat(const char *__restrict__ T, unsigned rowb, int gr, const int32_t *__restrict__ offs,
                                        const int32_t *__restrict__ idx, float *__restrict__ out, int d, int pool,
                                        const OutRoute ro, int s0, int s1, int *bag_ctr) {
     const int G = GT ? GT : gr;
@@ -633,144 +560,6 @@ __device__ __noinline__ void sched_flat(const char *__restrict__ T, unsigned row
             }
             while (b < se) finish_bag();  // the last bag(s) of the run, incl. trailing empty bags
         }
-    }
-}
-
-// ---- BULK family (sm_100a: TMA bulk-copy engine + mbarriers) ----------------
-// One warp walks a run of kFlatRun bags as one lookup range, like FLAT, but the
-// table rows are not loaded into registers: lane 0 issues one
-// cp.async.bulk.shared::cluster.global.mbarrier::complete_tx (UBLKCP) per row
-// into a ring of S stages of U rows in the warp's private slice of the CTA's
-// shared memory, and the warp consumes each stage (LDS.128 per lane, conflict
-// free) once its mbarrier completes.  Bytes in flight per warp = S*U rows,
-// independent of the register budget and not queued in the L1 load path.
-// S follows the shared memory the occupancy padding leaves (more stages at
-// lower k).  Rows of a bag are added in ascending lookup order.
-__device__ __forceinline__ unsigned smem_u32(const void *p) { return (unsigned)__cvta_generic_to_shared(p); }
-
-__device__ __forceinline__ void mbar_init(unsigned bar, unsigned count) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_expect_tx(unsigned bar, unsigned bytes) {
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(unsigned bar, unsigned parity) {
-    asm volatile(
-        "{\n\t.reg .pred p;\n\t"
-        "WAIT_%=:\n\t"
-        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
-        "@!p bra WAIT_%=;\n\t}" ::"r"(bar),
-        "r"(parity)
-        : "memory");
-}
-__device__ __forceinline__ void bulk_g2s(unsigned dst, const void *src, unsigned bytes, unsigned bar) {
-    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
-                 "l"(src), "r"(bytes), "r"(bar)
-                 : "memory");
-}
-
-constexpr int kBulkMaxStages = 8;
-constexpr int kBulkBarBytes = 8 * kBulkMaxStages;
-
-template <int U>
-__device__ __noinline__ void sched_bulk(const float *__restrict__ T, const int32_t *__restrict__ offs,
-                                       const int32_t *__restrict__ idx, float *__restrict__ out, int d, int pool,
-                                       const OutRoute ro, int s0, int s1, int *bag_ctr, unsigned char *wsmem,
-                                       int wbytes) {
-    const int lane = threadIdx.x & 31;
-    const unsigned rowb = (unsigned)d * 4u;
-    const unsigned stage_bytes = U * rowb;
-    int S = (int)((wbytes - kBulkBarBytes) / (int)stage_bytes);
-    S = S > kBulkMaxStages ? kBulkMaxStages : S;
-    const unsigned bar0 = smem_u32(wsmem);
-    const unsigned buf0 = bar0 + kBulkBarBytes;
-    const float *bufp = reinterpret_cast<const float *>(wsmem + kBulkBarBytes);
-    const bool ok = lane * 4 < d;
-    if (S < 1) {
-        // not even one stage fits (high occupancy leaves too little shared
-        // memory): same runs, rows through registers (warp per bag)
-        while (true) {
-            int v = 0;
-            if (lane == 0) v = atomicAdd(bag_ctr, kFlatRun);
-            const int s = s0 + __shfl_sync(0xffffffffu, v, 0);
-            if (s >= s1) return;
-            const int se = min(s1, s + kFlatRun);
-            for (int b = s; b < se; ++b)
-                group_bag<0, 32, 4, 1, 4>(reinterpret_cast<const char *>(T), (unsigned)d * 4u, idx, d, pool,
-                                          out_row(out, b, ro), ld_idx(offs + b), ld_idx(offs + b + 1), lane, 32);
-        }
-    }
-    if (lane == 0) {
-        for (int s = 0; s < S; ++s) mbar_init(bar0 + 8 * s, 1);
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    __syncwarp();
-    unsigned parity = 0;  // bit s = parity of stage s's next completion
-    while (true) {
-        int v = 0;
-        if (lane == 0) v = atomicAdd(bag_ctr, kFlatRun);
-        const int s = s0 + __shfl_sync(0xffffffffu, v, 0);
-        if (s >= s1) break;
-        const int se = min(s1, s + kFlatRun);
-        const int A = ld_idx(offs + s);
-        const int Z = ld_idx(offs + se);
-        // producer: issue stage `st` with rows [jp, jp+n)
-        int jp = A;
-        auto issue = [&](int st) {
-            const int n = min(U, Z - jp);
-            if (n <= 0) return;
-            const unsigned bar = bar0 + 8 * st;
-            if (lane == 0) mbar_expect_tx(bar, (unsigned)n * rowb);
-            __syncwarp();
-            if (lane < n) {  // lane r fetches row r of the stage: IDs and copies issue in parallel
-                const unsigned id = (unsigned)ld_idx(idx + jp + lane);
-                bulk_g2s(buf0 + (unsigned)st * stage_bytes + (unsigned)lane * rowb, T + (size_t)id * (unsigned)d, rowb,
-                         bar);
-            }
-            jp += n;
-        };
-#pragma unroll 1
-        for (int st = 0; st < S; ++st) issue(st);
-        float acc[4] = {0.f, 0.f, 0.f, 0.f};
-        int b = s, bstart = A, bend = ld_idx(offs + s + 1);
-        auto finish_bag = [&]() {
-            if (ok) {
-                pool_finish<4>(acc, pool, bend - bstart);
-                st_out<4>(out_row(out, b, ro) + lane * 4, acc);
-            }
-            acc[0] = acc[1] = acc[2] = acc[3] = 0.f;
-            ++b;
-            bstart = bend;
-            if (b < se) bend = ld_idx(offs + b + 1);
-        };
-        int jc = A;
-        int st = 0;
-        while (jc < Z) {
-            const int n = min(U, Z - jc);  // stages are consumed in issue order
-            mbar_wait(bar0 + 8 * st, (parity >> st) & 1u);
-            parity ^= 1u << st;
-            const float *rowp = bufp + (size_t)st * U * d + lane * 4;
-#pragma unroll
-            for (int r = 0; r < U; ++r) {
-                if (r < n) {
-                    float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
-                    if (ok) x = *reinterpret_cast<const float4 *>(rowp + r * d);
-                    while (jc + r >= bend) finish_bag();
-                    acc[0] += x.x;
-                    acc[1] += x.y;
-                    acc[2] += x.z;
-                    acc[3] += x.w;
-                }
-            }
-            jc += n;
-            __syncwarp();
-            // the stage's rows have been read: order those generic-proxy reads
-            // before the async-proxy writes that refill it
-            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-            issue(st);
-            st = (st + 1 == S) ? 0 : st + 1;
-        }
-        while (b < se) finish_bag();
     }
 }
 
@@ -845,7 +634,7 @@ static __device__ __noinline__ void sched_backward(const float *__restrict__ gra
 // xor-butterfly across the groups of a warp (every lane gets bit-identical
 // sums), then the 8 warp partials are summed in warp order from shared memory.
 template <int ET, int GT, int VEC, int C, int U>
-__device__ __noinline__ void sched_block(const char *__restrict__ T, unsigned rowb, int gr, const int32_t *__restrict__ offs,
+RECFLEX_SCHED_FN void sched_block(const char *__restrict__ T, unsigned rowb, int gr, const int32_t *__restrict__ offs,
                                         const int32_t *__restrict__ idx, float *__restrict__ out, int d, int pool,
                                         const OutRoute ro, int s0, int s1, float *red /* [8][SPAN] */) {
     const int G = GT ? GT : gr;

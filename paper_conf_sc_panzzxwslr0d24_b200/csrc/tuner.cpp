@@ -112,8 +112,6 @@ int64_t task_count(const FeatureDesc &d, int B, int64_t nnz) {
     if (B == 0) return 0;
     if (d.part == 0) {
         blocks = (B + d.per_block - 1) / d.per_block;
-    } else if (d.part == 2) {
-        blocks = d.per_block;
     } else {
         int64_t npb = d.per_block;
         const int64_t room = d.slots - 2;
@@ -121,6 +119,7 @@ int64_t task_count(const FeatureDesc &d, int B, int64_t nnz) {
         if (need > npb) npb = need;
         blocks = nnz / npb + 1;
     }
+    if (d.nalloc > 0) blocks = d.nalloc;
     if (d.cap > 0 && blocks > d.cap) blocks = d.cap;
     return blocks;
 }
@@ -151,7 +150,7 @@ struct Tuner {
     std::vector<TP> tps;
 
     DevBuf<FeatureDesc> d_desc;
-    DevBuf<int32_t> d_bs, d_npb, d_counter, d_ts, d_part1;
+    DevBuf<int32_t> d_bs, d_npb, d_need, d_counter, d_ts, d_part1;
     DevBuf<long long> d_timers;
     DevBuf<float> d_out;
     DevBuf<float> d_flush;
@@ -244,6 +243,7 @@ struct Tuner {
                 d.part = cands[f][c].part;
                 d.per_block = cands[f][c].per_block;
                 d.cap = 0;
+                d.nalloc = 0;
                 d.in_feature = c;
                 d.col = 0;
                 d.slot_base = 0;
@@ -253,6 +253,7 @@ struct Tuner {
                 check(d_desc.ensure(1));
                 check(d_bs.ensure(2));
                 check(d_npb.ensure(1));
+                check(d_need.ensure(1));
                 check(d_counter.ensure(4));
                 check(d_ts.ensure(std::max<int64_t>(d.part == 1 ? d.slots : 1, 1)));
                 check(d_part1.ensure(1));
@@ -266,6 +267,8 @@ struct Tuner {
                 ex.d_desc = d_desc.p;
                 ex.d_block_start = d_bs.p;
                 ex.d_npb_eff = d_npb.p;
+            ex.d_need = d_need.p;
+                ex.d_need = d_need.p;
                 ex.d_counter = d_counter.p;
                 ex.d_task_start = d_ts.p;
                 ex.d_part1 = d_part1.p;
@@ -322,6 +325,7 @@ struct Tuner {
                 while (got < target && ps < tp.pad_slots.size()) {
                     const int g = tp.pad_slots[ps];
                     FeatureDesc d = p->desc[g];
+                    d.nalloc = 0;
                     d.in_feature = n + (int)ps;
                     d.col = dump_col;
                     const int64_t nnz = bt.nnz(g);
@@ -344,6 +348,7 @@ struct Tuner {
                 d.part = cands[f][c].part;
                 d.per_block = cands[f][c].per_block;
                 d.cap = 0;
+                d.nalloc = 0;
                 d.in_feature = c;
                 d.col = c * base.dim;
                 d.rows = base.rows;
@@ -373,6 +378,7 @@ struct Tuner {
             check(d_desc.ensure(V));
             check(d_bs.ensure(V + 1));
             check(d_npb.ensure(V));
+            check(d_need.ensure(V));
             check(d_counter.ensure(4));
             check(d_ts.ensure(std::max<int64_t>(slot, 1)));
             check(d_part1.ensure(std::max<int64_t>((int64_t)part1.size(), 1)));
@@ -390,6 +396,7 @@ struct Tuner {
             ex.d_desc = d_desc.p;
             ex.d_block_start = d_bs.p;
             ex.d_npb_eff = d_npb.p;
+            ex.d_need = d_need.p;
             ex.d_counter = d_counter.p;
             ex.d_task_start = d_ts.p;
             ex.d_part1 = d_part1.p;
@@ -421,6 +428,7 @@ struct Tuner {
     void apply(const int32_t *choice) {
         for (int f = 0; f < p->F; ++f) {
             const recflex_schedule_t &s = cands[f][choice[f]];
+            if (p->desc[f].sched != s.sched_id) ++p->sched_version;
             p->desc[f].sched = s.sched_id;
             p->desc[f].part = s.part;
             p->desc[f].per_block = s.per_block;
@@ -483,7 +491,7 @@ struct Tuner {
                 const int sid = (int)(key / 100000 / 2), part = (int)(key / 100000 % 2);
                 const CatalogEntry &e = kCatalog[sid];
                 std::fprintf(stderr, " %dx[%s G%d V%d C%d U%d p%d/%ld]", hist[i].second,
-                             e.family == 3 ? "bulk" : (e.family == 2 ? "flat" : (e.family ? "block" : "group")),
+                             e.family == 2 ? "flat" : (e.family ? "block" : "group"),
                              e.G, e.VEC, e.C, e.U, part, key % 100000);
             }
             std::fprintf(stderr, "\n");
@@ -501,7 +509,7 @@ std::vector<recflex_schedule_t> candidates_for(const recflex_plan_s *p, int f, i
     const recflex_feature_spec_t &sp = p->specs[f];
     const FeatureDesc &d = p->desc[f];
     // the plan's current schedule is always candidate 0 (tie -> keep it)
-    out.push_back({d.sched, d.part, d.per_block});
+    out.push_back({d.sched, d.part, d.per_block, 0});
     const bool multi_hot = sp.max_len > 1.5f;
     auto add = [&](const recflex_schedule_t &s) {
         for (auto &o : out)
@@ -515,7 +523,7 @@ std::vector<recflex_schedule_t> candidates_for(const recflex_plan_s *p, int f, i
     for (int relax = 0; relax < 2 && out.size() <= 1; ++relax) {
         for (int id = 0; id < kCatalogSize; ++id) {
             const CatalogEntry &e = kCatalog[id];
-            recflex_schedule_t s = {id, 0, 1};
+            recflex_schedule_t s = {id, 0, 1, 0};
             s.per_block = samples_per_task_default(id, sp.mean_len, sp.coverage, p->task_lookups);
             if (!schedule_valid_for(s, d.dim, d.dtype, d.col, (int)p->d_tot)) continue;
             const int span = e.G * e.VEC * e.C;
@@ -523,7 +531,7 @@ std::vector<recflex_schedule_t> candidates_for(const recflex_plan_s *p, int f, i
             if (relax == 0 && (passes > 1 || e.C > 1)) continue;
             if (relax == 1 && passes > 2) continue;
             if (e.VEC == 1 && d.dim % 4 == 0) continue;  // scalar only where vectors cannot run
-            if (!multi_hot && (e.family == RECFLEX_FAMILY_BLOCK || e.family == RECFLEX_FAMILY_BULK)) continue;
+            if (!multi_hot && (e.family == RECFLEX_FAMILY_BLOCK)) continue;
             if (!multi_hot && e.family == RECFLEX_FAMILY_GROUP && e.U > 2) continue;  // one bag = one row
             add(s);
             if (multi_hot && e.family != RECFLEX_FAMILY_BLOCK) add({id, 1, std::max(128, p->task_lookups)});

@@ -140,6 +140,23 @@ class Plan:
             self._tables_key = key
         return self._tables_arr
 
+    # -------------------------------------------------------------- fusion compiler
+    def compile(self, occupancies: Optional[Sequence[int]] = None) -> dict:
+        """recflex_plan_compile: NVRTC-compile the plan-specialised fused kernel for the
+        current schedules (at the plan's occupancy, or each k given); returns jit_info."""
+        ks = [int(k) for k in occupancies] if occupancies else []
+        arr = (ctypes.c_int32 * max(1, len(ks)))(*ks) if ks else None
+        check(lib.recflex_plan_compile(self._h, arr, len(ks)), 'recflex_plan_compile')
+        return self.jit_info(ks[0] if len(ks) == 1 else 0)
+
+    def jit_info(self, k: int = 0) -> dict:
+        ji = _lib.JitInfo()
+        check(lib.recflex_jit_info(self._h, int(k), ctypes.byref(ji)), 'recflex_jit_info')
+        return {n: getattr(ji, n) for n, _ in _lib.JitInfo._fields_}
+
+    def set_jit(self, enable: bool) -> None:
+        check(lib.recflex_set_jit(self._h, 1 if enable else 0), 'recflex_set_jit')
+
     # -------------------------------------------------------------- hot path
     def forward(self, indices: torch.Tensor, offsets: torch.Tensor, B: int, tables: Sequence[torch.Tensor],
                 out: Optional[torch.Tensor] = None, stream=None) -> torch.Tensor:
@@ -169,6 +186,36 @@ class Plan:
         check(lib.recflex_forward_routed(self._h, idx_ptr, _dptr(offsets, torch.int32, 'offsets'), int(B), tarr, darr,
                                          len(dst_ptrs), int(rows_per_dst), int(dst_stride), int(col_base),
                                          _stream_ptr(stream)), 'recflex_forward_routed')
+
+    def forward_exchange(self, indices: torch.Tensor, offsets: torch.Tensor, B: int, tables: Sequence[torch.Tensor],
+                         world: int, rank: int, rows_per_dst: int, dst_stride: int, col_base: int,
+                         dst0: Sequence[int], dst1: Sequence[int], flags: Sequence[int], local_flags: int,
+                         stream=None) -> int:
+        """recflex_forward_exchange: routed forward into double-buffered destinations with a
+        device-side completion signal (no host barrier); returns the buffer index (0/1) this
+        step wrote -- see include/recflex.h for the lifetime rule."""
+        if offsets.numel() != self.F * B + 1:
+            raise ValueError('offsets must have F*B+1 entries')
+        tarr = self._tables(tables)
+        key = (tuple(dst0), tuple(dst1), tuple(flags))
+        if getattr(self, '_xkey', None) != key:
+            W = int(world)
+            self._xarrs = [(ctypes.c_void_p * W)(*[int(p) for p in dst0]), (ctypes.c_void_p * W)(*[int(p) for p in dst1]),
+                           (ctypes.c_void_p * W)(*[int(p) for p in flags])]
+            self._xkey = key
+        x = _lib.Exchange()
+        x.world, x.rank, x.rows_per_dst, x.dst_stride, x.col_base = (int(world), int(rank), int(rows_per_dst),
+                                                                      int(dst_stride), int(col_base))
+        x.dst[0] = ctypes.cast(self._xarrs[0], ctypes.c_void_p)
+        x.dst[1] = ctypes.cast(self._xarrs[1], ctypes.c_void_p)
+        x.flags = ctypes.cast(self._xarrs[2], ctypes.c_void_p)
+        x.local_flags = int(local_flags)
+        idx_ptr = _dptr(indices, torch.int32, 'indices') if indices.numel() else ctypes.c_void_p(offsets.data_ptr())
+        bi = ctypes.c_int32()
+        check(lib.recflex_forward_exchange(self._h, idx_ptr, _dptr(offsets, torch.int32, 'offsets'), int(B), tarr,
+                                           ctypes.byref(x), ctypes.byref(bi), _stream_ptr(stream)),
+              'recflex_forward_exchange')
+        return bi.value
 
     def forward_host(self, indices: torch.Tensor, offsets: torch.Tensor, B: int, tables: Sequence[torch.Tensor],
                      out: torch.Tensor, stream=None) -> torch.Tensor:
@@ -266,10 +313,11 @@ class Plan:
         s = _lib.Schedule()
         k = ctypes.c_int32()
         check(lib.recflex_get_schedule(self._h, f, ctypes.byref(s), ctypes.byref(k)), 'recflex_get_schedule')
-        return dict(sched_id=s.sched_id, part=s.part, per_block=s.per_block)
+        return dict(sched_id=s.sched_id, part=s.part, per_block=s.per_block, static_blocks=s.static_blocks)
 
-    def set_schedule(self, f: int, sched_id: int, part: int = 0, per_block: int = 256):
-        s = _lib.Schedule(int(sched_id), int(part), int(per_block))
+    def set_schedule(self, f: int, sched_id: int, part: int = 0, per_block: int = 256, static_blocks: int = 0):
+        """static_blocks > 0: the paper's static thread mapping with that many allocated tasks."""
+        s = _lib.Schedule(int(sched_id), int(part), int(per_block), int(static_blocks))
         check(lib.recflex_set_schedule(self._h, f, ctypes.byref(s)), 'recflex_set_schedule')
 
     @property
@@ -296,6 +344,19 @@ class Plan:
         check(lib.recflex_debug_task_map(self._h, _dptr(offsets, torch.int32, 'offsets'), int(B), bs, rg,
                                          max(2, 2 * total), _stream_ptr(stream)), 'recflex_debug_task_map')
         return list(bs), [(rg[2 * t], rg[2 * t + 1]) for t in range(total)]
+
+    def task_slots(self, f: int) -> int:
+        """recflex_get_task_slots: task-range slots reserved for feature f (reading C12)."""
+        v = ctypes.c_int32()
+        check(lib.recflex_get_task_slots(self._h, int(f), ctypes.byref(v)), 'recflex_get_task_slots')
+        return v.value
+
+    def debug_task_need(self) -> List[int]:
+        """recflex_debug_task_need: tasks every feature NEEDED in the last map (before a static
+        mapping folds them onto its allocated tasks)."""
+        nd = (ctypes.c_int32 * self.F)()
+        check(lib.recflex_debug_task_need(self._h, nd), 'recflex_debug_task_need')
+        return list(nd)
 
     def validate(self, indices: torch.Tensor, offsets: torch.Tensor, B: int, stream=None) -> int:
         """Returns the raw status (0 ok, 1 invalid offsets, 5 index out of range)."""
@@ -440,3 +501,32 @@ class KJTDist:
                                      _dptr(indices_out, torch.int32, 'indices_out') if indices_out.numel() else nul,
                                      _dptr(offsets_out, torch.int32, 'offsets_out'), _stream_ptr(stream)),
               'recflex_kjt_unpack')
+
+
+def jit_generate(sched_ids, dims, pools, k: int, dtypes=None):
+    """recflex_jit_generate (no GPU needed): (source, variant_of_feature, num_variants)."""
+    F = len(sched_ids)
+    A = ctypes.c_int32 * F
+    dt = A(*[dtype_code(d) for d in dtypes]) if dtypes is not None else None
+    n = ctypes.c_size_t()
+    nv = ctypes.c_int32()
+    var = A()
+    check(lib.recflex_jit_generate(A(*sched_ids), A(*dims), A(*pools), dt, F, int(k), None, 0, ctypes.byref(n),
+                                   var, ctypes.byref(nv)), 'recflex_jit_generate')
+    buf = ctypes.create_string_buffer(n.value + 1)
+    check(lib.recflex_jit_generate(A(*sched_ids), A(*dims), A(*pools), dt, F, int(k), buf, n.value + 1, None, None,
+                                   None), 'recflex_jit_generate')
+    return buf.value.decode(), list(var), nv.value
+
+
+def jit_compile_source(source: str):
+    """recflex_jit_compile_source (no GPU needed): (cubin bytes, NVRTC log, cache_hit)."""
+    n = ctypes.c_size_t()
+    log = ctypes.create_string_buffer(1 << 16)
+    hit = ctypes.c_int32()
+    check(lib.recflex_jit_compile_source(source.encode(), None, 0, ctypes.byref(n), log, 1 << 16, ctypes.byref(hit)),
+          'recflex_jit_compile_source')
+    buf = ctypes.create_string_buffer(n.value)
+    check(lib.recflex_jit_compile_source(source.encode(), buf, n.value, ctypes.byref(n), None, 0, None),
+          'recflex_jit_compile_source')
+    return buf.raw[:n.value], log.value.decode(errors='replace'), bool(hit.value)

@@ -25,6 +25,11 @@ from typing import List, Sequence
 import numpy as np
 
 
+def _nullcontext():
+    import contextlib
+    return contextlib.nullcontext()
+
+
 def row_bytes(dim: int, dtype: str = 'f32') -> int:
     """Bytes one lookup gathers: the stored row (int8: codes + scale + bias)."""
     return {'f32': 4 * dim, 'f16': 2 * dim, 'bf16': 2 * dim, 'i8': dim + 8, 'fp8': dim}[dtype]
@@ -289,8 +294,10 @@ class KJTInputDist:
         if self._send_idx.numel() < indices.numel():
             self._send_idx = torch.empty(indices.numel(), dtype=torch.int32, device=self.dev)
         self.kd.pack(indices, offsets, self.send_lengths, self._send_idx, self.dest_counts, stream=stream)
-        rl, ri, rc = exchange_kjt(self.send_lengths, self._send_idx, self.dest_counts, self.kd.send_length_counts,
-                                  self.kd.recv_length_counts, group)
+        # the collectives run on torch's current stream: make it the pack kernel's stream
+        with torch.cuda.stream(stream) if stream is not None else _nullcontext():
+            rl, ri, rc = exchange_kjt(self.send_lengths, self._send_idx, self.dest_counts,
+                                      self.kd.send_length_counts, self.kd.recv_length_counts, group)
         idx_out = torch.empty(sum(rc), dtype=torch.int32, device=self.dev)
         self.kd.unpack(rl, ri, idx_out, self.offsets_out, stream=stream)
         return idx_out, self.offsets_out
@@ -322,7 +329,9 @@ class ShardedEmbedding:
         out_local = self.plan.forward(indices, offsets, B, tables, out=out_local, stream=stream)
         if self.world == 1:
             return out_local
-        recv = exchange(out_local, self.dims_per_rank, B, group)
+        # the collective runs on torch's current stream: make it the kernel's stream
+        with torch.cuda.stream(stream) if stream is not None else _nullcontext():
+            recv = exchange(out_local, self.dims_per_rank, B, group)
         rows = B // self.world
         if out is None:
             out = torch.empty((rows, self.d_tot), dtype=torch.float32, device=out_local.device)
@@ -336,11 +345,19 @@ class FusedShardedEmbedding(ShardedEmbedding):
     each pooled row straight into the owning rank's final [B/W][D_tot] buffer
     through CUDA-IPC-mapped peer pointers (NVLink peer stores across GPUs of a
     node; plain stores when ranks share a device), so there is no separate
-    all-to-all pass and no relayout.  A collective barrier after the kernel
-    orders the destination's reads after every writer (stream-ordered
-    all_reduce on NCCL; host barrier on gloo)."""
+    all-to-all pass and no relayout (recflex_forward_exchange).
+
+    Per step there is no host or collective barrier: the destinations are
+    double-buffered (step n writes buffer n & 1 of every rank), the kernel's
+    last CTA publishes the step into every destination's flag array with a
+    system-scope release, and a one-warp wait kernel on this rank's stream
+    acquires all W flags before anything enqueued later runs.  The tensor
+    forward() returns is valid for work enqueued on the same stream before the
+    next-but-one forward() (include/recflex.h documents why); copy it to keep it
+    longer.  Setup (IPC handle exchange) uses the process group once."""
 
     def __init__(self, model, rank: int, world: int, device: int = 0, parts=None, group=None, dtype: str = 'f32'):
+        import torch
         import torch.distributed as dist
         from .plan import DeviceBuffer, ipc_handle, ipc_open
         super().__init__(model, rank, world, device, parts, dtype)
@@ -349,39 +366,44 @@ class FusedShardedEmbedding(ShardedEmbedding):
         self.group = group
         self.rows = model.batch // world
         self.col_base = sum(self.dims_per_rank[:rank])
-        self.buf = DeviceBuffer(self.rows, self.d_tot, device)
+        self.bufs = [DeviceBuffer(self.rows, self.d_tot, device) for _ in range(2)]
+        self.flags = DeviceBuffer(1, world, device)  # W uint32 (4-byte cells), zeroed below
+        self.flags.tensor.zero_()
+        torch.cuda.synchronize(device)
+        mine = (rank, [ipc_handle(b) for b in self.bufs], ipc_handle(self.flags))
         handles = [None] * world
-        dist.all_gather_object(handles, (rank, ipc_handle(self.buf)), group=group)
-        self.dst = [0] * world
+        dist.all_gather_object(handles, mine, group=group)
+        self.dst = [[0] * world, [0] * world]
+        self.flag_ptrs = [0] * world
         self._opened = []
-        for r, h in handles:
+        for r, bh, fh in handles:
             if r == rank:
-                self.dst[r] = self.buf.ptr.value
-            else:
-                p = ipc_open(h)
-                self.dst[r] = p
+                for b in range(2):
+                    self.dst[b][r] = self.bufs[b].ptr.value
+                self.flag_ptrs[r] = self.flags.ptr.value
+                continue
+            for b in range(2):
+                p = ipc_open(bh[b])
+                self.dst[b][r] = p
                 self._opened.append(p)
-        import torch
-        self._flag = torch.zeros(1, dtype=torch.float32, device=torch.device('cuda', device))
+            p = ipc_open(fh)
+            self.flag_ptrs[r] = p
+            self._opened.append(p)
+        dist.barrier(group=group)  # every rank's flags are zero before anyone's first step
 
     def forward(self, indices, offsets, B, tables, out_local=None, out=None, group=None, stream=None):
-        import torch
-        import torch.distributed as dist
         if B != self.model.batch:
             raise ValueError('the fused exchange buffers are sized for the model batch')
-        self.plan.forward_routed(indices, offsets, B, tables, self.dst, self.rows, self.d_tot, self.col_base,
-                                 stream=stream)
-        g = group if group is not None else self.group
-        if dist.get_backend(g) == 'nccl':
-            dist.all_reduce(self._flag, group=g)  # stream-ordered: every writer's kernel precedes it
-        else:
-            torch.cuda.current_stream().synchronize()
-            dist.barrier(group=g)
-        return self.buf.tensor
+        b = self.plan.forward_exchange(indices, offsets, B, tables, self.world, self.rank, self.rows, self.d_tot,
+                                       self.col_base, self.dst[0], self.dst[1], self.flag_ptrs, self.flags.ptr.value,
+                                       stream=stream)
+        return self.bufs[b].tensor
 
     def close(self):
         from .plan import ipc_close
         for p in self._opened:
             ipc_close(p)
         self._opened = []
-        self.buf.close()
+        for b in self.bufs:
+            b.close()
+        self.flags.close()

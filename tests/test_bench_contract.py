@@ -32,3 +32,36 @@ def test_reference_arm_json_line():
     assert cb['kind'] == 'oracle' and cb['cores'] >= 1 and cb['value'] == d['value'] and cb['sample']
     assert d['e2e']['h2d_bytes_per_step'] == 0 and d['e2e']['d2h_bytes_per_step'] == 0
     assert d['e2e']['value'] == d['value'] and d['e2e']['unit'] == d['unit']
+
+
+def _free_port():
+    import socket
+    s = socket.socket()
+    s.bind(('127.0.0.1', 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def test_reference_arm_under_torchrun_two_ranks():
+    """N > 1 launch (torchrun, 2 ranks, gloo on CPU): rank 0 alone prints one line
+    with n_gpus = 2 and the same workload config the GPU arm prints; rank 1 exits 0."""
+    cmd = [sys.executable, '-m', 'torch.distributed.run', '--nnodes=1', '--nproc-per-node', '2',
+           '--master-addr', '127.0.0.1', '--master-port', str(_free_port()), os.path.join(ROOT, 'bench.py'),
+           '--impl', 'reference', '--gpus', '2', '--config', 'tiny', '--steps', '2', '--warmup', '1',
+           '--ref-samples', '16']
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, cwd=ROOT)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith('{')]
+    assert len(lines) == 1, r.stdout
+    d = json.loads(lines[0])
+    assert d['n_gpus'] == 2 and d['impl'] == 'reference'
+    assert d['config']['parallelism'] == 'tablewise2'
+    sys.path.insert(0, ROOT)
+    import argparse
+
+    import bench
+    from paper_conf_sc_panzzxwslr0d24_b200 import synth
+    args = argparse.Namespace(config='tiny', dtype='f32', batches=3)
+    assert d['config'] == bench._workload_config(args, synth.make_model('tiny'), 2)
+    assert d['scaling'] == 'strong'

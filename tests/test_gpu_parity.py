@@ -102,15 +102,21 @@ def test_medium_full_int_and_float(name):
             check_tol(out, ref, lens, m.dims)
 
 
-def test_industrial_sampled():
+@pytest.mark.parametrize('mode', ['int', 'float'])
+def test_industrial_full_default_plan(mode):
+    """industrial (300 fields, SUM/MEAN mix) with the untuned plan: every one of the
+    4096 samples, integer tables bit-exact, U[-1,1) tables within tolerance.  (The tuned
+    plan is checked the same way in test_gpu_tuned_plans.)"""
+    from fullsize import sampled_oracle
     m = synth.make_model('industrial')
     b = synth.make_batch(m, 7)
-    case = Case(m, b, 'float')
+    case = Case(m, b, mode)
     _, out = run_plan(case)
-    rng = np.random.default_rng(0)
-    samples = np.unique(np.concatenate([[0, b.B - 1], rng.integers(0, b.B, 200)]))
-    ref, lens = case.oracle(samples)
-    check_tol(out[samples], ref, lens, m.dims)
+    ref, lens = sampled_oracle(m, b, np.arange(b.B), case.tables)
+    if mode == 'int':
+        assert bitexact(out, ref)
+    else:
+        check_tol(out, ref, lens, m.dims)
 
 
 @pytest.mark.parametrize('name', ['heavy', 'sharded1000'])
@@ -131,9 +137,10 @@ def test_full_size_sampled(name, plan_src, mode):
                             f'{name}_w1_r0.json')
         plan.import_(json.load(open(path)))
     _, out = run_plan(case, plan)
+    from fullsize import sampled_oracle
     rng = np.random.default_rng(1)
-    samples = np.unique(np.concatenate([[0, b.B - 1], rng.integers(0, b.B, 48)]))
-    ref, lens = case.oracle(samples)
+    samples = np.unique(np.concatenate([[0, b.B - 1], rng.choice(b.B, 1024, replace=False)]))
+    ref, lens = sampled_oracle(m, b, samples, case.tables)
     if mode == 'int':
         assert bitexact(out[samples], ref)
     else:
@@ -155,36 +162,74 @@ def _mixed_model():
     return synth.custom_model('mixed', feats, 301)
 
 
-@pytest.mark.parametrize('part', [0, 1, 2])
-def test_every_catalog_entry_int_bitexact(part):
+# per_block values per mapping: sample-partitioned (samples per task), lookup-
+# partitioned (lookups per task), static (part 0 with 7 samples per needed
+# task -> 43 needed tasks folded onto 3 or 17 allocated ones)
+_MAPPINGS = {'part0': [(0, 7, 0), (0, 64, 0)], 'part1': [(1, 5, 0), (1, 300, 0)],
+             'static': [(0, 7, 3), (1, 40, 17)]}
+
+
+def _every_entry(mapping, jit):
     P = _plan_mod()
     m = _mixed_model()
     b = synth.make_batch(m, 3)
     case = Case(m, b, 'int')
     ref, lens = case.oracle()
-    plan = P.Plan.from_model(m, max_batch=b.B)
     cat = P.catalog()
     col = np.cumsum([0] + m.dims)
     tested = 0
     for e in cat:
-        for per_block in {0: (7, 64), 1: (5, 300), 2: (3, 17)}[part]:
+        for part, per_block, nalloc in _MAPPINGS[mapping]:
+            plan = P.Plan.from_model(m, max_batch=b.B)
             used = []
             for f, feat in enumerate(m.features):
                 try:
-                    plan.set_schedule(f, e['id'], part, per_block)
+                    plan.set_schedule(f, e['id'], part, per_block, nalloc)
                     used.append(f)
                 except Exception:
                     pass  # entry not valid for this dim
             if not used:
                 continue
+            if jit:
+                info = plan.compile()
+                assert info['active'] == 1, info
             _, out = run_plan(case, plan)
             for f in used:
                 a, z = col[f], col[f + 1]
-                assert bitexact(out[:, a:z], ref[:, a:z]), (e, f, per_block)
+                assert bitexact(out[:, a:z], ref[:, a:z]), (e, f, part, per_block, nalloc, jit)
             tested += 1
-            # restore defaults for the next entry
-            plan = P.Plan.from_model(m, max_batch=b.B)
     assert tested >= 40
+
+
+@pytest.mark.parametrize('mapping', ['part0', 'part1'])
+def test_every_catalog_entry_int_bitexact(mapping):
+    """Every catalog entry in the precompiled catalog kernel, both runtime mappings."""
+    _every_entry(mapping, jit=False)
+
+
+@pytest.mark.parametrize('mapping', ['part0', 'part1', 'static'])
+def test_every_catalog_entry_jit_int_bitexact(mapping):
+    """Every catalog entry in a plan-specialised (NVRTC) kernel: both runtime
+    mappings and the paper's static mapping, integer tables, vs the oracle."""
+    _every_entry(mapping, jit=True)
+
+
+def test_static_mapping_needs_compiled_kernel():
+    """The static mapping (ablation straw man) is compiled only into plan-specialised
+    kernels: without recflex_plan_compile the forward refuses (no silent runtime mapping)."""
+    P = _plan_mod()
+    m = _mixed_model()
+    b = synth.make_batch(m, 3)
+    case = Case(m, b, 'int')
+    plan = P.Plan.from_model(m, max_batch=b.B)
+    s = plan.get_schedule(4)
+    plan.set_schedule(4, s['sched_id'], 0, 5, 2)
+    with pytest.raises(Exception):
+        run_plan(case, plan)
+    plan.compile()
+    _, out = run_plan(case, plan)
+    ref, _ = case.oracle()
+    assert bitexact(out, ref)
 
 
 @pytest.mark.parametrize('k', range(1, 9))
@@ -210,43 +255,61 @@ def test_occupancy_api_matches_k(k):
 
 # ---------------------------------------------------------------------------- thread map
 
-@pytest.mark.parametrize('seed', range(3))
+@pytest.mark.parametrize('seed', range(4))
 def test_task_map_bitexact_vs_oracle(seed):
+    _task_map_case(seed)
+
+
+def _task_map_case(seed):
+    """Device map kernel (+ fill kernel) vs the oracle's Fig. 8 task map: block
+    counts, needed counts, block_start, and lookup-partitioned task ranges --
+    incl. small per-task lookup counts that exceed the plan's reserved task slots
+    (the npb raise of reading C12) and static mappings."""
     P = _plan_mod()
     rng = np.random.default_rng(seed)
     m = _mixed_model()
     b = synth.make_batch(m, 11 + seed)
     plan = P.Plan.from_model(m, max_batch=b.B)
-    mode, pb = [], []
+    mode, pb, st, slots = [], [], [], []
     for f, feat in enumerate(m.features):
         s = plan.get_schedule(f)
         r = rng.random()
-        if r < 0.4:
+        nalloc = int(rng.integers(1, 40)) if rng.random() < 0.25 else 0
+        if r < 0.5:
             s['part'] = 1
-            # >= 128 lookups per task: within the plan's reserved task slots
-            # (max_batch * max_len / 128), so the map never raises npb (C12)
-            s['per_block'] = int(rng.integers(128, 700))
-        elif r < 0.6:
-            s['part'] = 2  # static mapping: fixed task count
-            s['per_block'] = int(rng.integers(1, 40))
+            # small windows force more tasks than the reserved slots hold for the
+            # long-bag features -> the map raises npb (C12)
+            s['per_block'] = int(rng.choice([1, 2, 3, 64, 128, 700]))
         else:
             s['part'] = 0
             s['per_block'] = int(rng.integers(1, 300))
-        plan.set_schedule(f, s['sched_id'], s['part'], s['per_block'])
+        plan.set_schedule(f, s['sched_id'], s['part'], s['per_block'], nalloc)
         mode.append(s['part'])
         pb.append(s['per_block'])
+        st.append(nalloc)
+        slots.append(plan.task_slots(f))
     off = torch.from_numpy(b.offsets).cuda()
     bs, ranges = plan.debug_task_map(off, b.B, ranges=True)
-    blocks, tf, tr = oracle.task_map(b.B, mode, pb, b.offsets)
+    need_gpu = plan.debug_task_need()
+    blocks, tf, tr, need, npb = oracle.task_map(b.B, mode, pb, b.offsets, slots=slots, static_blocks=st, full=True)
     exp_bs = oracle.block_start_from_task_map(m.F, tf)
     assert bs == exp_bs.tolist()
+    assert need_gpu == need.tolist()
+    raised = 0
     for f in range(m.F):
-        if mode[f] != 1:
+        if mode[f] != 1 or st[f] > 0:
             continue
-        s0, s1 = oracle.nnz_task_ranges(b.B, pb[f], b.offsets[f * b.B:(f + 1) * b.B + 1], int(blocks[f]))
+        raised += int(npb[f] > pb[f])
+        s0, s1 = oracle.nnz_task_ranges(b.B, int(npb[f]), b.offsets[f * b.B:(f + 1) * b.B + 1], int(blocks[f]))
         got = ranges[bs[f]:bs[f + 1]]
         assert [g[0] for g in got] == s0.tolist()
         assert [g[1] for g in got] == s1.tolist()
+    return raised
+
+
+def test_task_map_npb_raise_is_exercised():
+    """The slot-limited case of C12 actually occurs in the seeds above."""
+    assert sum(_task_map_case(s) for s in range(4)) > 0
 
 
 # ---------------------------------------------------------------------------- edge cases
@@ -424,9 +487,10 @@ def test_sharded1000_rank_plans_sampled():
     m = synth.make_model('sharded1000')
     b = synth.make_batch(m, 7)
     case = Case(m, b, 'int')
+    from fullsize import sampled_oracle
     rng = np.random.default_rng(2)
-    samples = np.unique(np.concatenate([[0, b.B - 1], rng.integers(0, b.B, 24)]))
-    ref, _ = case.oracle(samples)
+    samples = np.unique(np.concatenate([[0, b.B - 1], rng.choice(b.B, 1024, replace=False)]))
+    ref, _ = sampled_oracle(m, b, samples, case.tables)
     col = np.cumsum([0] + m.dims)
     dev = torch.device('cuda', 0)
     for W in (2, 4, 8):
@@ -434,6 +498,7 @@ def test_sharded1000_rank_plans_sampled():
         for r in range(W):
             sh = ShardedEmbedding(m, r, W, device=0, parts=parts)
             sh.plan.import_(json.load(open(os.path.join(tuned, f'sharded1000_w{W}_r{r}.json'))))
+            sh.plan.compile()  # the plan-specialised kernel bench.py runs
             idx, off = shard_batch(b, sh.features)
             out = sh.plan.forward(torch.from_numpy(idx).to(dev), torch.from_numpy(off).to(dev), b.B,
                                   [case.tables[f] for f in sh.features]).cpu().numpy()

@@ -2,8 +2,8 @@
 cuda:0, each runs its own fused plan over its features, the pooled outputs are
 exchanged (gloo, staged through host memory -- NCCL refuses two ranks on one
 device) and relayouted by the library's recflex_shard_concat kernel.  The
-result must equal the 1-GPU output restricted to the rank's samples, columns
-grouped by owning rank, bit for bit on integer-valued tables."""
+result must equal the ORACLE's output (fp64, integer-valued tables: bit for
+bit) restricted to the rank's samples, columns grouped by owning rank."""
 import os
 import socket
 
@@ -57,8 +57,18 @@ def _worker(rank, world, port, q):
         dist.destroy_process_group()
 
 
+def _oracle_full(seed=5):
+    """fp64 oracle output of the whole model and batch (integer-valued host tables)."""
+    import oracle
+    from paper_conf_sc_panzzxwslr0d24_b200 import synth
+    m = _model()
+    b = synth.make_batch(m, seed)
+    tabs = [synth.make_table(f.table, f.rows, f.dim, 'int').numpy() for f in m.features]
+    return m, b, oracle.embedding_bag(tabs, m.dims, [f.pool for f in m.features], b.indices, b.offsets, b.B)
+
+
 @pytest.mark.parametrize('world', [2, 3])
-def test_sharded_forward_matches_single_gpu(world):
+def test_sharded_forward_matches_oracle(world):
     from paper_conf_sc_panzzxwslr0d24_b200 import synth
     from paper_conf_sc_panzzxwslr0d24_b200.plan import Plan
     from paper_conf_sc_panzzxwslr0d24_b200.shard import column_order
@@ -72,17 +82,14 @@ def test_sharded_forward_matches_single_gpu(world):
     for p in procs:
         p.join(timeout=120)
         assert p.exitcode == 0
-    m = _model()
-    b = synth.make_batch(m, 5)
-    dev = torch.device('cuda', 0)
-    tables = [synth.make_table(f.table, f.rows, f.dim, 'int', device=dev) for f in m.features]
-    plan = Plan.from_model(m)
-    full = plan.forward(torch.from_numpy(b.indices).to(dev), torch.from_numpy(b.offsets).to(dev), b.B,
-                        tables).cpu().numpy()
+    m, b, full = _oracle_full()
     rows = b.B // world
     for rank, got, parts in res:
         order = column_order(m, parts)
-        assert np.array_equal(got, full[rank * rows:(rank + 1) * rows][:, order])
+        assert np.array_equal(got, full[rank * rows:(rank + 1) * rows][:, order].astype(np.float32))
+
+
+STEPS, SEEDS = 7, (5, 6, 8)
 
 
 def _worker_fused(rank, world, port, q):
@@ -95,19 +102,24 @@ def _worker_fused(rank, world, port, q):
     try:
         dev = torch.device('cuda', 0)
         m = _model()
-        b = synth.make_batch(m, 5)
         parts = partition_model(m, world)
         sh = FusedShardedEmbedding(m, rank, world, device=0, parts=parts)
         tables = [synth.make_table(m.features[f].table, m.features[f].rows, m.features[f].dim, 'int', device=dev)
                   for f in sh.features]
-        idx, off = shard_batch(b, sh.features)
-        res = []
-        for _ in range(2):  # twice: the routed pointer table is cached after the first call
-            out = sh.forward(torch.from_numpy(idx).to(dev), torch.from_numpy(off).to(dev), b.B, tables)
-            torch.cuda.synchronize()
-            res.append(out.cpu().numpy().copy())
-            dist.barrier()
-        q.put((rank, res, parts))
+        inputs = []
+        for sd in SEEDS:
+            idx, off = shard_batch(synth.make_batch(m, sd), sh.features)
+            inputs.append((torch.from_numpy(idx).to(dev), torch.from_numpy(off).to(dev)))
+        torch.cuda.synchronize()
+        # a step loop with NO host or collective barrier: double-buffered destinations and
+        # the device-side completion flags alone order writers and readers; each step's
+        # result is consumed (copied) on the same stream before the next-but-one step
+        outs = []
+        for i in range(STEPS):
+            o = sh.forward(*inputs[i % len(SEEDS)], m.batch, tables)
+            outs.append(o.clone())
+        torch.cuda.synchronize()
+        q.put((rank, [o.cpu().numpy() for o in outs], parts))
         dist.barrier()
         sh.close()
     finally:
@@ -115,11 +127,10 @@ def _worker_fused(rank, world, port, q):
 
 
 @pytest.mark.parametrize('world', [2, 3])
-def test_fused_exchange_matches_single_gpu(world):
+def test_fused_exchange_matches_oracle(world):
     """NEXT #1: the all-to-all folded into the fused kernel's store epilogue
-    (peer stores through CUDA-IPC-mapped buffers)."""
-    from paper_conf_sc_panzzxwslr0d24_b200 import synth
-    from paper_conf_sc_panzzxwslr0d24_b200.plan import Plan
+    (peer stores through CUDA-IPC-mapped buffers), over a barrier-free step loop
+    with changing batches: every step's received rows equal the oracle's."""
     from paper_conf_sc_panzzxwslr0d24_b200.shard import column_order
     ctx = mp.get_context('spawn')
     q = ctx.Queue()
@@ -127,18 +138,15 @@ def test_fused_exchange_matches_single_gpu(world):
     procs = [ctx.Process(target=_worker_fused, args=(r, world, port, q)) for r in range(world)]
     for p in procs:
         p.start()
-    res = [q.get(timeout=300) for _ in range(world)]
+    res = [q.get(timeout=600) for _ in range(world)]
     for p in procs:
         p.join(timeout=120)
         assert p.exitcode == 0
-    m = _model()
-    b = synth.make_batch(m, 5)
-    dev = torch.device('cuda', 0)
-    tables = [synth.make_table(f.table, f.rows, f.dim, 'int', device=dev) for f in m.features]
-    full = Plan.from_model(m).forward(torch.from_numpy(b.indices).to(dev), torch.from_numpy(b.offsets).to(dev), b.B,
-                                      tables).cpu().numpy()
-    rows = b.B // world
+    refs = {sd: _oracle_full(sd) for sd in SEEDS}
     for rank, outs, parts in res:
-        exp = full[rank * rows:(rank + 1) * rows][:, column_order(m, parts)]
-        for got in outs:
-            assert np.array_equal(got, exp)
+        assert len(outs) == STEPS
+        for i, got in enumerate(outs):
+            m, b, full = refs[SEEDS[i % len(SEEDS)]]
+            rows = b.B // world
+            exp = full[rank * rows:(rank + 1) * rows][:, column_order(m, parts)].astype(np.float32)
+            assert np.array_equal(got, exp), (rank, i)

@@ -244,18 +244,21 @@ def test_thread_count_does_not_change_result():
 
 # ---------------------------------------------------------------- task map (Fig. 8) pins
 
-def _brute_task_map(B, mode, pb, off, cap):
+def _brute_task_map(B, mode, pb, off, cap, slots, static):
     F = len(mode)
     tasks = []
     blocks = []
     for f in range(F):
         if mode[f] == 0:
             n = -(-B // pb[f])
-        elif mode[f] == 2:  # static mapping: fixed block count
-            n = pb[f]
         else:
             nnz = int(off[(f + 1) * B]) - int(off[f * B])
-            n = nnz // pb[f] + 1
+            npb = pb[f]
+            if slots[f] > 0:
+                npb = max(npb, -(-nnz // (slots[f] - 2)))
+            n = nnz // npb + 1
+        if static[f] > 0:  # static mapping: fixed allocated block count
+            n = static[f]
         if cap[f] > 0:
             n = min(n, cap[f])
         blocks.append(n)
@@ -269,15 +272,61 @@ def test_task_map_vs_brute_force(seed):
     F, B = int(rng.integers(1, 9)), int(rng.integers(1, 70))
     lens = rng.integers(0, 30, size=(F, B))
     b = synth.batch_from_lengths(lens, [100] * F, seed=seed)
-    mode = rng.integers(0, 3, size=F).tolist()
+    mode = rng.integers(0, 2, size=F).tolist()
     pb = [int(rng.integers(1, 40)) for _ in range(F)]
     cap = [int(rng.integers(0, 4)) if rng.random() < 0.3 else 0 for _ in range(F)]
-    blocks, tf, tr = oracle.task_map(B, mode, pb, b.offsets, cap)
-    eb, et = _brute_task_map(B, mode, pb, b.offsets, cap)
+    slots = [int(rng.integers(3, 12)) if rng.random() < 0.5 else 0 for _ in range(F)]
+    static = [int(rng.integers(1, 6)) if rng.random() < 0.3 else 0 for _ in range(F)]
+    blocks, tf, tr = oracle.task_map(B, mode, pb, b.offsets, cap, slots, static)
+    eb, et = _brute_task_map(B, mode, pb, b.offsets, cap, slots, static)
     assert blocks.tolist() == eb
     assert list(zip(tf.tolist(), tr.tolist())) == et
     bs = oracle.block_start_from_task_map(F, tf)
     assert bs[-1] == sum(eb) and np.all(np.diff(bs) == np.asarray(eb))
+
+
+def test_worked_static_mapping_p338():
+    """P:338 golden: 2 allocated blocks, 3 needed -> allocated block 0 performs needed
+    blocks 0 and 2 one after another, block 1 performs needed block 1."""
+    g = _gold()['task_map_p338_static']
+    off = np.zeros(g['B'] + 1, np.int32)
+    blocks, tf, tr, need, _ = oracle.task_map(g['B'], [0], [g['per_block']], off, static_blocks=[g['static_blocks']],
+                                              full=True)
+    assert need.tolist() == [g['need']] and blocks.tolist() == [g['blocks_map']]
+    assert tr.tolist() == list(range(g['blocks_map']))
+    alloc, seq = oracle.static_assignment(g['need'], g['static_blocks'])
+    assert alloc.tolist() == g['alloc_of'] and seq.tolist() == g['seq_of']
+    # the sample ranges each allocated block walks, in order
+    got = [[] for _ in range(g['blocks_map'])]
+    for q in sorted(range(g['need']), key=lambda q: (alloc[q], seq[q])):
+        got[alloc[q]].append([q * g['per_block'], min(g['B'], (q + 1) * g['per_block'])])
+    assert got == g['samples_of_allocated']
+
+
+def test_static_assignment_invariants():
+    for need in range(0, 20):
+        for nalloc in range(1, 8):
+            a, q = oracle.static_assignment(need, nalloc)
+            pairs = sorted(zip(a.tolist(), q.tolist()))
+            assert len(set(pairs)) == need                      # each needed block exactly once
+            for blk in range(nalloc):                            # each allocated block: steps 0, 1, 2, ...
+                steps = sorted(s for x, s in pairs if x == blk)
+                assert steps == list(range(len(steps)))
+            if need:
+                loads = np.bincount(a, minlength=nalloc)
+                assert loads.max() - loads.min() <= 1             # balanced round robin
+                assert loads.max() == -(-need // nalloc)
+
+
+def test_worked_nnz_partitioned_task_map():
+    """Hand-worked lookup-partitioned map incl. the npb raise for short task slots (C12)."""
+    g = _gold()['task_map_nnz_partitioned']
+    off = np.asarray(g['offsets'], np.int32)
+    for c in g['cases']:
+        blocks, tf, tr, need, npb = oracle.task_map(g['B'], [1], [c['per_block']], off, slots=[c['slots']], full=True)
+        assert npb.tolist() == [c['npb_eff']] and need.tolist() == [c['need']] and blocks.tolist() == [c['need']]
+        s0, s1 = oracle.nnz_task_ranges(g['B'], c['npb_eff'], off, c['need'])
+        assert [[a, b] for a, b in zip(s0.tolist(), s1.tolist())] == c['ranges']
 
 
 def test_nnz_task_ranges_partition():

@@ -61,11 +61,13 @@ def ablation_mapping(config, lines):
     plan = Plan.from_model(m, max_batch=tail_B)
     runtime = [plan.get_schedule(f) for f in range(m.F)]
     hist = [synth.make_batch(m, 100 + i, B=hist_B) for i in range(4)]
-    # blocks per feature under the runtime mapping on the historical batches
+    # tasks each feature needs under the runtime mapping on the historical batches
+    # ("we first run the runtime thread mapping kernels to collect the thread block
+    # usages")
     per_batch = []
     for hb in hist:
-        bs, _ = plan.debug_task_map(dev_batch(hb)[1], hist_B)
-        per_batch.append(np.diff(np.asarray(bs)))
+        plan.debug_task_map(dev_batch(hb)[1], hist_B)
+        per_batch.append(np.asarray(plan.debug_task_need()))
     per_batch = np.asarray(per_batch)
     static_avg = np.maximum(1, np.rint(per_batch.mean(axis=0))).astype(int)
     static_max = per_batch.max(axis=0).astype(int)
@@ -73,7 +75,9 @@ def ablation_mapping(config, lines):
              (f'long-tail request (B={tail_B}, P:340)', synth.make_batch(m, 8, B=tail_B), tail_B)]
     lines += [f'## Runtime vs static thread mapping ({config}, Fig. 13 / P:328-340)', '',
               'Static block counts per feature are the runtime mapping\'s counts averaged / maxed over 4 '
-              'historical batches of 512 samples; the schedules are identical, only the mapping differs.', '',
+              'historical batches of 512 samples; the schedules are identical, only the mapping differs. '
+              'Under the static mapping allocated block a performs the needed blocks a, a + n, a + 2n, ... '
+              'one after another (P:338, reading C31); every mode runs its plan-specialised kernel.', '',
               '| batch | runtime mapping (ms) | static avg (ms) | static max (ms) | slowdown avg | slowdown max |',
               '|---|---|---|---|---|---|']
     for label, b, B in tests:
@@ -82,10 +86,8 @@ def ablation_mapping(config, lines):
         for mode, counts in (('runtime', None), ('avg', static_avg), ('max', static_max)):
             for f in range(m.F):
                 s = runtime[f]
-                if counts is None:
-                    plan.set_schedule(f, s['sched_id'], s['part'], s['per_block'])
-                else:
-                    plan.set_schedule(f, s['sched_id'], 2, int(counts[f]))
+                plan.set_schedule(f, s['sched_id'], s['part'], s['per_block'], 0 if counts is None else int(counts[f]))
+            plan.compile()
             res[mode] = timer(plan, bd, B, tables, out, flush)
         lines.append(f"| {label} | {res['runtime']:.3f} | {res['avg']:.3f} | {res['max']:.3f} | "
                      f"{res['avg'] / res['runtime']:.2f}x | {res['max'] / res['runtime']:.2f}x |")
