@@ -569,6 +569,7 @@ def main():
 
     # the north-star target configuration (>= 70 % of HBM on the large multi-hot
     # model), timed in the same run at N = 1 (the headline stays the config above)
+    launch_desc = 'CUDA graph replay per step' if graphs else 'eager'
     heavy = None
     if world == 1 and args.config != 'heavy' and not args.no_heavy and not args.profile_only:
         del tables, phys, batches, graphs
@@ -597,7 +598,7 @@ def main():
             'impl_config': {'plan': plan_src, 'occupancy': plan.occupancy,
                             **({'dist_backend': backend} if world > 1 else {}),
                             'exchange': (args.exchange if world > 1 else 'none'),
-                            'launch': 'CUDA graph replay per step' if graphs else 'eager',
+                            'launch': launch_desc,
                             'kernel': (f"plan-specialised (NVRTC, {jit['variants']} variants, {jit['registers']} "
                                        f"regs, {jit['local_bytes']} B local)" if jit and jit['active'] else 'catalog'),
                             'input': ('data-parallel local batches + KJT input dist in the timed step'

@@ -212,13 +212,17 @@ typedef struct {
     int32_t verbose;         /* 1: print per-stage summaries to stderr                     */
     int32_t skip_guard;      /* 0: also time the incoming schedules at every k and keep
                                 them if faster than the two-stage result (K extra evals)   */
-    int32_t skip_refine;     /* 0: after selection, try every candidate per cluster of
+    int32_t refine;          /* 1: after selection, try every candidate per cluster of
                                 same-dim / same-length-class features in the real fused
-                                forward at the chosen k; keep if > 0.5% faster     */
+                                forward at the chosen k; keep if > 0.5% faster.
+                                Outside O(F*K + K); off by default, reported apart        */
     int32_t local_mode;      /* 0: interference-simulated co-execution with padding (the
                                 paper's method); 1: separate-combine straw man -- each
                                 candidate timed alone in a non-padded launch (P:73, P:324,
                                 for the Fig. 11 ablation)                                   */
+    int32_t stage2_catalog;  /* 0: stage 2 (and guard / refinement) time the plan-
+                                specialised kernel each choice compiles to (NVRTC, the
+                                kernel forwards run); 1: the precompiled catalog kernel   */
 } recflex_tune_options_t;
 
 typedef struct {
@@ -233,6 +237,11 @@ typedef struct {
     double tune_seconds;
     int64_t refine_evals;     /* cluster-refinement forwards timed                 */
     double refine_gain;       /* latency before refinement / after (>= 1)          */
+    double two_stage_ms;      /* stage-2 latency of the two-stage choice alone     */
+    double incoming_ms;       /* best guard latency of the incoming schedules      */
+    int64_t jit_compiles;     /* plan-specialised kernels compiled (or cache hits) */
+    double compile_seconds;   /* wall time spent compiling them                    */
+    double refine_seconds;    /* wall time of the refinement stage                 */
 } recflex_tune_stats_t;
 
 /* Two-stage interference-simulated tuning over num_batches historical batches

@@ -38,8 +38,8 @@ class CatalogInfo(ctypes.Structure):
 class TuneOptions(ctypes.Structure):
     _fields_ = [('num_occupancies', ctypes.c_int32), ('occupancies', ctypes.c_int32 * 8),
                 ('reps', ctypes.c_int32), ('pad_waves', ctypes.c_int32), ('max_candidates', ctypes.c_int32),
-                ('verbose', ctypes.c_int32), ('skip_guard', ctypes.c_int32), ('skip_refine', ctypes.c_int32),
-                ('local_mode', ctypes.c_int32)]
+                ('verbose', ctypes.c_int32), ('skip_guard', ctypes.c_int32), ('refine', ctypes.c_int32),
+                ('local_mode', ctypes.c_int32), ('stage2_catalog', ctypes.c_int32)]
 
 
 class TuneStats(ctypes.Structure):
@@ -47,7 +47,9 @@ class TuneStats(ctypes.Structure):
                 ('local_evals', ctypes.c_int64), ('global_evals', ctypes.c_int64),
                 ('guard_evals', ctypes.c_int64), ('guard_won', ctypes.c_int32),
                 ('best_occupancy', ctypes.c_int32), ('best_ms', ctypes.c_double), ('tune_seconds', ctypes.c_double),
-                ('refine_evals', ctypes.c_int64), ('refine_gain', ctypes.c_double)]
+                ('refine_evals', ctypes.c_int64), ('refine_gain', ctypes.c_double),
+                ('two_stage_ms', ctypes.c_double), ('incoming_ms', ctypes.c_double), ('jit_compiles', ctypes.c_int64),
+                ('compile_seconds', ctypes.c_double), ('refine_seconds', ctypes.c_double)]
 
 
 class JitInfo(ctypes.Structure):

@@ -58,7 +58,8 @@ constexpr int kStageSlots = 4;
 struct JitKernel {
     void *module = nullptr;    // CUmodule
     void *function = nullptr;  // CUfunction
-    int64_t version = -1;      // plan->sched_version it was generated from
+    uint64_t sig = 0;          // schedule signature it was generated from (jit_plan_sig)
+    int32_t *d_var = nullptr;  // device: variant id of every feature (this kernel's numbering)
     int variants = 0;
     int smem = 0, occ = 0, carveout = 0;
     int regs = 0, local_bytes = 0;
@@ -131,8 +132,9 @@ struct recflex_plan_s {
     // plan-specialised fused kernels (jit.cpp): used by forwards at occupancy k
     // while jit[k].version == sched_version (any schedule change bumps it)
     recflex::JitKernel jit[recflex::kMaxOcc + 1];
-    int32_t *jit_var = nullptr;  // device: variant id of every feature
     int64_t sched_version = 0;
+    int64_t sig_version = -1;    // sched_version the cached signature belongs to
+    uint64_t sig_cached = 0;
     int num_static = 0;          // features with a static thread mapping (P:338 ablation)
     bool use_jit = true;
 };
@@ -157,8 +159,9 @@ int find_catalog(int family, int G, int VEC, int C, int U, int ET = 0);
 int samples_per_task_default(int sched_id, float mean_len, float coverage, int target);
 int slots_for(int max_batch, float max_len);
 // plan-specialised fused kernel (jit.cpp)
-bool jit_ready(const recflex_plan_s *p, int k);
-int jit_launch(const recflex_plan_s *p, int k, const FusedArgs &a, bool pdl, cudaStream_t stream);
+bool jit_ready(recflex_plan_s *p, int k);
+uint64_t jit_plan_sig(recflex_plan_s *p);
+int jit_launch(recflex_plan_s *p, int k, const FusedArgs &a, bool pdl, cudaStream_t stream);
 recflex_status_t jit_compile_plan(recflex_plan_s *p, const int *ks, int nk);
 void jit_release(recflex_plan_s *p);
 

@@ -132,6 +132,9 @@ struct Tuner {
     int reps = 7;
     int pad_waves = 4;
     bool separate = false;  // local_mode 1: separate-combine straw man (ablation)
+    bool jit = true;            // stage 2 / guard / refinement time the plan-specialised kernel
+    int64_t jit_compiles = 0;
+    double compile_seconds = 0;
     int verbose = 0;
     std::vector<std::vector<recflex_schedule_t>> cands;  // per feature
     recflex_status_t err = RECFLEX_OK;
@@ -447,6 +450,17 @@ struct Tuner {
             fail(st);
             return 1e30;
         }
+        if (jit && !jit_ready(p, k)) {
+            // the kernel this choice compiles to is the one forwards will run
+            const auto t0 = std::chrono::steady_clock::now();
+            st = jit_compile_plan(p, &k, 1);
+            compile_seconds += std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+            ++jit_compiles;
+            if (st != RECFLEX_OK) {
+                fail(st);
+                return 1e30;
+            }
+        }
         double total = 0;
         for (const Batch &bt : batches) {
             check(d_out.ensure((int64_t)bt.B * p->d_tot));
@@ -568,6 +582,7 @@ extern "C" recflex_status_t recflex_tune_ex(recflex_plan_t p, int32_t N, const i
     if (opt && opt->pad_waves > 0) T.pad_waves = opt->pad_waves;
     if (opt) T.verbose = opt->verbose;
     if (opt) T.separate = opt->local_mode == 1;
+    if (opt) T.jit = opt->stage2_catalog == 0;
     const int max_c = opt ? opt->max_candidates : 0;
     for (int i = 0; i < N; ++i) {
         if (batch_sizes[i] <= 0 || batch_sizes[i] > p->max_batch || !indices[i] || !offsets[i])
@@ -620,12 +635,24 @@ extern "C" recflex_status_t recflex_tune_ex(recflex_plan_t p, int32_t N, const i
     // schedules (candidate 0 of every feature) at each k; keep whichever is
     // faster (an untuned-or-previous plan is never made slower by tuning).
     double best_ms = T.global_cost(best_k, choice.data());
+    const double two_stage_ms = best_ms;
+    double incoming_ms = 0;
     int64_t guard_evals = 0;
     if (!(opt && opt->skip_guard)) {
         std::vector<int32_t> zero(p->F, 0);
+        if (T.jit) {  // the incoming schedules at every k: one concurrent compile
+            T.apply(zero.data());
+            const auto t0 = std::chrono::steady_clock::now();
+            st = jit_compile_plan(p, T.ks.data(), (int)T.ks.size());
+            T.compile_seconds += std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+            T.jit_compiles += (int64_t)T.ks.size();
+            if (st != RECFLEX_OK) return st;
+        }
+        incoming_ms = std::numeric_limits<double>::infinity();
         for (int ki = 0; ki < (int)T.ks.size(); ++ki) {
             const double c0 = T.global_cost(ki, zero.data());
             ++guard_evals;
+            incoming_ms = std::min(incoming_ms, c0);
             if (c0 < best_ms) {
                 best_ms = c0;
                 best_k = ki;
@@ -643,7 +670,8 @@ extern "C" recflex_status_t recflex_tune_ex(recflex_plan_t p, int32_t N, const i
     // DRAM cost a schedule imposes on everyone else.
     int64_t refine_evals = 0;
     const double before_refine = best_ms;
-    if (!(opt && opt->skip_refine)) {
+    const auto t_refine = std::chrono::steady_clock::now();
+    if (opt && opt->refine) {
         std::vector<std::vector<int>> clusters;
         std::vector<long> keys;
         for (int f = 0; f < p->F; ++f) {
@@ -680,11 +708,21 @@ extern "C" recflex_status_t recflex_tune_ex(recflex_plan_t p, int32_t N, const i
             if (T.err != RECFLEX_OK) return T.err;
         }
     }
+    const double refine_seconds = std::chrono::duration<double>(std::chrono::steady_clock::now() - t_refine).count();
     T.apply(choice.data());
     p->k = T.ks[best_k];
     st = upload_desc(p, stream);
     if (st != RECFLEX_OK) return st;
+    if (T.jit && !jit_ready(p, p->k)) {  // leave the chosen kernel compiled (disk-cache hit)
+        st = jit_compile_plan(p, &p->k, 1);
+        if (st != RECFLEX_OK) return st;
+    }
     recflex_tune_stats_t s = {};
+    s.two_stage_ms = two_stage_ms;
+    s.incoming_ms = incoming_ms;
+    s.jit_compiles = T.jit_compiles;
+    s.compile_seconds = T.compile_seconds;
+    s.refine_seconds = refine_seconds;
     s.refine_evals = refine_evals;
     s.refine_gain = before_refine > 0 ? before_refine / best_ms : 1.0;
     s.local_launches = T.local_launches;

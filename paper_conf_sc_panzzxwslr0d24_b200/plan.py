@@ -282,7 +282,7 @@ class Plan:
     # -------------------------------------------------------------- tuner
     def tune(self, batches: Sequence[tuple], tables: Sequence[torch.Tensor], occupancies: Optional[List[int]] = None,
              reps: int = 7, pad_waves: int = 4, max_candidates: int = 0, verbose: bool = False, guard: bool = True,
-             refine: bool = True, separate: bool = False, stream=None) -> dict:
+             refine: bool = False, separate: bool = False, stage2_catalog: bool = False, stream=None) -> dict:
         """recflex_tune_ex over historical batches [(indices, offsets, B), ...]."""
         N = len(batches)
         idx_arr = (ctypes.c_void_p * N)(*[b[0].data_ptr() for b in batches])
@@ -298,15 +298,18 @@ class Plan:
         opt.max_candidates = max_candidates
         opt.verbose = 1 if verbose else 0
         opt.skip_guard = 0 if guard else 1
-        opt.skip_refine = 0 if refine else 1
+        opt.refine = 1 if refine else 0
         opt.local_mode = 1 if separate else 0
+        opt.stage2_catalog = 1 if stage2_catalog else 0
         st = _lib.TuneStats()
         check(lib.recflex_tune_ex(self._h, N, idx_arr, off_arr, bs_arr, self._tables(tables), _stream_ptr(stream),
                                   ctypes.byref(opt), ctypes.byref(st)), 'recflex_tune_ex')
         return dict(local_launches=st.local_launches, global_launches=st.global_launches,
                     local_evals=st.local_evals, global_evals=st.global_evals, guard_evals=st.guard_evals,
                     guard_won=bool(st.guard_won), refine_evals=st.refine_evals, refine_gain=st.refine_gain,
-                    best_occupancy=st.best_occupancy, best_ms=st.best_ms, tune_seconds=st.tune_seconds)
+                    best_occupancy=st.best_occupancy, best_ms=st.best_ms, tune_seconds=st.tune_seconds,
+                    two_stage_ms=st.two_stage_ms, incoming_ms=st.incoming_ms, jit_compiles=st.jit_compiles,
+                    compile_seconds=st.compile_seconds, refine_seconds=st.refine_seconds)
 
     # -------------------------------------------------------------- schedules
     def get_schedule(self, f: int) -> dict:

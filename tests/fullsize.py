@@ -31,7 +31,7 @@ def sampled_oracle(model, batch, samples, tables, dtype='f32', chunk=None):
     """fp64 oracle rows [len(samples)][D_tot] and bag lengths [len(samples)][F].
 
     tables[f]: the feature's stored table on the device (rows gathered per chunk of
-    samples; by default chunks hold ~256 MB of gathered rows)."""
+    samples; by default chunks hold ~1 GB of gathered rows)."""
     samples = np.asarray(samples, np.int64)
     F = batch.F
     if chunk is None:
@@ -39,7 +39,7 @@ def sampled_oracle(model, batch, samples, tables, dtype='f32', chunk=None):
         offs = batch.offsets.astype(np.int64)
         per_f = (offs[np.arange(1, F + 1) * batch.B] - offs[np.arange(F) * batch.B]) / max(1, batch.B)
         per_sample = float((per_f * row_b).sum()) + 1.0
-        chunk = int(max(16, min(samples.size, 256e6 / per_sample)))
+        chunk = int(max(16, min(samples.size, 1e9 / per_sample)))
     outs, lens_all = [], []
     for c0 in range(0, samples.size, chunk):
         sm = samples[c0:c0 + chunk]

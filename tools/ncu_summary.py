@@ -1,9 +1,12 @@
-"""Summarise an ncu --set full report of recflex_fused_kernel into profiles/.
+"""Summarise an ncu --set full report of the fused kernel into profiles/.
 
-    python tools/ncu_summary.py gpurun_out/prof_heavy.ncu-rep heavy r01 [--alg-bytes N]
+    python tools/ncu_summary.py gpurun_out/prof_heavy.ncu-rep heavy r02 [--dtype f32] [--suffix _w2_r0]
 
 Writes profiles/<tag>_ncu_<config>.md (human summary) and
-profiles/ncu_traffic_<config>.json (dram bytes per launch, read by bench.py).
+profiles/ncu_traffic_<config>[_dtype][suffix].json (dram bytes per launch, read
+by bench.py).  Algorithmic bytes (C26) and algorithmic ROW bytes are the mean
+over the bench's rotating batches (seeds 7, 8, 9); sector efficiency (SURVEY
+§8d) = algorithmic row bytes / (global-load sectors x 32).
 """
 import argparse
 import csv
@@ -61,11 +64,27 @@ def main():
     ap.add_argument('config')
     ap.add_argument('tag')
     ap.add_argument('--alg-bytes', type=float, default=None)
+    ap.add_argument('--dtype', default='f32')
+    ap.add_argument('--suffix', default='', help="e.g. '_w2_r0' for a rank plan")
     a = ap.parse_args()
+    row_bytes = None
+    if a.alg_bytes is None:
+        sys.path.insert(0, ROOT)
+        from paper_conf_sc_panzzxwslr0d24_b200 import synth
+        m = synth.make_model(a.config)
+        al, rb = [], []
+        for i in range(3):
+            ab = synth.algorithmic_bytes(m, synth.make_batch(m, 7 + i), a.dtype)
+            al.append(ab['total'])
+            rb.append(ab.get('rows', ab['total']))
+        a.alg_bytes = sum(al) / len(al)
+        row_bytes = sum(rb) / len(rb)
     hdr, units, launches = raw(a.rep)
     unit = dict(zip(hdr, units))
     os.makedirs(os.path.join(ROOT, 'profiles'), exist_ok=True)
-    lines = [f'# ncu --set full: recflex_fused_kernel, config `{a.config}` ({a.tag})', '',
+    L0 = launches[-1]
+    kname = L0.get('Kernel Name', 'recflex fused kernel')
+    lines = [f'# ncu --set full: `{kname}`, config `{a.config}` ({a.tag})', '',
              f'source: `{os.path.basename(a.rep)}` ({len(launches)} launch(es) profiled, '
              '`--clock-control none`, cold L2 per replay)', '']
     L = launches[-1]
@@ -93,9 +112,22 @@ def main():
     if a.alg_bytes:
         lines += ['', f'Algorithmic bytes per launch (C26): {a.alg_bytes / 1e9:.3f} GB; DRAM traffic '
                       f'{traffic / 1e9:.3f} GB = {traffic / a.alg_bytes:.3f}x algorithmic.']
+    sect = num(L.get('l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum'))
+    if row_bytes and sect:
+        sect *= {'sector': 1, 'Ksector': 1e3, 'Msector': 1e6, 'Gsector': 1e9}.get(
+            unit.get('l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum'), 1)
+        lines += [f'Sector efficiency (SURVEY §8d): algorithmic row bytes {row_bytes / 1e9:.3f} GB / '
+                  f'(global-load sectors x 32 = {sect * 32 / 1e9:.3f} GB) = {row_bytes / (sect * 32):.3f} '
+                  '(the global-load sectors also count the lookup-ID and offset loads).']
+        loc = num(L.get('l1tex__t_sectors_pipe_lsu_mem_local_op_ld.sum'))
+        if loc is not None:
+            loc *= {'sector': 1, 'Ksector': 1e3, 'Msector': 1e6, 'Gsector': 1e9}.get(
+                unit.get('l1tex__t_sectors_pipe_lsu_mem_local_op_ld.sum'), 1)
+            lines += [f'Local-memory (spill) load sectors / global-load sectors = {loc / sect:.4f}.']
     with open(os.path.join(ROOT, 'profiles', f'{a.tag}_ncu_{a.config}.md'), 'w') as fh:
         fh.write('\n'.join(lines) + '\n')
-    with open(os.path.join(ROOT, 'profiles', f'ncu_traffic_{a.config}.json'), 'w') as fh:
+    tname = f'ncu_traffic_{a.config}' + ('' if a.dtype == 'f32' else f'_{a.dtype}') + a.suffix + '.json'
+    with open(os.path.join(ROOT, 'profiles', tname), 'w') as fh:
         json.dump({'dram_bytes_per_launch': traffic, 'dram_read_bytes': rd_b, 'dram_write_bytes': wr_b,
                    'source': os.path.basename(a.rep), 'tag': a.tag}, fh, indent=1)
     print('\n'.join(lines))
