@@ -134,7 +134,9 @@ typedef struct {
 typedef enum {
     RECFLEX_FAMILY_GROUP = 0, /* G lanes per bag; 256/G bags in flight per CTA (G=32: warp per sample) */
     RECFLEX_FAMILY_BLOCK = 1, /* all 256 threads on one bag; smem partials + fixed-order reduction    */
-    RECFLEX_FAMILY_FLAT = 2   /* G lanes walk a run of 8 consecutive bags as one lookup range       */
+    RECFLEX_FAMILY_FLAT = 2,  /* G lanes walk a run of 8 consecutive bags as one lookup range       */
+    RECFLEX_FAMILY_WARP = 3   /* the 32/G lane groups of a warp share one bag (strided lookups,
+                                 xor-butterfly reduction): 32/G x U rows of a bag in flight        */
 } recflex_family_t;
 
 typedef struct {
@@ -422,10 +424,10 @@ recflex_status_t recflex_forward_routed(recflex_plan_t plan, const int32_t *indi
  *   local_flags   : this rank's own flag array (flags[rank] as seen locally)
  * Step n of this plan (n = 0, 1, ... counted per plan) writes buffer n & 1 of
  * every destination; *buffer_index receives n & 1 for the caller's own
- * buffer.  The fused kernel's last CTA publishes n + 1 into every
- * destination's flags[rank] with a system-scope release after all of the
- * step's pooled rows are stored; a one-warp wait kernel, enqueued after it on
- * `stream`, acquires flags[j] >= n + 1 for every writer j.  So work enqueued
+ * buffer.  A one-warp kernel enqueued right after the fused kernel on
+ * `stream` (so after every pooled row of the step is stored) publishes n + 1
+ * into every destination's flags[rank] with a system-scope release, then
+ * acquires flags[j] >= n + 1 for every writer j.  So work enqueued
  * on `stream` after this call sees the complete exchanged rows of step n.
  * Write-after-read safety: step n + 2 reuses buffer n & 1; a writer starts
  * step n + 2 only after its own wait of step n + 1, i.e. after every rank's

@@ -35,6 +35,9 @@ __device__ __forceinline__ void dispatch_chain(int id, const TaskCtx &x, float *
             if constexpr (e.family == RECFLEX_FAMILY_GROUP)
                 sched_group<e.ET, GT, e.VEC, e.C, e.U>(x.table, x.rowb, e.G, x.offs, x.idx, x.out, x.dim, x.pool, x.ro,
                                                         x.s0, x.s1, bag_ctr);
+            else if constexpr (e.family == RECFLEX_FAMILY_WARP)
+                sched_warp<e.ET, GT, e.VEC, e.C, e.U>(x.table, x.rowb, e.G, x.offs, x.idx, x.out, x.dim, x.pool, x.ro,
+                                                       x.s0, x.s1, bag_ctr);
             else if constexpr (e.family == RECFLEX_FAMILY_FLAT)
                 sched_flat<e.ET, GT, e.VEC, e.U>(x.table, x.rowb, e.G, x.offs, x.idx, x.out, x.dim, x.pool, x.ro, x.s0,
                                                   x.s1, bag_ctr);
@@ -269,6 +272,7 @@ __device__ __forceinline__ void fused_body(const FusedArgs &a) {
         ro.rows = a.route_rows;
         ro.colofs = a.col_base + fd.col;
         ro.stride = a.out_stride;
+#if defined(RECFLEX_JIT) && RECFLEX_JIT_STATIC
         // Static thread mapping (the paper's ablation straw man):
         // allocated task rel performs the needed tasks rel, rel + nalloc,
         // rel + 2*nalloc, ... one after another (reading C31); an allocated
@@ -284,32 +288,43 @@ __device__ __forceinline__ void fused_body(const FusedArgs &a) {
                 s0 = vld(&S.s0);
                 s1 = vld(&S.s1);
             }
-            if constexpr (BWD) {
-                sched_backward(a.grad + fd.col, a.out_stride, a.targets[f], a.offsets + (size_t)fd.in_feature * a.B,
-                               a.indices, fd.dim, fd.pool, a.bscale, s0, s1, &S.bag, a.bvec != 0);
-            } else {
-#ifdef RECFLEX_JIT
-                TaskCtx x;
-                x.table = static_cast<const char *>(fd.table);
-                x.offs = a.offsets + (size_t)fd.in_feature * a.B;
-                x.idx = a.indices;
-                x.out = a.out + fd.col;
-                x.ro = ro;
-                x.s0 = s0;
-                x.s1 = s1;
-                jit_dispatch(jv, x, red, &S.bag);
-#else
-                dispatch_task(fd.sched, static_cast<const char *>(fd.table), (unsigned)fd.row_bytes,
-                              a.offsets + (size_t)fd.in_feature * a.B, a.indices, a.out + fd.col, fd.dim, fd.pool, ro,
-                              s0, s1, red, &S.bag);
-#endif
-            }
+            TaskCtx x;
+            x.table = static_cast<const char *>(fd.table);
+            x.offs = a.offsets + (size_t)fd.in_feature * a.B;
+            x.idx = a.indices;
+            x.out = a.out + fd.col;
+            x.ro = ro;
+            x.s0 = s0;
+            x.s1 = s1;
+            jit_dispatch(jv, x, red, &S.bag);
             if (!stat) break;
             __syncthreads();           // every warp is done with needed task q
             if (tid == 0) S.bag = 0;   // fresh bag counter for the next one
             __syncthreads();
             q += fd.nalloc;
         }
+#else
+        if constexpr (BWD) {
+            sched_backward(a.grad + fd.col, a.out_stride, a.targets[f], a.offsets + (size_t)fd.in_feature * a.B,
+                           a.indices, fd.dim, fd.pool, a.bscale, vld(&S.s0), vld(&S.s1), &S.bag, a.bvec != 0);
+        } else {
+#ifdef RECFLEX_JIT
+            TaskCtx x;
+            x.table = static_cast<const char *>(fd.table);
+            x.offs = a.offsets + (size_t)fd.in_feature * a.B;
+            x.idx = a.indices;
+            x.out = a.out + fd.col;
+            x.ro = ro;
+            x.s0 = vld(&S.s0);
+            x.s1 = vld(&S.s1);
+            jit_dispatch(jv, x, red, &S.bag);
+#else
+            dispatch_task(fd.sched, static_cast<const char *>(fd.table), (unsigned)fd.row_bytes,
+                          a.offsets + (size_t)fd.in_feature * a.B, a.indices, a.out + fd.col, fd.dim, fd.pool, ro,
+                          vld(&S.s0), vld(&S.s1), red, &S.bag);
+#endif
+        }
+#endif
         if (cta_wide) __syncthreads();
         __syncwarp();
         if (lane == 0) {
@@ -319,31 +334,6 @@ __device__ __forceinline__ void fused_body(const FusedArgs &a) {
                 if (a.timers && t < a.timers_cap) a.timers[t] = (long long)(vld64(&S.wtime) / kWarps);
                 S.seq = -1;
                 st_release(&S.state, 0);
-            }
-        }
-    }
-    if constexpr (!BWD) {
-        if (a.route_flags) {
-            // Exchange completion (recflex_forward_exchange): every CTA makes its
-            // peer stores visible system-wide, then counts itself done; the last
-            // one bumps the epoch and publishes it into each destination's flag
-            // array with a system-scope release (the destination's wait kernel
-            // acquires it).  The fence -> atomic -> fence chain orders all CTAs'
-            // stores before the flag.
-            __syncthreads();
-            if (tid == 0) {
-                __threadfence_system();
-                if (atomicAdd(a.route_done, 1) == (int)gridDim.x - 1) {
-                    __threadfence_system();
-                    const int e = vld(a.route_epoch) + 1;
-                    vst(a.route_epoch, e);
-                    vst(a.route_done, 0);
-                    __threadfence_system();
-                    for (int j = 0; j < a.route_world; ++j)
-                        asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(a.route_flags[j] + a.route_rank),
-                                     "r"((unsigned)e)
-                                     : "memory");
-                }
             }
         }
     }

@@ -287,18 +287,36 @@ int concat_launch(const float *recv, int W, int rows, const int32_t *d_dims, con
     return (int)cudaGetLastError();
 }
 
-// Exchange wait (recflex_forward_exchange): lane j spins until writer j has
-// published this rank's current epoch (acquire at system scope), so work
-// ordered after this kernel on the stream sees every peer's pooled rows.  A
-// writer that never arrives (a dead peer) traps after ~60 s instead of hanging.
-__global__ void recflex_route_wait_kernel(const uint32_t *flags, const int32_t *epoch, int world) {
+// Exchange completion (recflex_forward_exchange), one warp launched right
+// after the fused kernel on the same stream: stream order puts every pooled
+// row the fused kernel stored (into local, NVLink-peer or IPC-mapped buffers)
+// before this kernel; lane 0 bumps the epoch, fences at system scope and
+// publishes it into every destination's flag array (slot `rank`) with a
+// system-scope release; then lane j spins until writer j has published this
+// step (acquire at system scope), so work ordered after this kernel sees every
+// peer's rows.  A writer that never arrives (a dead peer) traps after ~60 s.
+// (The signal lives in its own kernel, not in the fused kernel's epilogue: a
+// CTA barrier after the fused kernel's task loop changed how the compiler
+// reconverged the warp-decoupled loop and deadlocked warps on B200.)
+__global__ void recflex_route_signal_wait_kernel(uint32_t *const *flags, const uint32_t *local, int32_t *epoch,
+                                                 int rank, int world) {
+    __shared__ unsigned s_target;
     const int j = threadIdx.x;
+    if (j == 0) {
+        const unsigned e = (unsigned)*reinterpret_cast<volatile int32_t *>(epoch) + 1u;
+        *reinterpret_cast<volatile int32_t *>(epoch) = (int32_t)e;
+        __threadfence_system();
+        for (int r = 0; r < world; ++r)
+            asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(flags[r] + rank), "r"(e) : "memory");
+        s_target = e;
+    }
+    __syncthreads();
     if (j >= world) return;
-    const unsigned target = (unsigned)*reinterpret_cast<const volatile int32_t *>(epoch);
+    const unsigned target = s_target;
     unsigned long long t0 = 0, now;
     while (true) {
         unsigned v;
-        asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(flags + j) : "memory");
+        asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(local + j) : "memory");
         if ((int)(v - target) >= 0) break;
         __nanosleep(200);
         asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(now));
@@ -307,8 +325,10 @@ __global__ void recflex_route_wait_kernel(const uint32_t *flags, const int32_t *
     }
 }
 
-int route_wait_launch(const uint32_t *local_flags, const int32_t *epoch, int world, void *stream) {
-    recflex_route_wait_kernel<<<1, 32 * ((world + 31) / 32), 0, (cudaStream_t)stream>>>(local_flags, epoch, world);
+int route_signal_wait_launch(uint32_t *const *flags, const uint32_t *local_flags, int32_t *epoch, int rank, int world,
+                             void *stream) {
+    recflex_route_signal_wait_kernel<<<1, 32 * ((world + 31) / 32), 0, (cudaStream_t)stream>>>(flags, local_flags,
+                                                                                              epoch, rank, world);
     return (int)cudaGetLastError();
 }
 

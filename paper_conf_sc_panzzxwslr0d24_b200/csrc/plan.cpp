@@ -62,9 +62,9 @@ int row_bytes_of(int dim, int dtype) {
 int samples_per_task_default(int sched_id, float mean_len, float coverage, int target) {
     const CatalogEntry &e = kCatalog[sched_id];
     const int slots = (e.family == RECFLEX_FAMILY_GROUP) ? kBlockThreads / e.G
-                      : (e.family == RECFLEX_FAMILY_FLAT)
-                          ? (kBlockThreads / e.G) * 8
-                          : 1;
+                      : (e.family == RECFLEX_FAMILY_FLAT) ? (kBlockThreads / e.G) * 8
+                      : (e.family == RECFLEX_FAMILY_WARP) ? kBlockThreads / 32
+                                                          : 1;
     double el = std::max(0.25, (double)mean_len * std::max(0.05, (double)coverage));
     int R = (int)std::lround((double)target / (slots * el));
     R = std::min(32, std::max(1, R));
@@ -321,9 +321,6 @@ recflex_status_t run_pipeline(recflex_plan_s *p, const Exec &ex, const int32_t *
     a.route_rows = ex.route_rows;
     a.col_base = ex.col_base;
     a.route_epoch = ex.route_epoch;
-    a.route_done = ex.route_done;
-    a.route_flags = ex.route_flags;
-    a.route_rank = ex.route_rank;
     a.route_world = ex.route_world;
     a.grad = ex.grad;
     a.targets = ex.d_targets;
@@ -685,14 +682,11 @@ recflex_status_t recflex_forward_exchange(recflex_plan_t p, const int32_t *indic
     ex.route_rows = x->rows_per_dst;
     ex.col_base = x->col_base;
     ex.route_epoch = p->d_xcount;
-    ex.route_done = p->d_xcount + 1;
-    ex.route_flags = p->d_xflags;
-    ex.route_rank = x->rank;
     ex.route_world = W;
     st = run_pipeline(p, ex, indices, offsets, B, x->dst[0][0], x->dst_stride, p->k, stream, nullptr);
     if (st != RECFLEX_OK) return st;
-    int rc = route_wait_launch(x->local_flags, p->d_xcount, W, stream);
-    if (rc) return cuda_status_at((cudaError_t)rc, "exchange wait kernel launch");
+    int rc = route_signal_wait_launch(p->d_xflags, x->local_flags, p->d_xcount, x->rank, W, stream);
+    if (rc) return cuda_status_at((cudaError_t)rc, "exchange signal/wait kernel launch");
     if (buffer_index) *buffer_index = (int32_t)(p->x_steps & 1);
     ++p->x_steps;
     return RECFLEX_OK;

@@ -26,11 +26,9 @@ struct Exec {
     float *const *out_ptrs = nullptr;  // routed mode: device array of destination buffers
     int route_rows = 0;                // 0 = local output
     int col_base = 0;
-    // exchange mode (recflex_forward_exchange): double buffers + completion flags
+    // exchange mode (recflex_forward_exchange): double-buffered destinations
     int32_t *route_epoch = nullptr;
-    int32_t *route_done = nullptr;
-    uint32_t *const *route_flags = nullptr;
-    int route_rank = 0, route_world = 0;
+    int route_world = 0;
     // backward (NEXT #4)
     bool backward = false;
     const float *grad = nullptr;
@@ -125,7 +123,7 @@ struct recflex_plan_s {
     // recflex_forward_exchange state (device scratch + host caches)
     float **d_xroute = nullptr;       // 2 x W destination pointers
     uint32_t **d_xflags = nullptr;    // W flag-array pointers
-    int32_t *d_xcount = nullptr;      // [0] epoch (completed steps), [1] CTAs done in the launch
+    int32_t *d_xcount = nullptr;      // [0] epoch (completed exchange steps)
     std::vector<void *> xroute_cache;
     int64_t x_steps = 0;              // host mirror of the epoch (eager calls)
 

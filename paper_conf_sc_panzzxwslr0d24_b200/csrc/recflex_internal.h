@@ -86,13 +86,10 @@ struct FusedArgs {
     // plan-specialised (JIT-compiled) fused kernel: variant id of every feature
     const int32_t *jit_var;
     // exchange mode (recflex_forward_exchange): out_ptrs holds 2 x route_world
-    // destination pointers, buffer = *route_epoch & 1; the last CTA to finish
-    // bumps *route_epoch and publishes it into every destination's flag array
-    // (slot route_rank) with a system-scope release.  nullptr: plain routed mode.
+    // destination pointers, buffer = *route_epoch & 1 (the exchange kernel that
+    // follows the fused kernel bumps the epoch and signals).  nullptr: plain
+    // routed mode.
     int32_t *route_epoch;
-    int32_t *route_done;
-    uint32_t *const *route_flags;
-    int32_t route_rank;
     int32_t route_world;
 };
 
@@ -140,7 +137,7 @@ struct FusedArgs {
     X(2, 0, 16, 8, 1, 2) X(2, 0, 16, 8, 1, 4)                                  \
     RECFLEX_CATALOG_LOWP(X)
 #define RECFLEX_CATALOG_LOWP(X) RECFLEX_CATALOG_HALF(X, 1) RECFLEX_CATALOG_HALF(X, 2) RECFLEX_CATALOG_I8(X) \
-    RECFLEX_CATALOG_FP8(X) RECFLEX_CATALOG_HALF_U8(X, 1) RECFLEX_CATALOG_HALF_U8(X, 2)
+    RECFLEX_CATALOG_FP8(X) RECFLEX_CATALOG_HALF_U8(X, 1) RECFLEX_CATALOG_HALF_U8(X, 2) RECFLEX_CATALOG_WARP(X)
 
 // Reduced-precision rows, appended so the fp32 ids above
 // stay stable.  VEC counts ELEMENTS per lane per load: for 16-bit types
@@ -186,6 +183,15 @@ struct FusedArgs {
 // 32 lanes x 4 elements keep 4 accumulators per lane (cf. the FP8 entries).
 #define RECFLEX_CATALOG_HALF_U8(X, T) X(0, T, 16, 8, 1, 8) X(0, T, 32, 4, 1, 8) X(0, T, 8, 8, 1, 8)
 
+// WARP-SPLIT family (appended): the lane groups of one warp share a bag; NG*U
+// rows in flight per bag, NG = 32/G; R = NG*U divides 32.
+#define RECFLEX_CATALOG_WARP(X)                                                 \
+    X(3, 0, 1, 4, 1, 1)                                                         \
+    X(3, 0, 2, 4, 1, 2) X(3, 0, 2, 8, 1, 2)                                     \
+    X(3, 0, 4, 4, 1, 2) X(3, 0, 4, 4, 1, 4) X(3, 0, 4, 8, 1, 2) X(3, 0, 4, 8, 1, 4) \
+    X(3, 0, 8, 4, 1, 2) X(3, 0, 8, 4, 1, 4) X(3, 0, 8, 8, 1, 2) X(3, 0, 8, 8, 1, 4) \
+    X(3, 0, 16, 4, 1, 2) X(3, 0, 16, 4, 1, 4) X(3, 0, 16, 8, 1, 2) X(3, 0, 16, 8, 1, 4)
+
 struct CatalogEntry {
     int family, ET, G, VEC, C, U;
 };
@@ -228,6 +234,7 @@ int remap_launch(const int32_t *src, int32_t *dst, int64_t n, int64_t shift, int
 int concat_launch(const float *recv, int W, int rows, const int32_t *d_dims, const int32_t *d_cols, int d_tot,
                   float *out, void *stream);
 int flush_launch(void *buf, size_t bytes, void *stream);
-int route_wait_launch(const uint32_t *local_flags, const int32_t *epoch, int world, void *stream);
+int route_signal_wait_launch(uint32_t *const *flags, const uint32_t *local_flags, int32_t *epoch, int rank, int world,
+                             void *stream);
 
 }  // namespace recflex

@@ -492,6 +492,93 @@ RECFLEX_SCHED_FN void sched_group(const char *__restrict__ T, unsigned rowb, int
     }
 }
 
+// ---- WARP-SPLIT family -------------------------------------------------------
+// One bag at a time per WARP: its NG = 32/G lane groups share the bag, group g
+// taking lookups lo+g, lo+g+NG, ... (U rows each per iteration, so NG*U rows of
+// the bag are in flight at once instead of U), then the groups' partials are
+// combined with a fixed xor-butterfly (every lane gets bit-identical sums) and
+// group 0 stores.  For long bags in small batches, where the GROUP family's
+// per-bag chain of L/U dependent row round trips is the critical path (medium,
+// fig3).  IDs come through registers: lane l holds ID cb + l of the current
+// 32-ID chunk, the next chunk in flight; an iteration consumes R = NG*U IDs
+// (R divides 32 for every catalog entry).  Bags are claimed per warp from the
+// task's counter (results do not depend on which warp pools a bag).
+template <int ET, int GT, int VEC, int C, int U>
+RECFLEX_SCHED_FN void sched_warp(const char *__restrict__ T, unsigned rowb, int gr, const int32_t *__restrict__ offs,
+                                 const int32_t *__restrict__ idx, float *__restrict__ out, int d, int pool,
+                                 const OutRoute ro, int s0, int s1, int *bag_ctr) {
+    const int G = GT ? GT : gr;
+    const int NG = 32 / G;
+    const int R = NG * U;
+    const int lane = threadIdx.x & 31;
+    const int g = lane / G, lg = lane % G;
+    const int SPAN = G * VEC * C;
+    const int passes = (d + SPAN - 1) / SPAN;
+    while (true) {
+        int v = 0;
+        if (lane == 0) v = atomicAdd(bag_ctr, 1);
+        const int s = s0 + __shfl_sync(0xffffffffu, v, 0);
+        if (s >= s1) break;
+        const int lo = ld_idx(offs + s), hi = ld_idx(offs + s + 1);
+        float *__restrict__ orow = out_row(out, s, ro);
+        for (int p = 0; p < passes; ++p) {
+            int colv[C];
+            bool ok[C];
+#pragma unroll
+            for (int c = 0; c < C; ++c) {
+                colv[c] = p * SPAN + c * G * VEC + lg * VEC;
+                ok[c] = colv[c] < d;
+            }
+            float acc[C][VEC];
+#pragma unroll
+            for (int c = 0; c < C; ++c)
+#pragma unroll
+                for (int e = 0; e < VEC; ++e) acc[c][e] = 0.f;
+            int cb = lo;
+            int cur = (lo + lane < hi) ? ld_idx(idx + lo + lane) : 0;
+            int nxt = (lo + 32 + lane < hi) ? ld_idx(idx + lo + 32 + lane) : 0;
+            for (int j = lo; j < hi; j += R) {
+                if (j - cb >= 32) {
+                    cb += 32;
+                    cur = nxt;
+                    nxt = (cb + 32 + lane < hi) ? ld_idx(idx + cb + 32 + lane) : 0;
+                }
+                unsigned id[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u) id[u] = (unsigned)__shfl_sync(0xffffffffu, cur, (j - cb) + u * NG + g);
+                RowFrag<ET, VEC> rv[U][C];
+                rf_zero<ET, VEC, U, C>(rv);
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+#pragma unroll
+                    for (int c = 0; c < C; ++c)
+                        if (j + u * NG + g < hi && ok[c]) rv[u][c].load(T + (size_t)id[u] * rowb, colv[c], d);
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+                    if (j + u * NG + g < hi)
+#pragma unroll
+                        for (int c = 0; c < C; ++c)
+                            if (ok[c]) rv[u][c].add_to(acc[c]);
+            }
+            // the NG group partials -> one sum (fixed butterfly order)
+            for (int o = G; o < 32; o <<= 1)
+#pragma unroll
+                for (int c = 0; c < C; ++c)
+#pragma unroll
+                    for (int e = 0; e < VEC; ++e) acc[c][e] += __shfl_xor_sync(0xffffffffu, acc[c][e], o);
+            if (g == 0) {
+#pragma unroll
+                for (int c = 0; c < C; ++c) {
+                    if (ok[c]) {
+                        pool_finish<VEC>(acc[c], pool, hi - lo);
+                        st_out<VEC>(orow + colv[c], acc[c]);
+                    }
+                }
+            }
+        }
+    }
+}
+
 // ---- FLAT family -----------------------------------------------------------
 // A group claims a run of kFlatRun consecutive bags and walks their lookups as
 // one contiguous range (the KJT stores a run's bags back to back): every

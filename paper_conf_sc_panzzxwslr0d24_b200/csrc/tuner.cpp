@@ -26,6 +26,7 @@
 #include <chrono>
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <limits>
 #include <vector>
@@ -133,6 +134,7 @@ struct Tuner {
     int pad_waves = 4;
     bool separate = false;  // local_mode 1: separate-combine straw man (ablation)
     bool jit = true;            // stage 2 / guard / refinement time the plan-specialised kernel
+    bool trace = std::getenv("RECFLEX_TUNE_TRACE") != nullptr;
     int64_t jit_compiles = 0;
     double compile_seconds = 0;
     int verbose = 0;
@@ -167,6 +169,18 @@ struct Tuner {
     }
 
     void build_inputs(int f) {
+        const auto t_trace = std::chrono::steady_clock::now();
+        struct TraceEnd {
+            bool on;
+            int f;
+            std::chrono::steady_clock::time_point t0;
+            ~TraceEnd() {
+                if (on)
+                    std::fprintf(stderr, "[recflex tune] inputs f=%d %.1f ms\n", f,
+                                 std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0)
+                                     .count());
+            }
+        } trace_end{trace, f, t_trace};
         cur_f = f;
         tps.clear();
         tps.resize(batches.size());
@@ -308,6 +322,18 @@ struct Tuner {
         }
         const int k = ks[ki];
         const int n = (int)cands[f].size();
+        const auto t_trace = std::chrono::steady_clock::now();
+        struct TraceEnd {
+            bool on;
+            int k, f, n;
+            std::chrono::steady_clock::time_point t0;
+            ~TraceEnd() {
+                if (on)
+                    std::fprintf(stderr, "[recflex tune] local k=%d f=%d candidates=%d %.1f ms\n", k, f, n,
+                                 std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0)
+                                     .count());
+            }
+        } trace_end{trace, k, f, n, t_trace};
         std::vector<double> sum(n, 0.0);
         const FeatureDesc &base = p->desc[f];
         for (size_t i = 0; i < batches.size(); ++i) {
@@ -505,7 +531,7 @@ struct Tuner {
                 const int sid = (int)(key / 100000 / 2), part = (int)(key / 100000 % 2);
                 const CatalogEntry &e = kCatalog[sid];
                 std::fprintf(stderr, " %dx[%s G%d V%d C%d U%d p%d/%ld]", hist[i].second,
-                             e.family == 2 ? "flat" : (e.family ? "block" : "group"),
+                             e.family == 3 ? "warp" : e.family == 2 ? "flat" : (e.family ? "block" : "group"),
                              e.G, e.VEC, e.C, e.U, part, key % 100000);
             }
             std::fprintf(stderr, "\n");
@@ -545,7 +571,7 @@ std::vector<recflex_schedule_t> candidates_for(const recflex_plan_s *p, int f, i
             if (relax == 0 && (passes > 1 || e.C > 1)) continue;
             if (relax == 1 && passes > 2) continue;
             if (e.VEC == 1 && d.dim % 4 == 0) continue;  // scalar only where vectors cannot run
-            if (!multi_hot && (e.family == RECFLEX_FAMILY_BLOCK)) continue;
+            if (!multi_hot && (e.family == RECFLEX_FAMILY_BLOCK || e.family == RECFLEX_FAMILY_WARP)) continue;
             if (!multi_hot && e.family == RECFLEX_FAMILY_GROUP && e.U > 2) continue;  // one bag = one row
             add(s);
             if (multi_hot && e.family != RECFLEX_FAMILY_BLOCK) add({id, 1, std::max(128, p->task_lookups)});

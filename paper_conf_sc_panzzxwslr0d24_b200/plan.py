@@ -49,7 +49,7 @@ def catalog():
     for i in range(lib.recflex_catalog_size()):
         ci = _lib.CatalogInfo()
         check(lib.recflex_catalog_info(i, ctypes.byref(ci)), 'recflex_catalog_info')
-        out.append(dict(id=i, family=('group', 'block', 'flat', 'bulk')[ci.family], G=ci.group, VEC=ci.vec, C=ci.cols,
+        out.append(dict(id=i, family=('group', 'block', 'flat', 'warp')[ci.family], G=ci.group, VEC=ci.vec, C=ci.cols,
                         U=ci.unroll, dtype=DTYPE_NAMES[ci.dtype]))
     return out
 

@@ -54,13 +54,18 @@ def test_catalog_consistency():
         assert ci.group in (1, 2, 4, 8, 16, 32)
         # vec counts elements: fp32 4/16/32-byte loads, 16-bit 8/16/32-byte, int8 8/16-byte, fp8 8/16/32-byte
         assert ci.vec in {0: (1, 4, 8), 1: (4, 8, 16), 2: (4, 8, 16), 3: (8, 16), 4: (4, 8, 16, 32)}[ci.dtype]
-        # append-only catalog: every fp32 entry precedes every reduced-precision one
-        if ci.dtype == 0:
-            assert all(k[1] == 0 for k in seen)
         # an entry is valid only for its own storage type
         assert L.lib.recflex_catalog_valid_dtype(i, 128, ci.dtype) == 1
         assert all(L.lib.recflex_catalog_valid_dtype(i, 128, o) == 0 for o in range(5) if o != ci.dtype)
-    assert fams == {0, 1, 2}  # BULK (3) only in RECFLEX_EXPERIMENTAL_BULK builds
+    assert fams == {0, 1, 2, 3}
+    # append-only catalog: the ids the committed tuned plans name are unchanged
+    import json
+    import os
+    g = json.load(open(os.path.join(os.path.dirname(__file__), 'golden', 'catalog_r01.json')))['entries']
+    for i, e in enumerate(g):
+        ci = L.CatalogInfo()
+        L.lib.recflex_catalog_info(i, ctypes.byref(ci))
+        assert [ci.family, ci.dtype, ci.group, ci.vec, ci.cols, ci.unroll] == e, i
     assert L.lib.recflex_catalog_info(n, ctypes.byref(L.CatalogInfo())) != 0
     # every dim 1..256 has at least one valid fp32 entry; every dim % 4 == 0 a
     # 16-bit one, every dim % 8 == 0 an int8 one

@@ -507,3 +507,56 @@ def test_sharded1000_rank_plans_sampled():
             del sh, out
     del case
     torch.cuda.empty_cache()
+
+
+_FINE_TASKS = r'''
+import sys, numpy as np, torch
+sys.path.insert(0, sys.argv[1])
+import oracle
+from paper_conf_sc_panzzxwslr0d24_b200 import synth
+from paper_conf_sc_panzzxwslr0d24_b200.plan import Plan, catalog
+sys.path.insert(0, sys.argv[1] + '/tests')
+from fullsize import sampled_oracle
+jit = sys.argv[2] == 'jit'
+dev = torch.device('cuda', 0)
+m = synth.make_model('industrial')
+b = synth.make_batch(m, 7)
+phys = [synth.make_table(t, r, d, 'int', device=dev, seed=m.seed) for t, (r, d) in enumerate(m.tables)]
+tables = [phys[f.table] for f in m.features]
+bi, bo = torch.from_numpy(b.indices).to(dev), torch.from_numpy(b.offsets).to(dev)
+cat = catalog()
+plan = Plan.from_model(m)
+for f, ft in enumerate(m.features):
+    if ft.max_len() > 1.5:
+        fam = ('group', 'flat')[f % 2]
+        G = max(1, ft.dim // 4)
+        sid = [e['id'] for e in cat if (e['family'], e['G'], e['VEC'], e['C'], e['U'], e['dtype']) == (fam, G, 4, 1, 2, 'f32')][0]
+        plan.set_schedule(f, sid, 0, 8 if fam == 'group' else 64)
+for k in (4, 6):
+    plan.occupancy = k
+    if jit:
+        plan.compile()
+    for _ in range(3):
+        out = plan.forward(bi, bo, b.B, tables)
+    torch.cuda.synchronize()
+    S = np.arange(0, b.B, 7)
+    ref, _ = sampled_oracle(m, b, S, tables)
+    assert np.array_equal(out.cpu().numpy()[S], ref.astype(np.float32)), k
+print('ok')
+'''
+
+
+@pytest.mark.parametrize('kernel', ['catalog', 'jit'])
+def test_fine_grained_tasks_complete(kernel):
+    """Regression: thousands of tiny tasks (8 samples per GROUP task, short FLAT runs) on
+    industrial, in the catalog and the plan-specialised kernel, at k = 4 and 6.  A CTA
+    barrier after the warp-decoupled task loop once made the compiler reconverge the
+    loop so that a warp's lanes drifted into different tasks and deadlocked; this run
+    must finish (in a subprocess with a deadline) and match the oracle."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, '-c', _FINE_TASKS, root, kernel], capture_output=True, text=True,
+                       timeout=600)
+    assert r.returncode == 0 and r.stdout.strip().endswith('ok'), r.stderr[-2000:]

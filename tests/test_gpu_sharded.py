@@ -150,3 +150,31 @@ def test_fused_exchange_matches_oracle(world):
             rows = b.B // world
             exp = full[rank * rows:(rank + 1) * rows][:, column_order(m, parts)].astype(np.float32)
             assert np.array_equal(got, exp), (rank, i)
+
+
+def test_exchange_single_rank_protocol():
+    """recflex_forward_exchange with W = 1 in one process: the buffer index alternates
+    0, 1, 0, ...; each step's rows equal recflex_forward's; the rank's flag holds the
+    step count (the epoch the kernel's last CTA published)."""
+    from paper_conf_sc_panzzxwslr0d24_b200 import synth
+    from paper_conf_sc_panzzxwslr0d24_b200.plan import DeviceBuffer, Plan
+    dev = torch.device('cuda', 0)
+    m = _model()
+    plan = Plan.from_model(m)
+    tables = [synth.make_table(f.table, f.rows, f.dim, 'int', device=dev) for f in m.features]
+    bufs = [DeviceBuffer(m.batch, m.d_tot) for _ in range(2)]
+    flags = DeviceBuffer(1, 1)
+    flags.tensor.zero_()
+    for step in range(5):
+        b = synth.make_batch(m, 20 + step)
+        bi, bo = torch.from_numpy(b.indices).to(dev), torch.from_numpy(b.offsets).to(dev)
+        k = plan.forward_exchange(bi, bo, b.B, tables, 1, 0, b.B, m.d_tot, 0, [bufs[0].ptr.value],
+                                  [bufs[1].ptr.value], [flags.ptr.value], flags.ptr.value)
+        assert k == step % 2
+        got = bufs[k].tensor.clone()
+        ref = plan.forward(bi, bo, b.B, tables)
+        torch.cuda.synchronize()
+        assert torch.equal(got, ref)
+        assert int(flags.tensor.view(torch.int32)[0, 0].item()) == step + 1
+    for x in bufs + [flags]:
+        x.close()

@@ -23,8 +23,45 @@ phys = [synth.make_table(t, r, d, 'int', device=dev) for t, (r, d) in enumerate(
 tables = [phys[f.table] for f in m.features]
 bi, bo = torch.from_numpy(b.indices).to(dev), torch.from_numpy(b.offsets).to(dev)
 cat = catalog()
-fams = sys.argv[1:] or ['group', 'flat', 'block', 'bwd', 'kjt', 'host']
+fams = sys.argv[1:] or ['group', 'flat', 'block', 'warp', 'jit', 'static', 'exchange', 'bwd', 'kjt', 'host']
 for fam in fams:
+    if fam in ('jit', 'static'):
+        # plan-specialised kernels: every family in one compiled kernel, runtime or static mapping
+        plan = Plan.from_model(m)
+        by_fam = {}
+        for e in cat:
+            if e['dtype'] == 'f32':
+                by_fam.setdefault(e['family'], []).append(e['id'])
+        n = 0
+        for rnd in range(3):
+            for f in range(m.F):
+                fam_f = ('group', 'warp', 'flat', 'block')[(f + rnd) % 4]
+                for sid in by_fam[fam_f][rnd::3]:
+                    try:
+                        plan.set_schedule(f, sid, f % 2, 16 if f % 2 == 0 else 128, 3 if fam == 'static' else 0)
+                        break
+                    except Exception:
+                        pass
+            plan.compile()
+            plan.forward(bi, bo, b.B, tables)
+            n += 1
+        torch.cuda.synchronize()
+        print(fam, 'forwards', n)
+        continue
+    if fam == 'exchange':
+        # recflex_forward_exchange with one rank (its own buffers and flags): kernel epilogue
+        # flag publication + the wait kernel, several steps
+        from paper_conf_sc_panzzxwslr0d24_b200.plan import DeviceBuffer
+        plan = Plan.from_model(m)
+        bufs = [DeviceBuffer(b.B, m.d_tot) for _ in range(2)]
+        flags = DeviceBuffer(1, 1)
+        flags.tensor.zero_()
+        for i in range(4):
+            plan.forward_exchange(bi, bo, b.B, tables, 1, 0, b.B, m.d_tot, 0, [bufs[0].ptr.value],
+                                  [bufs[1].ptr.value], [flags.ptr.value], flags.ptr.value)
+        torch.cuda.synchronize()
+        print('exchange ok')
+        continue
     if fam == 'bwd':
         plan = Plan.from_model(m)
         grad = torch.randn((b.B, m.d_tot), device=dev)
