@@ -225,6 +225,10 @@ typedef struct {
     int32_t stage2_catalog;  /* 0: stage 2 (and guard / refinement) time the plan-
                                 specialised kernel each choice compiles to (NVRTC, the
                                 kernel forwards run); 1: the precompiled catalog kernel   */
+    int32_t no_tail;         /* 0: stage-1 cost = W_c / (#SM*k) + max(0, Lmax_c - T_est)
+                                (tail-aware, reading C33; T_est = measured latency of the
+                                incoming plan at k, K*N extra timed forwards); 1: the
+                                paper's plain sum of block times W_c (Eq. 3)              */
 } recflex_tune_options_t;
 
 typedef struct {

@@ -39,7 +39,7 @@ class TuneOptions(ctypes.Structure):
     _fields_ = [('num_occupancies', ctypes.c_int32), ('occupancies', ctypes.c_int32 * 8),
                 ('reps', ctypes.c_int32), ('pad_waves', ctypes.c_int32), ('max_candidates', ctypes.c_int32),
                 ('verbose', ctypes.c_int32), ('skip_guard', ctypes.c_int32), ('refine', ctypes.c_int32),
-                ('local_mode', ctypes.c_int32), ('stage2_catalog', ctypes.c_int32)]
+                ('local_mode', ctypes.c_int32), ('stage2_catalog', ctypes.c_int32), ('no_tail', ctypes.c_int32)]
 
 
 class TuneStats(ctypes.Structure):

@@ -134,6 +134,13 @@ struct Tuner {
     int pad_waves = 4;
     bool separate = false;  // local_mode 1: separate-combine straw man (ablation)
     bool jit = true;            // stage 2 / guard / refinement time the plan-specialised kernel
+    // Tail-aware stage-1 cost (reading C33): a candidate costs its
+    // CTA-time share W_c / (#SM * k) plus the part of its longest task that
+    // would outlast the whole kernel, max(0, Lmax_c - T_est), T_est = the
+    // measured latency of the incoming plan at k on the batch (cycles).
+    bool tail = true;
+    std::vector<std::vector<double>> t_est;  // [k index][batch] cycles
+    double clock_khz = 1.965e6;
     bool trace = std::getenv("RECFLEX_TUNE_TRACE") != nullptr;
     int64_t jit_compiles = 0;
     double compile_seconds = 0;
@@ -444,14 +451,57 @@ struct Tuner {
             check(cudaMemcpyAsync(bs.data(), d_bs.p, sizeof(int32_t) * (V + 1), cudaMemcpyDeviceToHost, stream));
             check(cudaStreamSynchronize(stream));
             if (err) return;
+            const double P = (double)p->num_sms * k;
+            const double T_est = (tail && ki < (int)t_est.size() && i < t_est[ki].size()) ? t_est[ki][i] : 0.0;
             for (int c = 0; c < n; ++c) {
                 const int v = cand_first + c;
-                double s = 0;
-                for (int64_t t = bs[v]; t < bs[v + 1]; ++t) s += (double)tm[t];
-                sum[c] += s;
+                double s = 0, mx = 0;
+                for (int64_t t = bs[v]; t < bs[v + 1]; ++t) {
+                    s += (double)tm[t];
+                    mx = std::max(mx, (double)tm[t]);
+                }
+                sum[c] += s / P + (T_est > 0 ? std::max(0.0, mx - T_est) : 0.0);
             }
         }
         for (int c = 0; c < n; ++c) costs[c] = sum[c];
+    }
+
+    // Latency of the plan's incoming schedules at occupancy ks[ki] on every batch
+    // (median of `reps` timed forwards after an L2 flush), in SM cycles.
+    void measure_incoming(int ki) {
+        const int k = ks[ki];
+        p->k = k;
+        recflex_status_t st = upload_desc(p, stream);
+        if (st != RECFLEX_OK) {
+            fail(st);
+            return;
+        }
+        if ((int)t_est.size() <= ki) t_est.resize(ki + 1);
+        t_est[ki].assign(batches.size(), 0.0);
+        for (size_t i = 0; i < batches.size(); ++i) {
+            const Batch &bt = batches[i];
+            check(d_out.ensure((int64_t)bt.B * p->d_tot));
+            if (err) return;
+            std::vector<float> ms;
+            for (int r = 0; r < std::max(3, reps / 2) + 1; ++r) {
+                int rc = flush_launch(d_flush.p, sizeof(float) * d_flush.cap, stream);
+                if (rc) fail(cuda_status((cudaError_t)rc));
+                check(cudaEventRecord(e0, stream));
+                st = run_pipeline(p, p->ex, bt.d_idx, bt.d_off, bt.B, d_out.p, (int)p->d_tot, k, stream, nullptr);
+                if (st != RECFLEX_OK) {
+                    fail(st);
+                    return;
+                }
+                check(cudaEventRecord(e1, stream));
+                check(cudaEventSynchronize(e1));
+                float t = 0;
+                cudaEventElapsedTime(&t, e0, e1);
+                ++global_launches;
+                if (r > 0) ms.push_back(t);
+            }
+            std::sort(ms.begin(), ms.end());
+            t_est[ki][i] = ms[ms.size() / 2] * clock_khz;  // ms x kHz = cycles
+        }
     }
 
     void apply(const int32_t *choice) {
@@ -643,6 +693,16 @@ extern "C" recflex_status_t recflex_tune_ex(recflex_plan_t p, int32_t N, const i
     if (T.d_flush.ensure(64 << 20) != cudaSuccess) return RECFLEX_ERR_OOM;  // 256 MB = 2x L2
     cudaEventCreate(&T.e0);
     cudaEventCreate(&T.e1);
+    if (opt && opt->no_tail) T.tail = false;
+    if (T.tail) {
+        int khz = 0;
+        if (cudaDeviceGetAttribute(&khz, cudaDevAttrClockRate, p->device) == cudaSuccess && khz > 0)
+            T.clock_khz = (double)khz;
+        const int k0 = p->k;
+        for (int ki = 0; ki < (int)T.ks.size(); ++ki) T.measure_incoming(ki);
+        p->k = k0;
+        if (T.err != RECFLEX_OK) return T.err;
+    }
     std::vector<int32_t> choice(p->F);
     int32_t best_k = 0;
     int64_t lc = 0, gc = 0;
