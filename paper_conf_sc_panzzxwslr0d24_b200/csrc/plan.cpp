@@ -275,6 +275,7 @@ recflex_status_t run_pipeline(recflex_plan_s *p, const Exec &ex, const int32_t *
     recflex_status_t st = prepare_occupancy(p, k);
     if (st != RECFLEX_OK) return st;
     if (ev) cudaEventRecord(ev->e0, stream);
+    NvtxRange nvtx_map("recflex pipeline (map, fill, fused)");
     MapArgs ma;
     ma.desc = ex.d_desc;
     ma.offsets = offsets;
@@ -566,6 +567,7 @@ struct DeviceGuard {
 
 recflex_status_t recflex_forward(recflex_plan_t p, const int32_t *indices, const int32_t *offsets, int32_t B,
                                  const void *const *tables, float *out, void *stream_) {
+    NvtxRange nvtx("recflex_forward");
     if (!p || !tables) return RECFLEX_ERR_INVALID_ARG;
     if (B < 0 || B > p->max_batch) return RECFLEX_ERR_INVALID_ARG;
     if (B == 0) return RECFLEX_OK;
@@ -596,6 +598,7 @@ recflex_status_t recflex_forward(recflex_plan_t p, const int32_t *indices, const
 recflex_status_t recflex_forward_routed(recflex_plan_t p, const int32_t *indices, const int32_t *offsets, int32_t B,
                                         const void *const *tables, float *const *host_dst, int32_t num_dst,
                                         int32_t rows_per_dst, int32_t dst_stride, int32_t col_base, void *stream_) {
+    NvtxRange nvtx("recflex_forward_routed");
     if (!p || !tables || !host_dst || num_dst <= 0 || num_dst > 1024 || rows_per_dst <= 0 || dst_stride <= 0 ||
         col_base < 0 || col_base + p->d_tot > dst_stride)
         return RECFLEX_ERR_INVALID_ARG;
@@ -633,6 +636,7 @@ recflex_status_t recflex_forward_routed(recflex_plan_t p, const int32_t *indices
 recflex_status_t recflex_forward_exchange(recflex_plan_t p, const int32_t *indices, const int32_t *offsets, int32_t B,
                                           const void *const *tables, const recflex_exchange_t *x,
                                           int32_t *buffer_index, void *stream_) {
+    NvtxRange nvtx("recflex_forward_exchange");
     if (!p || !tables || !x) return RECFLEX_ERR_INVALID_ARG;
     const int W = x->world;
     if (W <= 0 || W > 1024 || x->rank < 0 || x->rank >= W || x->rows_per_dst <= 0 || x->dst_stride <= 0 ||
@@ -694,6 +698,7 @@ recflex_status_t recflex_forward_exchange(recflex_plan_t p, const int32_t *indic
 
 recflex_status_t recflex_backward(recflex_plan_t p, const int32_t *indices, const int32_t *offsets, int32_t B,
                                   const float *grad, float *const *targets, float scale, void *stream_) {
+    NvtxRange nvtx("recflex_backward");
     if (!p || !targets || B < 0 || B > p->max_batch) return RECFLEX_ERR_INVALID_ARG;
     if (B == 0) return RECFLEX_OK;
     if (!indices || !offsets || !grad || ((uintptr_t)grad) % 16) return RECFLEX_ERR_INVALID_ARG;

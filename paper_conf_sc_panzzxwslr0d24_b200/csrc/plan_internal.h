@@ -1,6 +1,7 @@
 // plan_internal.h -- host-side plan state shared by plan.cpp and tuner.cpp.
 #pragma once
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include <string>
 #include <vector>
@@ -8,6 +9,13 @@
 #include "recflex_internal.h"
 
 namespace recflex {
+
+// NVTX range for the host-side timeline of an API call (header-only NVTX3: a
+// no-op unless a profiler injects itself, e.g. nsys / ncu --nvtx).
+struct NvtxRange {
+    explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+};
 
 // Device-side state one pipeline launch (map -> fill -> fused) reads.
 struct Exec {

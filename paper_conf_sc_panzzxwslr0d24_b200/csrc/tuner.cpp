@@ -637,6 +637,7 @@ extern "C" recflex_status_t recflex_tune_ex(recflex_plan_t p, int32_t N, const i
                                             const int32_t *const *offsets, const int32_t *batch_sizes,
                                             const void *const *tables, void *stream_,
                                             const recflex_tune_options_t *opt, recflex_tune_stats_t *stats) {
+    NvtxRange nvtx("recflex_tune");
     if (!p || N <= 0 || !indices || !offsets || !batch_sizes || !tables) return RECFLEX_ERR_INVALID_ARG;
     auto t_start = std::chrono::steady_clock::now();
     cudaStream_t stream = (cudaStream_t)stream_;

@@ -296,8 +296,10 @@ class KJTInputDist:
         self.kd.pack(indices, offsets, self.send_lengths, self._send_idx, self.dest_counts, stream=stream)
         # the collectives run on torch's current stream: make it the pack kernel's stream
         with torch.cuda.stream(stream) if stream is not None else _nullcontext():
+            torch.cuda.nvtx.range_push('recflex KJT all-to-all')
             rl, ri, rc = exchange_kjt(self.send_lengths, self._send_idx, self.dest_counts,
                                       self.kd.send_length_counts, self.kd.recv_length_counts, group)
+            torch.cuda.nvtx.range_pop()
         idx_out = torch.empty(sum(rc), dtype=torch.int32, device=self.dev)
         self.kd.unpack(rl, ri, idx_out, self.offsets_out, stream=stream)
         return idx_out, self.offsets_out
@@ -331,7 +333,9 @@ class ShardedEmbedding:
             return out_local
         # the collective runs on torch's current stream: make it the kernel's stream
         with torch.cuda.stream(stream) if stream is not None else _nullcontext():
+            torch.cuda.nvtx.range_push('recflex pooled-output all-to-all')
             recv = exchange(out_local, self.dims_per_rank, B, group)
+            torch.cuda.nvtx.range_pop()
         rows = B // self.world
         if out is None:
             out = torch.empty((rows, self.d_tot), dtype=torch.float32, device=out_local.device)

@@ -26,7 +26,9 @@ Layout produced (KJT feature-major CSR):
 from __future__ import annotations
 
 import dataclasses
+import json
 import math
+import os
 from typing import List, Optional
 
 import numpy as np
@@ -103,75 +105,85 @@ def _log_uniform(rng, lo, hi, size=None):
     return np.exp(rng.uniform(math.log(lo), math.log(hi), size=size))
 
 
-def make_model(name: str, seed: int = MODEL_SEED) -> Model:
+MODEL_DIR = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), 'configs', 'models')
+
+
+def _draw(rng, spec):
+    """A scalar from a recipe spec: {"fixed": v} | {"uniform": [a, b]} | {"log_uniform": [a, b]}."""
+    if 'fixed' in spec:
+        return spec['fixed']
+    if 'uniform' in spec:
+        return float(rng.uniform(*spec['uniform']))
+    if 'log_uniform' in spec:
+        return float(_log_uniform(rng, *spec['log_uniform']))
+    raise ValueError(f'bad spec {spec}')
+
+
+def load_recipe(name: str) -> dict:
+    path = os.path.join(MODEL_DIR, f'{name}.json')
+    if not os.path.exists(path):
+        raise ValueError(f'unknown model {name!r} (no {path})')
+    with open(path) as fh:
+        return json.load(fh)
+
+
+def make_model(name: str, seed: int = MODEL_SEED, recipe: Optional[dict] = None) -> Model:
+    """The synthetic model of a BASELINE config from its recipe configs/models/<name>.json
+    (SURVEY §8d).  Draws, per field in order: the dim (if chosen at random), the rows (if
+    log-uniform), then the coverage (one-hot) or the mean length and the coverage
+    (multi-hot); the one-hot set is a random permutation prefix drawn first when the
+    recipe says so.  tests/golden/models_r02.json pins the result."""
+    r = recipe if recipe is not None else load_recipe(name)
     rng = np.random.Generator(np.random.PCG64([seed, _name_key(name)]))
     feats: List[Feature] = []
-    if name == 'tiny':
-        # 4 fields (2 one-hot, 2 multi-hot L<=8 incl. empty bags), 1k rows, dim 16, sum, B=64
-        for f in range(4):
-            if f < 2:
-                feats.append(Feature(rows=1000, dim=16, pool=POOL_SUM, kind='onehot', coverage=1.0, lmax=1, table=f))
+    if 'explicit' in r:
+        feats = [Feature(**f) for f in r['explicit']]
+        B = int(r['batch'])
+    else:
+        F = int(r['fields'])
+        oh = r['onehot']
+        if oh['rule'] == 'random':
+            onehot = set(rng.permutation(F)[:oh['count']].tolist())
+        elif oh['rule'] == 'even':
+            onehot = set(range(0, F, 2))
+        elif oh['rule'] == 'first':
+            onehot = set(range(oh['count']))
+        else:
+            onehot = set()
+        mh = r.get('multihot', {})
+        for f in range(F):
+            ds = r['dim']
+            if 'choice' in ds:
+                dim = int(rng.choice(ds['choice'], p=ds['p']))
+            elif 'cycle' in ds:
+                dim = int(ds['cycle'][f % len(ds['cycle'])])
             else:
-                feats.append(Feature(rows=1000, dim=16, pool=POOL_SUM, kind='uniform', lo=0, hi=8, lmax=8, table=f))
-        B = 64
-    elif name == 'medium':
-        # 50 fields alternating one-hot / multi-hot, dims cycle 16/32/64, 1M rows, sum, B=1024
-        for f in range(50):
-            dim = (16, 32, 64)[f % 3]
-            if f % 2 == 0:
-                feats.append(Feature(rows=1_000_000, dim=dim, pool=POOL_SUM, kind='onehot',
-                                     coverage=float(rng.uniform(0.9, 1.0)), lmax=1, table=f))
-            else:
-                mu = float(rng.uniform(5, 50))
-                feats.append(Feature(rows=1_000_000, dim=dim, pool=POOL_SUM, kind='normal', mu=mu, sigma=mu / 4,
-                                     coverage=float(rng.uniform(0.3, 1.0)), lmax=int(round(3 * mu)), table=f))
-        B = 1024
-    elif name == 'industrial':
-        # 300 fields (120 one-hot / 180 multi-hot), skewed lognormal lengths 1..200,
-        # dims {8,16,32,64,128} p=.3/.3/.2/.1/.1, rows log-uniform [1e4, 2e6], even f sum / odd f mean
-        onehot = set(rng.permutation(300)[:120].tolist())
-        for f in range(300):
-            dim = int(rng.choice([8, 16, 32, 64, 128], p=[.3, .3, .2, .1, .1]))
-            rows = int(_log_uniform(rng, 1e4, 2e6))
-            pool = POOL_SUM if f % 2 == 0 else POOL_MEAN
+                dim = int(ds['fixed'])
+            rows = int(_draw(rng, r['rows']))
+            pool = {'sum': POOL_SUM, 'mean': POOL_MEAN}.get(r['pool'])
+            if pool is None:  # even_sum_odd_mean
+                pool = POOL_SUM if f % 2 == 0 else POOL_MEAN
+            tspec = r.get('tables', 'per_field')
+            table = f % int(tspec['alias_mod']) if isinstance(tspec, dict) else f
             if f in onehot:
                 feats.append(Feature(rows=rows, dim=dim, pool=pool, kind='onehot',
-                                     coverage=float(rng.uniform(0.5, 1.0)), lmax=1, table=f))
+                                     coverage=float(_draw(rng, r['onehot_coverage'])), lmax=1, table=table))
+            elif mh['kind'] == 'uniform':
+                feats.append(Feature(rows=rows, dim=dim, pool=pool, kind='uniform', lo=int(mh['lo']), hi=int(mh['hi']),
+                                     lmax=int(mh['hi']), table=table))
             else:
-                mu = float(_log_uniform(rng, 2, 200))
-                feats.append(Feature(rows=rows, dim=dim, pool=pool, kind='lognormal', mu=mu, sigma=0.9,
-                                     coverage=float(rng.uniform(0.3, 1.0)), lmax=200, table=f))
-        B = 4096
-    elif name == 'heavy':
-        # 100 multi-hot fields, lognormal mean 100 sigma .9 clipped [1,1000], coverage 1, dim 128,
-        # 10M-row index ranges aliased onto 16 physical tables (C25), sum, B=8192
-        for f in range(100):
-            feats.append(Feature(rows=10_000_000, dim=128, pool=POOL_SUM, kind='lognormal', mu=100.0, sigma=0.9,
-                                 coverage=1.0, lmax=1000, table=f % 16))
-        B = 8192
-    elif name == 'sharded1000':
-        # model-A-shaped 1000 fields (500/500), dims {4..128}, rows log-uniform [1e4, 1e6], sum, B=16384
-        onehot = set(rng.permutation(1000)[:500].tolist())
-        for f in range(1000):
-            dim = int(rng.choice([4, 8, 16, 32, 64, 128], p=[.1, .25, .25, .2, .1, .1]))
-            rows = int(_log_uniform(rng, 1e4, 1e6))
-            if f in onehot:
-                feats.append(Feature(rows=rows, dim=dim, pool=POOL_SUM, kind='onehot',
-                                     coverage=float(rng.uniform(0.5, 1.0)), lmax=1, table=f))
-            else:
-                mu = float(_log_uniform(rng, 2, 100))
-                feats.append(Feature(rows=rows, dim=dim, pool=POOL_SUM, kind='normal', mu=mu, sigma=mu / 4,
-                                     coverage=float(rng.uniform(0.3, 1.0)), lmax=max(1, int(round(3 * mu))),
-                                     table=f))
-        B = 16384
-    elif name == 'fig3':
-        # Fig. 3: two dim-32 fields; f0 N(50,10^2) at coverage 0.3, f1 fixed 50
-        feats.append(Feature(rows=1_000_000, dim=32, pool=POOL_SUM, kind='normal', mu=50, sigma=10,
-                             coverage=0.3, lmax=100, table=0))
-        feats.append(Feature(rows=1_000_000, dim=32, pool=POOL_SUM, kind='fixed', mu=50, lmax=50, table=1))
-        B = 512
-    else:
-        raise ValueError(f'unknown model {name!r}')
+                mu = _draw(rng, mh['mu'])
+                sigma = mu * mh['sigma_over_mu'] if 'sigma_over_mu' in mh else float(mh['sigma'])
+                cov = float(_draw(rng, mh['coverage']))
+                if 'lmax_over_mu' in mh:
+                    lmax = int(round(mh['lmax_over_mu'] * mu))
+                    if 'lmax_min' in mh:
+                        lmax = max(int(mh['lmax_min']), lmax)
+                else:
+                    lmax = int(mh['lmax'])
+                feats.append(Feature(rows=rows, dim=dim, pool=pool, kind=mh['kind'], mu=mu, sigma=sigma, coverage=cov,
+                                     lmax=lmax, table=table))
+        B = int(r['batch'])
     ntab = max(f.table for f in feats) + 1
     tables = [None] * ntab
     for f in feats:

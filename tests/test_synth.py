@@ -107,3 +107,25 @@ def test_oracle_and_product_do_not_import_each_other():
             src = open(os.path.join(ROOT, 'oracle', fn)).read()
             assert 'csrc' not in src and 'recflex.h' not in src, fn
             assert not re.search(r'paper_conf_sc_panzzxwslr0d24_b200\.(_lib|plan|shard)', src), fn
+
+
+def test_models_from_recipes_match_golden():
+    """configs/models/<name>.json recipes reproduce the models the tuned plans were made for."""
+    import dataclasses
+    import json
+    import os
+    g = json.load(open(os.path.join(os.path.dirname(__file__), 'golden', 'models_r02.json')))['models']
+    for n in synth.CONFIG_NAMES:
+        m = synth.make_model(n)
+        assert m.batch == g[n]['batch'], n
+        assert [list(t) for t in m.tables] == g[n]['tables'], n
+        assert [list(dataclasses.astuple(f)) for f in m.features] == g[n]['features'], n
+
+
+def test_recipe_variant_changes_model():
+    """A recipe is data: changing it changes the model (no hidden hard-coded config)."""
+    r = synth.load_recipe('medium')
+    r['batch'] = 256
+    r['dim'] = {'cycle': [8]}
+    m = synth.make_model('medium', recipe=r)
+    assert m.batch == 256 and set(m.dims) == {8} and m.F == 50
