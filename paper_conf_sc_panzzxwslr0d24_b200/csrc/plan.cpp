@@ -83,7 +83,7 @@ int task_lookups_target(const recflex_feature_spec_t *specs, int F, int max_batc
     return (int)std::min(4096.0, std::max(256.0, t));
 }
 
-recflex_schedule_t default_schedule(const recflex_feature_spec_t &spec, int target) {
+recflex_schedule_t default_schedule(const recflex_feature_spec_t &spec, int target, bool small_batch) {
     recflex_schedule_t s = {0, 0, 1, 0};
     const int d = spec.dim;
     int id = -1;
@@ -108,6 +108,21 @@ recflex_schedule_t default_schedule(const recflex_feature_spec_t &spec, int targ
         s.sched_id = id;
         s.per_block = id >= 0 ? samples_per_task_default(id, spec.mean_len, spec.coverage, target) : 1;
         return s;
+    }
+    // Small batches (the whole batch is well under 8 waves of 512-lookup tasks:
+    // medium, fig3) are latency-bound: a multi-hot bag pooled by one lane group is
+    // a chain of L/U dependent row round trips.  Split such bags across the lane
+    // groups of a warp (WARP-SPLIT family, 32/G x U rows of the bag in flight)
+    // with 4 bags per warp per task (measured on B200: medium 0.072 -> 0.038 ms
+    // fused, tools/latency_probe.py).
+    if (small_batch && spec.mean_len >= 8.f && d % 4 == 0 && d >= 8 && d <= 64) {
+        id = find_catalog(RECFLEX_FAMILY_WARP, d / 4, 4, 1, d / 4 <= 2 ? 2 : 4);
+        if (id >= 0) {
+            s.sched_id = id;
+            s.part = 0;
+            s.per_block = 32;
+            return s;
+        }
     }
     // Untuned defaults follow what the tuner picks most on B200 (sharded1000 /
     // heavy): rows up to 64 floats -> 256-bit loads with d/8 lanes per bag
@@ -485,8 +500,14 @@ recflex_status_t recflex_plan_create(const recflex_feature_spec_t *specs, int32_
     }
     p->slots_total = slot;
     p->task_lookups = task_lookups_target(specs, F, max_batch, p->num_sms);
+    {
+        double tot = 0;
+        for (int f = 0; f < F; ++f)
+            tot += (double)max_batch * std::max(0.25, (double)specs[f].mean_len * std::max(0.05, (double)specs[f].coverage));
+        p->small_batch = tot < 8.0 * p->num_sms * 4 * 512;
+    }
     for (int f = 0; f < F; ++f) {
-        recflex_schedule_t s = default_schedule(specs[f], p->task_lookups);
+        recflex_schedule_t s = default_schedule(specs[f], p->task_lookups, p->small_batch);
         if (!schedule_valid_for(s, p->desc[f].dim, p->desc[f].dtype, p->desc[f].col, (int)d_tot)) {
             if (specs[f].dtype != RECFLEX_DTYPE_F32) {
                 // reduced-precision entries need a 16-byte-aligned output column

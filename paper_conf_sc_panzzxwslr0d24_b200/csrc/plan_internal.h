@@ -87,6 +87,7 @@ struct recflex_plan_s {
     std::vector<const void *> tables;        // cached table pointers
     int k = 4;
     int task_lookups = 4096;  // lookups per task targeted by the default schedules
+    bool small_batch = false; // the expected batch is < 8 waves of 512-lookup tasks (latency-bound)
     bool desc_dirty = true;
     bool pdl = true;
     bool force_smem_pad = false;  // RECFLEX_SMEM_PAD=1: always pad shared memory to k CTAs/SM (A/B)
@@ -160,7 +161,7 @@ recflex_status_t upload_desc(recflex_plan_s *p, cudaStream_t stream);
 recflex_status_t staged_copy(recflex_plan_s *p, void *d_dst, const void *src, size_t bytes, cudaStream_t stream);
 bool schedule_valid_for(const recflex_schedule_t &s, int dim, int dtype, int col, int d_tot);
 int row_bytes_of(int dim, int dtype);
-recflex_schedule_t default_schedule(const recflex_feature_spec_t &spec, int target);
+recflex_schedule_t default_schedule(const recflex_feature_spec_t &spec, int target, bool small_batch);
 int find_catalog(int family, int G, int VEC, int C, int U, int ET = 0);
 int samples_per_task_default(int sched_id, float mean_len, float coverage, int target);
 int slots_for(int max_batch, float max_len);

@@ -144,7 +144,7 @@ def ablation_swap(config, lines, nfeat=3, seed=0):
     lines.append('')
 
 
-def ablation_tuning(config, lines, ks=(4,)):
+def ablation_tuning(config, lines, ks=(3, 4, 5, 6)):
     """Fig. 11 / P:324: two-stage interference-simulated tuning vs the
     separate-combine straw man (each candidate timed alone, non-padded)."""
     import time
@@ -156,23 +156,30 @@ def ablation_tuning(config, lines, ks=(4,)):
     test = dev_batch(synth.make_batch(m, 50))
     rows = []
     for label, kw in (('default heuristic (untuned)', None),
-                      ('separate-combine (straw man 1)', dict(separate=True, guard=False, refine=False)),
-                      ('two-stage co-execution (paper)', dict(separate=False, guard=False, refine=False)),
-                      ('two-stage + guard + cluster refinement (ours)', dict(separate=False, guard=True, refine=True))):
+                      ('separate-combine (straw man 1, P:73)', dict(separate=True, guard=False, refine=False)),
+                      ("two-stage co-execution, the paper's Eq. 3 cost", dict(tail=False, guard=False, refine=False)),
+                      ('two-stage, tail-aware stage 1 (C33)', dict(tail=True, guard=False, refine=False)),
+                      ('two-stage, tail-aware + guard (default)', dict(tail=True, guard=True, refine=False)),
+                      ('... + cluster refinement (opt-in, outside O(F*K+K))', dict(tail=True, guard=True,
+                                                                                     refine=True))):
         plan = Plan.from_model(m)
-        plan.occupancy = ks[0]
+        plan.occupancy = 4
         t0 = time.time()
         st = plan.tune(hist_dev, tables, occupancies=list(ks), reps=5, **kw) if kw is not None else {}
         tt = time.time() - t0
+        plan.compile()  # every plan timed in its plan-specialised kernel
         ms = timer(plan, test, m.batch, tables, out, flush)
-        rows.append((label, ms, tt, st.get('local_launches', 0)))
+        rows.append((label, ms, tt, st.get('local_launches', 0), st.get('global_launches', 0),
+                     st.get('compile_seconds', 0.0), st.get('refine_evals', 0), plan.occupancy))
         print(label, ms, tt, flush=True)
     base = rows[0][1]
     lines += [f'## Tuning strategies ({config}, k in {list(ks)}; Fig. 11 / P:324)', '',
-              'Each plan is tuned on 2 historical batches and timed on a held-out batch (median of 7, L2 flushed).',
-              '', '| tuner | fused forward (ms) | vs untuned | tuning time (s) | local launches |', '|---|---|---|---|---|']
-    for label, ms, tt, ll in rows:
-        lines.append(f'| {label} | {ms:.3f} | {base / ms:.2f}x | {tt:.0f} | {ll} |')
+              'Each plan is tuned on 2 historical batches and timed on a held-out batch (median of 7, L2 flushed) in '
+              'its plan-specialised kernel.', '',
+              '| tuner | k | fused forward (ms) | vs untuned | tuning time (s) | of which NVRTC (s) | local launches | '
+              'global launches | refinement forwards |', '|---|---|---|---|---|---|---|---|---|']
+    for label, ms, tt, ll, gl, cs, re, k in rows:
+        lines.append(f'| {label} | {k} | {ms:.3f} | {base / ms:.2f}x | {tt:.0f} | {cs:.0f} | {ll} | {gl} | {re} |')
     lines.append('')
 
 
