@@ -12,6 +12,8 @@
 //   block_start = exclusive scan of feature_blocks in feature order.
 #include <cuda_runtime.h>
 
+#include <algorithm>
+
 #include "recflex_internal.h"
 
 namespace recflex {
@@ -263,27 +265,45 @@ int remap_launch(const int32_t *src, int32_t *dst, int64_t n, int64_t shift, int
     return (int)cudaGetLastError();
 }
 
-// Relayout after the pooled-output all-to-all: chunk i [rows][dims[i]] -> columns
-__global__ void recflex_concat_kernel(const float *recv, int W, int rows, const int32_t *dims, const int32_t *cols,
-                                      int d_tot, float *out) {
-    const int64_t n = (int64_t)rows * d_tot;
-    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x) {
-        const int r = (int)(e / d_tot);
-        const int q = (int)(e % d_tot);
-        int i = 0;
-        while (i + 1 < W && cols[i + 1] <= q) ++i;
-        const int64_t chunk_base = (int64_t)rows * cols[i];  // chunks are contiguous in rank order
-        out[e] = recv[chunk_base + (int64_t)r * dims[i] + (q - cols[i])];
+// Relayout after the pooled-output all-to-all: received chunk i is rank i's
+// [rows][dims[i]] block (chunks contiguous in rank order); it goes to columns
+// [cols[i], cols[i] + dims[i]) of out [rows][d_tot].  blockIdx.y = chunk (no
+// per-element rank search); 16-byte copies when the chunk and the layout are
+// 4-float aligned (every config), else scalar.  Dims travel by value.
+__global__ void __launch_bounds__(256) recflex_concat_kernel(const float *__restrict__ recv, float *__restrict__ out,
+                                                             ConcatArgs a) {
+    const int i = blockIdx.y;
+    const int d = a.dims[i];
+    const int64_t n = (int64_t)a.rows * d;
+    const float *src = recv + (int64_t)a.rows * a.cols[i];
+    float *dst = out + a.cols[i];
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    const int64_t t0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (((d | a.cols[i] | a.d_tot) & 3) == 0) {
+        const int d4 = d >> 2;
+        const int64_t n4 = n >> 2;
+        for (int64_t e = t0; e < n4; e += stride) {
+            const int64_t r = e / d4;
+            const int c = (int)(e - r * d4);
+            const float4 v = __ldg(reinterpret_cast<const float4 *>(src) + e);
+            *reinterpret_cast<float4 *>(dst + r * a.d_tot + 4 * c) = v;
+        }
+    } else {
+        for (int64_t e = t0; e < n; e += stride) {
+            const int64_t r = e / d;
+            const int c = (int)(e - r * d);
+            dst[r * a.d_tot + c] = src[e];
+        }
     }
 }
 
-int concat_launch(const float *recv, int W, int rows, const int32_t *d_dims, const int32_t *d_cols, int d_tot,
-                  float *out, void *stream) {
-    const int64_t n = (int64_t)rows * d_tot;
-    if (n == 0) return 0;
-    int grid = (int)((n + 255) / 256);
-    if (grid > 148 * 16) grid = 148 * 16;
-    recflex_concat_kernel<<<grid, 256, 0, (cudaStream_t)stream>>>(recv, W, rows, d_dims, d_cols, d_tot, out);
+int concat_launch(const float *recv, const ConcatArgs &a, float *out, void *stream) {
+    if (a.W <= 0 || a.rows <= 0 || a.d_tot <= 0) return 0;
+    int64_t max_n = 0;
+    for (int i = 0; i < a.W; ++i) max_n = std::max<int64_t>(max_n, (int64_t)a.rows * a.dims[i]);
+    int gx = (int)std::min<int64_t>((max_n / 4 + 255) / 256, 148 * 8 / std::max(1, a.W) + 1);
+    gx = std::max(gx, 1);
+    recflex_concat_kernel<<<dim3(gx, a.W), 256, 0, (cudaStream_t)stream>>>(recv, out, a);
     return (int)cudaGetLastError();
 }
 

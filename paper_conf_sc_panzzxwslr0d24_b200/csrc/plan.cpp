@@ -547,9 +547,24 @@ recflex_status_t recflex_plan_create(const recflex_feature_spec_t *specs, int32_
     return RECFLEX_OK;
 }
 
+namespace {
+// Makes the plan's device current for the call and restores the caller's.
+struct DeviceGuard {
+    int prev = -1;
+    explicit DeviceGuard(int dev) {
+        if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+        if (prev != dev) cudaSetDevice(dev);
+    }
+    ~DeviceGuard() {
+        int cur = -1;
+        if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+    }
+};
+}  // namespace
+
 void recflex_destroy(recflex_plan_t p) {
     if (!p) return;
-    cudaSetDevice(p->device);
+    DeviceGuard guard(p->device);
     plan_free_device(p);
     delete p;
 }
@@ -571,20 +586,6 @@ static recflex_status_t sync_tables(recflex_plan_s *p, const void *const *tables
     return RECFLEX_OK;
 }
 
-namespace {
-// Makes the plan's device current for the call and restores the caller's.
-struct DeviceGuard {
-    int prev = -1;
-    explicit DeviceGuard(int dev) {
-        if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
-        if (prev != dev) cudaSetDevice(dev);
-    }
-    ~DeviceGuard() {
-        int cur = -1;
-        if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
-    }
-};
-}  // namespace
 
 recflex_status_t recflex_forward(recflex_plan_t p, const int32_t *indices, const int32_t *offsets, int32_t B,
                                  const void *const *tables, float *out, void *stream_) {
@@ -726,7 +727,7 @@ recflex_status_t recflex_backward(recflex_plan_t p, const int32_t *indices, cons
     for (int f = 0; f < p->F; ++f)
         if (!targets[f] || ((uintptr_t)targets[f]) % 16) return RECFLEX_ERR_INVALID_ARG;
     cudaStream_t stream = (cudaStream_t)stream_;
-    cudaSetDevice(p->device);
+    DeviceGuard guard(p->device);
     // the task map reads the descriptors (schedules, part); tables are not read
     if (p->desc_dirty) {
         recflex_status_t st = upload_desc(p, stream);
@@ -797,7 +798,7 @@ recflex_status_t recflex_forward_host(recflex_plan_t p, const int32_t *h_indices
     if (B == 0) return RECFLEX_OK;
     if (!h_offsets || !h_out || (nnz > 0 && !h_indices)) return RECFLEX_ERR_INVALID_ARG;
     cudaStream_t stream = (cudaStream_t)stream_;
-    cudaSetDevice(p->device);
+    DeviceGuard guard(p->device);
     const int64_t n_off = (int64_t)p->F * B + 1;
     const int64_t n_out = (int64_t)B * p->d_tot;
     cudaError_t e = cudaSuccess;
@@ -898,7 +899,7 @@ recflex_status_t recflex_debug_task_map(recflex_plan_t p, const int32_t *offsets
                                         int32_t *h_ranges, int64_t cap, void *stream_) {
     if (!p || !offsets || !h_bs || B < 0 || B > p->max_batch) return RECFLEX_ERR_INVALID_ARG;
     cudaStream_t stream = (cudaStream_t)stream_;
-    cudaSetDevice(p->device);
+    DeviceGuard guard(p->device);
     if (p->desc_dirty || p->ex.num_part1 != 0 || true) {
         // descriptors may be stale if no forward ran yet (tables not known): upload with null tables
         for (int f = 0; f < p->F; ++f) p->desc[f].table = p->tables[f];
@@ -968,7 +969,7 @@ recflex_status_t recflex_get_task_slots(recflex_plan_t p, int32_t f, int32_t *sl
 
 recflex_status_t recflex_debug_task_need(recflex_plan_t p, int32_t *host_need) {
     if (!p || !host_need) return RECFLEX_ERR_INVALID_ARG;
-    cudaSetDevice(p->device);
+    DeviceGuard guard(p->device);
     cudaError_t e = cudaMemcpy(host_need, p->ex.d_need, sizeof(int32_t) * p->F, cudaMemcpyDeviceToHost);
     return e == cudaSuccess ? RECFLEX_OK : cuda_status(e);
 }
@@ -978,7 +979,7 @@ recflex_status_t recflex_validate(recflex_plan_t p, const int32_t *indices, cons
     if (!p || !offsets || B < 0 || B > p->max_batch) return RECFLEX_ERR_INVALID_ARG;
     if (B == 0) return RECFLEX_OK;
     cudaStream_t stream = (cudaStream_t)stream_;
-    cudaSetDevice(p->device);
+    DeviceGuard guard(p->device);
     recflex_status_t st = upload_desc(p, stream);
     if (st != RECFLEX_OK) return st;
     int32_t *d_flag = nullptr;
@@ -1152,23 +1153,20 @@ recflex_status_t recflex_plan_import(recflex_plan_t p, const char *json) {
 
 recflex_status_t recflex_shard_concat(const float *recv, int32_t W, int32_t rows, const int32_t *host_dims, float *out,
                                       void *stream_) {
-    if (!recv || !out || !host_dims || W <= 0 || rows < 0) return RECFLEX_ERR_INVALID_ARG;
-    cudaStream_t stream = (cudaStream_t)stream_;
-    std::vector<int32_t> h(2 * W);
-    int32_t tot = 0;
+    if (!recv || !out || !host_dims || W <= 0 || W > kMaxConcatRanks || rows < 0) return RECFLEX_ERR_INVALID_ARG;
+    ConcatArgs a;
+    a.W = W;
+    a.rows = rows;
+    int64_t tot = 0;
     for (int i = 0; i < W; ++i) {
         if (host_dims[i] < 0) return RECFLEX_ERR_INVALID_ARG;
-        h[i] = host_dims[i];
-        h[W + i] = tot;
+        a.dims[i] = host_dims[i];
+        a.cols[i] = (int32_t)tot;
         tot += host_dims[i];
     }
-    int32_t *d = nullptr;
-    cudaError_t e = cudaMallocAsync(&d, sizeof(int32_t) * 2 * W, stream);
-    if (e != cudaSuccess) return cuda_status(e);
-    e = cudaMemcpyAsync(d, h.data(), sizeof(int32_t) * 2 * W, cudaMemcpyHostToDevice, stream);
-    if (e != cudaSuccess) return cuda_status(e);
-    int rc = concat_launch(recv, W, rows, d, d + W, tot, out, stream);
-    cudaFreeAsync(d, stream);
+    if (tot >= (int64_t(1) << 31)) return RECFLEX_ERR_INVALID_ARG;
+    a.d_tot = (int32_t)tot;
+    int rc = concat_launch(recv, a, out, stream_);
     if (rc) return cuda_status((cudaError_t)rc);
     return RECFLEX_OK;
 }

@@ -231,8 +231,13 @@ int fill_launch(const FillArgs &a, int grid_x, bool pdl, void *stream);
 int validate_launch(const FeatureDesc *desc, int F, int in_F, const int32_t *indices, const int32_t *offsets, int B,
                     int32_t *flag, void *stream);
 int remap_launch(const int32_t *src, int32_t *dst, int64_t n, int64_t shift, int64_t rows, void *stream);
-int concat_launch(const float *recv, int W, int rows, const int32_t *d_dims, const int32_t *d_cols, int d_tot,
-                  float *out, void *stream);
+constexpr int kMaxConcatRanks = 64;
+struct ConcatArgs {
+    int32_t W, rows, d_tot;
+    int32_t dims[kMaxConcatRanks];
+    int32_t cols[kMaxConcatRanks];
+};
+int concat_launch(const float *recv, const ConcatArgs &a, float *out, void *stream);
 int flush_launch(void *buf, size_t bytes, void *stream);
 int route_signal_wait_launch(uint32_t *const *flags, const uint32_t *local_flags, int32_t *epoch, int rank, int world,
                              void *stream);
