@@ -332,8 +332,13 @@ def main():
         plan.occupancy = args.occupancy
     # the paper's fusion compiler: the plan's schedules inlined into one kernel (NVRTC)
     jit = None
+    ksel = None
     if not args.no_jit:
         jit = plan.compile()
+        # stage 2 over the plan's two kernels (plan-specialised vs catalog) on the first batch
+        ksel = plan.select_kernel(batches[0][0], batches[0][1], B, tables, reps=5)
+        if not plan.jit_enabled:
+            jit = dict(jit, active=0)
 
     out_local = torch.empty((B, sh.d_local), dtype=torch.float32, device=dev)
     out_x = torch.empty((B // world, sh.d_tot), dtype=torch.float32, device=dev) if world > 1 else None
@@ -472,7 +477,7 @@ def main():
         send = rows * sh.d_local * 4 * (world - 1)
         recv = rows * (sh.d_tot - sh.d_local) * 4
         a2a_bytes = max(send, recv)
-        nvlink = 900e9
+        nvlink = 770e9  # measured peer copy per direction (B200_PROFILING.md; nominal 900 GB/s)
         a2a_ms = a2a_bytes / nvlink * 1e3
         relayout_ms = (2.0 * rows * sh.d_tot * 4) / (peak * 1e9) * 1e3 if args.exchange == 'nccl' else 0.0
         comp_max = max_over_ranks(comp_ms)
@@ -485,6 +490,7 @@ def main():
             'exchange': ('NCCL alltoallv + relayout kernel' if args.exchange == 'nccl' else
                          'peer stores in the fused kernel epilogue + device-side flags (recflex_forward_exchange)'),
             'nvlink': {'a2a_bytes_max_rank': max_over_ranks(a2a_bytes), 'gbs_per_direction': nvlink / 1e9,
+                       'gbs_source': 'measured B200 peer copy, B200_PROFILING.md (nominal 900)',
                        'a2a_ms_at_peak': a2a_max, 'relayout_ms_at_hbm_peak': max_over_ranks(relayout_ms),
                        'serial_bound_ms': comp_max + a2a_max + max_over_ranks(relayout_ms),
                        'overlapped_bound_ms': max(comp_max, a2a_max),
@@ -601,6 +607,7 @@ def main():
                             'launch': launch_desc,
                             'kernel': (f"plan-specialised (NVRTC, {jit['variants']} variants, {jit['registers']} "
                                        f"regs, {jit['local_bytes']} B local)" if jit and jit['active'] else 'catalog'),
+                            'kernel_selection': ksel,
                             'input': ('data-parallel local batches + KJT input dist in the timed step'
                                       if args.input_dist else 'table-wise KJT resident per rank'),
                             'l2': 'flushed between steps' if flush_between else
@@ -649,12 +656,13 @@ def time_config(config, args, dev, peak, steps=20, warmup=5, nbatches=3):
     if os.path.exists(path):
         with open(path) as fh:
             plan.import_(json.load(fh))
-    info = plan.compile()
+    plan.compile()
     bts, alg = [], []
     for i in range(nbatches):
         b = synth.make_batch(m, 7 + i)
         bts.append((torch.from_numpy(b.indices).to(dev), torch.from_numpy(b.offsets).to(dev)))
         alg.append(synth.algorithmic_bytes(m, b, 'f32')['total'])
+    ksel = plan.select_kernel(bts[0][0], bts[0][1], m.batch, tables, reps=5)
     alg_b = float(np.mean(alg))
     out = torch.empty((m.batch, m.d_tot), dtype=torch.float32, device=dev)
     for i in range(warmup):
@@ -695,9 +703,9 @@ def time_config(config, args, dev, peak, steps=20, warmup=5, nbatches=3):
            'effective_hbm_gbs': alg_b / (ms / 1e3) / 1e9, 'pct_of_8tbs': 100.0 * alg_b / (ms / 1e3) / 8e12,
            'roofline': {'bound': 'hbm', 'achieved': alg_b / (fused_ms / 1e3) / 1e9, 'peak': peak, 'unit': 'GB/s',
                         'frac': alg_b / (fused_ms / 1e3) / 1e9 / peak, 'fused_ms': fused_ms,
-                        'kernel': f'recflex_fused_jit_k{plan.occupancy}' if info['active'] else 'recflex_fused_kernel',
+                        'kernel': f'recflex_fused_jit_k{plan.occupancy}' if plan.jit_enabled else 'recflex_fused_kernel',
                         'algorithmic_bytes_per_launch': alg_b},
-           'plan': os.path.relpath(path, ROOT), 'occupancy': plan.occupancy,
+           'plan': os.path.relpath(path, ROOT), 'occupancy': plan.occupancy, 'kernel_selection': ksel,
            'l2': f'inputs > L2 ({alg_b / 1e9:.1f} GB algorithmic per step, {nbatches} rotating batches)',
            'launch': 'CUDA graph replay per step', 'clocks': clk}
     del graphs, tables, phys, bts

@@ -333,8 +333,18 @@ typedef struct {
 } recflex_jit_info_t;
 /* k = 0: the plan's current occupancy. */
 recflex_status_t recflex_jit_info(recflex_plan_t plan, int32_t k, recflex_jit_info_t *info);
-/* enable = 0: forwards ignore compiled kernels (A/B against the catalog kernel). */
+/* enable = 0: forwards ignore compiled kernels (A/B against the catalog kernel).
+ * The choice is part of the plan's exported state ("kernel"). */
 recflex_status_t recflex_set_jit(recflex_plan_t plan, int32_t enable);
+recflex_status_t recflex_get_jit(recflex_plan_t plan, int32_t *enabled);
+/* Stage 2 over the plan's two kernels: compiles the plan-specialised kernel
+ * for the current schedules and k (if needed), times it and the catalog kernel
+ * on one batch (device pointers; median of reps forwards, L2 flushed before
+ * each) and keeps the faster for later forwards.  *jit_ms / *catalog_ms
+ * (nullable) receive the medians.  Blocking; allocates scratch. */
+recflex_status_t recflex_select_kernel(recflex_plan_t plan, const int32_t *indices, const int32_t *offsets,
+                                       int32_t batch_size, const void *const *tables, int32_t reps, float *jit_ms,
+                                       float *catalog_ms, void *stream);
 /* Directory for cached cubins (created on first write); NULL or "" = none. */
 recflex_status_t recflex_set_jit_cache_dir(const char *dir);
 /* The generator alone (no GPU needed): CUDA source of the specialised kernel

@@ -125,6 +125,9 @@ SIGNATURES = {
     'recflex_get_task_slots': (c_int32, [c_void_p, c_int32, P(c_int32)]),
     'recflex_jit_info': (c_int32, [c_void_p, c_int32, P(JitInfo)]),
     'recflex_set_jit': (c_int32, [c_void_p, c_int32]),
+    'recflex_get_jit': (c_int32, [c_void_p, P(c_int32)]),
+    'recflex_select_kernel': (c_int32, [c_void_p, c_void_p, c_void_p, c_int32, P(c_void_p), c_int32,
+                                        P(ctypes.c_float), P(ctypes.c_float), c_void_p]),
     'recflex_set_jit_cache_dir': (c_int32, [ctypes.c_char_p]),
     'recflex_jit_generate': (c_int32, [P(c_int32), P(c_int32), P(c_int32), P(c_int32), c_int32, c_int32,
                                        ctypes.c_char_p, ctypes.c_size_t, P(ctypes.c_size_t), P(c_int32), P(c_int32)]),

@@ -1073,7 +1073,9 @@ recflex_status_t recflex_plan_export(recflex_plan_t p, char *buf, size_t cap, si
         if (p->desc[f].nalloc > 0) s += ", " + std::to_string(p->desc[f].nalloc);
         s += "]";
     }
-    s += "]}";
+    s += "], \"kernel\": \"";
+    s += p->use_jit ? "plan-specialised" : "catalog";
+    s += "\"}";
     if (len) *len = s.size() + 1;
     if (buf && cap > 0) {
         size_t n = std::min(cap - 1, s.size());
@@ -1148,6 +1150,12 @@ recflex_status_t recflex_plan_import(recflex_plan_t p, const char *json) {
     }
     for (int f = 0; f < p->F; ++f) recflex_set_schedule(p, f, &ss[f]);
     p->k = k;
+    // optional: which kernel the plan runs (recflex_select_kernel's choice)
+    if (const char *kc = std::strstr(json, "\"kernel\"")) {
+        const char *v = std::strchr(kc + 8, '"');  // opening quote of the value
+        if (v && !std::strncmp(v, "\"catalog\"", 9)) p->use_jit = false;
+        else if (v && !std::strncmp(v, "\"plan-specialised\"", 18)) p->use_jit = true;
+    }
     return RECFLEX_OK;
 }
 

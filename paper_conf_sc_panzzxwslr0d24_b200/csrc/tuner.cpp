@@ -800,8 +800,12 @@ extern "C" recflex_status_t recflex_tune_ex(recflex_plan_t p, int32_t N, const i
     p->k = T.ks[best_k];
     st = upload_desc(p, stream);
     if (st != RECFLEX_OK) return st;
-    if (T.jit && !jit_ready(p, p->k)) {  // leave the chosen kernel compiled (disk-cache hit)
-        st = jit_compile_plan(p, &p->k, 1);
+    if (T.jit) {
+        // stage 2 over the plan's two kernels for the final choice: the
+        // plan-specialised kernel (compiled; usually a disk-cache hit) vs the
+        // catalog kernel, on the first historical batch
+        st = recflex_select_kernel(p, T.batches[0].d_idx, T.batches[0].d_off, T.batches[0].B, p->tables.data(),
+                                   T.reps, nullptr, nullptr, stream);
         if (st != RECFLEX_OK) return st;
     }
     recflex_tune_stats_t s = {};

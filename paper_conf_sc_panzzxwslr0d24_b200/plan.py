@@ -157,6 +157,23 @@ class Plan:
     def set_jit(self, enable: bool) -> None:
         check(lib.recflex_set_jit(self._h, 1 if enable else 0), 'recflex_set_jit')
 
+    @property
+    def jit_enabled(self) -> bool:
+        v = ctypes.c_int32()
+        check(lib.recflex_get_jit(self._h, ctypes.byref(v)), 'recflex_get_jit')
+        return bool(v.value)
+
+    def select_kernel(self, indices: torch.Tensor, offsets: torch.Tensor, B: int, tables: Sequence[torch.Tensor],
+                      reps: int = 7, stream=None) -> dict:
+        """recflex_select_kernel: time the plan-specialised and the catalog kernel on this
+        batch and keep the faster (part of the exported plan)."""
+        j, c = ctypes.c_float(), ctypes.c_float()
+        check(lib.recflex_select_kernel(self._h, _dptr(indices, torch.int32, 'indices'),
+                                        _dptr(offsets, torch.int32, 'offsets'), int(B), self._tables(tables),
+                                        int(reps), ctypes.byref(j), ctypes.byref(c), _stream_ptr(stream)),
+              'recflex_select_kernel')
+        return dict(jit_ms=j.value, catalog_ms=c.value, kernel='plan-specialised' if self.jit_enabled else 'catalog')
+
     # -------------------------------------------------------------- hot path
     def forward(self, indices: torch.Tensor, offsets: torch.Tensor, B: int, tables: Sequence[torch.Tensor],
                 out: Optional[torch.Tensor] = None, stream=None) -> torch.Tensor:

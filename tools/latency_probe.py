@@ -27,6 +27,9 @@ def main():
     ap.add_argument('--spbs', default='8,16,32,64')
     ap.add_argument('--no-tuned', action='store_true')
     ap.add_argument('--no-jit', action='store_true', help='time the catalog kernel instead')
+    ap.add_argument('--onehot', action='store_true',
+                    help='sweep the ONE-HOT features instead (multi-hot features keep the plan\'s schedules)')
+    ap.add_argument('--base', default='tuned', choices=['tuned', 'default'])
     a = ap.parse_args()
     import torch
     from paper_conf_sc_panzzxwslr0d24_b200 import synth
@@ -39,7 +42,8 @@ def main():
     dev_b = [(torch.from_numpy(b.indices).to(dev), torch.from_numpy(b.offsets).to(dev)) for b in bts]
     plan = Plan.from_model(m)
     tuned = os.path.join(ROOT, 'configs', 'tuned', f'{a.config}_w1_r0.json')
-    plan.import_(json.load(open(tuned)))
+    if a.base == 'tuned':
+        plan.import_(json.load(open(tuned)))
     base = [plan.get_schedule(f) for f in range(m.F)]
     cat = catalog()
     out = torch.empty((m.batch, m.d_tot), device=dev)
@@ -68,7 +72,7 @@ def main():
                 return e['id']
         return None
 
-    multi = [f for f, ft in enumerate(m.features) if ft.max_len() > 1.5]
+    multi = [f for f, ft in enumerate(m.features) if (ft.max_len() > 1.5) != a.onehot]
     shapes = [] if a.no_tuned else [('tuned', None, None, None, None)]
     for fam in a.families.split(','):
         for V in [int(x) for x in a.vs.split(',')]:

@@ -27,6 +27,7 @@ def main():
     ap.add_argument('config', nargs='?', default='sharded1000')
     ap.add_argument('--worlds', default='1,2,4,8')
     ap.add_argument('--reps', type=int, default=10)
+    ap.add_argument('--no-jit', action='store_true')
     a = ap.parse_args()
     import torch
     from paper_conf_sc_panzzxwslr0d24_b200 import synth
@@ -49,6 +50,8 @@ def main():
             tuned = os.path.exists(path)
             if tuned:
                 sh.plan.import_(json.load(open(path)))
+            if not a.no_jit:
+                sh.plan.compile()  # the plan-specialised kernel bench.py runs
             tables = [phys[model.features[f].table] for f in sh.features]
             idx, off = shard_batch(full, sh.features)
             bi, bo = torch.from_numpy(idx).to(dev), torch.from_numpy(off).to(dev)
@@ -64,7 +67,7 @@ def main():
                 if rep >= 2:
                     ts.append(e0.elapsed_time(e1))
             per_rank.append(dict(rank=r, features=len(sh.features), d_local=sh.d_local, ms=float(np.median(ts)),
-                                 tuned=tuned, occupancy=sh.plan.occupancy))
+                                 tuned=tuned, occupancy=sh.plan.occupancy, jit=not a.no_jit))
             del sh, bi, bo, out
             torch.cuda.empty_cache()
         comp = max(p['ms'] for p in per_rank)
