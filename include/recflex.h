@@ -219,9 +219,13 @@ typedef struct {
                                 forward at the chosen k; keep if > 0.5% faster.
                                 Outside O(F*K + K); off by default, reported apart        */
     int32_t local_mode;      /* 0: interference-simulated co-execution with padding (the
-                                paper's method); 1: separate-combine straw man -- each
-                                candidate timed alone in a non-padded launch (P:73, P:324,
-                                for the Fig. 11 ablation)                                   */
+                                paper's method: all candidates of a feature in one padded
+                                launch, cost = their own block times); 1: separate-combine
+                                straw man -- each candidate timed alone in a non-padded
+                                launch (for the Fig. 11 ablation); 2: isolated
+                                co-execution -- one padded launch per candidate, cost = the
+                                launch's total block time, i.e. its own blocks plus the
+                                slowdown it inflicts on the padding (reading C34)          */
     int32_t stage2_catalog;  /* 0: stage 2 (and guard / refinement) time the plan-
                                 specialised kernel each choice compiles to (NVRTC, the
                                 kernel forwards run); 1: the precompiled catalog kernel   */

@@ -133,6 +133,7 @@ struct Tuner {
     int reps = 7;
     int pad_waves = 4;
     bool separate = false;  // local_mode 1: separate-combine straw man (ablation)
+    bool isolated = false;      // local_mode 2: one padded co-execution launch per candidate (C34)
     bool jit = true;            // stage 2 / guard / refinement time the plan-specialised kernel
     // Tail-aware stage-1 cost (reading C33): a candidate costs its
     // CTA-time share W_c / (#SM * k) plus the part of its longest task that
@@ -343,7 +344,19 @@ struct Tuner {
         } trace_end{trace, k, f, n, t_trace};
         std::vector<double> sum(n, 0.0);
         const FeatureDesc &base = p->desc[f];
-        for (size_t i = 0; i < batches.size(); ++i) {
+        // co-execution groups: all candidates in one padded launch (the paper's
+        // Eq. 3), or -- isolated mode -- one padded launch per candidate, whose
+        // cost is then the launch's TOTAL block time (own tasks + the slowdown it
+        // inflicts on the identical padding; reading C34)
+        std::vector<std::vector<int>> groups;
+        if (isolated) {
+            for (int c = 0; c < n; ++c) groups.push_back({c});
+        } else {
+            groups.emplace_back();
+            for (int c = 0; c < n; ++c) groups.back().push_back(c);
+        }
+        for (size_t i = 0; i < batches.size(); ++i)
+        for (const std::vector<int> &grp : groups) {
             const Batch &bt = batches[i];
             TP &tp = tps[i];
             const int B = bt.B;
@@ -378,7 +391,7 @@ struct Tuner {
             };
             add_pad(pre_target);
             const int cand_first = (int)ds.size();
-            for (int c = 0; c < n; ++c) {
+            for (int c : grp) {
                 FeatureDesc d = base;
                 d.sched = cands[f][c].sched_id;
                 d.part = cands[f][c].part;
@@ -453,14 +466,22 @@ struct Tuner {
             if (err) return;
             const double P = (double)p->num_sms * k;
             const double T_est = (tail && ki < (int)t_est.size() && i < t_est[ki].size()) ? t_est[ki][i] : 0.0;
-            for (int c = 0; c < n; ++c) {
-                const int v = cand_first + c;
+            double pad_sum = 0;  // isolated mode: the padding's block time in this launch
+            if (isolated) {
+                for (int v = 0; v < V; ++v) {
+                    if (v >= cand_first && v < cand_first + (int)grp.size()) continue;
+                    for (int64_t t = bs[v]; t < bs[v + 1]; ++t) pad_sum += (double)tm[t];
+                }
+            }
+            for (size_t gi = 0; gi < grp.size(); ++gi) {
+                const int c = grp[gi];
+                const int v = cand_first + (int)gi;
                 double s = 0, mx = 0;
                 for (int64_t t = bs[v]; t < bs[v + 1]; ++t) {
                     s += (double)tm[t];
                     mx = std::max(mx, (double)tm[t]);
                 }
-                sum[c] += s / P + (T_est > 0 ? std::max(0.0, mx - T_est) : 0.0);
+                sum[c] += (s + pad_sum) / P + (T_est > 0 ? std::max(0.0, mx - T_est) : 0.0);
             }
         }
         for (int c = 0; c < n; ++c) costs[c] = sum[c];
@@ -659,6 +680,7 @@ extern "C" recflex_status_t recflex_tune_ex(recflex_plan_t p, int32_t N, const i
     if (opt && opt->pad_waves > 0) T.pad_waves = opt->pad_waves;
     if (opt) T.verbose = opt->verbose;
     if (opt) T.separate = opt->local_mode == 1;
+    if (opt) T.isolated = opt->local_mode == 2;
     if (opt) T.jit = opt->stage2_catalog == 0;
     const int max_c = opt ? opt->max_candidates : 0;
     for (int i = 0; i < N; ++i) {

@@ -300,7 +300,7 @@ class Plan:
     def tune(self, batches: Sequence[tuple], tables: Sequence[torch.Tensor], occupancies: Optional[List[int]] = None,
              reps: int = 7, pad_waves: int = 4, max_candidates: int = 0, verbose: bool = False, guard: bool = True,
              refine: bool = False, separate: bool = False, stage2_catalog: bool = False, tail: bool = True,
-             stream=None) -> dict:
+             isolated: bool = False, stream=None) -> dict:
         """recflex_tune_ex over historical batches [(indices, offsets, B), ...]."""
         N = len(batches)
         idx_arr = (ctypes.c_void_p * N)(*[b[0].data_ptr() for b in batches])
@@ -317,7 +317,7 @@ class Plan:
         opt.verbose = 1 if verbose else 0
         opt.skip_guard = 0 if guard else 1
         opt.refine = 1 if refine else 0
-        opt.local_mode = 1 if separate else 0
+        opt.local_mode = 1 if separate else (2 if isolated else 0)
         opt.stage2_catalog = 1 if stage2_catalog else 0
         opt.no_tail = 0 if tail else 1
         st = _lib.TuneStats()

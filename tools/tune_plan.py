@@ -31,6 +31,7 @@ def main():
     ap.add_argument('--no-guard', action='store_true')
     ap.add_argument('--stage2-catalog', action='store_true', help='stage 2 on the catalog kernel (no NVRTC)')
     ap.add_argument('--no-tail', action='store_true', help="stage 1 = the paper's plain block-time sum")
+    ap.add_argument('--isolated', action='store_true', help='stage 1: one padded launch per candidate (C34)')
     a = ap.parse_args()
     import torch
     from paper_conf_sc_panzzxwslr0d24_b200 import synth
@@ -60,7 +61,7 @@ def main():
         t0 = time.time()
         st = sh.plan.tune(hist, tables, occupancies=ks, reps=a.reps, max_candidates=a.max_candidates, verbose=True,
                           refine=a.refine, guard=not a.no_guard, stage2_catalog=a.stage2_catalog,
-                          tail=not a.no_tail)
+                          tail=not a.no_tail, isolated=a.isolated)
         st['wall_s'] = time.time() - t0
         state = sh.plan.export()
         name = f'{a.config}_w{a.world}_r{r}' if a.dtype == 'f32' else f'{a.config}_{a.dtype}_w{a.world}_r{r}'
