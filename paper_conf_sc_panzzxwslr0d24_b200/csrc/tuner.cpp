@@ -466,6 +466,16 @@ struct Tuner {
             if (err) return;
             const double P = (double)p->num_sms * k;
             const double T_est = (tail && ki < (int)t_est.size() && i < t_est[ki].size()) ? t_est[ki][i] : 0.0;
+            // latency-bound batch (the incoming plan fills < 2 waves of tasks): the
+            // kernel time is the longest task chain, so a candidate costs its
+            // longest task (a separable surrogate of max_f Lmax_f); otherwise its
+            // CTA-time share plus the tail beyond T_est (reading C33)
+            bool latency_bound = false;
+            if (tail) {
+                double tasks = 0;
+                for (int g = 0; g < p->F; ++g) tasks += (double)task_count(p->desc[g], B, bt.nnz(g));
+                latency_bound = tasks < 2.0 * P;
+            }
             double pad_sum = 0;  // isolated mode: the padding's block time in this launch
             if (isolated) {
                 for (int v = 0; v < V; ++v) {
@@ -481,7 +491,7 @@ struct Tuner {
                     s += (double)tm[t];
                     mx = std::max(mx, (double)tm[t]);
                 }
-                sum[c] += (s + pad_sum) / P + (T_est > 0 ? std::max(0.0, mx - T_est) : 0.0);
+                sum[c] += latency_bound ? mx : (s + pad_sum) / P + (T_est > 0 ? std::max(0.0, mx - T_est) : 0.0);
             }
         }
         for (int c = 0; c < n; ++c) costs[c] = sum[c];
