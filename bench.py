@@ -117,6 +117,15 @@ def _cpu_model():
     return platform.processor() or 'unknown'
 
 
+def task_order_name(plan):
+    """Which order the plan's tasks are claimed in (reading C35): a heuristic's name or 'custom'."""
+    order = plan.task_order
+    for kind in plan.ORDER_KINDS:
+        if order == plan.task_order_heuristic(kind):
+            return kind
+    return 'custom'
+
+
 def _workload_config(args, model, world):
     """The `config` dict both arms print (identical keys and values for the same run):
     the workload only -- implementation details go to `impl_config`."""
@@ -608,6 +617,10 @@ def main():
                             'kernel': (f"plan-specialised (NVRTC, {jit['variants']} variants, {jit['registers']} "
                                        f"regs, {jit['local_bytes']} B local)" if jit and jit['active'] else 'catalog'),
                             'kernel_selection': ksel,
+                            'task_order': task_order_name(plan),
+                            'output_columns': ('task order (features concatenated in the order their tasks '
+                                               'run; recflex_get_columns)' if plan.export().get('columns')
+                                               else 'feature order'),
                             'input': ('data-parallel local batches + KJT input dist in the timed step'
                                       if args.input_dist else 'table-wise KJT resident per rank'),
                             'l2': 'flushed between steps' if flush_between else
@@ -706,6 +719,8 @@ def time_config(config, args, dev, peak, steps=20, warmup=5, nbatches=3):
                         'kernel': f'recflex_fused_jit_k{plan.occupancy}' if plan.jit_enabled else 'recflex_fused_kernel',
                         'algorithmic_bytes_per_launch': alg_b},
            'plan': os.path.relpath(path, ROOT), 'occupancy': plan.occupancy, 'kernel_selection': ksel,
+           'task_order': task_order_name(plan),
+           'output_columns': 'task order' if plan.export().get('columns') else 'feature order',
            'l2': f'inputs > L2 ({alg_b / 1e9:.1f} GB algorithmic per step, {nbatches} rotating batches)',
            'launch': 'CUDA graph replay per step', 'clocks': clk}
     del graphs, tables, phys, bts

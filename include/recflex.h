@@ -66,7 +66,7 @@ typedef unsigned long long uintptr_t;
 extern "C" {
 #endif
 
-#define RECFLEX_ABI_VERSION 3
+#define RECFLEX_ABI_VERSION 4
 #define RECFLEX_MAX_OCCUPANCY 8          /* CTAs of 256 threads per SM: K = 8 (reading C14) */
 
 typedef struct recflex_plan_s *recflex_plan_t; /* opaque, library-owned */
@@ -233,6 +233,8 @@ typedef struct {
                                 (tail-aware, reading C33; T_est = measured latency of the
                                 incoming plan at k, K*N extra timed forwards); 1: the
                                 paper's plain sum of block times W_c (Eq. 3)              */
+    int32_t keep_order;      /* 0: after kernel selection, recflex_select_task_order on the
+                                first batch (3 x reps forwards); 1: keep the plan's order  */
 } recflex_tune_options_t;
 
 typedef struct {
@@ -252,6 +254,7 @@ typedef struct {
     int64_t jit_compiles;     /* plan-specialised kernels compiled (or cache hits) */
     double compile_seconds;   /* wall time spent compiling them                    */
     double refine_seconds;    /* wall time of the refinement stage                 */
+    int32_t task_order;       /* RECFLEX_ORDER_* kept by the order selection, -1 = not run */
 } recflex_tune_stats_t;
 
 /* Two-stage interference-simulated tuning over num_batches historical batches
@@ -370,8 +373,10 @@ recflex_status_t recflex_jit_compile_source(const char *source, void *cubin_buf,
 /* ---- introspection / validation / persistence ---------------------------- */
 
 /* Runs the map (+ fill) kernels for offsets (device) and copies the task map
- * to the host: host_block_start[F+1] (exclusive scan of feature_blocks, Fig. 8
- * d_task_map in compressed form); host_task_range (nullable) receives, for
+ * to the host: host_block_start[F+1] (exclusive scan of feature_blocks taken
+ * in the plan's TASK ORDER -- entry e belongs to feature order[e] of
+ * recflex_get_task_order; Fig. 8 d_task_map in compressed form);
+ * host_task_range (nullable) receives, for
  * lookup-partitioned features, [s0, s1) of every task as 2*total ints
  * (-1 for sample-partitioned tasks).  Blocking. */
 recflex_status_t recflex_debug_task_map(recflex_plan_t plan, const int32_t *offsets, int32_t batch_size,
@@ -389,6 +394,45 @@ recflex_status_t recflex_get_task_slots(recflex_plan_t plan, int32_t f, int32_t 
  * the feature's task count unless a static mapping (static_blocks > 0) folds
  * them onto fewer.  host_need[F].  Blocking. */
 recflex_status_t recflex_debug_task_need(recflex_plan_t plan, int32_t *host_need);
+
+/* ---- task order (reading C35; a B200 addition, not in the paper) ---------
+ * The persistent CTAs claim tasks from one counter in task-map order, and the
+ * task map concatenates the features in the plan's task order (the paper:
+ * feature order, as blockIdx.x).  The order changes neither what a task
+ * computes nor where it stores (outputs are bitwise identical under every
+ * order); it changes which work overlaps and how long the kernel's tail is.
+ * Heuristics over the estimated bytes per task (per_block bags of
+ * coverage * mean_len rows, or per_block lookups, times the row pitch):    */
+#define RECFLEX_ORDER_FEATURE 0 /* feature order (the paper's)                    */
+#define RECFLEX_ORDER_LPT 1     /* longest estimated task first (stable)          */
+#define RECFLEX_ORDER_SPT 2     /* shortest estimated task first (stable)         */
+#define RECFLEX_NUM_ORDERS 3
+/* order[F]: a permutation of 0..F-1 (position -> feature) or NULL = feature
+ * order.  INVALID_ARG if not a permutation.  Setup call: synchronises the
+ * device.  Part of the exported plan ("order"). */
+recflex_status_t recflex_set_task_order(recflex_plan_t plan, const int32_t *order);
+/* Output layout: follow_task_order = 0 (default) -> out[s][col_f..col_f+d_f)
+ * with the features concatenated in feature order (the paper's); 1 -> in the
+ * plan's task order, so features whose tasks run back to back write adjacent
+ * columns (a later recflex_set_task_order moves the columns with it).
+ * NOT_SUPPORTED if a feature's schedule needs a 16-byte aligned column it
+ * would not get.  Setup call: synchronises the device.  col[F] of
+ * recflex_get_columns receives every feature's first output column. */
+recflex_status_t recflex_set_column_order(recflex_plan_t plan, int32_t follow_task_order);
+recflex_status_t recflex_get_columns(recflex_plan_t plan, int64_t *col);
+/* order[F] receives the plan's current task order. */
+recflex_status_t recflex_get_task_order(recflex_plan_t plan, int32_t *order);
+/* order[F] receives heuristic `kind` (RECFLEX_ORDER_*) for the plan's current
+ * schedules, without applying it. */
+recflex_status_t recflex_task_order_heuristic(recflex_plan_t plan, int32_t kind, int32_t *order);
+/* Times the plan's current kernel under every heuristic order on one batch
+ * (device pointers; median of reps forwards, L2 flushed before each), keeps
+ * the fastest (ties: the lower kind).  *chosen (nullable) receives its kind,
+ * ms[RECFLEX_NUM_ORDERS] (nullable) the medians.  Blocking; allocates
+ * scratch; the plan keeps its previous order on error. */
+recflex_status_t recflex_select_task_order(recflex_plan_t plan, const int32_t *indices, const int32_t *offsets,
+                                           int32_t batch_size, const void *const *tables, int32_t reps,
+                                           int32_t *chosen, float *ms, void *stream);
 
 /* Checks offsets (offsets[0]==0, monotone, F*B+1 entries) and that every ID of
  * feature f is in [0, rows_f).  Blocking.  RECFLEX_ERR_INDEX_OOB / INVALID_ARG. */

@@ -39,7 +39,8 @@ class TuneOptions(ctypes.Structure):
     _fields_ = [('num_occupancies', ctypes.c_int32), ('occupancies', ctypes.c_int32 * 8),
                 ('reps', ctypes.c_int32), ('pad_waves', ctypes.c_int32), ('max_candidates', ctypes.c_int32),
                 ('verbose', ctypes.c_int32), ('skip_guard', ctypes.c_int32), ('refine', ctypes.c_int32),
-                ('local_mode', ctypes.c_int32), ('stage2_catalog', ctypes.c_int32), ('no_tail', ctypes.c_int32)]
+                ('local_mode', ctypes.c_int32), ('stage2_catalog', ctypes.c_int32), ('no_tail', ctypes.c_int32),
+                ('keep_order', ctypes.c_int32)]
 
 
 class TuneStats(ctypes.Structure):
@@ -49,7 +50,8 @@ class TuneStats(ctypes.Structure):
                 ('best_occupancy', ctypes.c_int32), ('best_ms', ctypes.c_double), ('tune_seconds', ctypes.c_double),
                 ('refine_evals', ctypes.c_int64), ('refine_gain', ctypes.c_double),
                 ('two_stage_ms', ctypes.c_double), ('incoming_ms', ctypes.c_double), ('jit_compiles', ctypes.c_int64),
-                ('compile_seconds', ctypes.c_double), ('refine_seconds', ctypes.c_double)]
+                ('compile_seconds', ctypes.c_double), ('refine_seconds', ctypes.c_double),
+                ('task_order', ctypes.c_int32)]
 
 
 class JitInfo(ctypes.Structure):
@@ -128,6 +130,13 @@ SIGNATURES = {
     'recflex_get_jit': (c_int32, [c_void_p, P(c_int32)]),
     'recflex_select_kernel': (c_int32, [c_void_p, c_void_p, c_void_p, c_int32, P(c_void_p), c_int32,
                                         P(ctypes.c_float), P(ctypes.c_float), c_void_p]),
+    'recflex_set_task_order': (c_int32, [c_void_p, P(c_int32)]),
+    'recflex_get_task_order': (c_int32, [c_void_p, P(c_int32)]),
+    'recflex_set_column_order': (c_int32, [c_void_p, c_int32]),
+    'recflex_get_columns': (c_int32, [c_void_p, P(c_int64)]),
+    'recflex_task_order_heuristic': (c_int32, [c_void_p, c_int32, P(c_int32)]),
+    'recflex_select_task_order': (c_int32, [c_void_p, c_void_p, c_void_p, c_int32, P(c_void_p), c_int32,
+                                            P(c_int32), P(ctypes.c_float), c_void_p]),
     'recflex_set_jit_cache_dir': (c_int32, [ctypes.c_char_p]),
     'recflex_jit_generate': (c_int32, [P(c_int32), P(c_int32), P(c_int32), P(c_int32), c_int32, c_int32,
                                        ctypes.c_char_p, ctypes.c_size_t, P(ctypes.c_size_t), P(c_int32), P(c_int32)]),

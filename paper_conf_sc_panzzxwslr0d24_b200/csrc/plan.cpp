@@ -269,12 +269,16 @@ recflex_status_t staged_copy(recflex_plan_s *p, void *d_dst, const void *src, si
     return RECFLEX_OK;
 }
 
+// The device descriptor array lists the features in task order (C35).
 recflex_status_t upload_desc(recflex_plan_s *p, cudaStream_t stream) {
     for (int f = 0; f < p->F; ++f) p->desc[f].table = p->tables[f];
     p->part1.clear();
-    for (int f = 0; f < p->F; ++f)
-        if (p->desc[f].part == 1) p->part1.push_back(f);
-    recflex_status_t st = staged_copy(p, p->ex.d_desc, p->desc.data(), sizeof(FeatureDesc) * p->F, stream);
+    std::vector<FeatureDesc> dv(p->F);
+    for (int e = 0; e < p->F; ++e) {
+        dv[e] = p->desc[feature_at(p, e)];
+        if (dv[e].part == 1) p->part1.push_back(e);
+    }
+    recflex_status_t st = staged_copy(p, p->ex.d_desc, dv.data(), sizeof(FeatureDesc) * p->F, stream);
     if (st != RECFLEX_OK) return st;
     if (!p->part1.empty()) {
         st = staged_copy(p, p->ex.d_part1, p->part1.data(), sizeof(int32_t) * p->part1.size(), stream);
@@ -361,6 +365,100 @@ recflex_status_t run_pipeline(recflex_plan_s *p, const Exec &ex, const int32_t *
     if (rc) return cuda_status_at((cudaError_t)rc, ex.backward ? "backward kernel launch" : "fused kernel launch");
     if (ev) cudaEventRecord(ev->e2, stream);
     return RECFLEX_OK;
+}
+
+// Estimated bytes one task of feature f moves under its schedule (hotness
+// stats only): sample-partitioned tasks hold per_block bags of mean length
+// coverage * mean_len, lookup-partitioned tasks per_block lookups.
+static double task_bytes_estimate(const recflex_plan_s *p, int f) {
+    const FeatureDesc &d = p->desc[f];
+    const recflex_feature_spec_t &sp = p->specs[f];
+    const double rb = (double)d.row_bytes;
+    if (d.part == 1) return (double)d.per_block * rb;
+    const double L = std::max(0.05, (double)sp.mean_len * (double)sp.coverage);
+    return (double)d.per_block * L * rb;
+}
+
+void task_order_of_kind(const recflex_plan_s *p, int kind, std::vector<int32_t> &out) {
+    out.resize(p->F);
+    for (int f = 0; f < p->F; ++f) out[f] = f;
+    if (kind == RECFLEX_ORDER_FEATURE) return;
+    std::vector<double> est(p->F);
+    for (int f = 0; f < p->F; ++f) est[f] = task_bytes_estimate(p, f);
+    if (kind == RECFLEX_ORDER_LPT)
+        std::stable_sort(out.begin(), out.end(), [&](int a, int b) { return est[a] > est[b]; });
+    else
+        std::stable_sort(out.begin(), out.end(), [&](int a, int b) { return est[a] < est[b]; });
+}
+
+// Installs a task order (empty = feature order), the column mode and --
+// optionally -- new schedules as one change: every schedule is validated at
+// the output column it would get first (vector stores need col % 4 == 0), and
+// on error nothing changes.  Setup call: waits for the device (no forward of
+// the old layout still reads the plan's arrays), re-uploads the order-
+// dependent arrays of compiled kernels, marks the descriptors dirty.
+recflex_status_t set_layout(recflex_plan_s *p, const std::vector<int32_t> &order, bool follow,
+                            const std::vector<recflex_schedule_t> *scheds) {
+    std::vector<int32_t> col(p->F);
+    int64_t c = 0;
+    for (int e = 0; e < p->F; ++e) {
+        const int f = (follow && !order.empty()) ? order[e] : e;
+        col[f] = (int32_t)c;
+        c += p->desc[f].dim;
+    }
+    for (int f = 0; f < p->F; ++f) {
+        const FeatureDesc &d = p->desc[f];
+        const recflex_schedule_t s = scheds ? (*scheds)[f] : recflex_schedule_t{d.sched, d.part, d.per_block, d.nalloc};
+        if (!schedule_valid_for(s, d.dim, d.dtype, col[f], (int)p->d_tot)) {
+            if (scheds) return RECFLEX_ERR_INVALID_ARG;
+            set_last_error("column order: a feature's schedule needs a 16-byte aligned output column");
+            return RECFLEX_ERR_NOT_SUPPORTED;
+        }
+    }
+    cudaError_t e = cudaDeviceSynchronize();
+    if (e != cudaSuccess) return cuda_status(e);
+    if (scheds)
+        for (int f = 0; f < p->F; ++f) {
+            const recflex_schedule_t &s = (*scheds)[f];
+            FeatureDesc &d = p->desc[f];
+            if (d.sched != s.sched_id || (d.nalloc > 0) != (s.static_blocks > 0)) ++p->sched_version;
+            p->num_static += (s.static_blocks > 0 ? 1 : 0) - (d.nalloc > 0 ? 1 : 0);
+            d.sched = s.sched_id;
+            d.part = s.part;
+            d.per_block = s.per_block;
+            d.nalloc = s.static_blocks;
+        }
+    for (int f = 0; f < p->F; ++f) p->desc[f].col = col[f];
+    const bool order_changed = order != p->order;
+    p->order = order;
+    p->columns_follow_order = follow;
+    p->desc_dirty = true;
+    p->targets_cache.clear();
+    return order_changed ? jit_upload_var(p) : RECFLEX_OK;
+}
+
+// order: permutation of 0..F-1 (position -> feature) or nullptr = feature order.
+recflex_status_t normalize_order(const recflex_plan_s *p, const int32_t *order, std::vector<int32_t> &o) {
+    o.clear();
+    if (!order) return RECFLEX_OK;
+    std::vector<char> seen(p->F, 0);
+    bool identity = true;
+    for (int e = 0; e < p->F; ++e) {
+        const int32_t f = order[e];
+        if (f < 0 || f >= p->F || seen[f]) return RECFLEX_ERR_INVALID_ARG;
+        seen[f] = 1;
+        identity = identity && f == e;
+    }
+    if (!identity) o.assign(order, order + p->F);
+    return RECFLEX_OK;
+}
+
+recflex_status_t apply_task_order(recflex_plan_s *p, const int32_t *order) {
+    std::vector<int32_t> o;
+    recflex_status_t st = normalize_order(p, order, o);
+    if (st != RECFLEX_OK) return st;
+    if (o == p->order) return RECFLEX_OK;
+    return set_layout(p, o, p->columns_follow_order, nullptr);
 }
 
 }  // namespace recflex
@@ -741,9 +839,10 @@ recflex_status_t recflex_backward(recflex_plan_t p, const int32_t *indices, cons
             if (e != cudaSuccess) return cuda_status(e);
         }
         p->targets_cache.assign(targets, targets + p->F);
-        cudaError_t e = cudaMemcpyAsync(p->d_targets, p->targets_cache.data(), sizeof(float *) * p->F,
-                                        cudaMemcpyHostToDevice, stream);
-        if (e != cudaSuccess) return cuda_status(e);
+        std::vector<float *> tv(p->F);  // device table in task order (C35)
+        for (int e = 0; e < p->F; ++e) tv[e] = p->targets_cache[feature_at(p, e)];
+        recflex_status_t st = staged_copy(p, p->d_targets, tv.data(), sizeof(float *) * p->F, stream);
+        if (st != RECFLEX_OK) return st;
     }
     Exec ex = p->ex;
     ex.backward = true;
@@ -945,9 +1044,10 @@ recflex_status_t recflex_debug_task_map(recflex_plan_t p, const int32_t *offsets
             e = cudaMemcpy(ts.data(), p->ex.d_task_start, sizeof(int32_t) * p->slots_total, cudaMemcpyDeviceToHost);
             if (e != cudaSuccess) return cuda_status(e);
         }
-        for (int f = 0; f < p->F; ++f) {
-            for (int64_t t = h_bs[f]; t < h_bs[f + 1]; ++t) {
-                const int rel = (int)(t - h_bs[f]);
+        for (int e = 0; e < p->F; ++e) {
+            const int f = feature_at(p, e);  // block_start lists task-order positions (C35)
+            for (int64_t t = h_bs[e]; t < h_bs[e + 1]; ++t) {
+                const int rel = (int)(t - h_bs[e]);
                 if (p->desc[f].part == 1 && p->desc[f].nalloc == 0) {
                     h_ranges[2 * t] = ts[p->desc[f].slot_base + rel];
                     h_ranges[2 * t + 1] = ts[p->desc[f].slot_base + rel + 1];
@@ -970,8 +1070,109 @@ recflex_status_t recflex_get_task_slots(recflex_plan_t p, int32_t f, int32_t *sl
 recflex_status_t recflex_debug_task_need(recflex_plan_t p, int32_t *host_need) {
     if (!p || !host_need) return RECFLEX_ERR_INVALID_ARG;
     DeviceGuard guard(p->device);
-    cudaError_t e = cudaMemcpy(host_need, p->ex.d_need, sizeof(int32_t) * p->F, cudaMemcpyDeviceToHost);
-    return e == cudaSuccess ? RECFLEX_OK : cuda_status(e);
+    std::vector<int32_t> need(p->F);
+    cudaError_t e = cudaMemcpy(need.data(), p->ex.d_need, sizeof(int32_t) * p->F, cudaMemcpyDeviceToHost);
+    if (e != cudaSuccess) return cuda_status(e);
+    for (int i = 0; i < p->F; ++i) host_need[feature_at(p, i)] = need[i];  // back to feature order
+    return RECFLEX_OK;
+}
+
+recflex_status_t recflex_set_task_order(recflex_plan_t p, const int32_t *order) {
+    if (!p) return RECFLEX_ERR_INVALID_ARG;
+    DeviceGuard guard(p->device);
+    return apply_task_order(p, order);
+}
+
+recflex_status_t recflex_set_column_order(recflex_plan_t p, int32_t follow_task_order) {
+    if (!p || follow_task_order < 0 || follow_task_order > 1) return RECFLEX_ERR_INVALID_ARG;
+    DeviceGuard guard(p->device);
+    if ((follow_task_order != 0) == p->columns_follow_order) return RECFLEX_OK;
+    return set_layout(p, p->order, follow_task_order != 0, nullptr);
+}
+
+recflex_status_t recflex_get_columns(recflex_plan_t p, int64_t *col) {
+    if (!p || !col) return RECFLEX_ERR_INVALID_ARG;
+    for (int f = 0; f < p->F; ++f) col[f] = p->desc[f].col;
+    return RECFLEX_OK;
+}
+
+recflex_status_t recflex_get_task_order(recflex_plan_t p, int32_t *order) {
+    if (!p || !order) return RECFLEX_ERR_INVALID_ARG;
+    for (int e = 0; e < p->F; ++e) order[e] = feature_at(p, e);
+    return RECFLEX_OK;
+}
+
+recflex_status_t recflex_task_order_heuristic(recflex_plan_t p, int32_t kind, int32_t *order) {
+    if (!p || !order || kind < 0 || kind >= RECFLEX_NUM_ORDERS) return RECFLEX_ERR_INVALID_ARG;
+    std::vector<int32_t> o;
+    task_order_of_kind(p, kind, o);
+    std::copy(o.begin(), o.end(), order);
+    return RECFLEX_OK;
+}
+
+// Measured choice among the task-order heuristics (C35): time the plan's
+// current kernel under each order on the caller's batch (median of reps
+// forwards, L2 flushed before each), keep the fastest (ties: the lower kind).
+recflex_status_t recflex_select_task_order(recflex_plan_t p, const int32_t *indices, const int32_t *offsets,
+                                           int32_t B, const void *const *tables, int32_t reps, int32_t *chosen,
+                                           float *ms_out, void *stream_) {
+    if (!p || !indices || !offsets || !tables || B <= 0 || B > p->max_batch) return RECFLEX_ERR_INVALID_ARG;
+    NvtxRange nvtx("recflex_select_task_order");
+    DeviceGuard guard(p->device);
+    cudaStream_t stream = (cudaStream_t)stream_;
+    if (p->use_jit && !jit_ready(p, p->k)) {
+        int k = p->k;
+        recflex_status_t st = jit_compile_plan(p, &k, 1);
+        if (st != RECFLEX_OK) return st;
+    }
+    float *out = nullptr, *flush = nullptr;
+    const size_t flush_bytes = size_t(256) << 20;  // 2x L2
+    cudaError_t e = cudaMalloc(&out, sizeof(float) * (size_t)B * p->d_tot);
+    if (e == cudaSuccess) e = cudaMalloc(&flush, flush_bytes);
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+    if (e == cudaSuccess) e = cudaEventCreate(&e0);
+    if (e == cudaSuccess) e = cudaEventCreate(&e1);
+    recflex_status_t st = e == cudaSuccess ? RECFLEX_OK : cuda_status(e);
+    const std::vector<int32_t> keep = p->order;
+    float med[RECFLEX_NUM_ORDERS] = {0.f};
+    std::vector<std::vector<int32_t>> orders(RECFLEX_NUM_ORDERS);
+    for (int kind = 0; kind < RECFLEX_NUM_ORDERS && st == RECFLEX_OK; ++kind) {
+        task_order_of_kind(p, kind, orders[kind]);
+        st = apply_task_order(p, orders[kind].data());
+        std::vector<float> ms;
+        for (int r = 0; r < std::max(3, reps) + 1 && st == RECFLEX_OK; ++r) {
+            flush_launch(flush, flush_bytes, stream);
+            cudaEventRecord(e0, stream);
+            st = recflex_forward(p, indices, offsets, B, tables, out, stream);
+            cudaEventRecord(e1, stream);
+            e = cudaEventSynchronize(e1);
+            if (e != cudaSuccess) st = cuda_status(e);
+            float t = 0;
+            cudaEventElapsedTime(&t, e0, e1);
+            if (r > 0) ms.push_back(t);
+        }
+        if (!ms.empty()) {
+            std::sort(ms.begin(), ms.end());
+            med[kind] = ms[ms.size() / 2];
+        }
+    }
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    cudaFree(out);
+    cudaFree(flush);
+    if (st != RECFLEX_OK) {
+        apply_task_order(p, keep.empty() ? nullptr : keep.data());
+        return st;
+    }
+    int best = 0;
+    for (int kind = 1; kind < RECFLEX_NUM_ORDERS; ++kind)
+        if (med[kind] < med[best]) best = kind;
+    st = apply_task_order(p, orders[best].data());
+    if (st != RECFLEX_OK) return st;
+    if (chosen) *chosen = best;
+    if (ms_out)
+        for (int kind = 0; kind < RECFLEX_NUM_ORDERS; ++kind) ms_out[kind] = med[kind];
+    return RECFLEX_OK;
 }
 
 recflex_status_t recflex_validate(recflex_plan_t p, const int32_t *indices, const int32_t *offsets, int32_t B,
@@ -1073,7 +1274,14 @@ recflex_status_t recflex_plan_export(recflex_plan_t p, char *buf, size_t cap, si
         if (p->desc[f].nalloc > 0) s += ", " + std::to_string(p->desc[f].nalloc);
         s += "]";
     }
-    s += "], \"kernel\": \"";
+    s += "]";
+    if (!p->order.empty()) {
+        s += ", \"order\": [";
+        for (int e = 0; e < p->F; ++e) s += (e ? ", " : "") + std::to_string(p->order[e]);
+        s += "]";
+    }
+    if (p->columns_follow_order) s += ", \"columns\": \"task-order\"";
+    s += ", \"kernel\": \"";
     s += p->use_jit ? "plan-specialised" : "catalog";
     s += "\"}";
     if (len) *len = s.size() + 1;
@@ -1145,10 +1353,31 @@ recflex_status_t recflex_plan_import(recflex_plan_t p, const char *json) {
             c = save;
         }
         ss[f] = {(int32_t)a, (int32_t)b, (int32_t)d, (int32_t)st};
-        if (!schedule_valid_for(ss[f], p->desc[f].dim, p->desc[f].dtype, p->desc[f].col, (int)p->d_tot))
-            return RECFLEX_ERR_INVALID_ARG;
     }
-    for (int f = 0; f < p->F; ++f) recflex_set_schedule(p, f, &ss[f]);
+    // optional: the task order and column layout (C35); absent = feature order
+    std::vector<int32_t> order;
+    if (const char *oc = std::strstr(json, "\"order\"")) {
+        oc = std::strchr(oc, '[');
+        if (!oc) return RECFLEX_ERR_INVALID_ARG;
+        ++oc;
+        std::vector<int32_t> raw(p->F);
+        for (int e = 0; e < p->F; ++e) {
+            long f = 0;
+            if (!parse_int_after(oc, &f) || f < 0 || f >= p->F) return RECFLEX_ERR_INVALID_ARG;
+            raw[e] = (int32_t)f;
+        }
+        if (normalize_order(p, raw.data(), order) != RECFLEX_OK) return RECFLEX_ERR_INVALID_ARG;
+    }
+    bool follow = false;
+    if (const char *cc = std::strstr(json, "\"columns\"")) {
+        const char *v = std::strchr(cc + 9, '"');
+        follow = v && !std::strncmp(v, "\"task-order\"", 12);
+    }
+    {
+        DeviceGuard guard(p->device);
+        recflex_status_t st = set_layout(p, order, follow, &ss);  // validates every schedule at its column
+        if (st != RECFLEX_OK) return st;
+    }
     p->k = k;
     // optional: which kernel the plan runs (recflex_select_kernel's choice)
     if (const char *kc = std::strstr(json, "\"kernel\"")) {

@@ -65,7 +65,8 @@ struct JitKernel {
     void *module = nullptr;    // CUmodule
     void *function = nullptr;  // CUfunction
     uint64_t sig = 0;          // schedule signature it was generated from (jit_plan_sig)
-    int32_t *d_var = nullptr;  // device: variant id of every feature (this kernel's numbering)
+    int32_t *d_var = nullptr;  // device: variant id per task-order position (this kernel's numbering)
+    std::vector<int32_t> h_var;  // host: variant id per feature (feature order)
     int variants = 0;
     int smem = 0, occ = 0, carveout = 0;
     int regs = 0, local_bytes = 0;
@@ -82,8 +83,17 @@ struct recflex_plan_s {
     int num_sms = 148;
     int64_t d_tot = 0;
     std::vector<recflex_feature_spec_t> specs;
-    std::vector<recflex::FeatureDesc> desc;  // host mirror
-    std::vector<int32_t> part1;              // features with part == 1
+    std::vector<recflex::FeatureDesc> desc;  // host mirror, feature order
+    // Task order (reading C35): the device descriptor array -- and with it the
+    // task map, every per-feature device array (need, npb_eff, block_start,
+    // variant ids, backward targets) and the order in which the persistent
+    // CTAs claim tasks -- lists the features in this order: position e holds
+    // feature order[e].  Empty = feature order (the paper's).
+    std::vector<int32_t> order;
+    // Output layout (C35): false = features concatenated in feature order (the
+    // paper's), true = concatenated in task order (recflex_get_columns).
+    bool columns_follow_order = false;
+    std::vector<int32_t> part1;              // task-order positions with part == 1
     std::vector<const void *> tables;        // cached table pointers
     int k = 4;
     int task_lookups = 4096;  // lookups per task targeted by the default schedules
@@ -160,6 +170,15 @@ recflex_status_t run_pipeline(recflex_plan_s *p, const Exec &ex, const int32_t *
 recflex_status_t upload_desc(recflex_plan_s *p, cudaStream_t stream);
 recflex_status_t staged_copy(recflex_plan_s *p, void *d_dst, const void *src, size_t bytes, cudaStream_t stream);
 bool schedule_valid_for(const recflex_schedule_t &s, int dim, int dtype, int col, int d_tot);
+// feature at task-order position e
+inline int feature_at(const recflex_plan_s *p, int e) { return p->order.empty() ? e : p->order[e]; }
+// task-order heuristics (RECFLEX_ORDER_*): out = permutation, position -> feature
+void task_order_of_kind(const recflex_plan_s *p, int kind, std::vector<int32_t> &out);
+recflex_status_t apply_task_order(recflex_plan_s *p, const int32_t *order);
+recflex_status_t normalize_order(const recflex_plan_s *p, const int32_t *order, std::vector<int32_t> &o);
+recflex_status_t set_layout(recflex_plan_s *p, const std::vector<int32_t> &order, bool follow,
+                            const std::vector<recflex_schedule_t> *scheds);
+recflex_status_t jit_upload_var(recflex_plan_s *p);
 int row_bytes_of(int dim, int dtype);
 recflex_schedule_t default_schedule(const recflex_feature_spec_t &spec, int target, bool small_batch);
 int find_catalog(int family, int G, int VEC, int C, int U, int ET = 0);

@@ -292,7 +292,6 @@ struct Tuner {
                 ex.d_desc = d_desc.p;
                 ex.d_block_start = d_bs.p;
                 ex.d_npb_eff = d_npb.p;
-            ex.d_need = d_need.p;
                 ex.d_need = d_need.p;
                 ex.d_counter = d_counter.p;
                 ex.d_task_start = d_ts.p;
@@ -840,7 +839,15 @@ extern "C" recflex_status_t recflex_tune_ex(recflex_plan_t p, int32_t N, const i
                                    T.reps, nullptr, nullptr, stream);
         if (st != RECFLEX_OK) return st;
     }
+    int32_t order_kind = -1;
+    if (!(opt && opt->keep_order)) {
+        // the task order the final kernel runs fastest under (C35)
+        st = recflex_select_task_order(p, T.batches[0].d_idx, T.batches[0].d_off, T.batches[0].B, p->tables.data(),
+                                       T.reps, &order_kind, nullptr, stream);
+        if (st != RECFLEX_OK) return st;
+    }
     recflex_tune_stats_t s = {};
+    s.task_order = order_kind;
     s.two_stage_ms = two_stage_ms;
     s.incoming_ms = incoming_ms;
     s.jit_compiles = T.jit_compiles;

@@ -174,6 +174,53 @@ class Plan:
               'recflex_select_kernel')
         return dict(jit_ms=j.value, catalog_ms=c.value, kernel='plan-specialised' if self.jit_enabled else 'catalog')
 
+    # -------------------------------------------------------------- task order (reading C35)
+    ORDER_KINDS = ('feature', 'lpt', 'spt')  # RECFLEX_ORDER_*
+
+    @property
+    def task_order(self) -> List[int]:
+        """recflex_get_task_order: position -> feature (the order tasks are claimed in)."""
+        o = (ctypes.c_int32 * self.F)()
+        check(lib.recflex_get_task_order(self._h, o), 'recflex_get_task_order')
+        return list(o)
+
+    @task_order.setter
+    def task_order(self, order: Optional[Sequence[int]]):
+        """recflex_set_task_order: a permutation of range(F), or None = feature order."""
+        if order is not None and len(order) != self.F:
+            raise ValueError('task order: need a permutation of range(F)')
+        arr = None if order is None else (ctypes.c_int32 * self.F)(*[int(f) for f in order])
+        check(lib.recflex_set_task_order(self._h, arr), 'recflex_set_task_order')
+
+    def set_column_order(self, follow_task_order: bool):
+        """recflex_set_column_order: concatenate the pooled outputs in task order (True) or
+        feature order (False, default)."""
+        check(lib.recflex_set_column_order(self._h, 1 if follow_task_order else 0), 'recflex_set_column_order')
+
+    @property
+    def columns(self) -> List[int]:
+        """recflex_get_columns: first output column of every feature."""
+        c = (ctypes.c_int64 * self.F)()
+        check(lib.recflex_get_columns(self._h, c), 'recflex_get_columns')
+        return list(c)
+
+    def task_order_heuristic(self, kind: str) -> List[int]:
+        o = (ctypes.c_int32 * self.F)()
+        check(lib.recflex_task_order_heuristic(self._h, self.ORDER_KINDS.index(kind), o),
+              'recflex_task_order_heuristic')
+        return list(o)
+
+    def select_task_order(self, indices: torch.Tensor, offsets: torch.Tensor, B: int,
+                          tables: Sequence[torch.Tensor], reps: int = 7, stream=None) -> dict:
+        """recflex_select_task_order: time every heuristic order on this batch, keep the fastest."""
+        chosen = ctypes.c_int32()
+        ms = (ctypes.c_float * len(self.ORDER_KINDS))()
+        check(lib.recflex_select_task_order(self._h, _dptr(indices, torch.int32, 'indices'),
+                                            _dptr(offsets, torch.int32, 'offsets'), int(B), self._tables(tables),
+                                            int(reps), ctypes.byref(chosen), ms, _stream_ptr(stream)),
+              'recflex_select_task_order')
+        return dict(order=self.ORDER_KINDS[chosen.value], ms={k: ms[i] for i, k in enumerate(self.ORDER_KINDS)})
+
     # -------------------------------------------------------------- hot path
     def forward(self, indices: torch.Tensor, offsets: torch.Tensor, B: int, tables: Sequence[torch.Tensor],
                 out: Optional[torch.Tensor] = None, stream=None) -> torch.Tensor:
@@ -300,7 +347,7 @@ class Plan:
     def tune(self, batches: Sequence[tuple], tables: Sequence[torch.Tensor], occupancies: Optional[List[int]] = None,
              reps: int = 7, pad_waves: int = 4, max_candidates: int = 0, verbose: bool = False, guard: bool = True,
              refine: bool = False, separate: bool = False, stage2_catalog: bool = False, tail: bool = True,
-             isolated: bool = False, stream=None) -> dict:
+             isolated: bool = False, select_order: bool = True, stream=None) -> dict:
         """recflex_tune_ex over historical batches [(indices, offsets, B), ...]."""
         N = len(batches)
         idx_arr = (ctypes.c_void_p * N)(*[b[0].data_ptr() for b in batches])
@@ -320,6 +367,7 @@ class Plan:
         opt.local_mode = 1 if separate else (2 if isolated else 0)
         opt.stage2_catalog = 1 if stage2_catalog else 0
         opt.no_tail = 0 if tail else 1
+        opt.keep_order = 0 if select_order else 1
         st = _lib.TuneStats()
         check(lib.recflex_tune_ex(self._h, N, idx_arr, off_arr, bs_arr, self._tables(tables), _stream_ptr(stream),
                                   ctypes.byref(opt), ctypes.byref(st)), 'recflex_tune_ex')
@@ -328,7 +376,8 @@ class Plan:
                     guard_won=bool(st.guard_won), refine_evals=st.refine_evals, refine_gain=st.refine_gain,
                     best_occupancy=st.best_occupancy, best_ms=st.best_ms, tune_seconds=st.tune_seconds,
                     two_stage_ms=st.two_stage_ms, incoming_ms=st.incoming_ms, jit_compiles=st.jit_compiles,
-                    compile_seconds=st.compile_seconds, refine_seconds=st.refine_seconds)
+                    compile_seconds=st.compile_seconds, refine_seconds=st.refine_seconds,
+                    task_order=self.ORDER_KINDS[st.task_order] if st.task_order >= 0 else None)
 
     # -------------------------------------------------------------- schedules
     def get_schedule(self, f: int) -> dict:
@@ -354,6 +403,8 @@ class Plan:
 
     # -------------------------------------------------------------- introspection
     def debug_task_map(self, offsets: torch.Tensor, B: int, ranges: bool = False, stream=None):
+        """block_start[F+1] over the task order (entry e = feature task_order[e]) and, with
+        ranges, every task's [s0, s1) (lookup-partitioned features; else (-1, -1))."""
         bs = (ctypes.c_int32 * (self.F + 1))()
         if not ranges:
             check(lib.recflex_debug_task_map(self._h, _dptr(offsets, torch.int32, 'offsets'), int(B), bs, None, 0,

@@ -158,7 +158,11 @@ def model_parts(model, W: int, dtype: str = 'f32', config: str = '', tuned_dir: 
 
 
 def column_order(model, parts: List[List[int]]) -> np.ndarray:
-    """Global column index of every column of the exchanged [B/W][D_tot'] output."""
+    """Global column index of every column of the exchanged [B/W][D_tot'] output.
+
+    parts[r] lists rank r's features in its LOCAL column order: the partition's
+    order for plans with feature-order columns, ShardedEmbedding.column_features
+    for a rank plan whose outputs follow its task order (recflex_set_column_order)."""
     col = np.cumsum([0] + model.dims)
     order = []
     for part in parts:
@@ -324,6 +328,12 @@ class ShardedEmbedding:
         self.plan = Plan(specs, model.batch, device)
         self.d_local = self.dims_per_rank[rank]
         self.d_tot = sum(self.dims_per_rank)
+
+    @property
+    def column_features(self) -> List[int]:
+        """This rank's (global) features in the order of their local output columns."""
+        cols = self.plan.columns
+        return [self.features[i] for i in sorted(range(len(self.features)), key=lambda i: cols[i])]
 
     def forward(self, indices, offsets, B, tables, out_local=None, out=None, group=None, stream=None):
         import torch

@@ -65,6 +65,16 @@ def bitexact(gpu, ref):
     return np.array_equal(gpu, ref.astype(np.float32))
 
 
+def feature_columns(out, plan, dims):
+    """The plan's output reassembled in feature-order concatenation (the oracle's layout):
+    a plan whose outputs follow its task order (reading C35) places feature f at
+    plan.columns[f]."""
+    cols = plan.columns
+    if cols == np.cumsum([0] + list(dims))[:-1].tolist():
+        return out
+    return np.concatenate([out[:, c:c + d] for c, d in zip(cols, dims)], axis=1)
+
+
 def run_plan(case, plan=None, stream=None):
     P = _plan_mod()
     if plan is None:
@@ -141,10 +151,11 @@ def test_full_size_sampled(name, plan_src, mode):
     rng = np.random.default_rng(1)
     samples = np.unique(np.concatenate([[0, b.B - 1], rng.choice(b.B, 1024, replace=False)]))
     ref, lens = sampled_oracle(m, b, samples, case.tables)
+    got = feature_columns(out[samples], plan, m.dims)
     if mode == 'int':
-        assert bitexact(out[samples], ref)
+        assert bitexact(got, ref)
     else:
-        check_tol(out[samples], ref, lens, m.dims)
+        check_tol(got, ref, lens, m.dims)
     del case
     torch.cuda.empty_cache()
 
@@ -502,7 +513,7 @@ def test_sharded1000_rank_plans_sampled():
             idx, off = shard_batch(b, sh.features)
             out = sh.plan.forward(torch.from_numpy(idx).to(dev), torch.from_numpy(off).to(dev), b.B,
                                   [case.tables[f] for f in sh.features]).cpu().numpy()
-            cols = np.concatenate([np.arange(col[f], col[f + 1]) for f in sh.features])
+            cols = np.concatenate([np.arange(col[f], col[f + 1]) for f in sh.column_features])
             assert bitexact(out[samples], ref[:, cols]), (W, r)
             del sh, out
     del case

@@ -18,7 +18,7 @@ import torch
 
 from fullsize import sampled_oracle
 from paper_conf_sc_panzzxwslr0d24_b200 import synth
-from test_gpu_parity import bitexact, check_tol
+from test_gpu_parity import bitexact, check_tol, feature_columns
 
 pytestmark = pytest.mark.gpu
 
@@ -78,7 +78,7 @@ def test_tuned_plan_both_kernels_vs_oracle(config, dtype, mode):
     assert torch.equal(out_cat, out_jit), 'plan-specialised kernel differs from the catalog kernel'
     samples = _samples(b.B)
     ref, lens = sampled_oracle(m, b, samples, tables, dtype)
-    got = out_jit[torch.as_tensor(samples, device=dev)].cpu().numpy()
+    got = feature_columns(out_jit[torch.as_tensor(samples, device=dev)].cpu().numpy(), plan, m.dims)
     if mode == 'int':
         assert bitexact(got, ref)
     else:

@@ -7,6 +7,7 @@ import re
 import pytest
 
 from paper_conf_sc_panzzxwslr0d24_b200 import plan as P
+from paper_conf_sc_panzzxwslr0d24_b200._lib import JIT_CACHE, check, lib
 
 
 def _ids():
@@ -50,12 +51,18 @@ def test_generate_rejects_invalid_entry():
         P.jit_generate([find('group', 4, 4, 1, 4)], [16], [0], 9)    # k outside 1..8
 
 
-def test_compiles_for_sm100a_without_spills_at_k4():
+def test_compiles_for_sm100a_without_spills_at_k4(tmp_path):
     """A heavy-like plan (one GROUP G32 V4 U4 variant, d = 128) compiles with NVRTC
     for sm_100a and keeps everything in registers at the k = 4 cap (64 registers)."""
     find = _ids()
     src, _, _ = P.jit_generate([find('group', 32, 4, 1, 4)] * 3, [128] * 3, [0, 0, 0], 4)
-    cubin, log, _ = P.jit_compile_source(src)
+    # an empty cache directory: a cache hit would return the cubin without the ptxas log
+    check(lib.recflex_set_jit_cache_dir(str(tmp_path).encode()), 'recflex_set_jit_cache_dir')
+    try:
+        cubin, log, hit = P.jit_compile_source(src)
+    finally:
+        check(lib.recflex_set_jit_cache_dir(JIT_CACHE.encode()), 'recflex_set_jit_cache_dir')
+    assert not hit
     assert cubin[:4] == b'\x7fELF'
     m = re.search(r'(\d+) bytes spill stores, (\d+) bytes spill loads', log)
     assert m and m.group(1) == '0' and m.group(2) == '0', log
