@@ -28,6 +28,8 @@ def main():
     ap.add_argument('--worlds', default='1,2,4,8')
     ap.add_argument('--reps', type=int, default=10)
     ap.add_argument('--no-jit', action='store_true')
+    ap.add_argument('--tuned-dir', default=os.path.join(ROOT, 'configs', 'tuned'),
+                    help='where the per-rank plans <config>_w<W>_r<R>.json are read from')
     a = ap.parse_args()
     import torch
     from paper_conf_sc_panzzxwslr0d24_b200 import synth
@@ -46,7 +48,7 @@ def main():
         per_rank = []
         for r in range(W):
             sh = ShardedEmbedding(model, r, W, device=0, parts=parts)
-            path = os.path.join(ROOT, 'configs', 'tuned', f'{a.config}_w{W}_r{r}.json')
+            path = os.path.join(a.tuned_dir, f'{a.config}_w{W}_r{r}.json')
             tuned = os.path.exists(path)
             if tuned:
                 sh.plan.import_(json.load(open(path)))
