@@ -184,22 +184,37 @@ int map_launch(const MapArgs &a, void *stream) {
 // ---------------------------------------------------------------------------
 // Fill kernel (only for lookup-partitioned features): task_start[q] = first
 // sample whose bag starts in lookup window q (Fig. 8's d_task_map payload for
-// adaptive tasks).  Thread per (feature, sample); disjoint writes.
+// adaptive tasks).  CTA (chunk, k): part-1 feature k, samples [chunk * kFillSpan,
+// +kFillSpan), kFillPer per thread with independent coalesced offset loads (one
+// wave instead of a thread per sample -- the per-sample form was a chain of
+// dependent loads repeated over ~10 waves: 29 us on sharded1000).  Disjoint writes.
 // ---------------------------------------------------------------------------
+constexpr int kFillPer = 16;
+constexpr int kFillSpan = 256 * kFillPer;
+
 __global__ void __launch_bounds__(256) recflex_fill_kernel(FillArgs a) {
     asm volatile("griddepcontrol.wait;" ::: "memory");
-    const int k = blockIdx.y;
-    const int f = a.part1_features[k];
+    const int f = a.part1_features[blockIdx.y];
     const FeatureDesc &fd = a.desc[f];
-    const int s = blockIdx.x * blockDim.x + threadIdx.x;
-    if (s < a.B) {
-        const int32_t *offs = a.offsets + (size_t)fd.in_feature * a.B;
-        const int base = offs[0];
-        const int npb = a.npb_eff[f];
-        const int blocks = a.need[f];  // needed tasks (a static feature allocates a different count)
-        int32_t *ts = a.task_start + fd.slot_base;
-        const int q_hi = (offs[s] - base) / npb;
-        const int q_lo = (s == 0) ? -1 : (offs[s - 1] - base) / npb;
+    const int32_t *offs = a.offsets + (size_t)fd.in_feature * a.B;
+    const int base = offs[0];
+    const int npb = a.npb_eff[f];
+    const int blocks = a.need[f];  // needed tasks (a static feature allocates a different count)
+    int32_t *ts = a.task_start + fd.slot_base;
+    const int s0 = blockIdx.x * kFillSpan + threadIdx.x;
+    int cur[kFillPer], prev[kFillPer];
+#pragma unroll
+    for (int i = 0; i < kFillPer; ++i) {
+        const int s = s0 + i * 256;
+        cur[i] = s < a.B ? offs[s] : 0;
+        prev[i] = (s < a.B && s > 0) ? offs[s - 1] : base;
+    }
+#pragma unroll
+    for (int i = 0; i < kFillPer; ++i) {
+        const int s = s0 + i * 256;
+        if (s >= a.B) break;
+        const int q_hi = (cur[i] - base) / npb;
+        const int q_lo = (s == 0) ? -1 : (prev[i] - base) / npb;
         for (int q = q_lo + 1; q <= q_hi && q <= blocks; ++q) ts[q] = s;
         if (s == a.B - 1)
             for (int q = q_hi + 1; q <= blocks; ++q) ts[q] = a.B;
@@ -207,9 +222,9 @@ __global__ void __launch_bounds__(256) recflex_fill_kernel(FillArgs a) {
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
 }
 
-int fill_launch(const FillArgs &a, int grid_x, bool pdl, void *stream) {
+int fill_launch(const FillArgs &a, int B, bool pdl, void *stream) {
     cudaLaunchConfig_t lc = {};
-    lc.gridDim = dim3(grid_x, a.num_part1);
+    lc.gridDim = dim3((B + kFillSpan - 1) / kFillSpan, a.num_part1);
     lc.blockDim = dim3(256);
     lc.stream = (cudaStream_t)stream;
     cudaLaunchAttribute attr[1];

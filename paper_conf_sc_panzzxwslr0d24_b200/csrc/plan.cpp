@@ -318,7 +318,7 @@ recflex_status_t run_pipeline(recflex_plan_s *p, const Exec &ex, const int32_t *
         fa.num_part1 = ex.num_part1;
         fa.B = B;
         fa.task_start = ex.d_task_start;
-        rc = fill_launch(fa, (B + 255) / 256, p->pdl, stream);
+        rc = fill_launch(fa, B, p->pdl, stream);
         if (rc) return cuda_status_at((cudaError_t)rc, "fill kernel launch");
     }
     if (ev) cudaEventRecord(ev->e1, stream);
@@ -1028,7 +1028,7 @@ recflex_status_t recflex_debug_task_map(recflex_plan_t p, const int32_t *offsets
         fa.num_part1 = p->ex.num_part1;
         fa.B = B;
         fa.task_start = p->ex.d_task_start;
-        rc = fill_launch(fa, (B + 255) / 256, false, stream);
+        rc = fill_launch(fa, B, false, stream);
         if (rc) return cuda_status((cudaError_t)rc);
     }
     cudaError_t e = cudaMemcpyAsync(h_bs, p->ex.d_block_start, sizeof(int32_t) * (p->F + 1), cudaMemcpyDeviceToHost,

@@ -227,7 +227,7 @@ int backward_launch(int k, const FusedArgs &a, const LaunchCfg &cfg, void *strea
 int fused_prepare(int k, int device, int smem_bytes, int carveout);                              // cudaFuncSetAttribute
 int fused_occupancy(int k, int smem_bytes, int *blocks, int *regs, int *spill);
 int map_launch(const MapArgs &a, void *stream);
-int fill_launch(const FillArgs &a, int grid_x, bool pdl, void *stream);
+int fill_launch(const FillArgs &a, int B, bool pdl, void *stream);
 int validate_launch(const FeatureDesc *desc, int F, int in_F, const int32_t *indices, const int32_t *offsets, int B,
                     int32_t *flag, void *stream);
 int remap_launch(const int32_t *src, int32_t *dst, int64_t n, int64_t shift, int64_t rows, void *stream);

@@ -32,6 +32,9 @@ def main():
     ap.add_argument('--stage2-catalog', action='store_true', help='stage 2 on the catalog kernel (no NVRTC)')
     ap.add_argument('--no-tail', action='store_true', help="stage 1 = the paper's plain block-time sum")
     ap.add_argument('--isolated', action='store_true', help='stage 1: one padded launch per candidate (C34)')
+    ap.add_argument('--from-tuned', action='store_true',
+                    help='start from configs/tuned/<name>.json (its schedules, task order and column layout '
+                         'are the incoming plan the guard compares against)')
     a = ap.parse_args()
     import torch
     from paper_conf_sc_panzzxwslr0d24_b200 import synth
@@ -54,6 +57,11 @@ def main():
                 rows, dim = model.tables[t]
                 phys[t] = synth.make_table_stored(t, rows, dim, a.dtype, 'float', device=dev, seed=model.seed)
         tables = [phys[model.features[f].table] for f in feats]
+        name = f'{a.config}_w{a.world}_r{r}' if a.dtype == 'f32' else f'{a.config}_{a.dtype}_w{a.world}_r{r}'
+        src = os.path.join(ROOT, 'configs', 'tuned', name + '.json')
+        if a.from_tuned and os.path.exists(src):
+            with open(src) as fh:
+                sh.plan.import_(json.load(fh))
         hist = []
         for full in fulls:
             idx, off = shard_batch(full, feats)
@@ -64,7 +72,6 @@ def main():
                           tail=not a.no_tail, isolated=a.isolated)
         st['wall_s'] = time.time() - t0
         state = sh.plan.export()
-        name = f'{a.config}_w{a.world}_r{r}' if a.dtype == 'f32' else f'{a.config}_{a.dtype}_w{a.world}_r{r}'
         with open(os.path.join(a.out, name + '.json'), 'w') as fh:
             json.dump(state, fh)
         with open(os.path.join(a.out, name + '.log'), 'w') as fh:
