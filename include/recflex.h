@@ -235,6 +235,8 @@ typedef struct {
                                 paper's plain sum of block times W_c (Eq. 3)              */
     int32_t keep_order;      /* 0: after kernel selection, recflex_select_task_order on the
                                 first batch (3 x reps forwards); 1: keep the plan's order  */
+    int32_t keep_l2;         /* 0: then recflex_select_l2_policy (plan-specialised kernel
+                                only; <= 3 compiles + 3 x reps forwards); 1: keep it       */
 } recflex_tune_options_t;
 
 typedef struct {
@@ -255,6 +257,7 @@ typedef struct {
     double compile_seconds;   /* wall time spent compiling them                    */
     double refine_seconds;    /* wall time of the refinement stage                 */
     int32_t task_order;       /* RECFLEX_ORDER_* kept by the order selection, -1 = not run */
+    int32_t l2_policy;        /* recflex_select_l2_policy's choice, -1 = not run           */
 } recflex_tune_stats_t;
 
 /* Two-stage interference-simulated tuning over num_batches historical batches
@@ -420,6 +423,35 @@ recflex_status_t recflex_set_task_order(recflex_plan_t plan, const int32_t *orde
  * recflex_get_columns receives every feature's first output column. */
 recflex_status_t recflex_set_column_order(recflex_plan_t plan, int32_t follow_task_order);
 recflex_status_t recflex_get_columns(recflex_plan_t plan, int64_t *col);
+/* ---- L2 eviction priority of row loads (reading C36; a B200 addition) ----
+ * Within one batch the rows of a small table recur (sharded1000: 62 % of the
+ * gathered row bytes are repeats), but the rows of large tables stream
+ * through L2 and evict them.  The plan-specialised kernel can tag a feature's
+ * row loads with an L2 cache policy (createpolicy + ld...L2::cache_hint):    */
+#define RECFLEX_L2_DEFAULT 0
+#define RECFLEX_L2_EVICT_FIRST 1  /* stream: rows rarely recur within a batch   */
+#define RECFLEX_L2_EVICT_LAST 2   /* keep: small table, rows recur              */
+/* policy[F] (values above) or NULL = default for every feature.  Takes effect
+ * in the next compiled plan-specialised kernel (part of its signature; the
+ * catalog kernel ignores it).  INVALID_ARG on an unknown value.  Part of the
+ * exported plan ("l2"). */
+recflex_status_t recflex_set_l2_policy(recflex_plan_t plan, const int32_t *policy);
+recflex_status_t recflex_get_l2_policy(recflex_plan_t plan, int32_t *policy);
+/* The heuristic policy for an L2 of l2_bytes: evict_last when the table is at
+ * most l2_bytes / 4 and a batch looks each row up at least once on average
+ * (max_batch * mean_len * coverage >= rows); evict_first when the table is
+ * larger than the L2 or a batch looks up fewer than half its rows; else
+ * default.  Writes policy[F]; does not apply it. */
+recflex_status_t recflex_l2_policy_heuristic(recflex_plan_t plan, int64_t l2_bytes, int32_t *policy);
+/* Measured choice (plan-specialised kernel only; NOT_SUPPORTED otherwise):
+ * candidate 0 = no hints, 1 = the heuristic policy, 2 = its evict_last part
+ * alone; each compiled (NVRTC, disk cache) and timed on one batch (median of
+ * reps forwards, L2 flushed before each); the fastest is kept (ties: 0, then
+ * 2, then 1).  *chosen / ms[3] (nullable) receive the choice and the medians.
+ * Blocking; allocates scratch; the previous policy is kept on error. */
+recflex_status_t recflex_select_l2_policy(recflex_plan_t plan, const int32_t *indices, const int32_t *offsets,
+                                          int32_t batch_size, const void *const *tables, int32_t reps,
+                                          int64_t l2_bytes, int32_t *chosen, float *ms, void *stream);
 /* order[F] receives the plan's current task order. */
 recflex_status_t recflex_get_task_order(recflex_plan_t plan, int32_t *order);
 /* order[F] receives heuristic `kind` (RECFLEX_ORDER_*) for the plan's current

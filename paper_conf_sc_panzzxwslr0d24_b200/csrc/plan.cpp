@@ -1090,6 +1090,45 @@ recflex_status_t recflex_set_column_order(recflex_plan_t p, int32_t follow_task_
     return set_layout(p, p->order, follow_task_order != 0, nullptr);
 }
 
+recflex_status_t recflex_set_l2_policy(recflex_plan_t p, const int32_t *policy) {
+    if (!p) return RECFLEX_ERR_INVALID_ARG;
+    std::vector<int8_t> l2;
+    if (policy) {
+        bool any = false;
+        for (int f = 0; f < p->F; ++f) {
+            if (policy[f] < RECFLEX_L2_DEFAULT || policy[f] > RECFLEX_L2_EVICT_LAST) return RECFLEX_ERR_INVALID_ARG;
+            any = any || policy[f] != RECFLEX_L2_DEFAULT;
+        }
+        if (any) l2.assign(policy, policy + p->F);
+    }
+    if (l2 != p->l2) {
+        p->l2.swap(l2);
+        ++p->sched_version;  // the plan-specialised kernel compiles the policies in
+    }
+    return RECFLEX_OK;
+}
+
+recflex_status_t recflex_get_l2_policy(recflex_plan_t p, int32_t *policy) {
+    if (!p || !policy) return RECFLEX_ERR_INVALID_ARG;
+    for (int f = 0; f < p->F; ++f) policy[f] = p->l2.empty() ? 0 : p->l2[f];
+    return RECFLEX_OK;
+}
+
+recflex_status_t recflex_l2_policy_heuristic(recflex_plan_t p, int64_t l2_bytes, int32_t *policy) {
+    if (!p || !policy || l2_bytes <= 0) return RECFLEX_ERR_INVALID_ARG;
+    for (int f = 0; f < p->F; ++f) {
+        const recflex_feature_spec_t &sp = p->specs[f];
+        const double table = (double)sp.num_rows * (double)p->desc[f].row_bytes;
+        const double lookups = (double)p->max_batch * (double)sp.mean_len * (double)sp.coverage;
+        const double reuse = lookups / std::max(1.0, (double)sp.num_rows);  // lookups per row per batch
+        int pol = RECFLEX_L2_DEFAULT;
+        if (table <= 0.25 * (double)l2_bytes && reuse >= 1.0) pol = RECFLEX_L2_EVICT_LAST;
+        else if (table >= (double)l2_bytes || reuse < 0.5) pol = RECFLEX_L2_EVICT_FIRST;
+        policy[f] = pol;
+    }
+    return RECFLEX_OK;
+}
+
 recflex_status_t recflex_get_columns(recflex_plan_t p, int64_t *col) {
     if (!p || !col) return RECFLEX_ERR_INVALID_ARG;
     for (int f = 0; f < p->F; ++f) col[f] = p->desc[f].col;
@@ -1281,6 +1320,11 @@ recflex_status_t recflex_plan_export(recflex_plan_t p, char *buf, size_t cap, si
         s += "]";
     }
     if (p->columns_follow_order) s += ", \"columns\": \"task-order\"";
+    if (!p->l2.empty()) {
+        s += ", \"l2\": [";
+        for (int f = 0; f < p->F; ++f) s += (f ? ", " : "") + std::to_string((int)p->l2[f]);
+        s += "]";
+    }
     s += ", \"kernel\": \"";
     s += p->use_jit ? "plan-specialised" : "catalog";
     s += "\"}";
@@ -1368,6 +1412,19 @@ recflex_status_t recflex_plan_import(recflex_plan_t p, const char *json) {
         }
         if (normalize_order(p, raw.data(), order) != RECFLEX_OK) return RECFLEX_ERR_INVALID_ARG;
     }
+    // optional: L2 eviction priorities (C36); absent = default everywhere
+    std::vector<int32_t> l2;
+    if (const char *lc = std::strstr(json, "\"l2\"")) {
+        lc = std::strchr(lc, '[');
+        if (!lc) return RECFLEX_ERR_INVALID_ARG;
+        ++lc;
+        l2.resize(p->F);
+        for (int f = 0; f < p->F; ++f) {
+            long v = 0;
+            if (!parse_int_after(lc, &v) || v < 0 || v > 2) return RECFLEX_ERR_INVALID_ARG;
+            l2[f] = (int32_t)v;
+        }
+    }
     bool follow = false;
     if (const char *cc = std::strstr(json, "\"columns\"")) {
         const char *v = std::strchr(cc + 9, '"');
@@ -1378,6 +1435,7 @@ recflex_status_t recflex_plan_import(recflex_plan_t p, const char *json) {
         recflex_status_t st = set_layout(p, order, follow, &ss);  // validates every schedule at its column
         if (st != RECFLEX_OK) return st;
     }
+    recflex_set_l2_policy(p, l2.empty() ? nullptr : l2.data());
     p->k = k;
     // optional: which kernel the plan runs (recflex_select_kernel's choice)
     if (const char *kc = std::strstr(json, "\"kernel\"")) {

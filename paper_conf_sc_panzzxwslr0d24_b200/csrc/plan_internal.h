@@ -93,6 +93,9 @@ struct recflex_plan_s {
     // Output layout (C35): false = features concatenated in feature order (the
     // paper's), true = concatenated in task order (recflex_get_columns).
     bool columns_follow_order = false;
+    // L2 eviction priority of every feature's row loads in the plan-specialised
+    // kernel (C36): 0 default, 1 evict_first, 2 evict_last.  Empty = all 0.
+    std::vector<int8_t> l2;
     std::vector<int32_t> part1;              // task-order positions with part == 1
     std::vector<const void *> tables;        // cached table pointers
     int k = 4;

@@ -36,24 +36,47 @@ namespace recflex {
 // ---- loads ---------------------------------------------------------------
 // Rows are gathered once and never reused by the CTA: bypass L1 allocation so
 // the (reused) index lines stay resident.  `.nc` = read-only path.
-template <int VEC>
-__device__ __forceinline__ void ld_row(const float *p, float (&v)[VEC]);
+//
+// L2 eviction priority of a feature's row loads (reading C36), a compile-time
+// P of the plan-specialised kernel: 0 = default, 1 = evict_first (rows of
+// large tables that rarely recur within a batch: let them stream through L2),
+// 2 = evict_last (small tables whose rows recur: keep them across the stream).
+// The policy is a 64-bit operand built by createpolicy (a uniform value).
+template <int P>
+__device__ __forceinline__ uint64_t l2pol() {
+    uint64_t pol = 0;
+    if constexpr (P == 1) asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    else if constexpr (P == 2) asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
 
-template <>
-__device__ __forceinline__ void ld_row<1>(const float *p, float (&v)[1]) {
-    asm("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(v[0]) : "l"(p));
-}
-template <>
-__device__ __forceinline__ void ld_row<4>(const float *p, float (&v)[4]) {
-    asm("ld.global.nc.L1::no_allocate.v4.f32 {%0, %1, %2, %3}, [%4];"
-        : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3])
-        : "l"(p));
-}
-template <>
-__device__ __forceinline__ void ld_row<8>(const float *p, float (&v)[8]) {
-    asm("ld.global.nc.L1::no_allocate.v8.f32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
-        : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3]), "=f"(v[4]), "=f"(v[5]), "=f"(v[6]), "=f"(v[7])
-        : "l"(p));
+template <int VEC, int P = 0>
+__device__ __forceinline__ void ld_row(const float *p, float (&v)[VEC]) {
+    static_assert(VEC == 1 || VEC == 4 || VEC == 8, "1, 4 or 8 floats");
+    if constexpr (P == 0) {
+        if constexpr (VEC == 1)
+            asm("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(v[0]) : "l"(p));
+        else if constexpr (VEC == 4)
+            asm("ld.global.nc.L1::no_allocate.v4.f32 {%0, %1, %2, %3}, [%4];"
+                : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3])
+                : "l"(p));
+        else
+            asm("ld.global.nc.L1::no_allocate.v8.f32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
+                : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3]), "=f"(v[4]), "=f"(v[5]), "=f"(v[6]), "=f"(v[7])
+                : "l"(p));
+    } else {
+        const uint64_t pol = l2pol<P>();
+        if constexpr (VEC == 1)
+            asm("ld.global.nc.L1::no_allocate.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v[0]) : "l"(p), "l"(pol));
+        else if constexpr (VEC == 4)
+            asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.f32 {%0, %1, %2, %3}, [%4], %5;"
+                : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3])
+                : "l"(p), "l"(pol));
+        else
+            asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v8.f32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8], %9;"
+                : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3]), "=f"(v[4]), "=f"(v[5]), "=f"(v[6]), "=f"(v[7])
+                : "l"(p), "l"(pol));
+    }
 }
 
 __device__ __forceinline__ int ld_idx(const int32_t *p) { return __ldg(p); }
@@ -71,9 +94,25 @@ __device__ __forceinline__ int ld_idx(const int32_t *p) { return __ldg(p); }
 //          (bytes [d, d+8) of the row); value = fma(scale, q, bias) in fp32.
 //          q -> fp32 without I2F: the code byte is placed in the mantissa of
 //          2^23 (PRMT) and 2^23 + 128 subtracted (exact).
-template <int NW>
+template <int NW, int P = 0>
 __device__ __forceinline__ void ld_words(const void *p, unsigned (&w)[NW]) {
-    if constexpr (NW == 1) {
+    if constexpr (P != 0) {
+        const uint64_t pol = l2pol<P>();
+        if constexpr (NW == 1)
+            asm("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(w[0]) : "l"(p), "l"(pol));
+        else if constexpr (NW == 2)
+            asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.b32 {%0, %1}, [%2], %3;"
+                : "=r"(w[0]), "=r"(w[1])
+                : "l"(p), "l"(pol));
+        else if constexpr (NW == 4)
+            asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.b32 {%0, %1, %2, %3}, [%4], %5;"
+                : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3])
+                : "l"(p), "l"(pol));
+        else
+            asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8], %9;"
+                : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]), "=r"(w[4]), "=r"(w[5]), "=r"(w[6]), "=r"(w[7])
+                : "l"(p), "l"(pol));
+    } else if constexpr (NW == 1) {
         asm("ld.global.nc.L1::no_allocate.b32 %0, [%1];" : "=r"(w[0]) : "l"(p));
     } else if constexpr (NW == 2) {
         asm("ld.global.nc.L1::no_allocate.v2.b32 {%0, %1}, [%2];" : "=r"(w[0]), "=r"(w[1]) : "l"(p));
@@ -116,8 +155,9 @@ struct RowFrag<RECFLEX_DTYPE_F32, VEC> {
 #pragma unroll
         for (int e = 0; e < VEC; ++e) x[e] = 0.f;
     }
+    template <int P = 0>
     __device__ __forceinline__ void load(const char *row, int col, int) {
-        ld_row<VEC>(reinterpret_cast<const float *>(row) + col, x);
+        ld_row<VEC, P>(reinterpret_cast<const float *>(row) + col, x);
     }
     __device__ __forceinline__ void add_to(float (&acc)[VEC]) const {
 #pragma unroll
@@ -132,7 +172,8 @@ struct RowFrag<RECFLEX_DTYPE_F16, VEC> {
 #pragma unroll
         for (int e = 0; e < VEC / 2; ++e) w[e] = 0u;
     }
-    __device__ __forceinline__ void load(const char *row, int col, int) { ld_words<VEC / 2>(row + 2 * col, w); }
+    template <int P = 0>
+    __device__ __forceinline__ void load(const char *row, int col, int) { ld_words<VEC / 2, P>(row + 2 * col, w); }
     __device__ __forceinline__ void add_to(float (&acc)[VEC]) const {
 #pragma unroll
         for (int i = 0; i < VEC / 2; ++i) {
@@ -149,7 +190,8 @@ struct RowFrag<RECFLEX_DTYPE_BF16, VEC> {
 #pragma unroll
         for (int e = 0; e < VEC / 2; ++e) w[e] = 0u;
     }
-    __device__ __forceinline__ void load(const char *row, int col, int) { ld_words<VEC / 2>(row + 2 * col, w); }
+    template <int P = 0>
+    __device__ __forceinline__ void load(const char *row, int col, int) { ld_words<VEC / 2, P>(row + 2 * col, w); }
     __device__ __forceinline__ void add_to(float (&acc)[VEC]) const {
 #pragma unroll
         for (int i = 0; i < VEC / 2; ++i) {
@@ -179,7 +221,8 @@ struct RowFrag<RECFLEX_DTYPE_FP8, VEC> {
 #pragma unroll
         for (int e = 0; e < VEC / 4; ++e) w[e] = 0u;
     }
-    __device__ __forceinline__ void load(const char *row, int col, int) { ld_words<VEC / 4>(row + col, w); }
+    template <int P = 0>
+    __device__ __forceinline__ void load(const char *row, int col, int) { ld_words<VEC / 4, P>(row + col, w); }
     __device__ __forceinline__ void add_to(float (&acc)[VEC]) const {
 #pragma unroll
         for (int i = 0; i < VEC / 4; ++i) {
@@ -203,9 +246,10 @@ struct RowFrag<RECFLEX_DTYPE_I8, VEC> {
         for (int e = 0; e < VEC / 4; ++e) w[e] = 0u;
         sb[0] = sb[1] = 0u;
     }
+    template <int P = 0>
     __device__ __forceinline__ void load(const char *row, int col, int d) {
-        ld_words<VEC / 4>(row + col, w);
-        ld_words<2>(row + d, sb);  // 8-byte aligned: d % 8 == 0
+        ld_words<VEC / 4, P>(row + col, w);
+        ld_words<2, P>(row + d, sb);  // 8-byte aligned: d % 8 == 0
     }
     __device__ __forceinline__ void add_to(float (&acc)[VEC]) const {
         const float sc = __uint_as_float(sb[0]), bi = __uint_as_float(sb[1]);
@@ -307,7 +351,7 @@ struct TaskCtx {
 // ---- GROUP family --------------------------------------------------------
 // One bag [lo, hi) pooled by the G lanes of a group: lane lg holds columns
 // p*SPAN + c*G*VEC + lg*VEC (+0..VEC-1); U rows in flight per lane.
-template <int ET, int GT, int VEC, int C, int U>
+template <int ET, int GT, int VEC, int C, int U, int P = 0>
 __device__ __forceinline__ void group_bag(const char *__restrict__ T, unsigned rowb, const int32_t *__restrict__ idx, int d,
                                           int pool, float *__restrict__ orow, int lo, int hi, int lg, int gr) {
     const int G = GT ? GT : gr;  // GT == 0: lane-group size at run time (see kRuntimeG)
@@ -357,7 +401,7 @@ __device__ __forceinline__ void group_bag(const char *__restrict__ T, unsigned r
                     for (int u = 0; u < U; ++u)
 #pragma unroll
                         for (int c = 0; c < C; ++c)
-                            if (ok[c]) v[u][c].load(T + (size_t)id[u] * rowb, colv[c], d);
+                            if (ok[c]) v[u][c].template load<P>(T + (size_t)id[u] * rowb, colv[c], d);
 #pragma unroll
                     for (int u = 0; u < U; ++u)
 #pragma unroll
@@ -380,7 +424,7 @@ __device__ __forceinline__ void group_bag(const char *__restrict__ T, unsigned r
                     for (int u = 0; u < U; ++u)
 #pragma unroll
                         for (int c = 0; c < C; ++c)
-                            if (u < n && ok[c]) v[u][c].load(T + (size_t)id[u] * rowb, colv[c], d);
+                            if (u < n && ok[c]) v[u][c].template load<P>(T + (size_t)id[u] * rowb, colv[c], d);
 #pragma unroll
                     for (int u = 0; u < U; ++u)
                         if (u < n)
@@ -415,7 +459,7 @@ __device__ __forceinline__ void group_bag(const char *__restrict__ T, unsigned r
                 for (int u = 0; u < U; ++u)
 #pragma unroll
                     for (int c = 0; c < C; ++c)
-                        if (ok[c]) v[u][c].load(T + (size_t)id[u] * rowb, colv[c], d);
+                        if (ok[c]) v[u][c].template load<P>(T + (size_t)id[u] * rowb, colv[c], d);
 #pragma unroll
                 for (int u = 0; u < U; ++u)
 #pragma unroll
@@ -434,7 +478,7 @@ __device__ __forceinline__ void group_bag(const char *__restrict__ T, unsigned r
                 for (int u = 0; u < U; ++u)
 #pragma unroll
                     for (int c = 0; c < C; ++c)
-                        if (u < n && ok[c]) v[u][c].load(T + (size_t)id[u] * rowb, colv[c], d);
+                        if (u < n && ok[c]) v[u][c].template load<P>(T + (size_t)id[u] * rowb, colv[c], d);
 #pragma unroll
                 for (int u = 0; u < U; ++u)
                     if (u < n)
@@ -459,7 +503,7 @@ __device__ __forceinline__ void group_bag(const char *__restrict__ T, unsigned r
 // its own group; the next bag's offsets are loaded while the current bag is
 // pooled.  Which group pools a bag does not change the bag's arithmetic (rows
 // in ascending lookup order) -> results are independent of the claim order.
-template <int ET, int GT, int VEC, int C, int U>
+template <int ET, int GT, int VEC, int C, int U, int P = 0>
 RECFLEX_SCHED_FN void sched_group(const char *__restrict__ T, unsigned rowb, int gr, const int32_t *__restrict__ offs,
                                         const int32_t *__restrict__ idx, float *__restrict__ out, int d, int pool,
                                         const OutRoute ro, int s0, int s1, int *bag_ctr) {
@@ -485,7 +529,7 @@ RECFLEX_SCHED_FN void sched_group(const char *__restrict__ T, unsigned rowb, int
             lon = ld_idx(offs + sn);
             hin = ld_idx(offs + sn + 1);
         }
-        group_bag<ET, GT, VEC, C, U>(T, rowb, idx, d, pool, out_row(out, s, ro), lo, hi, lg, G);
+        group_bag<ET, GT, VEC, C, U, P>(T, rowb, idx, d, pool, out_row(out, s, ro), lo, hi, lg, G);
         s = sn;
         lo = lon;
         hi = hin;
@@ -503,7 +547,7 @@ RECFLEX_SCHED_FN void sched_group(const char *__restrict__ T, unsigned rowb, int
 // 32-ID chunk, the next chunk in flight; an iteration consumes R = NG*U IDs
 // (R divides 32 for every catalog entry).  Bags are claimed per warp from the
 // task's counter (results do not depend on which warp pools a bag).
-template <int ET, int GT, int VEC, int C, int U>
+template <int ET, int GT, int VEC, int C, int U, int P = 0>
 RECFLEX_SCHED_FN void sched_warp(const char *__restrict__ T, unsigned rowb, int gr, const int32_t *__restrict__ offs,
                                  const int32_t *__restrict__ idx, float *__restrict__ out, int d, int pool,
                                  const OutRoute ro, int s0, int s1, int *bag_ctr) {
@@ -552,7 +596,7 @@ RECFLEX_SCHED_FN void sched_warp(const char *__restrict__ T, unsigned rowb, int 
                 for (int u = 0; u < U; ++u)
 #pragma unroll
                     for (int c = 0; c < C; ++c)
-                        if (j + u * NG + g < hi && ok[c]) rv[u][c].load(T + (size_t)id[u] * rowb, colv[c], d);
+                        if (j + u * NG + g < hi && ok[c]) rv[u][c].template load<P>(T + (size_t)id[u] * rowb, colv[c], d);
 #pragma unroll
                 for (int u = 0; u < U; ++u)
                     if (j + u * NG + g < hi)
@@ -589,7 +633,7 @@ RECFLEX_SCHED_FN void sched_warp(const char *__restrict__ T, unsigned rowb, int 
 // ascending lookup order (same arithmetic as GROUP).
 constexpr int kFlatRun = 8;
 
-template <int ET, int GT, int VEC, int U>
+template <int ET, int GT, int VEC, int U, int P = 0>
 RECFLEX_SCHED_FN void sched_flat(const char *__restrict__ T, unsigned rowb, int gr, const int32_t *__restrict__ offs,
                                        const int32_t *__restrict__ idx, float *__restrict__ out, int d, int pool,
                                        const OutRoute ro, int s0, int s1, int *bag_ctr) {
@@ -636,7 +680,7 @@ RECFLEX_SCHED_FN void sched_flat(const char *__restrict__ T, unsigned rowb, int 
                 for (int u = 0; u < U; ++u) r[u].zero();
 #pragma unroll
                 for (int u = 0; u < U; ++u)
-                    if (j + u < Z && ok) r[u].load(T + (size_t)id[u] * rowb, col, d);
+                    if (j + u < Z && ok) r[u].template load<P>(T + (size_t)id[u] * rowb, col, d);
 #pragma unroll
                 for (int u = 0; u < U; ++u) {
                     if (j + u < Z) {
@@ -720,7 +764,7 @@ static __device__ __noinline__ void sched_backward(const float *__restrict__ gra
 // (adjacent groups read adjacent IDs: coalesced index loads).  Partials:
 // xor-butterfly across the groups of a warp (every lane gets bit-identical
 // sums), then the 8 warp partials are summed in warp order from shared memory.
-template <int ET, int GT, int VEC, int C, int U>
+template <int ET, int GT, int VEC, int C, int U, int P = 0>
 RECFLEX_SCHED_FN void sched_block(const char *__restrict__ T, unsigned rowb, int gr, const int32_t *__restrict__ offs,
                                         const int32_t *__restrict__ idx, float *__restrict__ out, int d, int pool,
                                         const OutRoute ro, int s0, int s1, float *red /* [8][SPAN] */) {
@@ -765,7 +809,7 @@ RECFLEX_SCHED_FN void sched_block(const char *__restrict__ T, unsigned rowb, int
                 for (int u = 0; u < U; ++u)
 #pragma unroll
                     for (int c = 0; c < C; ++c)
-                        if (ok[c]) v[u][c].load(T + (size_t)id[u] * rowb, colv[c], d);
+                        if (ok[c]) v[u][c].template load<P>(T + (size_t)id[u] * rowb, colv[c], d);
 #pragma unroll
                 for (int u = 0; u < U; ++u)
 #pragma unroll
@@ -783,7 +827,7 @@ RECFLEX_SCHED_FN void sched_block(const char *__restrict__ T, unsigned rowb, int
                 for (int u = 0; u < U; ++u)
 #pragma unroll
                     for (int c = 0; c < C; ++c)
-                        if (j + u * NG < hi && ok[c]) v[u][c].load(T + (size_t)id[u] * rowb, colv[c], d);
+                        if (j + u * NG < hi && ok[c]) v[u][c].template load<P>(T + (size_t)id[u] * rowb, colv[c], d);
 #pragma unroll
                 for (int u = 0; u < U; ++u)
                     if (j + u * NG < hi)

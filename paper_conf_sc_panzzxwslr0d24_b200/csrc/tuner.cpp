@@ -846,8 +846,16 @@ extern "C" recflex_status_t recflex_tune_ex(recflex_plan_t p, int32_t N, const i
                                        T.reps, &order_kind, nullptr, stream);
         if (st != RECFLEX_OK) return st;
     }
+    int32_t l2_choice = -1;
+    if (!(opt && opt->keep_l2) && T.jit && p->use_jit) {
+        // the L2 eviction priorities the final kernel runs fastest with (C36)
+        st = recflex_select_l2_policy(p, T.batches[0].d_idx, T.batches[0].d_off, T.batches[0].B, p->tables.data(),
+                                      T.reps, int64_t(126) << 20, &l2_choice, nullptr, stream);
+        if (st != RECFLEX_OK) return st;
+    }
     recflex_tune_stats_t s = {};
     s.task_order = order_kind;
+    s.l2_policy = l2_choice;
     s.two_stage_ms = two_stage_ms;
     s.incoming_ms = incoming_ms;
     s.jit_compiles = T.jit_compiles;

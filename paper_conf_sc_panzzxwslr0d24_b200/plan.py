@@ -204,6 +204,42 @@ class Plan:
         check(lib.recflex_get_columns(self._h, c), 'recflex_get_columns')
         return list(c)
 
+    # -------------------------------------------------------------- L2 policy (reading C36)
+    L2_POLICIES = ('default', 'evict_first', 'evict_last')  # RECFLEX_L2_*
+
+    @property
+    def l2_policy(self) -> List[int]:
+        """recflex_get_l2_policy: every feature's L2 eviction priority (0/1/2)."""
+        o = (ctypes.c_int32 * self.F)()
+        check(lib.recflex_get_l2_policy(self._h, o), 'recflex_get_l2_policy')
+        return list(o)
+
+    @l2_policy.setter
+    def l2_policy(self, policy: Optional[Sequence[int]]):
+        if policy is not None and len(policy) != self.F:
+            raise ValueError('l2 policy: one value per feature')
+        arr = None if policy is None else (ctypes.c_int32 * self.F)(*[int(v) for v in policy])
+        check(lib.recflex_set_l2_policy(self._h, arr), 'recflex_set_l2_policy')
+
+    def l2_policy_heuristic(self, l2_bytes: int = 126 * 2 ** 20) -> List[int]:
+        o = (ctypes.c_int32 * self.F)()
+        check(lib.recflex_l2_policy_heuristic(self._h, int(l2_bytes), o), 'recflex_l2_policy_heuristic')
+        return list(o)
+
+    L2_CANDIDATES = ('none', 'heuristic', 'evict_last_only')  # recflex_select_l2_policy
+
+    def select_l2_policy(self, indices: torch.Tensor, offsets: torch.Tensor, B: int,
+                         tables: Sequence[torch.Tensor], reps: int = 7, l2_bytes: int = 126 * 2 ** 20,
+                         stream=None) -> dict:
+        """recflex_select_l2_policy: time no hints / the heuristic / its evict_last part, keep the fastest."""
+        chosen = ctypes.c_int32()
+        ms = (ctypes.c_float * 3)()
+        check(lib.recflex_select_l2_policy(self._h, _dptr(indices, torch.int32, 'indices'),
+                                           _dptr(offsets, torch.int32, 'offsets'), int(B), self._tables(tables),
+                                           int(reps), int(l2_bytes), ctypes.byref(chosen), ms, _stream_ptr(stream)),
+              'recflex_select_l2_policy')
+        return dict(l2=self.L2_CANDIDATES[chosen.value], ms={k: ms[i] for i, k in enumerate(self.L2_CANDIDATES)})
+
     def task_order_heuristic(self, kind: str) -> List[int]:
         o = (ctypes.c_int32 * self.F)()
         check(lib.recflex_task_order_heuristic(self._h, self.ORDER_KINDS.index(kind), o),
@@ -347,7 +383,7 @@ class Plan:
     def tune(self, batches: Sequence[tuple], tables: Sequence[torch.Tensor], occupancies: Optional[List[int]] = None,
              reps: int = 7, pad_waves: int = 4, max_candidates: int = 0, verbose: bool = False, guard: bool = True,
              refine: bool = False, separate: bool = False, stage2_catalog: bool = False, tail: bool = True,
-             isolated: bool = False, select_order: bool = True, stream=None) -> dict:
+             isolated: bool = False, select_order: bool = True, select_l2: bool = True, stream=None) -> dict:
         """recflex_tune_ex over historical batches [(indices, offsets, B), ...]."""
         N = len(batches)
         idx_arr = (ctypes.c_void_p * N)(*[b[0].data_ptr() for b in batches])
@@ -368,6 +404,7 @@ class Plan:
         opt.stage2_catalog = 1 if stage2_catalog else 0
         opt.no_tail = 0 if tail else 1
         opt.keep_order = 0 if select_order else 1
+        opt.keep_l2 = 0 if select_l2 else 1
         st = _lib.TuneStats()
         check(lib.recflex_tune_ex(self._h, N, idx_arr, off_arr, bs_arr, self._tables(tables), _stream_ptr(stream),
                                   ctypes.byref(opt), ctypes.byref(st)), 'recflex_tune_ex')
@@ -377,7 +414,8 @@ class Plan:
                     best_occupancy=st.best_occupancy, best_ms=st.best_ms, tune_seconds=st.tune_seconds,
                     two_stage_ms=st.two_stage_ms, incoming_ms=st.incoming_ms, jit_compiles=st.jit_compiles,
                     compile_seconds=st.compile_seconds, refine_seconds=st.refine_seconds,
-                    task_order=self.ORDER_KINDS[st.task_order] if st.task_order >= 0 else None)
+                    task_order=self.ORDER_KINDS[st.task_order] if st.task_order >= 0 else None,
+                    l2_policy=self.L2_CANDIDATES[st.l2_policy] if st.l2_policy >= 0 else None)
 
     # -------------------------------------------------------------- schedules
     def get_schedule(self, f: int) -> dict:

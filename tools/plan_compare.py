@@ -14,7 +14,10 @@ sys.path.insert(0, ROOT)
 
 
 def main():
-    config, paths = sys.argv[1], sys.argv[2:]
+    args = sys.argv[1:]
+    catalog = '--catalog' in args      # time the precompiled catalog kernel instead
+    args = [x for x in args if x != '--catalog']
+    config, paths = args[0], args[1:]
     import torch
     from paper_conf_sc_panzzxwslr0d24_b200 import synth
     from paper_conf_sc_panzzxwslr0d24_b200.plan import Plan, l2_flush
@@ -32,6 +35,8 @@ def main():
         if path != 'default':
             plan.import_(json.load(open(path)))
         info = plan.compile()
+        if catalog:
+            plan.set_jit(False)
         ts = []
         for r in range(32):
             l2_flush(flush)
@@ -44,7 +49,8 @@ def main():
                 ts.append(e0.elapsed_time(e1))
         ms = float(np.median(ts))
         res.append((ms, path))
-        print(json.dumps(dict(config=config, plan=path, k=plan.occupancy, ms=round(ms, 4), regs=info['registers'],
+        print(json.dumps(dict(config=config, plan=path, kernel='catalog' if catalog else 'jit', k=plan.occupancy,
+                              ms=round(ms, 4), regs=info['registers'],
                               local_bytes=info['local_bytes'], variants=info['variants'])), flush=True)
     best = min(res)
     print(json.dumps(dict(config=config, best=best[1], ms=round(best[0], 4))), flush=True)

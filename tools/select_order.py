@@ -1,8 +1,8 @@
-"""Task-order selection (reading C35) for the tuned plans bench.py loads: load
+"""Task-order (reading C35) and L2-policy (C36) selection for the tuned plans bench.py loads: load
 configs/tuned/<config>[_<dtype>]_w<W>_r<R>.json, compile, keep the faster kernel
-(recflex_select_kernel), then recflex_select_task_order on a tuning batch (seed 8,
-as tools/tune_plan.py's second historical batch) and export the plan, its order
-included, to DIR (default gpurun_out/tuned).
+(recflex_select_kernel), then recflex_select_task_order and recflex_select_l2_policy
+on a tuning batch (seed 8, as tools/tune_plan.py's second historical batch) and export
+the plan, its order and L2 policy included, to DIR (default gpurun_out/tuned).
 
     python tools/select_order.py sharded1000 [--world W] [--dtype bf16] [--out DIR]
 """
@@ -56,11 +56,14 @@ def main():
         sh.plan.compile()
         ksel = sh.plan.select_kernel(bi, bo, model.batch, tables, reps=5)
         res = sh.plan.select_task_order(bi, bo, model.batch, tables, reps=a.reps)
+        l2 = sh.plan.select_l2_policy(bi, bo, model.batch, tables, reps=a.reps) if sh.plan.jit_enabled else None
         state = sh.plan.export()
         with open(os.path.join(a.out, name + '.json'), 'w') as fh:
             json.dump(state, fh)
         print(json.dumps(dict(plan=name, kernel=ksel['kernel'], order=res['order'],
                               columns=state.get('columns', 'feature'),
+                              l2=(l2['l2'] if l2 else 'n/a (catalog kernel)'),
+                              l2_ms=({k: round(v, 4) for k, v in l2['ms'].items()} if l2 else None),
                               ms={k: round(v, 4) for k, v in res['ms'].items()})), flush=True)
         del sh, tables, phys
         torch.cuda.empty_cache()
