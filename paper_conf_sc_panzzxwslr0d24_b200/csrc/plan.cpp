@@ -1096,7 +1096,7 @@ recflex_status_t recflex_set_l2_policy(recflex_plan_t p, const int32_t *policy) 
     if (policy) {
         bool any = false;
         for (int f = 0; f < p->F; ++f) {
-            if (policy[f] < RECFLEX_L2_DEFAULT || policy[f] > RECFLEX_L2_EVICT_LAST) return RECFLEX_ERR_INVALID_ARG;
+            if (policy[f] < RECFLEX_L2_DEFAULT || policy[f] > RECFLEX_L2_KEEP_L1) return RECFLEX_ERR_INVALID_ARG;
             any = any || policy[f] != RECFLEX_L2_DEFAULT;
         }
         if (any) l2.assign(policy, policy + p->F);
@@ -1421,7 +1421,7 @@ recflex_status_t recflex_plan_import(recflex_plan_t p, const char *json) {
         l2.resize(p->F);
         for (int f = 0; f < p->F; ++f) {
             long v = 0;
-            if (!parse_int_after(lc, &v) || v < 0 || v > 2) return RECFLEX_ERR_INVALID_ARG;
+            if (!parse_int_after(lc, &v) || v < 0 || v > RECFLEX_L2_KEEP_L1) return RECFLEX_ERR_INVALID_ARG;
             l2[f] = (int32_t)v;
         }
     }

@@ -42,11 +42,13 @@ namespace recflex {
 // large tables that rarely recur within a batch: let them stream through L2),
 // 2 = evict_last (small tables whose rows recur: keep them across the stream).
 // The policy is a 64-bit operand built by createpolicy (a uniform value).
+// P = 3 (small tables whose rows recur within a CTA's tasks): evict_last in L2
+// and the rows ALLOCATE in L1 (no .L1::no_allocate).
 template <int P>
 __device__ __forceinline__ uint64_t l2pol() {
     uint64_t pol = 0;
     if constexpr (P == 1) asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
-    else if constexpr (P == 2) asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+    else if constexpr (P == 2 || P == 3) asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
     return pol;
 }
 
@@ -64,6 +66,18 @@ __device__ __forceinline__ void ld_row(const float *p, float (&v)[VEC]) {
             asm("ld.global.nc.L1::no_allocate.v8.f32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
                 : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3]), "=f"(v[4]), "=f"(v[5]), "=f"(v[6]), "=f"(v[7])
                 : "l"(p));
+    } else if constexpr (P == 3) {
+        const uint64_t pol = l2pol<P>();
+        if constexpr (VEC == 1)
+            asm("ld.global.nc.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v[0]) : "l"(p), "l"(pol));
+        else if constexpr (VEC == 4)
+            asm("ld.global.nc.L2::cache_hint.v4.f32 {%0, %1, %2, %3}, [%4], %5;"
+                : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3])
+                : "l"(p), "l"(pol));
+        else
+            asm("ld.global.nc.L2::cache_hint.v8.f32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8], %9;"
+                : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3]), "=f"(v[4]), "=f"(v[5]), "=f"(v[6]), "=f"(v[7])
+                : "l"(p), "l"(pol));
     } else {
         const uint64_t pol = l2pol<P>();
         if constexpr (VEC == 1)
@@ -96,7 +110,21 @@ __device__ __forceinline__ int ld_idx(const int32_t *p) { return __ldg(p); }
 //          2^23 (PRMT) and 2^23 + 128 subtracted (exact).
 template <int NW, int P = 0>
 __device__ __forceinline__ void ld_words(const void *p, unsigned (&w)[NW]) {
-    if constexpr (P != 0) {
+    if constexpr (P == 3) {
+        const uint64_t pol = l2pol<P>();
+        if constexpr (NW == 1)
+            asm("ld.global.nc.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(w[0]) : "l"(p), "l"(pol));
+        else if constexpr (NW == 2)
+            asm("ld.global.nc.L2::cache_hint.v2.b32 {%0, %1}, [%2], %3;" : "=r"(w[0]), "=r"(w[1]) : "l"(p), "l"(pol));
+        else if constexpr (NW == 4)
+            asm("ld.global.nc.L2::cache_hint.v4.b32 {%0, %1, %2, %3}, [%4], %5;"
+                : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3])
+                : "l"(p), "l"(pol));
+        else
+            asm("ld.global.nc.L2::cache_hint.v8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8], %9;"
+                : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]), "=r"(w[4]), "=r"(w[5]), "=r"(w[6]), "=r"(w[7])
+                : "l"(p), "l"(pol));
+    } else if constexpr (P != 0) {
         const uint64_t pol = l2pol<P>();
         if constexpr (NW == 1)
             asm("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(w[0]) : "l"(p), "l"(pol));

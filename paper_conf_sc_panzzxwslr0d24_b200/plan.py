@@ -205,7 +205,7 @@ class Plan:
         return list(c)
 
     # -------------------------------------------------------------- L2 policy (reading C36)
-    L2_POLICIES = ('default', 'evict_first', 'evict_last')  # RECFLEX_L2_*
+    L2_POLICIES = ('default', 'evict_first', 'evict_last', 'keep_l1')  # RECFLEX_L2_*
 
     @property
     def l2_policy(self) -> List[int]:

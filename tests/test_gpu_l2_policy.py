@@ -34,7 +34,7 @@ def test_every_policy_bitexact(mapping):
         plan.set_schedule(f, s['sched_id'], 1 if mapping == 'part1' else 0, 40 if mapping == 'part1' else 16)
     rng = np.random.default_rng(0)
     variants = None
-    for pol in ([0] * m.F, [1] * m.F, [2] * m.F, rng.integers(0, 3, m.F).tolist()):
+    for pol in ([0] * m.F, [1] * m.F, [2] * m.F, [3] * m.F, rng.integers(0, 4, m.F).tolist()):
         plan.l2_policy = pol
         assert plan.l2_policy == pol
         info = plan.compile()
@@ -55,7 +55,7 @@ def test_lowp_rows_with_policies_bitexact():
         b = synth.make_batch(m, 4)
         case = TypedCase(m, b, dtype, 'int')
         plan = case.plan()
-        plan.l2_policy = [1 + (f % 2) for f in range(m.F)]
+        plan.l2_policy = [1 + (f % 3) for f in range(m.F)]
         plan.compile()
         out = case.run(plan)
         ref, _ = case.oracle()
@@ -79,7 +79,7 @@ def test_policy_export_import_invalid_and_heuristic():
     p2.import_(st)
     assert p2.l2_policy == [0] * m.F and 'l2' not in p2.export()
     with pytest.raises(RuntimeError):
-        plan.l2_policy = [3] * m.F
+        plan.l2_policy = [4] * m.F
     assert plan.l2_policy == h
 
 

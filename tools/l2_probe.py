@@ -42,6 +42,14 @@ def main():
             'first_only': [1 if p == 1 else 0 for p in heur],
             'last_only': [2 if p == 2 else 0 for p in heur],
             'all_first': [1] * m.F, 'all_last': [2] * m.F}
+    # rows of tables up to X MB with >= 1 lookup per row per batch also allocate in L1 (policy 3)
+    for mb in (1, 4, 16):
+        pol = list(heur)
+        for f, feat in enumerate(m.features):
+            tb = feat.rows * feat.dim * 4
+            if tb <= mb * 2 ** 20 and m.batch * feat.mean_len() * feat.coverage >= feat.rows:
+                pol[f] = 3
+        pols[f'l1_{mb}mb'] = pol
     print(json.dumps(dict(config=a.config, heuristic_counts={k: heur.count(i) for i, k in
                                                              enumerate(Plan.L2_POLICIES)})), flush=True)
     for name in a.variants.split(','):
