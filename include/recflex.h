@@ -237,6 +237,8 @@ typedef struct {
                                 first batch (3 x reps forwards); 1: keep the plan's order  */
     int32_t keep_l2;         /* 0: then recflex_select_l2_policy (plan-specialised kernel
                                 only; <= 3 compiles + 3 x reps forwards); 1: keep it       */
+    int32_t keep_task_size;  /* 0: before the order selection, recflex_select_task_size
+                                (3 x reps forwards); 1: keep the per-task sizes            */
 } recflex_tune_options_t;
 
 typedef struct {
@@ -258,6 +260,7 @@ typedef struct {
     double refine_seconds;    /* wall time of the refinement stage                 */
     int32_t task_order;       /* RECFLEX_ORDER_* kept by the order selection, -1 = not run */
     int32_t l2_policy;        /* recflex_select_l2_policy's choice, -1 = not run           */
+    int32_t task_size;        /* recflex_select_task_size's choice, -1 = not run           */
 } recflex_tune_stats_t;
 
 /* Two-stage interference-simulated tuning over num_batches historical batches
@@ -454,6 +457,17 @@ recflex_status_t recflex_l2_policy_heuristic(recflex_plan_t plan, int64_t l2_byt
 recflex_status_t recflex_select_l2_policy(recflex_plan_t plan, const int32_t *indices, const int32_t *offsets,
                                           int32_t batch_size, const void *const *tables, int32_t reps,
                                           int64_t l2_bytes, int32_t *chosen, float *ms, void *stream);
+/* ---- task granularity (reading C37) ---------------------------------------
+ * The default schedules size tasks for a plan-wide lookup target and the
+ * tuner keeps that size; with the task order and L2 policy in place the best
+ * size can move.  Times the plan with every feature's per_block scaled by 1,
+ * 1/2 and 2 (lookup-partitioned: >= 16 lookups per task; a heuristic task
+ * order is re-derived for each), on one batch (median of reps forwards, L2
+ * flushed before each), keeps the fastest (ties: 1, 1/2, 2).  *chosen (0, 1, 2
+ * = x1, x1/2, x2) and ms[3] (nullable).  Blocking; allocates scratch. */
+recflex_status_t recflex_select_task_size(recflex_plan_t plan, const int32_t *indices, const int32_t *offsets,
+                                          int32_t batch_size, const void *const *tables, int32_t reps,
+                                          int32_t *chosen, float *ms, void *stream);
 /* order[F] receives the plan's current task order. */
 recflex_status_t recflex_get_task_order(recflex_plan_t plan, int32_t *order);
 /* order[F] receives heuristic `kind` (RECFLEX_ORDER_*) for the plan's current

@@ -40,7 +40,7 @@ class TuneOptions(ctypes.Structure):
                 ('reps', ctypes.c_int32), ('pad_waves', ctypes.c_int32), ('max_candidates', ctypes.c_int32),
                 ('verbose', ctypes.c_int32), ('skip_guard', ctypes.c_int32), ('refine', ctypes.c_int32),
                 ('local_mode', ctypes.c_int32), ('stage2_catalog', ctypes.c_int32), ('no_tail', ctypes.c_int32),
-                ('keep_order', ctypes.c_int32), ('keep_l2', ctypes.c_int32)]
+                ('keep_order', ctypes.c_int32), ('keep_l2', ctypes.c_int32), ('keep_task_size', ctypes.c_int32)]
 
 
 class TuneStats(ctypes.Structure):
@@ -51,7 +51,7 @@ class TuneStats(ctypes.Structure):
                 ('refine_evals', ctypes.c_int64), ('refine_gain', ctypes.c_double),
                 ('two_stage_ms', ctypes.c_double), ('incoming_ms', ctypes.c_double), ('jit_compiles', ctypes.c_int64),
                 ('compile_seconds', ctypes.c_double), ('refine_seconds', ctypes.c_double),
-                ('task_order', ctypes.c_int32), ('l2_policy', ctypes.c_int32)]
+                ('task_order', ctypes.c_int32), ('l2_policy', ctypes.c_int32), ('task_size', ctypes.c_int32)]
 
 
 class JitInfo(ctypes.Structure):
@@ -131,6 +131,8 @@ SIGNATURES = {
     'recflex_select_kernel': (c_int32, [c_void_p, c_void_p, c_void_p, c_int32, P(c_void_p), c_int32,
                                         P(ctypes.c_float), P(ctypes.c_float), c_void_p]),
     'recflex_set_task_order': (c_int32, [c_void_p, P(c_int32)]),
+    'recflex_select_task_size': (c_int32, [c_void_p, c_void_p, c_void_p, c_int32, P(c_void_p), c_int32,
+                                           P(c_int32), P(ctypes.c_float), c_void_p]),
     'recflex_get_task_order': (c_int32, [c_void_p, P(c_int32)]),
     'recflex_set_column_order': (c_int32, [c_void_p, c_int32]),
     'recflex_get_columns': (c_int32, [c_void_p, P(c_int64)]),

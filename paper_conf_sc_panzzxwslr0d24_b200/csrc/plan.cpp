@@ -1149,6 +1149,99 @@ recflex_status_t recflex_task_order_heuristic(recflex_plan_t p, int32_t kind, in
     return RECFLEX_OK;
 }
 
+// Measured task granularity (C37): every feature's tasks scaled by 1, 1/2 or 2
+// (samples per task for sample-partitioned schedules, lookups per task for
+// lookup-partitioned ones, at least 16), the task order re-derived if it is a
+// heuristic's; the fastest scale is kept (ties: 1, then 1/2, then 2).
+recflex_status_t recflex_select_task_size(recflex_plan_t p, const int32_t *indices, const int32_t *offsets,
+                                          int32_t B, const void *const *tables, int32_t reps, int32_t *chosen,
+                                          float *ms_out, void *stream_) {
+    if (!p || !indices || !offsets || !tables || B <= 0 || B > p->max_batch) return RECFLEX_ERR_INVALID_ARG;
+    NvtxRange nvtx("recflex_select_task_size");
+    DeviceGuard guard(p->device);
+    cudaStream_t stream = (cudaStream_t)stream_;
+    // which heuristic (if any) the current order is, to re-derive it per candidate
+    int kind = -1;
+    for (int k = 0; k < RECFLEX_NUM_ORDERS && kind < 0; ++k) {
+        std::vector<int32_t> o;
+        task_order_of_kind(p, k, o);
+        std::vector<int32_t> cur(p->F);
+        for (int e = 0; e < p->F; ++e) cur[e] = feature_at(p, e);
+        if (o == cur) kind = k;
+    }
+    const std::vector<int32_t> keep_order = p->order;
+    std::vector<recflex_schedule_t> base(p->F);
+    for (int f = 0; f < p->F; ++f) base[f] = {p->desc[f].sched, p->desc[f].part, p->desc[f].per_block, p->desc[f].nalloc};
+    const int num = 2, den[3] = {2, 4, 1};  // scale = num / den: 1, 1/2, 2
+    auto scaled = [&](int c) {
+        std::vector<recflex_schedule_t> ss = base;
+        for (auto &x : ss) {
+            const int64_t v = (int64_t)x.per_block * num / den[c];
+            x.per_block = (int32_t)std::max<int64_t>(x.part == 1 ? 16 : 1, std::min<int64_t>(v, 1 << 30));
+        }
+        return ss;
+    };
+    auto apply = [&](int c) -> recflex_status_t {
+        std::vector<int32_t> o = keep_order;
+        std::vector<recflex_schedule_t> ss = scaled(c);
+        // schedules first (columns unchanged), then the re-derived order
+        recflex_status_t st = set_layout(p, p->order, p->columns_follow_order, &ss);
+        if (st != RECFLEX_OK || kind < 0) return st;
+        task_order_of_kind(p, kind, o);
+        return apply_task_order(p, o.data());
+    };
+    float *out = nullptr, *flush = nullptr;
+    const size_t flush_bytes = size_t(256) << 20;  // 2x L2
+    cudaError_t e = cudaMalloc(&out, sizeof(float) * (size_t)B * p->d_tot);
+    if (e == cudaSuccess) e = cudaMalloc(&flush, flush_bytes);
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+    if (e == cudaSuccess) e = cudaEventCreate(&e0);
+    if (e == cudaSuccess) e = cudaEventCreate(&e1);
+    recflex_status_t st = e == cudaSuccess ? RECFLEX_OK : cuda_status(e);
+    if (st == RECFLEX_OK && p->use_jit && !jit_ready(p, p->k)) {
+        int k = p->k;
+        st = jit_compile_plan(p, &k, 1);  // per-task sizes are not compiled in: one kernel serves all scales
+    }
+    float med[3] = {0.f, 0.f, 0.f};
+    for (int c = 0; c < 3 && st == RECFLEX_OK; ++c) {
+        st = apply(c);
+        std::vector<float> ms;
+        for (int r = 0; r < std::max(3, reps) + 1 && st == RECFLEX_OK; ++r) {
+            flush_launch(flush, flush_bytes, stream);
+            cudaEventRecord(e0, stream);
+            st = recflex_forward(p, indices, offsets, B, tables, out, stream);
+            cudaEventRecord(e1, stream);
+            e = cudaEventSynchronize(e1);
+            if (e != cudaSuccess) st = cuda_status(e);
+            float t = 0;
+            cudaEventElapsedTime(&t, e0, e1);
+            if (r > 0) ms.push_back(t);
+        }
+        if (!ms.empty()) {
+            std::sort(ms.begin(), ms.end());
+            med[c] = ms[ms.size() / 2];
+        }
+    }
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    cudaFree(out);
+    cudaFree(flush);
+    int best = 0;
+    if (st == RECFLEX_OK)
+        for (int c = 1; c < 3; ++c)
+            if (med[c] < med[best]) best = c;
+    if (st != RECFLEX_OK) {
+        set_layout(p, keep_order, p->columns_follow_order, &base);
+        return st;
+    }
+    st = apply(best);
+    if (st != RECFLEX_OK) return st;
+    if (chosen) *chosen = best;
+    if (ms_out)
+        for (int c = 0; c < 3; ++c) ms_out[c] = med[c];
+    return RECFLEX_OK;
+}
+
 // Measured choice among the task-order heuristics (C35): time the plan's
 // current kernel under each order on the caller's batch (median of reps
 // forwards, L2 flushed before each), keep the fastest (ties: the lower kind).

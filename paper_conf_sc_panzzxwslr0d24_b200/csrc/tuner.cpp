@@ -839,6 +839,13 @@ extern "C" recflex_status_t recflex_tune_ex(recflex_plan_t p, int32_t N, const i
                                    T.reps, nullptr, nullptr, stream);
         if (st != RECFLEX_OK) return st;
     }
+    int32_t size_choice = -1;
+    if (!(opt && opt->keep_task_size)) {
+        // the task granularity the final kernel runs fastest with (C37)
+        st = recflex_select_task_size(p, T.batches[0].d_idx, T.batches[0].d_off, T.batches[0].B, p->tables.data(),
+                                      T.reps, &size_choice, nullptr, stream);
+        if (st != RECFLEX_OK) return st;
+    }
     int32_t order_kind = -1;
     if (!(opt && opt->keep_order)) {
         // the task order the final kernel runs fastest under (C35)
@@ -856,6 +863,7 @@ extern "C" recflex_status_t recflex_tune_ex(recflex_plan_t p, int32_t N, const i
     recflex_tune_stats_t s = {};
     s.task_order = order_kind;
     s.l2_policy = l2_choice;
+    s.task_size = size_choice;
     s.two_stage_ms = two_stage_ms;
     s.incoming_ms = incoming_ms;
     s.jit_compiles = T.jit_compiles;

@@ -226,6 +226,19 @@ class Plan:
         check(lib.recflex_l2_policy_heuristic(self._h, int(l2_bytes), o), 'recflex_l2_policy_heuristic')
         return list(o)
 
+    TASK_SIZES = ('x1', 'x1/2', 'x2')  # recflex_select_task_size
+
+    def select_task_size(self, indices: torch.Tensor, offsets: torch.Tensor, B: int,
+                         tables: Sequence[torch.Tensor], reps: int = 7, stream=None) -> dict:
+        """recflex_select_task_size: every feature's per-task size x1, x1/2, x2 timed, the fastest kept."""
+        chosen = ctypes.c_int32()
+        ms = (ctypes.c_float * 3)()
+        check(lib.recflex_select_task_size(self._h, _dptr(indices, torch.int32, 'indices'),
+                                           _dptr(offsets, torch.int32, 'offsets'), int(B), self._tables(tables),
+                                           int(reps), ctypes.byref(chosen), ms, _stream_ptr(stream)),
+              'recflex_select_task_size')
+        return dict(task_size=self.TASK_SIZES[chosen.value], ms={k: ms[i] for i, k in enumerate(self.TASK_SIZES)})
+
     L2_CANDIDATES = ('none', 'heuristic', 'evict_last_only')  # recflex_select_l2_policy
 
     def select_l2_policy(self, indices: torch.Tensor, offsets: torch.Tensor, B: int,
@@ -383,7 +396,8 @@ class Plan:
     def tune(self, batches: Sequence[tuple], tables: Sequence[torch.Tensor], occupancies: Optional[List[int]] = None,
              reps: int = 7, pad_waves: int = 4, max_candidates: int = 0, verbose: bool = False, guard: bool = True,
              refine: bool = False, separate: bool = False, stage2_catalog: bool = False, tail: bool = True,
-             isolated: bool = False, select_order: bool = True, select_l2: bool = True, stream=None) -> dict:
+             isolated: bool = False, select_order: bool = True, select_l2: bool = True,
+             select_task_size: bool = True, stream=None) -> dict:
         """recflex_tune_ex over historical batches [(indices, offsets, B), ...]."""
         N = len(batches)
         idx_arr = (ctypes.c_void_p * N)(*[b[0].data_ptr() for b in batches])
@@ -405,6 +419,7 @@ class Plan:
         opt.no_tail = 0 if tail else 1
         opt.keep_order = 0 if select_order else 1
         opt.keep_l2 = 0 if select_l2 else 1
+        opt.keep_task_size = 0 if select_task_size else 1
         st = _lib.TuneStats()
         check(lib.recflex_tune_ex(self._h, N, idx_arr, off_arr, bs_arr, self._tables(tables), _stream_ptr(stream),
                                   ctypes.byref(opt), ctypes.byref(st)), 'recflex_tune_ex')
@@ -415,7 +430,8 @@ class Plan:
                     two_stage_ms=st.two_stage_ms, incoming_ms=st.incoming_ms, jit_compiles=st.jit_compiles,
                     compile_seconds=st.compile_seconds, refine_seconds=st.refine_seconds,
                     task_order=self.ORDER_KINDS[st.task_order] if st.task_order >= 0 else None,
-                    l2_policy=self.L2_CANDIDATES[st.l2_policy] if st.l2_policy >= 0 else None)
+                    l2_policy=self.L2_CANDIDATES[st.l2_policy] if st.l2_policy >= 0 else None,
+                    task_size=self.TASK_SIZES[st.task_size] if st.task_size >= 0 else None)
 
     # -------------------------------------------------------------- schedules
     def get_schedule(self, f: int) -> dict:

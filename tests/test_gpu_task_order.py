@@ -229,3 +229,26 @@ def test_column_order_full_size_sampled():
     ref, _ = sampled_oracle(m, b, samples, tables)
     assert plan.columns != np.cumsum([0] + m.dims)[:-1].tolist()
     assert bitexact(got, ref)
+
+
+@pytest.mark.parametrize('order', ['feature', 'lpt'])
+def test_select_task_size_keeps_parity(order):
+    """recflex_select_task_size (reading C37): the kept scale is applied to every
+    feature's per-task size, a heuristic order is re-derived, outputs stay bit-exact."""
+    P = _P()
+    m = synth.make_model('fig3')
+    b = synth.make_batch(m, 7)
+    case = Case(m, b, 'int')
+    plan = P.Plan.from_model(m)
+    plan.task_order = plan.task_order_heuristic(order)
+    before = [plan.get_schedule(f)['per_block'] for f in range(m.F)]
+    parts = [plan.get_schedule(f)['part'] for f in range(m.F)]
+    res = plan.select_task_size(case.idx, case.off, b.B, case.tables, reps=3)
+    assert res['task_size'] in plan.TASK_SIZES and all(v > 0 for v in res['ms'].values())
+    num, den = {'x1': (1, 1), 'x1/2': (1, 2), 'x2': (2, 1)}[res['task_size']]
+    after = [plan.get_schedule(f)['per_block'] for f in range(m.F)]
+    assert after == [max(16 if parts[f] else 1, before[f] * num // den) for f in range(m.F)]
+    assert plan.task_order == plan.task_order_heuristic(order)
+    _, out = run_plan(case, plan)
+    ref, _ = case.oracle()
+    assert bitexact(feature_columns(out, plan, m.dims), ref)

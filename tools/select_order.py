@@ -21,6 +21,7 @@ def main():
     ap.add_argument('--world', type=int, default=1)
     ap.add_argument('--dtype', default='f32', choices=['f32', 'f16', 'bf16', 'i8', 'fp8'])
     ap.add_argument('--reps', type=int, default=9)
+    ap.add_argument('--task-size', action='store_true', help='also recflex_select_task_size (C37) first')
     ap.add_argument('--columns', default='plan', choices=['plan', 'feature', 'task-order'],
                     help="output layout to select under: the plan file's, or set it")
     ap.add_argument('--out', default=os.path.join(ROOT, 'gpurun_out', 'tuned'))
@@ -55,6 +56,7 @@ def main():
             sh.plan.set_column_order(a.columns == 'task-order')
         sh.plan.compile()
         ksel = sh.plan.select_kernel(bi, bo, model.batch, tables, reps=5)
+        size = sh.plan.select_task_size(bi, bo, model.batch, tables, reps=a.reps) if a.task_size else None
         res = sh.plan.select_task_order(bi, bo, model.batch, tables, reps=a.reps)
         l2 = sh.plan.select_l2_policy(bi, bo, model.batch, tables, reps=a.reps) if sh.plan.jit_enabled else None
         state = sh.plan.export()
@@ -62,6 +64,8 @@ def main():
             json.dump(state, fh)
         print(json.dumps(dict(plan=name, kernel=ksel['kernel'], order=res['order'],
                               columns=state.get('columns', 'feature'),
+                              task_size=(size['task_size'] if size else None),
+                              size_ms=({k: round(v, 4) for k, v in size['ms'].items()} if size else None),
                               l2=(l2['l2'] if l2 else 'n/a (catalog kernel)'),
                               l2_ms=({k: round(v, 4) for k, v in l2['ms'].items()} if l2 else None),
                               ms={k: round(v, 4) for k, v in res['ms'].items()})), flush=True)
