@@ -44,7 +44,7 @@ def main():
         phys[t] = synth.make_table_stored(t, rows, dim, 'f32', 'float', device=dev, seed=model.seed)
     flush = torch.empty(64 << 20, device=dev)
     for W in [int(x) for x in a.worlds.split(',')]:
-        parts = model_parts(model, W, 'f32', a.config, os.path.join(ROOT, 'configs', 'tuned'))
+        parts = model_parts(model, W, 'f32', a.config, a.tuned_dir)
         per_rank = []
         for r in range(W):
             sh = ShardedEmbedding(model, r, W, device=0, parts=parts)

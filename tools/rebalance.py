@@ -37,6 +37,8 @@ def main():
     ap.add_argument('--tries', type=int, default=6, help='candidates tried per move')
     ap.add_argument('--reps', type=int, default=10)
     ap.add_argument('--out', default=os.path.join(ROOT, 'gpurun_out', 'rebalance'))
+    ap.add_argument('--catalog', action='store_true', help='measure the catalog kernel (round 1) instead of the '
+                                                           'plan-specialised one')
     a = ap.parse_args()
     import torch
     from paper_conf_sc_panzzxwslr0d24_b200 import synth
@@ -54,22 +56,45 @@ def main():
             for t, (rows, dim) in enumerate(model.tables)}
     flush = torch.empty(64 << 20, device=dev)
 
-    # per-feature schedule and per-rank occupancy from the tuned plans
-    sched, occ = {}, []
+    # per-feature schedule and L2 policy, per-rank occupancy, task-order kind and
+    # column layout from the tuned plans (a moved feature keeps its schedule and
+    # policy; the receiving rank re-derives its order heuristic)
+    sched, l2, occ, kinds, cols = {}, {}, [], [], []
     for r in range(W):
         st = json.load(open(os.path.join(tuned_dir, f'{a.config}_w{W}_r{r}.json')))
-        for f, s in zip(parts[r], st['schedules']):
+        pol = st.get('l2', [0] * len(parts[r]))
+        for f, s, q in zip(parts[r], st['schedules'], pol):
             sched[f] = s
+            l2[f] = q
         occ.append(st['occupancy'])
+        cols.append(st.get('columns'))
+        sh = ShardedEmbedding(model, r, W, device=0, parts=parts)
+        sh.plan.import_(st)
+        kinds.append(next((k for k in sh.plan.ORDER_KINDS if sh.plan.task_order == sh.plan.task_order_heuristic(k)),
+                          'feature'))
+        del sh
     catalog = st['catalog_size']
+    fingerprint = st.get('catalog_fingerprint')
 
-    def state(part, k):
-        return dict(abi=2, catalog_size=catalog, num_features=len(part), occupancy=k,
-                    schedules=[sched[f] for f in part])
+    def state(part, r):
+        d = dict(abi=2, catalog_size=catalog, num_features=len(part), occupancy=occ[r],
+                 schedules=[sched[f] for f in part], l2=[l2[f] for f in part])
+        if fingerprint is not None:
+            d['catalog_fingerprint'] = fingerprint
+        if cols[r]:
+            d['columns'] = cols[r]
+        return d
+
+    def rank_plan(parts_, r):
+        sh = ShardedEmbedding(model, r, W, device=0, parts=parts_)
+        sh.plan.import_(state(parts_[r], r))
+        sh.plan.task_order = sh.plan.task_order_heuristic(kinds[r])
+        if not a.catalog:
+            sh.plan.compile()  # the plan-specialised kernel bench.py runs
+        return sh
 
     def measure(parts_, r, k):
-        sh = ShardedEmbedding(model, r, W, device=0, parts=parts_)
-        sh.plan.import_(state(parts_[r], k))
+        sh = rank_plan(parts_, r)
         tables = [phys[model.features[f].table] for f in sh.features]
         idx, off = shard_batch(full, sh.features)
         bi, bo = torch.from_numpy(idx).to(dev), torch.from_numpy(off).to(dev)
@@ -98,8 +123,10 @@ def main():
         json.dump(dict(config=a.config, world=W, parts=parts, log=log,
                        note='tools/rebalance.py: measured refinement of the LPT partition'), fh)
     for r in range(W):  # every rank's plan follows the (possibly new) partition
+        sh = rank_plan(parts, r)
         with open(os.path.join(a.out, f'{a.config}_w{W}_r{r}.json'), 'w') as fh:
-            json.dump(state(parts[r], occ[r]), fh)
+            json.dump(sh.plan.export(), fh)
+        del sh
     print(json.dumps(dict(done=True, changed=sorted(changed), max=max(t), max_over_mean=max(t) * W / sum(t))), flush=True)
 
 
