@@ -34,7 +34,19 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, q):
+def _set_layout(sh, layout):
+    """'task-order': the rank plan runs its LPT task order with its outputs concatenated
+    in that order and mixed L2 policies (readings C35, C36) -- the global exchanged layout
+    then follows every rank's ShardedEmbedding.column_features."""
+    if layout == 'task-order':
+        sh.plan.set_column_order(True)
+        sh.plan.task_order = sh.plan.task_order_heuristic('lpt')
+        sh.plan.l2_policy = [(i % 3) for i in range(len(sh.features))]
+        sh.plan.compile()
+    return sh.column_features
+
+
+def _worker(rank, world, port, q, layout='feature'):
     import torch.distributed as dist
     from paper_conf_sc_panzzxwslr0d24_b200 import synth
     from paper_conf_sc_panzzxwslr0d24_b200.shard import ShardedEmbedding, partition_model, shard_batch
@@ -47,12 +59,13 @@ def _worker(rank, world, port, q):
         b = synth.make_batch(m, 5)
         parts = partition_model(m, world)
         sh = ShardedEmbedding(m, rank, world, device=0, parts=parts)
+        cols = _set_layout(sh, layout)
         tables = [synth.make_table(m.features[f].table, m.features[f].rows, m.features[f].dim, 'int', device=dev)
                   for f in sh.features]
         idx, off = shard_batch(b, sh.features)
         out = sh.forward(torch.from_numpy(idx).to(dev), torch.from_numpy(off).to(dev), b.B, tables)
         torch.cuda.synchronize()
-        q.put((rank, out.cpu().numpy(), parts))
+        q.put((rank, out.cpu().numpy(), cols))
     finally:
         dist.destroy_process_group()
 
@@ -67,32 +80,32 @@ def _oracle_full(seed=5):
     return m, b, oracle.embedding_bag(tabs, m.dims, [f.pool for f in m.features], b.indices, b.offsets, b.B)
 
 
+@pytest.mark.parametrize('layout', ['feature', 'task-order'])
 @pytest.mark.parametrize('world', [2, 3])
-def test_sharded_forward_matches_oracle(world):
-    from paper_conf_sc_panzzxwslr0d24_b200 import synth
-    from paper_conf_sc_panzzxwslr0d24_b200.plan import Plan
+def test_sharded_forward_matches_oracle(world, layout):
     from paper_conf_sc_panzzxwslr0d24_b200.shard import column_order
     ctx = mp.get_context('spawn')
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q, layout)) for r in range(world)]
     for p in procs:
         p.start()
-    res = [q.get(timeout=300) for _ in range(world)]
+    res = sorted([q.get(timeout=300) for _ in range(world)], key=lambda x: x[0])
     for p in procs:
         p.join(timeout=120)
         assert p.exitcode == 0
     m, b, full = _oracle_full()
     rows = b.B // world
-    for rank, got, parts in res:
-        order = column_order(m, parts)
+    cols = [c for _, _, c in res]   # every rank's features in its local column order
+    order = column_order(m, cols)
+    for rank, got, _ in res:
         assert np.array_equal(got, full[rank * rows:(rank + 1) * rows][:, order].astype(np.float32))
 
 
 STEPS, SEEDS = 7, (5, 6, 8)
 
 
-def _worker_fused(rank, world, port, q):
+def _worker_fused(rank, world, port, q, layout='feature'):
     import torch.distributed as dist
     from paper_conf_sc_panzzxwslr0d24_b200 import synth
     from paper_conf_sc_panzzxwslr0d24_b200.shard import FusedShardedEmbedding, partition_model, shard_batch
@@ -104,6 +117,7 @@ def _worker_fused(rank, world, port, q):
         m = _model()
         parts = partition_model(m, world)
         sh = FusedShardedEmbedding(m, rank, world, device=0, parts=parts)
+        cols = _set_layout(sh, layout)
         tables = [synth.make_table(m.features[f].table, m.features[f].rows, m.features[f].dim, 'int', device=dev)
                   for f in sh.features]
         inputs = []
@@ -119,15 +133,16 @@ def _worker_fused(rank, world, port, q):
             o = sh.forward(*inputs[i % len(SEEDS)], m.batch, tables)
             outs.append(o.clone())
         torch.cuda.synchronize()
-        q.put((rank, [o.cpu().numpy() for o in outs], parts))
+        q.put((rank, [o.cpu().numpy() for o in outs], cols))
         dist.barrier()
         sh.close()
     finally:
         dist.destroy_process_group()
 
 
+@pytest.mark.parametrize('layout', ['feature', 'task-order'])
 @pytest.mark.parametrize('world', [2, 3])
-def test_fused_exchange_matches_oracle(world):
+def test_fused_exchange_matches_oracle(world, layout):
     """NEXT #1: the all-to-all folded into the fused kernel's store epilogue
     (peer stores through CUDA-IPC-mapped buffers), over a barrier-free step loop
     with changing batches: every step's received rows equal the oracle's."""
@@ -135,20 +150,21 @@ def test_fused_exchange_matches_oracle(world):
     ctx = mp.get_context('spawn')
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker_fused, args=(r, world, port, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker_fused, args=(r, world, port, q, layout)) for r in range(world)]
     for p in procs:
         p.start()
-    res = [q.get(timeout=600) for _ in range(world)]
+    res = sorted([q.get(timeout=600) for _ in range(world)], key=lambda x: x[0])
     for p in procs:
         p.join(timeout=120)
         assert p.exitcode == 0
     refs = {sd: _oracle_full(sd) for sd in SEEDS}
-    for rank, outs, parts in res:
+    cols = [c for _, _, c in res]   # every rank's features in its local column order
+    for rank, outs, _ in res:
         assert len(outs) == STEPS
         for i, got in enumerate(outs):
             m, b, full = refs[SEEDS[i % len(SEEDS)]]
             rows = b.B // world
-            exp = full[rank * rows:(rank + 1) * rows][:, column_order(m, parts)].astype(np.float32)
+            exp = full[rank * rows:(rank + 1) * rows][:, column_order(m, cols)].astype(np.float32)
             assert np.array_equal(got, exp), (rank, i)
 
 
