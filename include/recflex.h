@@ -239,6 +239,9 @@ typedef struct {
                                 only; <= 3 compiles + 3 x reps forwards); 1: keep it       */
     int32_t keep_task_size;  /* 0: before the order selection, recflex_select_task_size
                                 (3 x reps forwards); 1: keep the per-task sizes            */
+    float switch_margin;     /* stage 1: a candidate other than the feature's incoming
+                                schedule must cost < (1 - margin) x the incoming one to be
+                                chosen (reading C38; 0 = the paper's plain argmin)         */
 } recflex_tune_options_t;
 
 typedef struct {

@@ -40,7 +40,8 @@ class TuneOptions(ctypes.Structure):
                 ('reps', ctypes.c_int32), ('pad_waves', ctypes.c_int32), ('max_candidates', ctypes.c_int32),
                 ('verbose', ctypes.c_int32), ('skip_guard', ctypes.c_int32), ('refine', ctypes.c_int32),
                 ('local_mode', ctypes.c_int32), ('stage2_catalog', ctypes.c_int32), ('no_tail', ctypes.c_int32),
-                ('keep_order', ctypes.c_int32), ('keep_l2', ctypes.c_int32), ('keep_task_size', ctypes.c_int32)]
+                ('keep_order', ctypes.c_int32), ('keep_l2', ctypes.c_int32), ('keep_task_size', ctypes.c_int32),
+                ('switch_margin', ctypes.c_float)]
 
 
 class TuneStats(ctypes.Structure):

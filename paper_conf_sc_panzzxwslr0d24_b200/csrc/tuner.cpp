@@ -146,6 +146,7 @@ struct Tuner {
     int64_t jit_compiles = 0;
     double compile_seconds = 0;
     int verbose = 0;
+    double switch_margin = 0.0;  // C38
     std::vector<std::vector<recflex_schedule_t>> cands;  // per feature
     recflex_status_t err = RECFLEX_OK;
     int64_t local_launches = 0, global_launches = 0;
@@ -621,7 +622,16 @@ struct Tuner {
     }
 };
 
-void cb_local(void *u, int32_t ki, int32_t f, double *costs) { static_cast<Tuner *>(u)->local_cost(ki, f, costs); }
+// Stage-1 costs as the selection sees them: with a switch margin (C38) every
+// candidate other than the incoming schedule (candidate 0) is charged
+// 1 / (1 - margin) x its measured cost, so a feature leaves its schedule only
+// for a predicted gain larger than the margin.
+void cb_local(void *u, int32_t ki, int32_t f, double *costs) {
+    Tuner *T = static_cast<Tuner *>(u);
+    T->local_cost(ki, f, costs);
+    if (T->switch_margin > 0.0)
+        for (int c = 1; c < (int)T->cands[f].size(); ++c) costs[c] /= (1.0 - T->switch_margin);
+}
 double cb_global(void *u, int32_t ki, const int32_t *choice) { return static_cast<Tuner *>(u)->global_cost(ki, choice); }
 
 std::vector<recflex_schedule_t> candidates_for(const recflex_plan_s *p, int f, int max_c) {
@@ -691,6 +701,10 @@ extern "C" recflex_status_t recflex_tune_ex(recflex_plan_t p, int32_t N, const i
     if (opt) T.separate = opt->local_mode == 1;
     if (opt) T.isolated = opt->local_mode == 2;
     if (opt) T.jit = opt->stage2_catalog == 0;
+    if (opt) {
+        if (!(opt->switch_margin >= 0.f && opt->switch_margin < 1.f)) return RECFLEX_ERR_INVALID_ARG;
+        T.switch_margin = opt->switch_margin;
+    }
     const int max_c = opt ? opt->max_candidates : 0;
     for (int i = 0; i < N; ++i) {
         if (batch_sizes[i] <= 0 || batch_sizes[i] > p->max_batch || !indices[i] || !offsets[i])

@@ -32,6 +32,8 @@ def main():
     ap.add_argument('--stage2-catalog', action='store_true', help='stage 2 on the catalog kernel (no NVRTC)')
     ap.add_argument('--no-tail', action='store_true', help="stage 1 = the paper's plain block-time sum")
     ap.add_argument('--isolated', action='store_true', help='stage 1: one padded launch per candidate (C34)')
+    ap.add_argument('--margin', type=float, default=0.0, help='stage-1 switch margin (reading C38)')
+    ap.add_argument('--no-post', action='store_true', help='skip the task-size / order / L2 selections')
     ap.add_argument('--from-tuned', action='store_true',
                     help='start from configs/tuned/<name>.json (its schedules, task order and column layout '
                          'are the incoming plan the guard compares against)')
@@ -69,7 +71,8 @@ def main():
         t0 = time.time()
         st = sh.plan.tune(hist, tables, occupancies=ks, reps=a.reps, max_candidates=a.max_candidates, verbose=True,
                           refine=a.refine, guard=not a.no_guard, stage2_catalog=a.stage2_catalog,
-                          tail=not a.no_tail, isolated=a.isolated)
+                          tail=not a.no_tail, isolated=a.isolated, switch_margin=a.margin,
+                          select_order=not a.no_post, select_l2=not a.no_post, select_task_size=not a.no_post)
         st['wall_s'] = time.time() - t0
         state = sh.plan.export()
         with open(os.path.join(a.out, name + '.json'), 'w') as fh:
