@@ -242,6 +242,9 @@ typedef struct {
     float switch_margin;     /* stage 1: a candidate other than the feature's incoming
                                 schedule must cost < (1 - margin) x the incoming one to be
                                 chosen (reading C38; 0 = the paper's plain argmin)         */
+    int32_t position_balance; /* 1: stage-1 launches list a feature's candidates in reverse
+                                on every other (batch, k), so no candidate always runs
+                                next to the pre- or the post-padding (reading C39)         */
 } recflex_tune_options_t;
 
 typedef struct {

@@ -41,7 +41,7 @@ class TuneOptions(ctypes.Structure):
                 ('verbose', ctypes.c_int32), ('skip_guard', ctypes.c_int32), ('refine', ctypes.c_int32),
                 ('local_mode', ctypes.c_int32), ('stage2_catalog', ctypes.c_int32), ('no_tail', ctypes.c_int32),
                 ('keep_order', ctypes.c_int32), ('keep_l2', ctypes.c_int32), ('keep_task_size', ctypes.c_int32),
-                ('switch_margin', ctypes.c_float)]
+                ('switch_margin', ctypes.c_float), ('position_balance', ctypes.c_int32)]
 
 
 class TuneStats(ctypes.Structure):

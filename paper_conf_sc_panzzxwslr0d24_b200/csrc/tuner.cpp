@@ -147,6 +147,7 @@ struct Tuner {
     double compile_seconds = 0;
     int verbose = 0;
     double switch_margin = 0.0;  // C38
+    bool position_balance = false;  // C39
     std::vector<std::vector<recflex_schedule_t>> cands;  // per feature
     recflex_status_t err = RECFLEX_OK;
     int64_t local_launches = 0, global_launches = 0;
@@ -356,7 +357,13 @@ struct Tuner {
             for (int c = 0; c < n; ++c) groups.back().push_back(c);
         }
         for (size_t i = 0; i < batches.size(); ++i)
-        for (const std::vector<int> &grp : groups) {
+        for (const std::vector<int> &grp0 : groups) {
+            // position balance (C39): the candidates' tasks follow one another in the
+            // launch, so the first ones overlap the pre-padding and the last ones the
+            // post-padding; every other (batch, k) lists them in reverse so each
+            // candidate sees both ends equally
+            std::vector<int> grp = grp0;
+            if (position_balance && ((i + (size_t)ki) & 1)) std::reverse(grp.begin(), grp.end());
             const Batch &bt = batches[i];
             TP &tp = tps[i];
             const int B = bt.B;
@@ -704,6 +711,7 @@ extern "C" recflex_status_t recflex_tune_ex(recflex_plan_t p, int32_t N, const i
     if (opt) {
         if (!(opt->switch_margin >= 0.f && opt->switch_margin < 1.f)) return RECFLEX_ERR_INVALID_ARG;
         T.switch_margin = opt->switch_margin;
+        T.position_balance = opt->position_balance != 0;
     }
     const int max_c = opt ? opt->max_candidates : 0;
     for (int i = 0; i < N; ++i) {

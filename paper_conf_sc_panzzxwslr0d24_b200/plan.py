@@ -397,7 +397,8 @@ class Plan:
              reps: int = 7, pad_waves: int = 4, max_candidates: int = 0, verbose: bool = False, guard: bool = True,
              refine: bool = False, separate: bool = False, stage2_catalog: bool = False, tail: bool = True,
              isolated: bool = False, select_order: bool = True, select_l2: bool = True,
-             select_task_size: bool = True, switch_margin: float = 0.0, stream=None) -> dict:
+             select_task_size: bool = True, switch_margin: float = 0.0, position_balance: bool = False,
+             stream=None) -> dict:
         """recflex_tune_ex over historical batches [(indices, offsets, B), ...]."""
         N = len(batches)
         idx_arr = (ctypes.c_void_p * N)(*[b[0].data_ptr() for b in batches])
@@ -421,6 +422,7 @@ class Plan:
         opt.keep_l2 = 0 if select_l2 else 1
         opt.keep_task_size = 0 if select_task_size else 1
         opt.switch_margin = float(switch_margin)
+        opt.position_balance = 1 if position_balance else 0
         st = _lib.TuneStats()
         check(lib.recflex_tune_ex(self._h, N, idx_arr, off_arr, bs_arr, self._tables(tables), _stream_ptr(stream),
                                   ctypes.byref(opt), ctypes.byref(st)), 'recflex_tune_ex')

@@ -34,6 +34,7 @@ def main():
     ap.add_argument('--isolated', action='store_true', help='stage 1: one padded launch per candidate (C34)')
     ap.add_argument('--margin', type=float, default=0.0, help='stage-1 switch margin (reading C38)')
     ap.add_argument('--no-post', action='store_true', help='skip the task-size / order / L2 selections')
+    ap.add_argument('--balance', action='store_true', help='stage 1: position-balanced candidates (reading C39)')
     ap.add_argument('--from-tuned', action='store_true',
                     help='start from configs/tuned/<name>.json (its schedules, task order and column layout '
                          'are the incoming plan the guard compares against)')
@@ -71,7 +72,7 @@ def main():
         t0 = time.time()
         st = sh.plan.tune(hist, tables, occupancies=ks, reps=a.reps, max_candidates=a.max_candidates, verbose=True,
                           refine=a.refine, guard=not a.no_guard, stage2_catalog=a.stage2_catalog,
-                          tail=not a.no_tail, isolated=a.isolated, switch_margin=a.margin,
+                          tail=not a.no_tail, isolated=a.isolated, switch_margin=a.margin, position_balance=a.balance,
                           select_order=not a.no_post, select_l2=not a.no_post, select_task_size=not a.no_post)
         st['wall_s'] = time.time() - t0
         state = sh.plan.export()
