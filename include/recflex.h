@@ -441,7 +441,10 @@ recflex_status_t recflex_get_columns(recflex_plan_t plan, int64_t *col);
 #define RECFLEX_L2_EVICT_FIRST 1  /* stream: rows rarely recur within a batch   */
 #define RECFLEX_L2_EVICT_LAST 2   /* keep: small table, rows recur              */
 #define RECFLEX_L2_KEEP_L1 3      /* keep, and allocate the rows in L1 as well  */
-/* policy[F] (values above) or NULL = default for every feature.  (KEEP_L1 was
+/* A new plan starts with the heuristic's EVICT_LAST part (below; L2 size from
+ * the device) and DEFAULT elsewhere; an imported plan without "l2" has
+ * DEFAULT everywhere.
+ * policy[F] (values above) or NULL = default for every feature.  (KEEP_L1 was
  * measured no better than EVICT_LAST on sharded1000 / industrial.)  Takes effect
  * in the next compiled plan-specialised kernel (part of its signature; the
  * catalog kernel ignores it).  INVALID_ARG on an unknown value.  Part of the

@@ -635,6 +635,18 @@ recflex_status_t recflex_plan_create(const recflex_feature_spec_t *specs, int32_
         delete p;
         return cuda_status(e);
     }
+    {
+        // default L2 policy (C36): the heuristic's evict_last part (recurring rows of
+        // small tables); evict_first is left to the measured selection
+        int l2 = 0;
+        cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, device);
+        std::vector<int32_t> pol(F);
+        if (l2 > 0 && recflex_l2_policy_heuristic(p, l2, pol.data()) == RECFLEX_OK) {
+            for (int32_t &v : pol)
+                if (v != RECFLEX_L2_EVICT_LAST) v = RECFLEX_L2_DEFAULT;
+            recflex_set_l2_policy(p, pol.data());
+        }
+    }
     if (const char *env = std::getenv("RECFLEX_OCCUPANCY")) {
         int k = std::atoi(env);
         if (k >= 1 && k <= kMaxOcc) p->k = k;

@@ -53,5 +53,5 @@ case $step in
     MARGINS="0 0.03 0.08" bash tools/tune_margin_study.sh
     MARGINS=0 EXTRA=--balance bash tools/tune_margin_study.sh
     bash tools/tune_catalog_study.sh ;;
-  *) sed -n 2,8p "$0"; echo "steps: order-probe l2-probe size-probe select select-ranks rebalance retune verify bench-all tuner-studies" ;;
+  *) sed -n 2,6p "$0"; echo "steps: order-probe l2-probe size-probe select select-ranks rebalance retune verify bench-all tuner-studies" ;;
 esac
