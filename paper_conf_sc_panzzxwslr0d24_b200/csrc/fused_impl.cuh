@@ -166,10 +166,12 @@ __device__ __forceinline__ void fill_slot(TaskSlot &S, int n, const FusedArgs &a
         S.f = f;
         S.s0 = s0;
         S.s1 = s1;
+        st_release(&S.state, 2);  // publish first: waiting warps need not wait for the prefetch below
 #ifndef RECFLEX_NO_L2PF
         if (s1 > s0) {
             // stage the task's contiguous lookup-ID range into L2 with one bulk
-            // prefetch (TMA engine)
+            // prefetch (TMA engine); its two offset loads are off the slot's
+            // publish path
             const int32_t *offs = a.offsets + (size_t)fd.in_feature * a.B;
             const int32_t j0 = __ldg(offs + s0), j1 = __ldg(offs + s1);
             const uintptr_t b = reinterpret_cast<uintptr_t>(a.indices + j0) & ~uintptr_t(15);
@@ -178,6 +180,7 @@ __device__ __forceinline__ void fill_slot(TaskSlot &S, int n, const FusedArgs &a
                 asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(b), "r"((unsigned)(e - b)) : "memory");
         }
 #endif
+        return;
     }
     st_release(&S.state, 2);
 }
