@@ -117,6 +117,12 @@ def _cpu_model():
     return platform.processor() or 'unknown'
 
 
+def l2_policy_summary(plan):
+    """How many features' row loads carry each L2 eviction priority (reading C36)."""
+    pol = plan.l2_policy
+    return {name: pol.count(i) for i, name in enumerate(plan.L2_POLICIES) if pol.count(i)}
+
+
 def task_order_name(plan):
     """Which order the plan's tasks are claimed in (reading C35): a heuristic's name or 'custom'."""
     order = plan.task_order
@@ -618,6 +624,7 @@ def main():
                                        f"regs, {jit['local_bytes']} B local)" if jit and jit['active'] else 'catalog'),
                             'kernel_selection': ksel,
                             'task_order': task_order_name(plan),
+                            'l2_policy': l2_policy_summary(plan),
                             'output_columns': ('task order (features concatenated in the order their tasks '
                                                'run; recflex_get_columns)' if plan.export().get('columns')
                                                else 'feature order'),
