@@ -303,3 +303,29 @@ def test_refine_partition_synthetic():
     p2, t2, log2 = refine_partition(parts, measure_fail, est, moves=3)
     assert p2 == parts and t2 == t  # every candidate of the slow rank skipped: nothing moves
     assert [e['step'] for e in log2] == ['start'] + ['skip'] * 6
+
+
+def test_column_order_with_task_order_columns():
+    """Rank plans whose outputs follow their task order (reading C35): the exchanged
+    layout lists each rank's features in LOCAL column order; column_order maps every
+    exchanged column back to its global column, for any per-rank permutation."""
+    m = synth.make_model('tiny')   # 4 fields of dim 16
+    col = np.cumsum([0] + m.dims)
+    rng = np.random.default_rng(0)
+    parts = [[0, 2], [3, 1]]
+    for _ in range(5):
+        local = [list(rng.permutation(p)) for p in parts]
+        order = column_order(m, local)
+        assert sorted(order.tolist()) == list(range(int(col[-1])))
+        pos = 0
+        for p in local:
+            for f in p:
+                assert order[pos:pos + m.dims[f]].tolist() == list(range(col[f], col[f + 1]))
+                pos += m.dims[f]
+    # exchanged rows regrouped by column_order reproduce the feature-order output
+    full = rng.standard_normal((4, int(col[-1])))
+    order = column_order(m, local)
+    exchanged = full[:, order]
+    back = np.empty_like(full)
+    back[:, order] = exchanged
+    assert np.array_equal(back, full)
