@@ -3,7 +3,8 @@ tasks are laid out in the task map -- and claimed by the persistent CTAs --
 must not change any output bit, in either kernel, for any mapping; the task map
 under an order is the oracle's per-feature task counts scanned in that order;
 the order travels with the exported plan; the backward scatters into the right
-tables under a permuted order."""
+tables under a permuted order.  (The full-size check of a plan with task-order columns is
+the tuned sharded1000 plan in test_gpu_parity / test_gpu_tuned_plans, which bench.py times.)"""
 import numpy as np
 import pytest
 import torch
@@ -202,33 +203,6 @@ def test_backward_under_order(mode):
     plan = P.Plan.from_model(m, max_batch=b.B)
     plan.task_order = np.random.default_rng(3).permutation(m.F).tolist()
     _check(_run(m, b, mode, plan=plan), mode)
-
-
-def test_column_order_full_size_sampled():
-    """sharded1000's tuned plan with its outputs in task order (the bench's
-    headline layout): sampled rows vs the oracle, reassembled by plan.columns."""
-    import json
-    import os
-    from fullsize import sampled_oracle
-    P = _P()
-    m = synth.make_model('sharded1000')
-    b = synth.make_batch(m, 9)
-    dev = torch.device('cuda', 0)
-    phys = [synth.make_table(t, r, d, 'int', device=dev, seed=m.seed) for t, (r, d) in enumerate(m.tables)]
-    tables = [phys[f.table] for f in m.features]
-    plan = P.Plan.from_model(m)
-    path = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), 'configs', 'tuned',
-                        'sharded1000_w1_r0.json')
-    plan.import_(json.load(open(path)))
-    plan.set_column_order(True)
-    plan.task_order = plan.task_order_heuristic('lpt')
-    plan.compile()
-    out = plan.forward(torch.from_numpy(b.indices).to(dev), torch.from_numpy(b.offsets).to(dev), b.B, tables)
-    samples = np.unique(np.concatenate([[0, b.B - 1], np.random.default_rng(0).choice(b.B, 1024, replace=False)]))
-    got = _to_feature_columns(out.cpu().numpy()[samples], plan, m.dims)
-    ref, _ = sampled_oracle(m, b, samples, tables)
-    assert plan.columns != np.cumsum([0] + m.dims)[:-1].tolist()
-    assert bitexact(got, ref)
 
 
 @pytest.mark.parametrize('order', ['feature', 'lpt'])
