@@ -421,7 +421,8 @@ recflex_status_t recflex_debug_task_need(recflex_plan_t plan, int32_t *host_need
 #define RECFLEX_NUM_ORDERS 3
 /* order[F]: a permutation of 0..F-1 (position -> feature) or NULL = feature
  * order.  INVALID_ARG if not a permutation.  Setup call: synchronises the
- * device.  Part of the exported plan ("order"). */
+ * device and uploads the plan's device arrays at once, so a CUDA graph captured
+ * earlier replays in the new order.  Part of the exported plan ("order"). */
 recflex_status_t recflex_set_task_order(recflex_plan_t plan, const int32_t *order);
 /* Output layout: follow_task_order = 0 (default) -> out[s][col_f..col_f+d_f)
  * with the features concatenated in feature order (the paper's); 1 -> in the

@@ -434,6 +434,15 @@ recflex_status_t set_layout(recflex_plan_s *p, const std::vector<int32_t> &order
     p->columns_follow_order = follow;
     p->desc_dirty = true;
     p->targets_cache.clear();
+    // the device descriptors (columns, schedules, order) and the compiled
+    // kernels' variant ids change together, now: a CUDA graph captured earlier
+    // replays on these arrays without an eager forward to upload them
+    recflex_status_t st = upload_desc(p, nullptr);
+    if (st == RECFLEX_OK) {
+        e = cudaStreamSynchronize(nullptr);
+        if (e != cudaSuccess) st = cuda_status(e);
+    }
+    if (st != RECFLEX_OK) return st;
     return order_changed ? jit_upload_var(p) : RECFLEX_OK;
 }
 

@@ -226,3 +226,31 @@ def test_select_task_size_keeps_parity(order):
     _, out = run_plan(case, plan)
     ref, _ = case.oracle()
     assert bitexact(feature_columns(out, plan, m.dims), ref)
+
+
+def test_order_change_under_captured_graph():
+    """A CUDA graph captured before recflex_set_task_order replays consistently after it:
+    the device descriptors and the compiled kernel's variant ids change together (the
+    descriptors are uploaded by the setter, not deferred to the next eager forward)."""
+    P = _P()
+    m = _mixed_model()
+    b = synth.make_batch(m, 8)
+    case = Case(m, b, 'int')
+    ref, _ = case.oracle()
+    plan = P.Plan.from_model(m, max_batch=b.B)
+    plan.compile()
+    out = torch.empty((b.B, m.d_tot), device='cuda')
+    plan.forward(case.idx, case.off, b.B, case.tables, out=out)   # uploads descriptors before capture
+    torch.cuda.synchronize()
+    s = torch.cuda.Stream()
+    s.wait_stream(torch.cuda.current_stream())
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        plan.forward(case.idx, case.off, b.B, case.tables, out=out, stream=s)
+    torch.cuda.current_stream().wait_stream(s)
+    for order in (np.random.default_rng(5).permutation(m.F).tolist(), list(range(m.F))[::-1], None):
+        plan.task_order = order
+        out.zero_()
+        g.replay()
+        torch.cuda.synchronize()
+        assert bitexact(out.cpu().numpy(), ref), order
