@@ -44,6 +44,15 @@ def main():
         'class_asc_lpt': list(np.lexsort((rank_lpt, cls))),
         'class_desc_lpt': list(np.lexsort((rank_lpt, -cls))),
     }
+    rng = np.random.default_rng(11)
+    for i in range(int(os.environ.get('ORDER_PROBE_RANDOM', '0'))):
+        orders[f'random{i}'] = list(rng.permutation(m.F))
+        # LPT with random swaps of neighbours (a local perturbation)
+        o = list(lpt)
+        for _ in range(m.F // 4):
+            a_ = int(rng.integers(0, m.F - 1))
+            o[a_], o[a_ + 1] = o[a_ + 1], o[a_]
+        orders[f'lpt_jitter{i}'] = o
     for name, order in orders.items():
         plan.task_order = [int(x) for x in order]
         ts = []
