@@ -351,7 +351,8 @@ def main():
     if not args.no_jit:
         jit = plan.compile()
         # stage 2 over the plan's two kernels (plan-specialised vs catalog) on the first batch
-        ksel = plan.select_kernel(batches[0][0], batches[0][1], B, tables, reps=5)
+        # small (latency-bound) steps are noisy at 5 repetitions: time them longer
+        ksel = plan.select_kernel(batches[0][0], batches[0][1], B, tables, reps=5 if alg_local > 1e9 else 31)
         if not plan.jit_enabled:
             jit = dict(jit, active=0)
 
