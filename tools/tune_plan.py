@@ -33,6 +33,7 @@ def main():
     ap.add_argument('--no-tail', action='store_true', help="stage 1 = the paper's plain block-time sum")
     ap.add_argument('--isolated', action='store_true', help='stage 1: one padded launch per candidate (C34)')
     ap.add_argument('--margin', type=float, default=0.0, help='stage-1 switch margin (reading C38)')
+    ap.add_argument('--pad-waves', type=int, default=4, help='stage-1 padding in waves of tasks (P:148)')
     ap.add_argument('--no-post', action='store_true', help='skip the task-size / order / L2 selections')
     ap.add_argument('--balance', action='store_true', help='stage 1: position-balanced candidates (reading C39)')
     ap.add_argument('--from-tuned', action='store_true',
@@ -72,7 +73,7 @@ def main():
         t0 = time.time()
         st = sh.plan.tune(hist, tables, occupancies=ks, reps=a.reps, max_candidates=a.max_candidates, verbose=True,
                           refine=a.refine, guard=not a.no_guard, stage2_catalog=a.stage2_catalog,
-                          tail=not a.no_tail, isolated=a.isolated, switch_margin=a.margin, position_balance=a.balance,
+                          tail=not a.no_tail, isolated=a.isolated, switch_margin=a.margin, position_balance=a.balance, pad_waves=a.pad_waves,
                           select_order=not a.no_post, select_l2=not a.no_post, select_task_size=not a.no_post)
         st['wall_s'] = time.time() - t0
         state = sh.plan.export()
