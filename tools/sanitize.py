@@ -1,4 +1,7 @@
-"""Small forwards for compute-sanitizer (memcheck / racecheck / synccheck / initcheck)."""
+"""Small forwards for compute-sanitizer (memcheck / racecheck / synccheck / initcheck).
+
+(compute-sanitizer is closed on the round-2 GPU pool; the families still run as plain
+forwards, and the GPU tests compare the same paths with the oracle.)"""
 import os
 import sys
 
@@ -23,7 +26,7 @@ phys = [synth.make_table(t, r, d, 'int', device=dev) for t, (r, d) in enumerate(
 tables = [phys[f.table] for f in m.features]
 bi, bo = torch.from_numpy(b.indices).to(dev), torch.from_numpy(b.offsets).to(dev)
 cat = catalog()
-fams = sys.argv[1:] or ['group', 'flat', 'block', 'warp', 'jit', 'static', 'exchange', 'bwd', 'kjt', 'host']
+fams = sys.argv[1:] or ['group', 'flat', 'block', 'warp', 'jit', 'static', 'order', 'exchange', 'bwd', 'kjt', 'host']
 for fam in fams:
     if fam in ('jit', 'static'):
         # plan-specialised kernels: every family in one compiled kernel, runtime or static mapping
@@ -47,6 +50,32 @@ for fam in fams:
             n += 1
         torch.cuda.synchronize()
         print(fam, 'forwards', n)
+        continue
+    if fam == 'order':
+        # task order (C35) with task-order columns, every L2 policy (C36), halved task sizes
+        # (C37) and lookup-partitioned features (the one-wave fill kernel), in both kernels
+        import numpy as np
+        plan = Plan.from_model(m)
+        for f in range(m.F):
+            s = plan.get_schedule(f)
+            plan.set_schedule(f, s['sched_id'], f % 2, 8 if f % 2 == 0 else 24)
+        rng = np.random.default_rng(1)
+        n = 0
+        for rnd, cols in enumerate((False, True)):
+            try:
+                plan.set_column_order(cols)
+            except Exception:
+                pass
+            for jit in (False, True):
+                plan.task_order = rng.permutation(m.F).tolist()
+                plan.l2_policy = [(f + rnd) % 4 for f in range(m.F)]
+                if jit:
+                    plan.compile()
+                plan.set_jit(jit)
+                plan.forward(bi, bo, b.B, tables)
+                n += 1
+        torch.cuda.synchronize()
+        print('order forwards', n)
         continue
     if fam == 'exchange':
         # recflex_forward_exchange with one rank (its own buffers and flags): kernel epilogue
